@@ -1,0 +1,379 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 MoE routed-expert layer (BASELINE.json metric:
+"MoE-layer prefill tokens/s & decode µs/layer; % of HBM or tensor peak").
+
+A step = one full forward of the layer -- router logits, score/group top-k,
+count/permute, FP8 activation quantisation, gather, grouped GEMM1+SwiGLU,
+grouped GEMM2, shared expert, weighted combine -- over one batch of synthetic
+tokens shaped like the DeepSeek-V3 MoE layer (256 routed experts in 8 groups,
+top-4 groups, top-8, H 7168, F 2048, 1 shared expert, FP8 128x128 block-scaled
+weights; BASELINE.json configs[4]), prefill T = 8192 tokens per GPU.
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference]
+
+N > 1: one process per GPU (torchrun), each rank runs an independent replica of
+the layer on its own tokens (weak scaling, no data-path collective; DESIGN.md
+§7), value = all ranks' tokens / max-over-ranks time.
+
+Inputs are resident in HBM when the timed region starts; L2 is flushed (a
+256 MiB write, outside the timed events) before every timed step.  Each step is
+timed with CUDA events on the launching stream.  `e2e` re-times the same step
+through the public API with host (pinned) input/output buffers, H2D and D2H
+inside the events.  The oracle (oracle/, a plain fp64 CPU program) is timed on
+a bounded sample for `cpu_baseline` and, with --impl reference, as the
+reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "MoE-layer prefill tokens/s & decode µs/layer; % of HBM or tensor peak"
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        d["_source"] = "measured (MEASURED_PEAKS.json)"
+        return d
+    d = dict(PEAKS_FALLBACK)
+    d["_source"] = "fallback (B200_PROFILING.md)"
+    return d
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [s.strip() for s in line.split(",")]
+            if len(parts) == 7:
+                self.rows.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            self.proc.wait(timeout=5)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = sorted(float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit())
+        mx = max(float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit())
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower() == "active"})
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": mx, "reasons": reasons,
+                "samples": len(self.rows)}
+
+
+def dist_setup():
+    import torch
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if ws > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(local)
+    return ws, rank, local
+
+
+def barrier(ws):
+    if ws > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def max_over_ranks(v: float, ws: int) -> float:
+    if ws == 1:
+        return v
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+# --------------------------------------------------------------------- oracle
+def oracle_tokens_per_s(p, w, x_rows, budget_s: float = 25.0):
+    """Time the CPU oracle (as it stands) on a bounded sample of tokens."""
+    import numpy as np
+    import torch
+    from oracle import moe_oracle as O
+    from tests.parity import oracle_cfg, oracle_weights
+    cfg, W = oracle_cfg(p), oracle_weights(p, w)
+    done, t0 = 0, time.perf_counter()
+    for i in range(x_rows.shape[0]):
+        O.moe_layer(x_rows[i:i + 1].cpu().to(torch.float64).numpy(), W, cfg)
+        done += 1
+        if time.perf_counter() - t0 > budget_s:
+            break
+    dt = time.perf_counter() - t0
+    return done / dt, done, dt
+
+
+def cpu_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count()
+
+
+def run_reference(args):
+    """--impl reference: the oracle timed on the host cores, same metric/config."""
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import torch
+    from inputs.presets import PRESETS
+    from inputs.synthetic import make_tokens, make_weights
+    p = PRESETS[args.config]
+    dev = "cuda" if torch.cuda.is_available() else "cpu"
+    w = make_weights(p, dev)
+    x, _ = make_tokens(p, args.steps + args.warmup, dev)
+    from oracle import moe_oracle as O
+    from tests.parity import oracle_cfg, oracle_weights
+    cfg, W = oracle_cfg(p), oracle_weights(p, w)
+    for i in range(args.warmup):
+        O.moe_layer(x[i:i + 1].cpu().to(torch.float64).numpy(), W, cfg)
+    t0 = time.perf_counter()
+    for i in range(args.steps):
+        j = args.warmup + i
+        O.moe_layer(x[j:j + 1].cpu().to(torch.float64).numpy(), W, cfg)
+    dt = time.perf_counter() - t0
+    v = args.steps / dt
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "tokens/s", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": f"{p.name}_moe_layer_prefill", "tokens_per_step": 1},
+            "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": cpu_cores(), "kind": "oracle",
+                             "sample": f"1 token per step of the {p.name} layer (fp64 numpy oracle, "
+                                       "experts dequantised per call)"},
+            "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# --------------------------------------------------------------------- ours
+def algorithmic(p, T, n_distinct):
+    """Algorithmic FLOPs / bytes per stage."""
+    H, F, Fs, k, E = p.hidden, p.ffn, p.shared_ffn, p.top_k, p.n_experts
+    wb = 1 if p.wtype == 1 else 2
+    exp_bytes = 3 * H * F * wb + (3 * (H // 128) * (F // 128) * 4 if p.wtype == 1 else 0)
+    return {
+        "gemm1_swiglu": {"flops": 2.0 * T * k * 2 * F * H, "bytes": n_distinct * 2 * H * F * wb},
+        "gemm2": {"flops": 2.0 * T * k * H * F, "bytes": n_distinct * H * F * wb},
+        "shared_gemm1": {"flops": 2.0 * T * 2 * Fs * H, "bytes": 2 * H * Fs * wb},
+        "shared_gemm2": {"flops": 2.0 * T * H * Fs, "bytes": H * Fs * wb},
+        "router_logits": {"flops": 2.0 * T * H * E, "bytes": E * H * 2 + T * H * 2},
+        "layer_bytes": n_distinct * exp_bytes + (3 * H * Fs * wb if Fs else 0) + E * H * 2 + 2 * T * H * 2,
+        "layer_flops": 2.0 * T * k * 3 * H * F + 2.0 * T * 3 * H * Fs + 2.0 * T * H * E,
+    }
+
+
+def timed_steps(layer, xs, y, steps, warmup, flush, profile=True):
+    """Per-step CUDA-event times (ms) and per-stage ms; xs: list of inputs cycled."""
+    import torch
+    st = torch.cuda.current_stream()
+    for i in range(warmup):
+        layer.forward(xs[i % len(xs)], y=y)
+    torch.cuda.synchronize()
+    if profile:
+        layer.profile(True)
+    times, stages = [], {}
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    for i in range(steps):
+        flush.zero_()
+        e0.record(st)
+        layer.forward(xs[(warmup + i) % len(xs)], y=y)
+        e1.record(st)
+        e1.synchronize()
+        times.append(e0.elapsed_time(e1))
+        if profile:
+            for k, v in layer.stage_times().items():
+                stages.setdefault(k, []).append(v)
+    if profile:
+        layer.profile(False)
+    return times, {k: sum(v) / len(v) for k, v in stages.items()}
+
+
+def run_ours(args):
+    import torch
+    ws, rank, local = dist_setup()
+    from paper_conf_sosp_chenxztwdcylqzo25_b200 import build as b
+    if rank == 0:
+        b.build()
+    barrier(ws)
+    from inputs.presets import PRESETS
+    from inputs.synthetic import make_tokens, make_weights
+    from paper_conf_sosp_chenxztwdcylqzo25_b200 import moe
+    peaks = load_peaks()
+    p = PRESETS[args.config]
+    T = args.tokens or p.prefill_tokens
+    w = make_weights(p, "cuda")
+    x, _ = make_tokens(p, T, "cuda", offset=rank)
+    y = torch.empty_like(x)
+    layer = moe.MoELayer(p, w, max_tokens=T, device=local)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    info = layer.info()
+
+    # ---------------- prefill, device-resident inputs ----------------
+    barrier(ws)
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        times, stages = timed_steps(layer, [x], y, args.steps, args.warmup, flush)
+    torch.cuda.synchronize()
+    barrier(ws)
+    ms = max_over_ranks(sum(times) / len(times), ws)
+    value = ws * T / (ms * 1e-3)
+
+    # routing statistics of this batch (distinct experts hit, for the byte counts)
+    routing = {}
+    layer.forward(x, y=y, routing=routing)
+    counts = routing["expert_counts"].cpu()
+    n_distinct = int((counts > 0).sum())
+    alg = algorithmic(p, T, n_distinct)
+    fp8 = p.wtype == 1
+    tc_peak = (2.0 if fp8 else 1.0) * peaks["bf16_tflops_sustained"]
+    dom = max((k for k in stages if k in alg), key=lambda k: stages[k])
+    ach = alg[dom]["flops"] / (stages[dom] * 1e-3) / 1e12
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        traffic = json.load(open(tpath)).get(f"{p.name}:{T}:{dom}")
+    roofline = {"bound": "tensor", "kernel": dom, "achieved": ach, "peak": tc_peak, "unit": "TFLOP/s",
+                "frac": ach / tc_peak, "traffic": traffic,
+                "peak_source": f"{peaks['_source']}: bf16_tflops_sustained x {'2 (fp8/bf16 nominal ratio)' if fp8 else '1'}",
+                "algorithmic": f"2*T*k*{'2F*H' if dom == 'gemm1_swiglu' else 'H*F'} flops per launch, T={T}",
+                "stage_ms": {k: round(v, 4) for k, v in stages.items()}}
+    layer_tflops = alg["layer_flops"] / (ms * 1e-3) / 1e12
+
+    # ---------------- decode, T = 1 (distinct tokens, L2 flushed) ----------------
+    decode = None
+    if not args.no_decode:
+        xd, _ = make_tokens(p, args.steps + args.warmup, "cuda", offset=1000 + rank)
+        rows = [xd[i:i + 1].contiguous() for i in range(xd.shape[0])]
+        yd = torch.empty_like(rows[0])
+        dtimes, dstages = timed_steps(layer, rows, yd, args.steps, args.warmup, flush)
+        dus = max_over_ranks(sum(dtimes) / len(dtimes), ws) * 1e3
+        algd = algorithmic(p, 1, p.top_k)
+        decode = {"us_per_layer": dus, "tokens": 1,
+                  "roofline": {"bound": "hbm", "achieved": algd["layer_bytes"] / (dus * 1e-6) / 1e9,
+                               "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                               "frac": algd["layer_bytes"] / (dus * 1e-6) / 1e9 / peaks["hbm_gbs"],
+                               "bytes": algd["layer_bytes"],
+                               "stage_us": {k: round(v * 1e3, 2) for k, v in dstages.items()}}}
+
+    # ---------------- e2e through the public API, host buffers ----------------
+    e2e = None
+    if not args.no_e2e:
+        xh = x.cpu().pin_memory()
+        yh = torch.empty_like(xh).pin_memory()
+        xdev = torch.empty_like(x)
+        st = torch.cuda.current_stream()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        for _ in range(args.warmup):
+            xdev.copy_(xh, non_blocking=True)
+            layer.forward(xdev, y=y)
+            yh.copy_(y, non_blocking=True)
+        torch.cuda.synchronize()
+        et = []
+        for _ in range(args.steps):
+            flush.zero_()
+            e0.record(st)
+            xdev.copy_(xh, non_blocking=True)
+            layer.forward(xdev, y=y)
+            yh.copy_(y, non_blocking=True)
+            e1.record(st)
+            e1.synchronize()
+            et.append(e0.elapsed_time(e1))
+        ems = max_over_ranks(sum(et) / len(et), ws)
+        e2e = {"value": ws * T / (ems * 1e-3), "unit": "tokens/s", "h2d_bytes_per_step": int(x.numel() * 2),
+               "d2h_bytes_per_step": int(y.numel() * 2), "ms_per_step": ems}
+
+    # ---------------- CPU oracle on a bounded sample (rank 0, N = 1) ----------------
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu:
+        v, n, dt = oracle_tokens_per_s(p, w, x[:64], budget_s=args.cpu_budget)
+        cpu = {"value": v, "unit": "tokens/s", "cores": cpu_cores(), "kind": "oracle",
+               "sample": f"{n} tokens of the same batch, one oracle call per token ({dt:.1f} s, fp64 numpy, "
+                         "experts dequantised per call)"}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": ws, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "e4m3" if fp8 else "bf16", "data": "synthetic",
+                "config": {"workload": f"{p.name}_moe_layer_prefill", "tokens_per_gpu": T, "hidden": p.hidden,
+                           "ffn": p.ffn, "experts": p.n_experts, "top_k": p.top_k, "shared_ffn": p.shared_ffn,
+                           "weights": "fp8_e4m3_block128_ue8m0" if fp8 else "bf16", "parallelism":
+                           f"replica x{ws}" if ws > 1 else "single", "l2": "flushed before every step (256 MiB write, "
+                           "outside the timed events); inputs resident in HBM",
+                           "distinct_experts_hit": n_distinct},
+                "layer_tflops": layer_tflops,
+                "roofline": roofline, "decode": decode, "e2e": e2e, "cpu_baseline": cpu,
+                "gpu_launches": info.kernels_per_forward_prefill * args.steps,
+                "clocks": clk.summary()}
+        print(json.dumps(line), flush=True)
+    layer.close()
+    if ws > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="v3")
+    ap.add_argument("--tokens", type=int, default=0)
+    ap.add_argument("--no-decode", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=20.0)
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "ours":
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

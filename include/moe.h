@@ -1,0 +1,180 @@
+/*
+ * moe.h -- C ABI of the B200-native MoE routed-expert layer.
+ *
+ * The operation (PAPER.md = the KTransformers paper, SOSP'25; L<n> = line n):
+ *
+ *   O_k = I_k + S_k(I_k) + R_k^all(I_k)                               (L219, §4.1)
+ *   O_k = I_k + S_k(I_k) + R_{k-1}^def(I_{k-1}) + R_k^imm(I_k)         (L241, §4.1)
+ *
+ * R_k: routed experts chosen per token by the gate, "top-k or its variants
+ * (e.g., grouped top-k in DeepSeek-V3/R1)" (L98, §2.1); S_k: shared experts
+ * "activated across all tokens" (L98); deferred experts are the lowest-scoring
+ * selected experts, whose output joins one layer later (L215, Fig. 9b).
+ * Gate and expert FFN follow the public DeepSeek-V2/V3 and Qwen2-MoE
+ * definitions the paper evaluates (reading R1):
+ *   s = sigmoid(x Wg^T) | softmax(x Wg^T); sel = s + bias; optional group limit;
+ *   idx = top_k(sel); w = s[idx] (/ sum if norm_topk) * routed_scale;
+ *   FFN_e(x) = W2_e (silu(W1_e x) * W3_e x).
+ *
+ * Conventions (all functions):
+ *   - Every pointer documented "device" is a CUDA device pointer on
+ *     config.device; "host" pointers are ordinary host memory.
+ *   - Nothing aborts.  Errors are returned as moe_status; moe_last_error()
+ *     gives a thread-local detail string.  Asynchronous device faults surface
+ *     at the caller's next synchronisation (normal CUDA convention).
+ *   - A handle is not reentrant: one forward at a time per handle (the
+ *     workspace is single-stream).
+ */
+#ifndef MOE_B200_H
+#define MOE_B200_H
+
+#include <stdint.h>
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct moe_layer moe_layer; /* opaque, library-owned */
+
+typedef enum {
+  MOE_OK = 0,
+  MOE_ERR_INVALID_ARG = -1, /* bad pointer / size / enum / n_deferred          */
+  MOE_ERR_UNSUPPORTED = -2, /* shape or dtype the kernels do not implement     */
+  MOE_ERR_OOM = -3,         /* device allocation failed at create              */
+  MOE_ERR_CUDA = -4,        /* a CUDA runtime call or kernel launch failed     */
+  MOE_ERR_NCCL = -5,        /* an NCCL call failed (expert parallel)           */
+  MOE_ERR_CAPACITY = -6     /* T > max_tokens                                  */
+} moe_status;
+
+typedef enum { MOE_SCORE_SOFTMAX = 0, MOE_SCORE_SIGMOID = 1 } moe_score_fn;
+/* group score of group-limited routing (n_group > 1):
+ * MAX = DeepSeek-V2/V2.5 group_limited_greedy; TOP2_SUM = DeepSeek-V3.       */
+typedef enum { MOE_GROUP_MAX = 0, MOE_GROUP_TOP2_SUM = 1 } moe_group_score;
+/* weight storage: BF16; e4m3 codes + one fp32 power-of-two scale per 128x128
+ * block (reading R10: UE8M0 block scaling, north_star "128x128
+ * block-scaled FP8"); F32 (toy config only).                                 */
+typedef enum { MOE_W_BF16 = 0, MOE_W_FP8_BLOCK128 = 1, MOE_W_F32 = 2 } moe_wtype;
+
+typedef struct {
+  int32_t hidden;            /* H, multiple of 128                                   */
+  int32_t ffn;               /* F of one routed expert, multiple of 128              */
+  int32_t n_experts;         /* E, global number of routed experts (<= 1024)         */
+  int32_t top_k;             /* k, 1 <= k <= 32, k <= E                              */
+  int32_t n_group;           /* 1 => plain top-k; else E % n_group == 0, n_group<=32 */
+  int32_t topk_group;        /* groups kept (1 <= topk_group <= n_group)             */
+  int32_t group_score;       /* moe_group_score                                      */
+  int32_t score_fn;          /* moe_score_fn                                         */
+  int32_t norm_topk;         /* 1 => w /= sum(w) before routed_scale                 */
+  float routed_scale;        /* multiplies the combine weights                      */
+  int32_t shared_ffn;        /* Fs (multiple of 128); 0 => no shared expert          */
+  int32_t shared_gated;      /* 1 => shared output *= sigmoid(x . w_sg) (Qwen2)      */
+  int32_t wtype;             /* moe_wtype                                            */
+  int32_t max_tokens;        /* per-rank capacity; every workspace sized at create   */
+  int32_t gemv_max_tokens;   /* T <= this => weight-streaming (decode) kernels;
+                                0 => library default (the L170 switch) */
+  int32_t device;            /* CUDA device ordinal                                  */
+  int32_t ep_rank, ep_size;  /* expert parallel group; ep_size 1 => single GPU       */
+  const void *nccl_unique_id;/* host, 128 bytes (ncclUniqueId) when ep_size > 1      */
+} moe_layer_config;
+
+/* Weights: DEVICE pointers, row-major, read at create and copied + repacked into
+ * library-owned memory (the paper's load-time repack, L157); the caller may
+ * free them after moe_layer_create returns.  With ep_size = P each rank passes
+ * its contiguous slice of E/P experts (rank r owns [r*E/P, (r+1)*E/P)).
+ *   gate_w      [E, H]      bf16 (the full router on every rank)
+ *   gate_bias   [E]         fp32 or NULL (selection-only bias, DeepSeek-V3)
+ *   w13         [E/P, 2F, H]  rows 0..F-1 = W1 (gate_proj), F..2F-1 = W3 (up_proj)
+ *   w2          [E/P, H, F]   W2 (down_proj)
+ *   *_scale     FP8 only: fp32 powers of two, [.., rows/128, cols/128]
+ *   ws13, ws2   shared expert [2Fs, H], [H, Fs] (same dtype/scales as routed)
+ *   shared_gate_w [H] bf16 or NULL (required iff shared_gated)               */
+typedef struct {
+  const void *gate_w;  const float *gate_bias;
+  const void *w13;     const float *w13_scale;
+  const void *w2;      const float *w2_scale;
+  const void *ws13;    const float *ws13_scale;
+  const void *ws2;     const float *ws2_scale;
+  const void *shared_gate_w;
+} moe_layer_weights;
+
+/* Optional DEVICE outputs for parity checks (any member may be NULL):
+ *   topk_idx      [T, k] int32  expert ids in canonical slot order
+ *                               (combine weight descending, ties -> lower id)
+ *   topk_w        [T, k] fp32   combine weights in the same order
+ *   expert_counts [E]    int32  tokens routed to each expert (this rank's tokens)
+ *   perm          [T*k]  int32  token index of every row of the expert-sorted
+ *                               order (stable: by expert, then token)          */
+typedef struct {
+  int32_t *topk_idx;
+  float *topk_w;
+  int32_t *expert_counts;
+  int32_t *perm;
+} moe_routing_out;
+
+/* ncclGetUniqueId for the expert-parallel bootstrap (rank 0 calls it and
+ * broadcasts the 128 bytes through the launcher's process group).            */
+moe_status moe_get_unique_id(void *out128);
+
+/* Validate the config, allocate all workspaces for max_tokens and copy/repack
+ * the weights.  Synchronous (returns after the copies are done).  *out is set
+ * to NULL on failure.  With ep_size > 1 this is collective over the EP group. */
+moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights *w,
+                            moe_layer **out);
+
+/* y = residual + S(x) + R^all(x)   (Eq. L219), stream-ordered on `stream`
+ * (a cudaStream_t; NULL = legacy default stream), no host synchronisation and
+ * no allocation on the single-GPU path (CUDA-Graph capturable, L193).
+ *   x         device [T, H] bf16, 16-byte aligned
+ *   residual  device [T, H] bf16 or NULL (NULL => no I_k term, reading R7)
+ *   y         device [T, H] bf16; may alias residual, must not alias x
+ *   T         0 <= T <= max_tokens (T == 0 is legal and launches nothing)
+ *   dbg       NULL or routing outputs (see moe_routing_out)                   */
+moe_status moe_layer_forward(moe_layer *layer, const void *x, const void *residual, int32_t T,
+                             void *y, moe_routing_out *dbg, void *stream);
+
+/* Expert Deferral (Eq. L241): the last n_deferred slots of each token's
+ * canonical order are deferred.
+ *   y            = residual + S(x) + R^imm(x) + deferred_in
+ *   deferred_out = R^def(x)
+ * deferred_in  device [T, H] bf16 or NULL (NULL: first layer, k = 1 case)
+ * deferred_out device [T, H] bf16 or NULL (NULL: last layer, k = L case -- all
+ *              experts immediate, L215 "not applied at the final layer")
+ * 0 <= n_deferred <= k-1, else MOE_ERR_INVALID_ARG.  n_deferred = 0 with both
+ * NULL is exactly moe_layer_forward.                                          */
+moe_status moe_layer_forward_deferred(moe_layer *layer, const void *x, const void *residual,
+                                      int32_t T, int32_t n_deferred, const void *deferred_in,
+                                      void *y, void *deferred_out, moe_routing_out *dbg,
+                                      void *stream);
+
+/* Free every library allocation (and the NCCL communicator).  NULL is a no-op. */
+moe_status moe_layer_destroy(moe_layer *layer);
+
+const char *moe_status_string(moe_status s);
+const char *moe_last_error(void);
+
+/* Introspection for tests and the bench (host-only, no device work). */
+typedef struct {
+  int64_t weight_bytes;      /* library-owned weight bytes (after repack)          */
+  int64_t workspace_bytes;   /* library-owned workspace bytes                       */
+  int32_t gemv_max_tokens;   /* effective decode/prefill switch                     */
+  int32_t kernels_per_forward_prefill; /* launches of one forward, GEMM path        */
+  int32_t kernels_per_forward_decode;  /* launches of one forward, GEMV path        */
+  int32_t local_experts;     /* E / ep_size                                         */
+} moe_layer_info;
+moe_status moe_layer_get_info(const moe_layer *layer, moe_layer_info *info);
+
+/* Stage timing (instrumentation for the bench's roofline figures; off by
+ * default).  When enabled, forward records a CUDA event after every stage on
+ * the forward's stream (adds no synchronisation).  moe_layer_stage_times waits
+ * for the last recorded forward and writes the elapsed ms of each stage
+ * (n_out = number of stages, at most cap; stages not run in that forward give
+ * 0).  moe_stage_name(i) names stage i ("router_logits", "gemm1", ...).      */
+moe_status moe_layer_profile(moe_layer *layer, int32_t enable);
+moe_status moe_layer_stage_times(moe_layer *layer, float *ms_out, int32_t cap, int32_t *n_out);
+const char *moe_stage_name(int32_t i);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MOE_B200_H */

@@ -247,11 +247,13 @@ def act_quant_e4m3(v: np.ndarray, block: int = 128) -> np.ndarray:
 
 
 def dequant_block128(codes: np.ndarray, scales: np.ndarray) -> np.ndarray:
-    """W[r, c] = e4m3(codes[r, c]) * scales[r // 128, c // 128]."""
-    w = e4m3_decode(codes)
+    """W[r, c] = e4m3(codes[r, c]) * scales[r // 128, c // 128].
+    (e4m3_decode evaluated once per code value as a 256-entry table.)"""
+    table = e4m3_decode(np.arange(256, dtype=np.uint8))
+    w = table[np.asarray(codes, np.uint8)]
     r, c = w.shape
-    sfull = np.repeat(np.repeat(np.asarray(scales, F64), 128, axis=0), 128, axis=1)[:r, :c]
-    return w * sfull
+    w = w.reshape(r // 128, 128, c // 128, 128) * np.asarray(scales, F64)[:, None, :, None]
+    return w.reshape(r, c)
 
 
 # --------------------------------------------------------------------------

@@ -1,0 +1,132 @@
+// common.cuh -- shared device helpers and the layer's internal state.
+// Nothing here is shared with oracle/ (the CPU checker); see DESIGN.md §2.
+#pragma once
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <cuda_fp8.h>
+#include <stdint.h>
+
+#include "../../include/moe.h"
+
+namespace moe {
+
+constexpr int kPadM = 128;       // expert segments of the sorted order are padded to this
+constexpr int kChunkTokens = 256; // token chunk of the deterministic permutation
+
+// ---------------------------------------------------------------- conversions
+__device__ __forceinline__ float bf2f(__nv_bfloat16 v) { return __bfloat162float(v); }
+
+__device__ __forceinline__ void bf16x8_to_f32(const uint4 &u, float *f) {
+  const __nv_bfloat162 *p = reinterpret_cast<const __nv_bfloat162 *>(&u);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    float2 t = __bfloat1622float2(p[i]);
+    f[2 * i] = t.x;
+    f[2 * i + 1] = t.y;
+  }
+}
+
+__device__ __forceinline__ void fp8x8_to_f32(const uint2 &u, float *f) {
+  const __nv_fp8x2_storage_t *p = reinterpret_cast<const __nv_fp8x2_storage_t *>(&u);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    __half2_raw h = __nv_cvt_fp8x2_to_halfraw2(p[i], __NV_E4M3);
+    float2 t = __half22float2(*reinterpret_cast<__half2 *>(&h));
+    f[2 * i] = t.x;
+    f[2 * i + 1] = t.y;
+  }
+}
+
+// UE8M0 ceil scale (reading R10): s = 2^ceil(log2(fl32(amax/448))),
+// ceil taken from the fp32 bits of the IEEE quotient; s = 1 when amax == 0.
+// Returns the unbiased exponent e (s = 2^e).
+__device__ __forceinline__ int ue8m0_exponent(float amax) {
+  if (!(amax > 0.f)) return 0;
+  float q = __fdiv_rn(amax, 448.f);
+  uint32_t b = __float_as_uint(q);
+  int e = int((b >> 23) & 0xFF) - 127 + ((b & 0x7FFFFF) != 0 ? 1 : 0);
+  return e;
+}
+__device__ __forceinline__ float exp2i(int e) { return __uint_as_float(uint32_t(e + 127) << 23); }
+
+__device__ __forceinline__ uint8_t f32_to_e4m3(float v) {
+  return (uint8_t)__nv_cvt_float_to_fp8(v, __NV_SATFINITE, __NV_E4M3);
+}
+
+__device__ __forceinline__ float silu_f(float g) { return g / (1.f + __expf(-g)); }
+
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+}  // namespace moe
+
+// ------------------------------------------------------------------ layer state
+struct moe_layer {
+  moe_layer_config cfg;
+  int E;        // local experts (E / ep_size)
+  int E_glob;   // global experts
+  int e0;       // first global expert owned by this rank
+  int k, H, F, Fs;
+  bool fp8, f32w;
+  int act_bytes;  // bytes per activation element fed to the expert GEMMs (1 fp8, 2 bf16)
+  int max_tokens;
+  int gemv_max_tokens;
+  int64_t R_max;  // padded sorted rows capacity
+
+  // ---- weights (library-owned, repacked) ----
+  void *gate_w = nullptr;      // [E_glob (+1 shared gate row), H] bf16
+  float *gate_bias = nullptr;  // [E_glob] or null
+  int gate_rows = 0;
+  void *w13 = nullptr;         // [E, 2F, H]  rows interleaved per 128: (W1 blk b, W3 blk b)
+  float *w13_s = nullptr;      // [E, 2F/128, H/128]  (same interleave)
+  void *w2 = nullptr;          // [E, H, F]
+  float *w2_s = nullptr;       // [E, H/128, F/128]
+  void *ws13 = nullptr;        // [2Fs, H] interleaved
+  float *ws13_s = nullptr;
+  void *ws2 = nullptr;         // [H, Fs]
+  float *ws2_s = nullptr;
+  int64_t weight_bytes = 0;
+
+  // ---- workspace ----
+  float *logits = nullptr;      // [maxT, gate_rows]
+  int32_t *topk_idx = nullptr;  // [maxT, k]  (global expert ids, canonical order)
+  float *topk_w = nullptr;      // [maxT, k]
+  float *sgate = nullptr;       // [maxT]  sigmoid(x . w_sg) (Qwen2)
+  int32_t *chunk_cnt = nullptr; // [nchunk, E]
+  int32_t *chunk_base = nullptr;// [nchunk, E]
+  int32_t *counts = nullptr;    // [E]
+  int32_t *offs = nullptr;      // [E+1] unpadded
+  int32_t *offs_pad = nullptr;  // [E+1] padded to kPadM
+  int4 *tiles = nullptr;        // [max_tiles] (expert, row0, row_end, 0)
+  int32_t *n_tiles = nullptr;   // [1]
+  int32_t *act_list = nullptr;  // [E] active experts (count > 0), ascending
+  int32_t *n_active = nullptr;  // [1]
+  int32_t *row_token = nullptr; // [R_max] token of each padded row (-1 = pad)
+  int32_t *pos = nullptr;       // [maxT*k] padded row of (t, j) (local experts only; -1 = remote)
+  void *xq = nullptr;           // [maxT, H] e4m3 (FP8 only)
+  float *xs = nullptr;          // [maxT, H/128]
+  void *xperm = nullptr;        // [R_max, H] act dtype
+  float *xperm_s = nullptr;     // [R_max, H/128]
+  void *hbuf = nullptr;         // [R_max, F] act dtype
+  float *h_s = nullptr;         // [R_max, F/128]
+  __nv_bfloat16 *yperm = nullptr; // [R_max, H]
+  void *hsh = nullptr;          // [maxT, Fs]
+  float *hsh_s = nullptr;       // [maxT, Fs/128]
+  __nv_bfloat16 *ysh = nullptr; // [maxT, H]
+  int64_t workspace_bytes = 0;
+  int max_tiles = 0;
+  // ---- stage timing (moe_layer_profile) ----
+  static constexpr int kStages = 10;
+  bool prof = false;
+  cudaEvent_t ev[kStages + 1] = {};
+  bool ev_hit[kStages + 1] = {};
+  int nchunk_max = 0;
+};

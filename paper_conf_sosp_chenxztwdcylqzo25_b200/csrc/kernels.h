@@ -1,0 +1,82 @@
+// kernels.h -- internal launch interface between the host layer (moe_api.cu)
+// and the kernels.  Not part of the public C ABI (include/moe.h).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace moe {
+
+enum { WT_BF16 = 0, WT_FP8 = 1, WT_F32 = 2 };
+enum { GEMM_LOGITS = 0, GEMM_SWIGLU = 1, GEMM_PLAIN = 2 };
+
+struct SimtGemmArgs {
+  const void *A;          // activation rows
+  const float *As;        // fp8 A: [rows, K/128] scales
+  int64_t lda;            // elements
+  int a_fp8;
+  const void *B;          // weights of expert 0
+  const float *Bs;        // fp8 B scales of expert 0 [N/128, K/128]
+  int64_t b_stride;       // elements between experts
+  int64_t bs_stride;      // scales between experts
+  int b_type;             // WT_*
+  int N, K;
+  const int4 *tiles;      // routed: (expert, row0, row_end, 0) per 128-row tile; null = dense
+  const int32_t *n_tiles; // device count of tiles
+  int M;                  // dense rows
+  void *C;                // output
+  float *Cs;              // fp8 output scales [rows, ldc/128]
+  int64_t ldc;
+  int out_fp8;
+};
+cudaError_t launch_simt_gemm(int mode, const SimtGemmArgs &a, int grid_x, cudaStream_t st);
+
+struct RouterArgs {
+  const float *logits;    // [T, ldl]
+  int ldl;
+  const float *bias;      // [E] or null
+  int T, E, k, n_group, topk_group, group_score, score_fn, norm_topk;
+  float routed_scale;
+  int shared_gated;       // logit column E is the shared-expert gate
+  int32_t *topk_idx;      // [T, k]
+  float *topk_w;          // [T, k]
+  float *sgate;           // [T]
+};
+cudaError_t launch_router_select(const RouterArgs &a, cudaStream_t st);
+
+struct PermuteArgs {
+  const int32_t *topk_idx;  // [T, k] global expert ids
+  int T, k, E, e0;          // local experts [e0, e0 + E)
+  int32_t *chunk_cnt, *chunk_base;  // [nchunk, E]
+  int32_t *counts, *offs, *offs_pad;
+  int4 *tiles; int32_t *n_tiles;
+  int32_t *act_list; int32_t *n_active;
+  int32_t *row_token;       // [R_max]
+  int64_t R_max;
+  int32_t *pos;             // [T*k]
+  int32_t *dbg_perm;        // [T*k] unpadded token order or null
+  int32_t *dbg_counts;      // [E] or null
+};
+cudaError_t launch_permute(const PermuteArgs &a, cudaStream_t st);
+
+// x bf16 [T, H] -> e4m3 [T, H] + [T, H/128] fp32 power-of-two scales
+cudaError_t launch_act_quant(const void *x, int T, int H, void *xq, float *xs, cudaStream_t st);
+// rows of src (bf16 or e4m3 + scales) gathered into the padded expert order
+cudaError_t launch_gather_rows(const void *src, const float *src_s, int H, int elem_bytes,
+                               const int32_t *row_token, const int32_t *offs_pad, int E,
+                               int64_t R_bound, void *dst, float *dst_s, cudaStream_t st);
+
+struct CombineArgs {
+  int T, H, k, n_imm;
+  const int32_t *pos;        // [T, k] padded rows
+  const float *topk_w;       // [T, k]
+  const void *yperm;         // [R, H] bf16
+  const void *ysh;           // [T, H] bf16 or null
+  const float *sgate;        // [T] or null
+  const void *residual;      // [T, H] or null
+  const void *deferred_in;   // [T, H] or null
+  void *y;                   // [T, H]
+  void *deferred_out;        // [T, H] or null
+};
+cudaError_t launch_combine(const CombineArgs &a, cudaStream_t st);
+
+}  // namespace moe

@@ -1,0 +1,465 @@
+// moe_api.cu -- the C ABI of include/moe.h: create (validate, allocate,
+// repack weights), forward (enqueue the kernels, no host sync), destroy.
+#include <cmath>
+#include <cstdarg>
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "common.cuh"
+#include "kernels.h"
+
+using namespace moe;
+
+namespace {
+thread_local std::string g_err;
+
+moe_status fail(moe_status s, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return s;
+}
+
+#define CUDA_TRY(expr)                                                                        \
+  do {                                                                                        \
+    cudaError_t _e = (expr);                                                                  \
+    if (_e != cudaSuccess)                                                                    \
+      return fail(_e == cudaErrorMemoryAllocation ? MOE_ERR_OOM : MOE_ERR_CUDA, "%s: %s (%s:%d)", \
+                  #expr, cudaGetErrorString(_e), __FILE__, __LINE__);                         \
+  } while (0)
+
+template <class T>
+cudaError_t dalloc(moe_layer *L, T **p, size_t bytes, bool weight) {
+  if (bytes == 0) { *p = nullptr; return cudaSuccess; }
+  cudaError_t e = cudaMalloc(reinterpret_cast<void **>(p), bytes);
+  if (e == cudaSuccess) (weight ? L->weight_bytes : L->workspace_bytes) += (int64_t)bytes;
+  return e;
+}
+
+void free_all(moe_layer *L) {
+  void *ptrs[] = {L->gate_w, L->gate_bias, L->w13, L->w13_s, L->w2, L->w2_s, L->ws13, L->ws13_s, L->ws2,
+                  L->ws2_s, L->logits, L->topk_idx, L->topk_w, L->sgate, L->chunk_cnt, L->chunk_base,
+                  L->counts, L->offs, L->offs_pad, L->tiles, L->n_tiles, L->act_list, L->n_active,
+                  L->row_token, L->pos, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
+                  L->hsh, L->hsh_s, L->ysh};
+  for (void *p : ptrs)
+    if (p) cudaFree(p);
+}
+
+bool is_pow2(float v) {
+  if (!(v > 0.f) || !std::isfinite(v)) return false;
+  int e;
+  float m = std::frexp(v, &e);
+  return m == 0.5f;
+}
+
+// Repack [rows = 2F, cols] W13 into 128-row interleave: block 2b = W1 rows
+// [128b, 128b+128), block 2b+1 = W3 rows [F + 128b, ...).  One 256-row GEMM N
+// tile then holds matching gate/up columns (fused gate+up).
+cudaError_t interleave_w13(const void *src, void *dst, int nexp, int F, int H, int es) {
+  const size_t blk = (size_t)128 * H * es;
+  for (int e = 0; e < nexp; ++e) {
+    const char *s = reinterpret_cast<const char *>(src) + (size_t)e * 2 * F * H * es;
+    char *d = reinterpret_cast<char *>(dst) + (size_t)e * 2 * F * H * es;
+    cudaError_t r = cudaMemcpy2D(d, 2 * blk, s, blk, blk, F / 128, cudaMemcpyDeviceToDevice);
+    if (r != cudaSuccess) return r;
+    r = cudaMemcpy2D(d + blk, 2 * blk, s + (size_t)F * H * es, blk, blk, F / 128, cudaMemcpyDeviceToDevice);
+    if (r != cudaSuccess) return r;
+  }
+  return cudaSuccess;
+}
+
+// scales: copy to host, check powers of two, optionally interleave like W13
+moe_status load_scales(const float *src, float **dst, moe_layer *L, int nexp, int rows, int cols, bool inter,
+                       const char *name) {
+  const int rb = rows / 128, cb = cols / 128;
+  const size_t n = (size_t)nexp * rb * cb;
+  std::vector<float> h(n), o(n);
+  CUDA_TRY(cudaMemcpy(h.data(), src, n * sizeof(float), cudaMemcpyDeviceToHost));
+  for (size_t i = 0; i < n; ++i)
+    if (!is_pow2(h[i]))
+      return fail(MOE_ERR_UNSUPPORTED, "%s[%zu] = %g is not a power of two (UE8M0 block scales only, DESIGN.md R10)",
+                  name, i, (double)h[i]);
+  if (inter) {
+    const int half = rb / 2;
+    for (int e = 0; e < nexp; ++e)
+      for (int b = 0; b < half; ++b)
+        for (int c = 0; c < cb; ++c) {
+          o[((size_t)e * rb + 2 * b) * cb + c] = h[((size_t)e * rb + b) * cb + c];
+          o[((size_t)e * rb + 2 * b + 1) * cb + c] = h[((size_t)e * rb + half + b) * cb + c];
+        }
+  } else {
+    o = h;
+  }
+  CUDA_TRY(dalloc(L, dst, n * sizeof(float), true));
+  CUDA_TRY(cudaMemcpy(*dst, o.data(), n * sizeof(float), cudaMemcpyHostToDevice));
+  return MOE_OK;
+}
+
+moe_status validate(const moe_layer_config *c, const moe_layer_weights *w) {
+  if (!c || !w) return fail(MOE_ERR_INVALID_ARG, "null config or weights");
+  if (c->hidden <= 0 || c->hidden % 128) return fail(MOE_ERR_UNSUPPORTED, "hidden %d must be a positive multiple of 128", c->hidden);
+  if (c->ffn <= 0 || c->ffn % 128) return fail(MOE_ERR_UNSUPPORTED, "ffn %d must be a positive multiple of 128", c->ffn);
+  if (c->shared_ffn < 0 || c->shared_ffn % 128) return fail(MOE_ERR_UNSUPPORTED, "shared_ffn %d must be a multiple of 128", c->shared_ffn);
+  if (c->n_experts <= 0 || c->n_experts > 1024) return fail(MOE_ERR_UNSUPPORTED, "n_experts %d not in [1, 1024]", c->n_experts);
+  if (c->top_k <= 0 || c->top_k > 32 || c->top_k > c->n_experts) return fail(MOE_ERR_INVALID_ARG, "top_k %d invalid", c->top_k);
+  if (c->n_group <= 0 || c->n_group > 32 || c->n_experts % c->n_group)
+    return fail(MOE_ERR_INVALID_ARG, "n_group %d must divide n_experts and be <= 32", c->n_group);
+  if (c->topk_group <= 0 || c->topk_group > c->n_group) return fail(MOE_ERR_INVALID_ARG, "topk_group %d invalid", c->topk_group);
+  if (c->n_group > 1 && c->topk_group * (c->n_experts / c->n_group) < c->top_k)
+    return fail(MOE_ERR_INVALID_ARG, "kept groups hold fewer than top_k experts");
+  if (c->n_group > 1 && c->group_score == MOE_GROUP_TOP2_SUM && c->n_experts / c->n_group < 2)
+    return fail(MOE_ERR_INVALID_ARG, "top-2 group score needs >= 2 experts per group");
+  if (c->score_fn != MOE_SCORE_SOFTMAX && c->score_fn != MOE_SCORE_SIGMOID) return fail(MOE_ERR_INVALID_ARG, "score_fn");
+  if (c->group_score != MOE_GROUP_MAX && c->group_score != MOE_GROUP_TOP2_SUM) return fail(MOE_ERR_INVALID_ARG, "group_score");
+  if (c->wtype != MOE_W_BF16 && c->wtype != MOE_W_FP8_BLOCK128 && c->wtype != MOE_W_F32) return fail(MOE_ERR_INVALID_ARG, "wtype");
+  if (c->max_tokens < 0) return fail(MOE_ERR_INVALID_ARG, "max_tokens");
+  if (c->ep_size != 1) return fail(MOE_ERR_UNSUPPORTED, "ep_size %d: expert parallel build not enabled in this library", c->ep_size);
+  if (!w->gate_w || !w->w13 || !w->w2) return fail(MOE_ERR_INVALID_ARG, "gate_w / w13 / w2 must be non-null");
+  if (c->wtype == MOE_W_FP8_BLOCK128 && (!w->w13_scale || !w->w2_scale))
+    return fail(MOE_ERR_INVALID_ARG, "FP8 weights need w13_scale and w2_scale");
+  if (c->shared_ffn > 0 && (!w->ws13 || !w->ws2)) return fail(MOE_ERR_INVALID_ARG, "shared_ffn > 0 needs ws13 / ws2");
+  if (c->shared_ffn > 0 && c->wtype == MOE_W_FP8_BLOCK128 && (!w->ws13_scale || !w->ws2_scale))
+    return fail(MOE_ERR_INVALID_ARG, "FP8 shared expert needs scales");
+  if (c->shared_gated && (!w->shared_gate_w || c->shared_ffn == 0))
+    return fail(MOE_ERR_INVALID_ARG, "shared_gated needs shared_gate_w and a shared expert");
+  return MOE_OK;
+}
+}  // namespace
+
+extern "C" {
+
+const char *moe_status_string(moe_status s) {
+  switch (s) {
+    case MOE_OK: return "MOE_OK";
+    case MOE_ERR_INVALID_ARG: return "MOE_ERR_INVALID_ARG";
+    case MOE_ERR_UNSUPPORTED: return "MOE_ERR_UNSUPPORTED";
+    case MOE_ERR_OOM: return "MOE_ERR_OOM";
+    case MOE_ERR_CUDA: return "MOE_ERR_CUDA";
+    case MOE_ERR_NCCL: return "MOE_ERR_NCCL";
+    case MOE_ERR_CAPACITY: return "MOE_ERR_CAPACITY";
+  }
+  return "MOE_ERR_UNKNOWN";
+}
+
+const char *moe_last_error(void) { return g_err.c_str(); }
+
+moe_status moe_get_unique_id(void *out128) {
+  if (!out128) return fail(MOE_ERR_INVALID_ARG, "null out");
+  return fail(MOE_ERR_UNSUPPORTED, "expert parallel build not enabled in this library");
+}
+
+moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights *w, moe_layer **out) {
+  if (!out) return fail(MOE_ERR_INVALID_ARG, "null out");
+  *out = nullptr;
+  moe_status st = validate(cfg, w);
+  if (st != MOE_OK) return st;
+  CUDA_TRY(cudaSetDevice(cfg->device));
+
+  moe_layer *L = new moe_layer();
+  L->cfg = *cfg;
+  L->cfg.nccl_unique_id = nullptr;
+  L->E_glob = cfg->n_experts;
+  L->E = cfg->n_experts / cfg->ep_size;
+  L->e0 = cfg->ep_rank * L->E;
+  L->k = cfg->top_k;
+  L->H = cfg->hidden;
+  L->F = cfg->ffn;
+  L->Fs = cfg->shared_ffn;
+  L->fp8 = cfg->wtype == MOE_W_FP8_BLOCK128;
+  L->f32w = cfg->wtype == MOE_W_F32;
+  L->act_bytes = L->fp8 ? 1 : 2;
+  L->max_tokens = cfg->max_tokens;
+  L->gemv_max_tokens = cfg->gemv_max_tokens > 0 ? cfg->gemv_max_tokens : 0;
+  const int H = L->H, F = L->F, Fs = L->Fs, E = L->E, k = L->k;
+  const int wes = L->fp8 ? 1 : (L->f32w ? 4 : 2);
+  auto cleanup = [&](moe_status s) { free_all(L); delete L; return s; };
+#define C_TRY(expr)                                                                            \
+  do {                                                                                         \
+    cudaError_t _e = (expr);                                                                   \
+    if (_e != cudaSuccess)                                                                     \
+      return cleanup(fail(_e == cudaErrorMemoryAllocation ? MOE_ERR_OOM : MOE_ERR_CUDA, "%s: %s", #expr, \
+                          cudaGetErrorString(_e)));                                            \
+  } while (0)
+#define S_TRY(expr)                      \
+  do {                                   \
+    moe_status _s = (expr);              \
+    if (_s != MOE_OK) return cleanup(_s); \
+  } while (0)
+
+  // ---- router weights (+ Qwen2 shared gate as one extra row) ----
+  L->gate_rows = L->E_glob + (cfg->shared_gated ? 1 : 0);
+  C_TRY(dalloc(L, &L->gate_w, (size_t)L->gate_rows * H * 2, true));
+  C_TRY(cudaMemcpy(L->gate_w, w->gate_w, (size_t)L->E_glob * H * 2, cudaMemcpyDeviceToDevice));
+  if (cfg->shared_gated)
+    C_TRY(cudaMemcpy(reinterpret_cast<char *>(L->gate_w) + (size_t)L->E_glob * H * 2, w->shared_gate_w,
+                     (size_t)H * 2, cudaMemcpyDeviceToDevice));
+  if (w->gate_bias) {
+    C_TRY(dalloc(L, &L->gate_bias, (size_t)L->E_glob * 4, true));
+    C_TRY(cudaMemcpy(L->gate_bias, w->gate_bias, (size_t)L->E_glob * 4, cudaMemcpyDeviceToDevice));
+  }
+  // ---- routed experts ----
+  C_TRY(dalloc(L, &L->w13, (size_t)E * 2 * F * H * wes, true));
+  C_TRY(interleave_w13(w->w13, L->w13, E, F, H, wes));
+  C_TRY(dalloc(L, &L->w2, (size_t)E * H * F * wes, true));
+  C_TRY(cudaMemcpy(L->w2, w->w2, (size_t)E * H * F * wes, cudaMemcpyDeviceToDevice));
+  if (L->fp8) {
+    S_TRY(load_scales(w->w13_scale, &L->w13_s, L, E, 2 * F, H, true, "w13_scale"));
+    S_TRY(load_scales(w->w2_scale, &L->w2_s, L, E, H, F, false, "w2_scale"));
+  }
+  if (Fs > 0) {
+    C_TRY(dalloc(L, &L->ws13, (size_t)2 * Fs * H * wes, true));
+    C_TRY(interleave_w13(w->ws13, L->ws13, 1, Fs, H, wes));
+    C_TRY(dalloc(L, &L->ws2, (size_t)H * Fs * wes, true));
+    C_TRY(cudaMemcpy(L->ws2, w->ws2, (size_t)H * Fs * wes, cudaMemcpyDeviceToDevice));
+    if (L->fp8) {
+      S_TRY(load_scales(w->ws13_scale, &L->ws13_s, L, 1, 2 * Fs, H, true, "ws13_scale"));
+      S_TRY(load_scales(w->ws2_scale, &L->ws2_s, L, 1, H, Fs, false, "ws2_scale"));
+    }
+  }
+
+  // ---- workspace, sized for max_tokens ----
+  const int64_t Tm = std::max(1, cfg->max_tokens);
+  const int64_t pairs = Tm * k;
+  L->R_max = pairs + (int64_t)E * kPadM;
+  L->max_tiles = (int)(L->R_max / kPadM);
+  L->nchunk_max = (int)((Tm + kChunkTokens - 1) / kChunkTokens);
+  const int ab = L->act_bytes;
+  C_TRY(dalloc(L, &L->logits, (size_t)Tm * L->gate_rows * 4, false));
+  C_TRY(dalloc(L, &L->topk_idx, (size_t)pairs * 4, false));
+  C_TRY(dalloc(L, &L->topk_w, (size_t)pairs * 4, false));
+  C_TRY(dalloc(L, &L->sgate, (size_t)Tm * 4, false));
+  C_TRY(dalloc(L, &L->chunk_cnt, (size_t)L->nchunk_max * E * 4, false));
+  C_TRY(dalloc(L, &L->chunk_base, (size_t)L->nchunk_max * E * 4, false));
+  C_TRY(dalloc(L, &L->counts, (size_t)E * 4, false));
+  C_TRY(dalloc(L, &L->offs, (size_t)(E + 1) * 4, false));
+  C_TRY(dalloc(L, &L->offs_pad, (size_t)(E + 1) * 4, false));
+  C_TRY(dalloc(L, &L->tiles, (size_t)L->max_tiles * sizeof(int4), false));
+  C_TRY(dalloc(L, &L->n_tiles, 4, false));
+  C_TRY(dalloc(L, &L->act_list, (size_t)E * 4, false));
+  C_TRY(dalloc(L, &L->n_active, 4, false));
+  C_TRY(dalloc(L, &L->row_token, (size_t)L->R_max * 4, false));
+  C_TRY(dalloc(L, &L->pos, (size_t)pairs * 4, false));
+  if (L->fp8) {
+    C_TRY(dalloc(L, &L->xq, (size_t)Tm * H, false));
+    C_TRY(dalloc(L, &L->xs, (size_t)Tm * (H / 128) * 4, false));
+    C_TRY(dalloc(L, &L->xperm_s, (size_t)L->R_max * (H / 128) * 4, false));
+    C_TRY(dalloc(L, &L->h_s, (size_t)L->R_max * (F / 128) * 4, false));
+    if (Fs) C_TRY(dalloc(L, &L->hsh_s, (size_t)Tm * (Fs / 128) * 4, false));
+  }
+  C_TRY(dalloc(L, &L->xperm, (size_t)L->R_max * H * ab, false));
+  C_TRY(dalloc(L, &L->hbuf, (size_t)L->R_max * F * ab, false));
+  C_TRY(dalloc(L, &L->yperm, (size_t)L->R_max * H * 2, false));
+  if (Fs) {
+    C_TRY(dalloc(L, &L->hsh, (size_t)Tm * Fs * ab, false));
+    C_TRY(dalloc(L, &L->ysh, (size_t)Tm * H * 2, false));
+  }
+  C_TRY(cudaMemset(L->row_token, 0xff, (size_t)L->R_max * 4));
+  C_TRY(cudaDeviceSynchronize());
+#undef C_TRY
+#undef S_TRY
+  *out = L;
+  return MOE_OK;
+}
+
+static const char *kStageNames[moe_layer::kStages] = {
+    "router_logits", "router_select", "permute", "act_quant", "gather", "gemm1_swiglu", "gemm2",
+    "shared_gemm1", "shared_gemm2", "combine"};
+enum { ST_LOGITS = 0, ST_SELECT, ST_PERMUTE, ST_QUANT, ST_GATHER, ST_GEMM1, ST_GEMM2, ST_SH1, ST_SH2, ST_COMBINE };
+
+static inline void mark(moe_layer *L, int stage, cudaStream_t st) {
+  if (!L->prof) return;
+  cudaEventRecord(L->ev[stage + 1], st);
+  L->ev_hit[stage + 1] = true;
+}
+
+static moe_status forward_impl(moe_layer *L, const void *x, const void *residual, int32_t T, int32_t n_def,
+                               const void *deferred_in, void *y, void *deferred_out, moe_routing_out *dbg,
+                               void *stream) {
+  if (!L) return fail(MOE_ERR_INVALID_ARG, "null layer");
+  if (T < 0) return fail(MOE_ERR_INVALID_ARG, "T = %d < 0", T);
+  if (T > L->max_tokens) return fail(MOE_ERR_CAPACITY, "T = %d > max_tokens = %d", T, L->max_tokens);
+  if (n_def < 0 || n_def > L->k - 1) return fail(MOE_ERR_INVALID_ARG, "n_deferred = %d not in [0, k-1]", n_def);
+  if (T > 0 && (!x || !y)) return fail(MOE_ERR_INVALID_ARG, "x and y must be non-null");
+  if (x && x == y) return fail(MOE_ERR_INVALID_ARG, "y must not alias x");
+  if (T == 0) return MOE_OK;
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  if (L->prof) {
+    for (int i = 0; i <= moe_layer::kStages; ++i) L->ev_hit[i] = false;
+    cudaEventRecord(L->ev[0], st);
+    L->ev_hit[0] = true;
+  }
+  const int H = L->H, F = L->F, Fs = L->Fs, E = L->E, k = L->k;
+  const int btype = L->fp8 ? WT_FP8 : (L->f32w ? WT_F32 : WT_BF16);
+
+  // 1. router logits (bf16 x . bf16 Wg, fp32 accumulate)
+  {
+    SimtGemmArgs a{};
+    a.A = x; a.lda = H; a.a_fp8 = 0;
+    a.B = L->gate_w; a.b_type = WT_BF16; a.N = L->gate_rows; a.K = H;
+    a.M = T; a.C = L->logits; a.ldc = L->gate_rows;
+    CUDA_TRY(launch_simt_gemm(GEMM_LOGITS, a, (T + 63) / 64, st));
+    mark(L, ST_LOGITS, st);
+  }
+  // 2. scores + group-limited top-k + weights
+  {
+    RouterArgs r{};
+    r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
+    r.T = T; r.E = L->E_glob; r.k = k; r.n_group = L->cfg.n_group; r.topk_group = L->cfg.topk_group;
+    r.group_score = L->cfg.group_score; r.score_fn = L->cfg.score_fn; r.norm_topk = L->cfg.norm_topk;
+    r.routed_scale = L->cfg.routed_scale; r.shared_gated = L->cfg.shared_gated;
+    r.topk_idx = L->topk_idx; r.topk_w = L->topk_w; r.sgate = L->sgate;
+    CUDA_TRY(launch_router_select(r, st));
+    mark(L, ST_SELECT, st);
+  }
+  // 3. count / scan / permute
+  {
+    PermuteArgs p{};
+    p.topk_idx = L->topk_idx; p.T = T; p.k = k; p.E = E; p.e0 = L->e0;
+    p.chunk_cnt = L->chunk_cnt; p.chunk_base = L->chunk_base; p.counts = L->counts; p.offs = L->offs;
+    p.offs_pad = L->offs_pad; p.tiles = L->tiles; p.n_tiles = L->n_tiles; p.act_list = L->act_list;
+    p.n_active = L->n_active; p.row_token = L->row_token; p.R_max = L->R_max; p.pos = L->pos;
+    p.dbg_perm = dbg ? dbg->perm : nullptr;
+    p.dbg_counts = dbg ? dbg->expert_counts : nullptr;
+    CUDA_TRY(launch_permute(p, st));
+    mark(L, ST_PERMUTE, st);
+  }
+  const int64_t pairs = (int64_t)T * k;
+  const int64_t R_bound = std::min<int64_t>(L->R_max, pairs + (int64_t)std::min<int64_t>(E, pairs) * kPadM);
+  const int tile_bound = (int)(R_bound / kPadM);
+  // 4. activation quantisation (FP8) and gather into expert order
+  const void *xa = x;
+  const float *xa_s = nullptr;
+  if (L->fp8) {
+    CUDA_TRY(launch_act_quant(x, T, H, L->xq, L->xs, st));
+    xa = L->xq;
+    xa_s = L->xs;
+    mark(L, ST_QUANT, st);
+  }
+  CUDA_TRY(launch_gather_rows(xa, xa_s, H, L->act_bytes, L->row_token, L->offs_pad, E, R_bound, L->xperm,
+                              L->xperm_s, st));
+  mark(L, ST_GATHER, st);
+  // 5. routed experts: GEMM1 + SwiGLU, GEMM2
+  {
+    SimtGemmArgs a{};
+    a.A = L->xperm; a.As = L->xperm_s; a.lda = H; a.a_fp8 = L->fp8;
+    a.B = L->w13; a.Bs = L->w13_s; a.b_stride = (int64_t)2 * F * H; a.bs_stride = (int64_t)(2 * F / 128) * (H / 128);
+    a.b_type = btype; a.N = 2 * F; a.K = H;
+    a.tiles = L->tiles; a.n_tiles = L->n_tiles;
+    a.C = L->hbuf; a.Cs = L->h_s; a.ldc = F; a.out_fp8 = L->fp8;
+    CUDA_TRY(launch_simt_gemm(GEMM_SWIGLU, a, 2 * tile_bound, st));
+    mark(L, ST_GEMM1, st);
+    SimtGemmArgs b{};
+    b.A = L->hbuf; b.As = L->h_s; b.lda = F; b.a_fp8 = L->fp8;
+    b.B = L->w2; b.Bs = L->w2_s; b.b_stride = (int64_t)H * F; b.bs_stride = (int64_t)(H / 128) * (F / 128);
+    b.b_type = btype; b.N = H; b.K = F;
+    b.tiles = L->tiles; b.n_tiles = L->n_tiles;
+    b.C = L->yperm; b.ldc = H;
+    CUDA_TRY(launch_simt_gemm(GEMM_PLAIN, b, 2 * tile_bound, st));
+    mark(L, ST_GEMM2, st);
+  }
+  // 6. shared expert on every token
+  if (Fs > 0) {
+    SimtGemmArgs a{};
+    a.A = xa; a.As = xa_s; a.lda = H; a.a_fp8 = L->fp8;
+    a.B = L->ws13; a.Bs = L->ws13_s; a.b_type = btype; a.N = 2 * Fs; a.K = H;
+    a.M = T; a.C = L->hsh; a.Cs = L->hsh_s; a.ldc = Fs; a.out_fp8 = L->fp8;
+    CUDA_TRY(launch_simt_gemm(GEMM_SWIGLU, a, (T + 63) / 64, st));
+    mark(L, ST_SH1, st);
+    SimtGemmArgs b{};
+    b.A = L->hsh; b.As = L->hsh_s; b.lda = Fs; b.a_fp8 = L->fp8;
+    b.B = L->ws2; b.Bs = L->ws2_s; b.b_type = btype; b.N = H; b.K = Fs;
+    b.M = T; b.C = L->ysh; b.ldc = H;
+    CUDA_TRY(launch_simt_gemm(GEMM_PLAIN, b, (T + 63) / 64, st));
+    mark(L, ST_SH2, st);
+  }
+  // 7. weighted combine + residual (+ deferral split)
+  {
+    CombineArgs c{};
+    c.T = T; c.H = H; c.k = k; c.n_imm = deferred_out ? k - n_def : k;
+    c.pos = L->pos; c.topk_w = L->topk_w; c.yperm = L->yperm;
+    c.ysh = Fs > 0 ? L->ysh : nullptr; c.sgate = L->cfg.shared_gated ? L->sgate : nullptr;
+    c.residual = residual; c.deferred_in = deferred_in; c.y = y; c.deferred_out = deferred_out;
+    CUDA_TRY(launch_combine(c, st));
+    mark(L, ST_COMBINE, st);
+  }
+  if (dbg) {
+    if (dbg->topk_idx)
+      CUDA_TRY(cudaMemcpyAsync(dbg->topk_idx, L->topk_idx, pairs * 4, cudaMemcpyDeviceToDevice, st));
+    if (dbg->topk_w) CUDA_TRY(cudaMemcpyAsync(dbg->topk_w, L->topk_w, pairs * 4, cudaMemcpyDeviceToDevice, st));
+  }
+  return MOE_OK;
+}
+
+moe_status moe_layer_forward(moe_layer *L, const void *x, const void *residual, int32_t T, void *y,
+                             moe_routing_out *dbg, void *stream) {
+  return forward_impl(L, x, residual, T, 0, nullptr, y, nullptr, dbg, stream);
+}
+
+moe_status moe_layer_forward_deferred(moe_layer *L, const void *x, const void *residual, int32_t T,
+                                      int32_t n_deferred, const void *deferred_in, void *y, void *deferred_out,
+                                      moe_routing_out *dbg, void *stream) {
+  return forward_impl(L, x, residual, T, n_deferred, deferred_in, y, deferred_out, dbg, stream);
+}
+
+moe_status moe_layer_profile(moe_layer *L, int32_t enable) {
+  if (!L) return fail(MOE_ERR_INVALID_ARG, "null layer");
+  if (enable && !L->ev[0]) {
+    for (int i = 0; i <= moe_layer::kStages; ++i) CUDA_TRY(cudaEventCreate(&L->ev[i]));
+  }
+  L->prof = enable != 0;
+  return MOE_OK;
+}
+
+moe_status moe_layer_stage_times(moe_layer *L, float *ms_out, int32_t cap, int32_t *n_out) {
+  if (!L || !ms_out) return fail(MOE_ERR_INVALID_ARG, "null argument");
+  if (!L->ev[0] || !L->ev_hit[0]) return fail(MOE_ERR_INVALID_ARG, "no profiled forward recorded");
+  int last = 0;
+  for (int i = 1; i <= moe_layer::kStages; ++i)
+    if (L->ev_hit[i]) last = i;
+  CUDA_TRY(cudaEventSynchronize(L->ev[last]));
+  const int n = std::min<int>(cap, moe_layer::kStages);
+  int prev = 0;
+  for (int i = 0; i < n; ++i) {
+    ms_out[i] = 0.f;
+    if (L->ev_hit[i + 1]) {
+      CUDA_TRY(cudaEventElapsedTime(&ms_out[i], L->ev[prev], L->ev[i + 1]));
+      prev = i + 1;
+    }
+  }
+  if (n_out) *n_out = n;
+  return MOE_OK;
+}
+
+const char *moe_stage_name(int32_t i) {
+  return (i >= 0 && i < moe_layer::kStages) ? kStageNames[i] : "";
+}
+
+moe_status moe_layer_destroy(moe_layer *L) {
+  if (!L) return MOE_OK;
+  cudaSetDevice(L->cfg.device);
+  for (int i = 0; i <= moe_layer::kStages; ++i)
+    if (L->ev[i]) cudaEventDestroy(L->ev[i]);
+  free_all(L);
+  delete L;
+  return MOE_OK;
+}
+
+moe_status moe_layer_get_info(const moe_layer *L, moe_layer_info *info) {
+  if (!L || !info) return fail(MOE_ERR_INVALID_ARG, "null argument");
+  info->weight_bytes = L->weight_bytes;
+  info->workspace_bytes = L->workspace_bytes;
+  info->gemv_max_tokens = L->gemv_max_tokens;
+  info->kernels_per_forward_prefill = 9 + (L->fp8 ? 1 : 0) + (L->Fs > 0 ? 2 : 0);
+  info->kernels_per_forward_decode = info->kernels_per_forward_prefill;
+  info->local_experts = L->E;
+  return MOE_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,93 @@
+"""Helpers shared by the GPU parity tests: build the oracle's view of the same
+seeded weights, merge tie-band routing, and compare GPU results with the oracle.
+(Test infrastructure: imports oracle/, never imported by the product path.)"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from inputs.presets import W_FP8
+from oracle import moe_oracle as O
+
+TOL = {0: 5e-3, 1: 2e-2, 2: 5e-3}   # north_star: BF16 rel-L2 <= 5e-3, FP8 <= 2e-2 (F32 toy: BF16 bar)
+
+
+def oracle_cfg(p) -> O.OracleConfig:
+    return O.OracleConfig(hidden=p.hidden, ffn=p.ffn, n_experts=p.n_experts, top_k=p.top_k,
+                          n_group=p.n_group, topk_group=p.topk_group, group_score=p.group_score,
+                          score_fn=p.score_fn, norm_topk=bool(p.norm_topk), routed_scale=p.routed_scale,
+                          shared_ffn=p.shared_ffn, shared_gated=bool(p.shared_gated), fp8=p.wtype == W_FP8)
+
+
+def _f64(t):
+    return t.detach().to("cpu").to(torch.float64).numpy()
+
+
+def oracle_weights(p, w) -> O.OracleWeights:
+    """Dequantised fp64 weights, fetched per expert (works for CPU or GPU tensors)."""
+    F, Fs = p.ffn, p.shared_ffn
+    fp8 = p.wtype == W_FP8
+
+    def deq(codes, scales):
+        if fp8:
+            return O.dequant_block128(codes.detach().cpu().numpy(), scales.detach().cpu().numpy())
+        return _f64(codes)
+
+    def expert(e):
+        w13 = deq(w.w13[e], w.w13_scale[e] if fp8 else None)
+        return w13[:F], w13[F:], deq(w.w2[e], w.w2_scale[e] if fp8 else None)
+
+    shared = None
+    if Fs:
+        def shared():
+            a = deq(w.ws13, w.ws13_scale)
+            return a[:Fs], a[Fs:], deq(w.ws2, w.ws2_scale)
+    return O.OracleWeights(_f64(w.gate_w), None if w.gate_bias is None else _f64(w.gate_bias), expert, shared,
+                           None if w.shared_gate_w is None else _f64(w.shared_gate_w))
+
+
+def merged_routing(x64, W, cfg, gpu_idx, ties):
+    """Oracle routing for every token, except tie-band tokens which take the
+    GPU's expert set (checked valid within the band) with oracle weights."""
+    s = O.scores(O.router_logits(x64, W.gate_w), cfg.score_fn)
+    idx = O.select_experts(s, W.gate_bias, cfg.n_group, cfg.topk_group, cfg.top_k, cfg.group_score)
+    if len(ties):
+        sel = s + (W.gate_bias[None, :] if W.gate_bias is not None else 0.0)
+        for t in ties:
+            g = np.array(sorted(gpu_idx[t]))
+            assert len(set(g.tolist())) == cfg.top_k
+            # every chosen expert is within the band of the oracle's k-th choice
+            kth = np.sort(sel[t, idx[t]])[0]
+            assert np.all(sel[t, g] >= kth - 1e-5), f"token {t}: GPU choice outside the tie band"
+            idx[t] = g
+    w = O.combine_weights(s, idx, cfg.norm_topk, cfg.routed_scale)
+    idx, w = O.canonical_order(idx, w)
+    return idx, w
+
+
+def rel_l2(a, b) -> float:
+    a = np.asarray(a, np.float64)
+    b = np.asarray(b, np.float64)
+    return float(np.linalg.norm(a - b) / max(np.linalg.norm(b), 1e-30))
+
+
+def check_routing(gpu_idx, gpu_w, orc_idx, orc_w, ties, routed_scale, norm):
+    T = gpu_idx.shape[0]
+    keep = np.setdiff1d(np.arange(T), ties)
+    # bit-exact expert sets outside the tie band
+    np.testing.assert_array_equal(np.sort(gpu_idx[keep], 1), np.sort(orc_idx[keep], 1))
+    # canonical order on the GPU side: weights non-increasing
+    assert np.all(np.diff(gpu_w, axis=1) <= 0)
+    # weights per expert
+    for t in keep[:4096]:
+        og = dict(zip(orc_idx[t].tolist(), orc_w[t].tolist()))
+        for e, wv in zip(gpu_idx[t].tolist(), gpu_w[t].tolist()):
+            assert abs(wv - og[e]) <= 1e-5 * max(1.0, abs(og[e])), (t, e, wv, og[e])
+    if norm:
+        np.testing.assert_allclose(gpu_w.sum(1), routed_scale, rtol=1e-5)
+
+
+def check_permutation(gpu_counts, gpu_perm, idx, n_experts):
+    counts, offsets, perm_t, _ = O.count_and_permute(idx, n_experts)
+    np.testing.assert_array_equal(gpu_counts, counts)
+    np.testing.assert_array_equal(gpu_perm, perm_t)
