@@ -1,0 +1,311 @@
+// umma_gemm.cu -- persistent grouped expert GEMM on the 5th-gen tensor cores.
+//
+//   routed:  C[rows of expert e] = A[rows of expert e] . B_e^T
+//   shared:  C[token rows]       = A[token rows] . B_s^T
+//
+// GEMM1 (EPI_SWIGLU): A = x_perm (tokens sorted by expert), B = W13 with rows
+// interleaved per 128 (W1 block b, W3 block b), so one 256-wide N tile holds
+// matching gate/up columns and the epilogue computes h = silu(g) * u from the
+// fp32 accumulators -- the fused gate+up batch of PAPER.md L179.  FP8: h is
+// requantised to e4m3 with a 1x128 UE8M0 scale straight from fp32 (DESIGN.md
+// reading R11), written together with the scale image GEMM2 consumes.
+// GEMM2 (EPI_PLAIN):  A = h, B = W2 -> bf16 rows.
+//
+// Work units = (expert m-tile of 128 rows, 256-wide n-block), ordered expert-
+// major then n-block then m-tile so CTAs running concurrently share one weight
+// slab through L2 (the device-side analog of PAPER.md L181's co-scheduling of
+// same-expert tasks).  Roles per CTA (192 threads, one CTA per SM):
+//   warp 0     TMA producer (A/B tiles, FP8 scale images) into a 4-stage ring
+//   warp 1     TMEM allocator + single-thread tcgen05.mma issuer
+//   warps 2-5  epilogue: tcgen05.ld -> registers -> global
+#include <cuda.h>
+
+#include "common.cuh"
+#include "kernels.h"
+#include "sm100.cuh"
+
+namespace moe {
+using namespace sm100;
+
+constexpr int UG_BM = 128, UG_BN = 256, UG_STAGES = 4, UG_THREADS = 192;
+constexpr int UG_A_BYTES = UG_BM * 128;        // 16 KB (128 rows x 128 B)
+constexpr int UG_B_BYTES = UG_BN * 128;        // 32 KB
+constexpr int UG_SFA_BYTES = 512;              // 128 rows x 4 B image
+constexpr int UG_SFB_BYTES = 1024;             // 256 rows x 4 B image
+constexpr uint32_t UG_TMEM_COLS = 512;
+constexpr uint32_t UG_SFA_COL = 256, UG_SFB_COL = 264;
+constexpr size_t UG_SMEM = 1024 + (size_t)UG_STAGES * (UG_A_BYTES + UG_B_BYTES + UG_SFA_BYTES + UG_SFB_BYTES) + 256;
+
+struct UnitInfo {
+  int valid, group, expert, row0, row_end, nb;
+};
+
+__device__ __forceinline__ UnitInfo decode_unit(const UmmaParams &p, int u, int n_routed_units) {
+  UnitInfo r{};
+  if (u < n_routed_units) {
+    const int nb_r = p.nb_r;
+    const int4 t_any = p.tiles[u / nb_r];
+    const int t0 = t_any.w & 0xFFFF, nt = t_any.w >> 16;
+    const int local = u - t0 * nb_r;
+    const int4 tl = p.tiles[t0 + local % nt];
+    r.valid = 1; r.group = 0; r.expert = tl.x; r.row0 = tl.y; r.row_end = tl.z; r.nb = local / nt;
+    return r;
+  }
+  const int us = u - n_routed_units;
+  const int mt = (p.T_shared + UG_BM - 1) / UG_BM;
+  if (p.T_shared > 0 && us < mt * p.nb_s) {
+    r.valid = 1; r.group = 1; r.expert = 0; r.nb = us / mt;
+    r.row0 = (us % mt) * UG_BM; r.row_end = p.T_shared;
+  }
+  return r;
+}
+
+// byte offset of the UE8M0 scale of (row, k-block) in a scale image
+__device__ __forceinline__ size_t sf_image_offset(int row, int kb, int tile_stride) {
+  const int tile = row >> 7, r = row & 127;
+  const int word = (r & 31) * 4 + (r >> 5);
+  return ((size_t)((kb >> 2) * tile_stride + tile) * 128 + word) * 4 + (kb & 3);
+}
+
+template <bool FP8, int EPI>
+__global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_constant__ UmmaParams p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t *sA = smem;
+  uint8_t *sB = sA + UG_STAGES * UG_A_BYTES;
+  uint8_t *sSFA = sB + UG_STAGES * UG_B_BYTES;
+  uint8_t *sSFB = sSFA + UG_STAGES * UG_SFA_BYTES;
+  uint64_t *full = reinterpret_cast<uint64_t *>(sSFB + UG_STAGES * UG_SFB_BYTES);
+  uint64_t *empty = full + UG_STAGES;
+  uint64_t *tmem_full = empty + UG_STAGES;
+  uint64_t *tmem_empty = tmem_full + 1;
+  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(tmem_empty + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int n_routed_units = p.tiles ? (*p.n_tiles) * p.nb_r : 0;
+
+  if (warp == 0 && lane == 0) {
+    prefetch_tmap(&p.g[0].a_map); prefetch_tmap(&p.g[0].b_map);
+    prefetch_tmap(&p.g[1].a_map); prefetch_tmap(&p.g[1].b_map);
+    for (int s = 0; s < UG_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+    mbar_init(tmem_full, 1);
+    mbar_init(tmem_empty, 128);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc(tmem_base_smem, UG_TMEM_COLS);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_base_smem;
+
+  if (warp == 0) {
+    // ============================ TMA producer ============================
+    if (lane == 0) {
+      int stage = 0; uint32_t phase = 0;
+      for (int u = blockIdx.x;; u += gridDim.x) {
+        const UnitInfo ui = decode_unit(p, u, n_routed_units);
+        if (!ui.valid) break;
+        const UmmaGroup &g = p.g[ui.group];
+        const int brow = ui.expert * g.n_total + ui.nb * UG_BN;
+        for (int kb = 0; kb < g.kblocks; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          uint32_t bytes = UG_A_BYTES + UG_B_BYTES;
+          if (FP8) bytes += UG_SFA_BYTES + UG_SFB_BYTES;
+          mbar_expect_tx(&full[stage], bytes);
+          const int kc = kb * (FP8 ? 128 : 64);   // element coordinate along K
+          tma_load_2d(sA + stage * UG_A_BYTES, &g.a_map, &full[stage], kc, ui.row0);
+          tma_load_2d(sB + stage * UG_B_BYTES, &g.b_map, &full[stage], kc, brow);
+          if (FP8) {
+            const uint8_t *sfa = g.sfa + ((size_t)(kb >> 2) * g.sfa_tile_stride + (ui.row0 >> 7)) * 512;
+            const uint8_t *sfb = g.sfb + (size_t)ui.expert * g.sfb_expert_stride +
+                                 ((size_t)(kb >> 2) * g.sfb_rb + ui.nb * 2) * 512;
+            bulk_load(sSFA + stage * UG_SFA_BYTES, sfa, UG_SFA_BYTES, &full[stage]);
+            bulk_load(sSFB + stage * UG_SFB_BYTES, sfb, UG_SFB_BYTES, &full[stage]);
+          }
+          if (++stage == UG_STAGES) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ============================ MMA issuer ============================
+    int stage = 0; uint32_t phase = 0; uint32_t acc_phase = 0;
+    for (int u = blockIdx.x;; u += gridDim.x) {
+      const UnitInfo ui = decode_unit(p, u, n_routed_units);
+      if (!ui.valid) break;
+      const int kblocks = p.g[ui.group].kblocks;
+      mbar_wait(tmem_empty, acc_phase ^ 1);
+      tc_fence_after();
+      for (int kb = 0; kb < kblocks; ++kb) {
+        mbar_wait(&full[stage], phase);
+        tc_fence_after();
+        if (lane == 0) {
+          const uint32_t a0 = smem_u32(sA + stage * UG_A_BYTES);
+          const uint32_t b0 = smem_u32(sB + stage * UG_B_BYTES);
+          if (FP8) {
+            tmem_cp_32x128b_x4(tmem + UG_SFA_COL, sf_desc(smem_u32(sSFA + stage * UG_SFA_BYTES)));
+            tmem_cp_32x128b_x4(tmem + UG_SFB_COL, sf_desc(smem_u32(sSFB + stage * UG_SFB_BYTES)));
+            tmem_cp_32x128b_x4(tmem + UG_SFB_COL + 4, sf_desc(smem_u32(sSFB + stage * UG_SFB_BYTES + 512)));
+          }
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const uint64_t ad = sw128_kmajor_desc(a0 + k * 32);
+            const uint64_t bd = sw128_kmajor_desc(b0 + k * 32);
+            const uint32_t acc = (kb | k) != 0;
+            if (FP8)
+              mma_mxf8(tmem, ad, bd, idesc_mxf8(UG_BM, UG_BN, kb & 3, kb & 3), acc, tmem + UG_SFA_COL,
+                       tmem + UG_SFB_COL);
+            else
+              mma_bf16(tmem, ad, bd, idesc_bf16(UG_BM, UG_BN), acc);
+          }
+          mma_commit(&empty[stage]);
+          if (kb == kblocks - 1) mma_commit(tmem_full);
+        }
+        __syncwarp();
+        if (++stage == UG_STAGES) { stage = 0; phase ^= 1; }
+      }
+      acc_phase ^= 1;
+    }
+  } else {
+    // ============================ epilogue ============================
+    const int q = warp & 3;                       // TMEM lane quadrant of this warp
+    const uint32_t lane_base = (uint32_t)(q * 32) << 16;
+    uint32_t acc_phase = 0;
+    for (int u = blockIdx.x;; u += gridDim.x) {
+      const UnitInfo ui = decode_unit(p, u, n_routed_units);
+      if (!ui.valid) break;
+      const UmmaGroup &g = p.g[ui.group];
+      mbar_wait(tmem_full, acc_phase);
+      tc_fence_after();
+      const int row = ui.row0 + q * 32 + lane;
+      const bool live = row < ui.row_end;
+      if constexpr (EPI == GEMM_SWIGLU) {
+        float h[128];
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+          uint32_t gr[32], ur[32];
+          tmem_ld_32x32b_x32(tmem + lane_base + c * 32, gr);
+          tmem_ld_32x32b_x32(tmem + lane_base + 128 + c * 32, ur);
+          tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 32; ++i) h[c * 32 + i] = silu_f(__uint_as_float(gr[i])) * __uint_as_float(ur[i]);
+        }
+        tc_fence_before();
+        mbar_arrive(tmem_empty);
+        if (FP8) {
+          float amax = 0.f;
+#pragma unroll
+          for (int i = 0; i < 128; ++i) amax = fmaxf(amax, fabsf(h[i]));
+          const int e = ue8m0_exponent(amax);
+          const float inv = exp2i(-e);
+          if (live) {
+            uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<uint8_t *>(g.out) + (size_t)row * g.ldc +
+                                                   ui.nb * 128);
+#pragma unroll
+            for (int v = 0; v < 8; ++v) {
+              uint32_t w[4];
+#pragma unroll
+              for (int j = 0; j < 4; ++j) {
+                const int b = v * 16 + j * 4;
+                w[j] = (uint32_t)f32_to_e4m3(h[b] * inv) | ((uint32_t)f32_to_e4m3(h[b + 1] * inv) << 8) |
+                       ((uint32_t)f32_to_e4m3(h[b + 2] * inv) << 16) | ((uint32_t)f32_to_e4m3(h[b + 3] * inv) << 24);
+              }
+              dst[v] = make_uint4(w[0], w[1], w[2], w[3]);
+            }
+            g.out_sf[sf_image_offset(row, ui.nb, g.out_sf_tile_stride)] = (uint8_t)(e + 127);
+          }
+        } else if (live) {
+          uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(g.out) + (size_t)row * g.ldc +
+                                                 ui.nb * 128);
+#pragma unroll
+          for (int v = 0; v < 16; ++v) {
+            uint32_t w[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              __nv_bfloat162 b2 = __floats2bfloat162_rn(h[v * 8 + 2 * j], h[v * 8 + 2 * j + 1]);
+              w[j] = *reinterpret_cast<uint32_t *>(&b2);
+            }
+            dst[v] = make_uint4(w[0], w[1], w[2], w[3]);
+          }
+        }
+      } else {
+        __nv_bfloat16 *crow = reinterpret_cast<__nv_bfloat16 *>(g.out) + (size_t)row * g.ldc + ui.nb * UG_BN;
+#pragma unroll 1
+        for (int c = 0; c < 8; ++c) {
+          uint32_t r[32];
+          tmem_ld_32x32b_x32(tmem + lane_base + c * 32, r);
+          tmem_ld_wait();
+          if (live) {
+            uint4 *dst = reinterpret_cast<uint4 *>(crow + c * 32);
+#pragma unroll
+            for (int v = 0; v < 4; ++v) {
+              uint32_t w[4];
+#pragma unroll
+              for (int j = 0; j < 4; ++j) {
+                __nv_bfloat162 b2 = __floats2bfloat162_rn(__uint_as_float(r[v * 8 + 2 * j]),
+                                                          __uint_as_float(r[v * 8 + 2 * j + 1]));
+                w[j] = *reinterpret_cast<uint32_t *>(&b2);
+              }
+              dst[v] = make_uint4(w[0], w[1], w[2], w[3]);
+            }
+          }
+        }
+        tc_fence_before();
+        mbar_arrive(tmem_empty);
+      }
+      acc_phase ^= 1;
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc(tmem, UG_TMEM_COLS);
+}
+
+template <bool FP8, int EPI>
+static cudaError_t launch_one(const UmmaParams &p, int grid, cudaStream_t st) {
+  auto k = umma_grouped_gemm<FP8, EPI>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)UG_SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  k<<<grid, UG_THREADS, UG_SMEM, st>>>(p);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st) {
+  if (grid <= 0) return cudaSuccess;
+  if (fp8) return epi == GEMM_SWIGLU ? launch_one<true, GEMM_SWIGLU>(p, grid, st) : launch_one<true, GEMM_PLAIN>(p, grid, st);
+  return epi == GEMM_SWIGLU ? launch_one<false, GEMM_SWIGLU>(p, grid, st) : launch_one<false, GEMM_PLAIN>(p, grid, st);
+}
+
+// ------------------------------------------------------------------ tensor maps
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    void *ptr = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
+  }
+  return fn;
+}
+
+// 2-D row-major [rows, cols] K-major operand, box = (128 bytes of K, box_rows), 128B swizzle
+bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows) {
+  auto enc = get_encode();
+  if (!enc) return false;
+  const int es = fp8 ? 1 : 2;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)(cols * es)};
+  cuuint32_t box[2] = {(cuuint32_t)(128 / es), (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(m, fp8 ? CU_TENSOR_MAP_DATA_TYPE_UINT8 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2,
+                   const_cast<void *>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+}  // namespace moe
