@@ -73,10 +73,13 @@ SMALL = {
     "toy": PRESETS["toy"],
     "v2lite_s": PRESETS["v2lite"].with_(name="v2lite_s", hidden=512, ffn=384, shared_ffn=768,
                                         prefill_tokens=200),
-    "qwen2_s": PRESETS["qwen2"].with_(name="qwen2_s", hidden=384, ffn=256, n_experts=16,
+    "qwen2_s": PRESETS["qwen2"].with_(name="qwen2_s", hidden=512, ffn=256, n_experts=16,
                                       shared_ffn=640, prefill_tokens=150),
     "v25_s": PRESETS["v25"].with_(name="v25_s", hidden=512, ffn=256, n_experts=32,
                                   shared_ffn=384, prefill_tokens=181),
+    # hidden 384 (not a multiple of 256) takes the CUDA-core GEMM path
+    "v2lite_h384": PRESETS["v2lite"].with_(name="v2lite_h384", hidden=384, ffn=256, n_experts=16,
+                                           shared_ffn=512, prefill_tokens=77),
     "v3_s": PRESETS["v3"].with_(name="v3_s", hidden=512, ffn=256, n_experts=64,
                                 shared_ffn=256, prefill_tokens=333),
 }

@@ -1,6 +1,7 @@
 // common.cuh -- shared device helpers and the layer's internal state.
 // Nothing here is shared with oracle/ (the CPU checker); see DESIGN.md §2.
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <cuda_fp8.h>
@@ -51,6 +52,17 @@ __device__ __forceinline__ float exp2i(int e) { return __uint_as_float(uint32_t(
 
 __device__ __forceinline__ uint8_t f32_to_e4m3(float v) {
   return (uint8_t)__nv_cvt_float_to_fp8(v, __NV_SATFINITE, __NV_E4M3);
+}
+
+// byte offset of the UE8M0 scale of (row, 128-col block kb) in a scale image:
+// per group of 4 k-blocks and 128-row tile, 512 B laid out as the
+// tcgen05.cp 32x128b.warpx4 source -- datapath l holds rows l, l+32, l+64,
+// l+96 (one 32-bit word each, one byte per k-block of the group).
+__device__ __forceinline__ size_t sf_img_off(int64_t row, int kb, int tile_stride) {
+  const int64_t tile = row >> 7;
+  const int r = (int)(row & 127);
+  const int word = (r & 31) * 4 + (r >> 5);
+  return ((size_t)((kb >> 2) * (int64_t)tile_stride + tile) * 128 + word) * 4 + (kb & 3);
 }
 
 __device__ __forceinline__ float silu_f(float g) { return g / (1.f + __expf(-g)); }
@@ -121,6 +133,14 @@ struct moe_layer {
   void *hsh = nullptr;          // [maxT, Fs]
   float *hsh_s = nullptr;       // [maxT, Fs/128]
   __nv_bfloat16 *ysh = nullptr; // [maxT, H]
+  // ---- tcgen05 path ----
+  bool umma = false;
+  uint8_t *w13_img = nullptr, *w2_img = nullptr, *ws13_img = nullptr, *ws2_img = nullptr;  // weight scale images
+  uint8_t *xperm_img = nullptr, *h_img = nullptr, *xq_img = nullptr, *hsh_img = nullptr;   // activation images
+  int img_tiles_sh = 0;         // ceil(maxT / 128)
+  int64_t w13_img_stride = 0, w2_img_stride = 0;
+  CUtensorMap map_xperm, map_h, map_w13, map_w2, map_xq, map_hsh, map_ws13, map_ws2;
+  int num_sms = 148;
   int64_t workspace_bytes = 0;
   int max_tiles = 0;
   // ---- stage timing (moe_layer_profile) ----

@@ -10,7 +10,8 @@ namespace moe {
 // (reading R10; north_star "128x128 block-scaled FP8" -- activations
 // take the 1x128 granularity).  One warp per (row, block): 4 values per lane.
 __global__ void __launch_bounds__(256) act_quant_kernel(const __nv_bfloat16 *__restrict__ x, int T, int H,
-                                                        uint8_t *__restrict__ xq, float *__restrict__ xs) {
+                                                        uint8_t *__restrict__ xq, float *__restrict__ xs,
+                                                        uint8_t *__restrict__ img, int img_stride) {
   const int nb = H / 128;
   const int64_t total = (int64_t)T * nb;
   const int lane = threadIdx.x & 31;
@@ -27,16 +28,20 @@ __global__ void __launch_bounds__(256) act_quant_kernel(const __nv_bfloat16 *__r
     uint32_t q = (uint32_t)f32_to_e4m3(v0.x * inv) | ((uint32_t)f32_to_e4m3(v0.y * inv) << 8) |
                  ((uint32_t)f32_to_e4m3(v1.x * inv) << 16) | ((uint32_t)f32_to_e4m3(v1.y * inv) << 24);
     *reinterpret_cast<uint32_t *>(xq + base) = q;
-    if (lane == 0) xs[row * nb + b] = exp2i(e);
+    if (lane == 0) {
+      xs[row * nb + b] = exp2i(e);
+      if (img) img[sf_img_off(row, (int)b, img_stride)] = (uint8_t)(e + 127);
+    }
   }
 }
 
-cudaError_t launch_act_quant(const void *x, int T, int H, void *xq, float *xs, cudaStream_t st) {
+cudaError_t launch_act_quant(const void *x, int T, int H, void *xq, float *xs, uint8_t *img, int img_stride,
+                             cudaStream_t st) {
   if (T <= 0) return cudaSuccess;
   const int64_t warps = (int64_t)T * (H / 128);
   const int grid = (int)std::min<int64_t>((warps + 7) / 8, 148 * 16);
   act_quant_kernel<<<grid, 256, 0, st>>>(reinterpret_cast<const __nv_bfloat16 *>(x), T, H,
-                                         reinterpret_cast<uint8_t *>(xq), xs);
+                                         reinterpret_cast<uint8_t *>(xq), xs, img, img_stride);
   return cudaGetLastError();
 }
 
@@ -46,7 +51,8 @@ __global__ void __launch_bounds__(256) gather_rows_kernel(const uint8_t *__restr
                                                           const float *__restrict__ src_s, int row_bytes,
                                                           int nscale, const int32_t *__restrict__ row_token,
                                                           const int32_t *__restrict__ offs_pad, int E,
-                                                          uint8_t *__restrict__ dst, float *__restrict__ dst_s) {
+                                                          uint8_t *__restrict__ dst, float *__restrict__ dst_s,
+                                                          uint8_t *__restrict__ dst_img, int img_stride) {
   const int64_t nrows = offs_pad[E];
   const int lane = threadIdx.x & 31;
   const int nvec = row_bytes / 16;
@@ -57,23 +63,30 @@ __global__ void __launch_bounds__(256) gather_rows_kernel(const uint8_t *__restr
       const uint4 *s = reinterpret_cast<const uint4 *>(src + (int64_t)t * row_bytes);
       for (int i = lane; i < nvec; i += 32) d[i] = __ldg(s + i);
       if (dst_s)
-        for (int i = lane; i < nscale; i += 32) dst_s[r * nscale + i] = src_s[(int64_t)t * nscale + i];
+        for (int i = lane; i < nscale; i += 32) {
+          const float s = src_s[(int64_t)t * nscale + i];
+          dst_s[r * nscale + i] = s;
+          if (dst_img) dst_img[sf_img_off(r, i, img_stride)] = (uint8_t)((__float_as_uint(s) >> 23) & 0xFF);
+        }
     } else {
       for (int i = lane; i < nvec; i += 32) d[i] = make_uint4(0, 0, 0, 0);
       if (dst_s)
-        for (int i = lane; i < nscale; i += 32) dst_s[r * nscale + i] = 1.f;
+        for (int i = lane; i < nscale; i += 32) {
+          dst_s[r * nscale + i] = 1.f;
+          if (dst_img) dst_img[sf_img_off(r, i, img_stride)] = 127;
+        }
     }
   }
 }
 
 cudaError_t launch_gather_rows(const void *src, const float *src_s, int H, int elem_bytes,
                                const int32_t *row_token, const int32_t *offs_pad, int E, int64_t R_bound,
-                               void *dst, float *dst_s, cudaStream_t st) {
+                               void *dst, float *dst_s, uint8_t *dst_img, int img_stride, cudaStream_t st) {
   if (R_bound <= 0) return cudaSuccess;
   const int grid = (int)std::min<int64_t>((R_bound + 7) / 8, 148 * 8);
   gather_rows_kernel<<<grid, 256, 0, st>>>(reinterpret_cast<const uint8_t *>(src), src_s, H * elem_bytes,
                                            H / 128, row_token, offs_pad, E,
-                                           reinterpret_cast<uint8_t *>(dst), dst_s);
+                                           reinterpret_cast<uint8_t *>(dst), dst_s, dst_img, img_stride);
   return cudaGetLastError();
 }
 

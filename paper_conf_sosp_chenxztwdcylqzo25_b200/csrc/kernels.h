@@ -1,6 +1,8 @@
 // kernels.h -- internal launch interface between the host layer (moe_api.cu)
 // and the kernels.  Not part of the public C ABI (include/moe.h).
 #pragma once
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -59,11 +61,14 @@ struct PermuteArgs {
 cudaError_t launch_permute(const PermuteArgs &a, cudaStream_t st);
 
 // x bf16 [T, H] -> e4m3 [T, H] + [T, H/128] fp32 power-of-two scales
-cudaError_t launch_act_quant(const void *x, int T, int H, void *xq, float *xs, cudaStream_t st);
+// (img != null: also the UE8M0 scale image of the T rows, tile stride img_stride)
+cudaError_t launch_act_quant(const void *x, int T, int H, void *xq, float *xs, uint8_t *img, int img_stride,
+                             cudaStream_t st);
 // rows of src (bf16 or e4m3 + scales) gathered into the padded expert order
 cudaError_t launch_gather_rows(const void *src, const float *src_s, int H, int elem_bytes,
                                const int32_t *row_token, const int32_t *offs_pad, int E,
-                               int64_t R_bound, void *dst, float *dst_s, cudaStream_t st);
+                               int64_t R_bound, void *dst, float *dst_s, uint8_t *dst_img, int img_stride,
+                               cudaStream_t st);
 
 struct CombineArgs {
   int T, H, k, n_imm;
@@ -78,5 +83,32 @@ struct CombineArgs {
   void *deferred_out;        // [T, H] or null
 };
 cudaError_t launch_combine(const CombineArgs &a, cudaStream_t st);
+
+// ---------------------------------------------------------------- tcgen05 GEMM
+struct UmmaGroup {              // one operand set: 0 = routed experts, 1 = shared expert
+  CUtensorMap a_map;            // A rows, K-major, box 128 B x 128 rows, SW128
+  CUtensorMap b_map;            // B rows of all experts stacked, box 128 B x 256 rows
+  const uint8_t *sfa;           // FP8: A scale image [K/512][tiles][512 B]
+  const uint8_t *sfb;           // FP8: B scale image [expert][K/512][N/128][512 B]
+  int64_t sfb_expert_stride;    // bytes
+  int sfa_tile_stride;          // 128-row tiles per k-group in the A image
+  int sfb_rb;                   // N/128
+  int n_total;                  // N (B rows per expert)
+  int kblocks;                  // K / 128 bytes
+  void *out;                    // C rows
+  int64_t ldc;                  // elements
+  uint8_t *out_sf;              // FP8 SwiGLU: scale image of h
+  int out_sf_tile_stride;
+};
+struct UmmaParams {
+  UmmaGroup g[2];
+  const int4 *tiles;            // routed tiles (expert, row0, row_end, t0 | nt << 16)
+  const int32_t *n_tiles;
+  int nb_r;                     // routed N blocks of 256
+  int T_shared;                 // shared-expert rows (0 = none)
+  int nb_s;                     // shared N blocks of 256
+};
+cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st);
+bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);
 
 }  // namespace moe

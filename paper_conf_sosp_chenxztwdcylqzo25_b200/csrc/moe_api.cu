@@ -47,7 +47,8 @@ void free_all(moe_layer *L) {
                   L->ws2_s, L->logits, L->topk_idx, L->topk_w, L->sgate, L->chunk_cnt, L->chunk_base,
                   L->counts, L->offs, L->offs_pad, L->tiles, L->n_tiles, L->act_list, L->n_active,
                   L->row_token, L->pos, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
-                  L->hsh, L->hsh_s, L->ysh};
+                  L->hsh, L->hsh_s, L->ysh, L->w13_img, L->w2_img, L->ws13_img, L->ws2_img,
+                  L->xperm_img, L->h_img, L->xq_img, L->hsh_img};
   for (void *p : ptrs)
     if (p) cudaFree(p);
 }
@@ -77,7 +78,7 @@ cudaError_t interleave_w13(const void *src, void *dst, int nexp, int F, int H, i
 
 // scales: copy to host, check powers of two, optionally interleave like W13
 moe_status load_scales(const float *src, float **dst, moe_layer *L, int nexp, int rows, int cols, bool inter,
-                       const char *name) {
+                       const char *name, std::vector<float> *host_out = nullptr) {
   const int rb = rows / 128, cb = cols / 128;
   const size_t n = (size_t)nexp * rb * cb;
   std::vector<float> h(n), o(n);
@@ -99,6 +100,38 @@ moe_status load_scales(const float *src, float **dst, moe_layer *L, int nexp, in
   }
   CUDA_TRY(dalloc(L, dst, n * sizeof(float), true));
   CUDA_TRY(cudaMemcpy(*dst, o.data(), n * sizeof(float), cudaMemcpyHostToDevice));
+  if (host_out) *host_out = std::move(o);
+  return MOE_OK;
+}
+
+// Scale image of a weight tensor for the tcgen05 block-scaled MMA: for every
+// expert, group of 4 K-blocks and 128-row block, 128 identical 32-bit words
+// holding the UE8M0 bytes of the 4 K-blocks (the tcgen05.cp source layout;
+// every row of a 128x128 block shares the block's scale, R10).
+moe_status build_weight_image(const std::vector<float> &s, int nexp, int rows, int cols, uint8_t **dst,
+                              moe_layer *L, int64_t *expert_stride) {
+  const int rb = rows / 128, kbn = cols / 128, G = (kbn + 3) / 4;
+  const size_t per_exp = (size_t)G * rb * 512;
+  std::vector<uint8_t> img((size_t)nexp * per_exp);
+  for (int e = 0; e < nexp; ++e)
+    for (int g = 0; g < G; ++g)
+      for (int r = 0; r < rb; ++r) {
+        uint8_t b[4];
+        for (int j = 0; j < 4; ++j) {
+          const int kb = 4 * g + j;
+          uint32_t bits = 127u << 23;
+          if (kb < kbn) {
+            float v = s[((size_t)e * rb + r) * kbn + kb];
+            memcpy(&bits, &v, 4);
+          }
+          b[j] = (uint8_t)((bits >> 23) & 0xFF);
+        }
+        uint8_t *d = img.data() + e * per_exp + ((size_t)g * rb + r) * 512;
+        for (int w = 0; w < 128; ++w) memcpy(d + 4 * w, b, 4);
+      }
+  CUDA_TRY(dalloc(L, dst, img.size(), true));
+  CUDA_TRY(cudaMemcpy(*dst, img.data(), img.size(), cudaMemcpyHostToDevice));
+  *expert_stride = (int64_t)per_exp;
   return MOE_OK;
 }
 
@@ -209,9 +242,12 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   C_TRY(interleave_w13(w->w13, L->w13, E, F, H, wes));
   C_TRY(dalloc(L, &L->w2, (size_t)E * H * F * wes, true));
   C_TRY(cudaMemcpy(L->w2, w->w2, (size_t)E * H * F * wes, cudaMemcpyDeviceToDevice));
+  L->umma = !L->f32w && (H % 256 == 0);
+  std::vector<float> hs13, hs2, hss13, hss2;
   if (L->fp8) {
-    S_TRY(load_scales(w->w13_scale, &L->w13_s, L, E, 2 * F, H, true, "w13_scale"));
-    S_TRY(load_scales(w->w2_scale, &L->w2_s, L, E, H, F, false, "w2_scale"));
+    if (!L->umma) return cleanup(fail(MOE_ERR_UNSUPPORTED, "FP8 weights need hidden %% 256 == 0"));
+    S_TRY(load_scales(w->w13_scale, &L->w13_s, L, E, 2 * F, H, true, "w13_scale", &hs13));
+    S_TRY(load_scales(w->w2_scale, &L->w2_s, L, E, H, F, false, "w2_scale", &hs2));
   }
   if (Fs > 0) {
     C_TRY(dalloc(L, &L->ws13, (size_t)2 * Fs * H * wes, true));
@@ -219,8 +255,8 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
     C_TRY(dalloc(L, &L->ws2, (size_t)H * Fs * wes, true));
     C_TRY(cudaMemcpy(L->ws2, w->ws2, (size_t)H * Fs * wes, cudaMemcpyDeviceToDevice));
     if (L->fp8) {
-      S_TRY(load_scales(w->ws13_scale, &L->ws13_s, L, 1, 2 * Fs, H, true, "ws13_scale"));
-      S_TRY(load_scales(w->ws2_scale, &L->ws2_s, L, 1, H, Fs, false, "ws2_scale"));
+      S_TRY(load_scales(w->ws13_scale, &L->ws13_s, L, 1, 2 * Fs, H, true, "ws13_scale", &hss13));
+      S_TRY(load_scales(w->ws2_scale, &L->ws2_s, L, 1, H, Fs, false, "ws2_scale", &hss2));
     }
   }
 
@@ -261,6 +297,44 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
     C_TRY(dalloc(L, &L->ysh, (size_t)Tm * H * 2, false));
   }
   C_TRY(cudaMemset(L->row_token, 0xff, (size_t)L->R_max * 4));
+
+  // ---- tcgen05 path: scale images and tensor maps ----
+  C_TRY(cudaDeviceGetAttribute(&L->num_sms, cudaDevAttrMultiProcessorCount, cfg->device));
+  if (L->umma) {
+    const bool f8 = L->fp8;
+    L->img_tiles_sh = (int)((Tm + 127) / 128);
+    if (f8) {
+      int64_t st;
+      S_TRY(build_weight_image(hs13, E, 2 * F, H, &L->w13_img, L, &st)); L->w13_img_stride = st;
+      S_TRY(build_weight_image(hs2, E, H, F, &L->w2_img, L, &st)); L->w2_img_stride = st;
+      if (Fs) {
+        S_TRY(build_weight_image(hss13, 1, 2 * Fs, H, &L->ws13_img, L, &st));
+        S_TRY(build_weight_image(hss2, 1, H, Fs, &L->ws2_img, L, &st));
+      }
+      const size_t g1 = (H / 128 + 3) / 4, g2 = (F / 128 + 3) / 4, gs = (Fs / 128 + 3) / 4;
+      C_TRY(dalloc(L, &L->xperm_img, g1 * L->max_tiles * 512, false));
+      C_TRY(dalloc(L, &L->h_img, g2 * L->max_tiles * 512, false));
+      C_TRY(dalloc(L, &L->xq_img, g1 * L->img_tiles_sh * 512, false));
+      C_TRY(cudaMemset(L->xperm_img, 127, g1 * L->max_tiles * 512));
+      C_TRY(cudaMemset(L->h_img, 127, g2 * L->max_tiles * 512));
+      C_TRY(cudaMemset(L->xq_img, 127, g1 * L->img_tiles_sh * 512));
+      if (Fs) {
+        C_TRY(dalloc(L, &L->hsh_img, gs * L->img_tiles_sh * 512, false));
+        C_TRY(cudaMemset(L->hsh_img, 127, gs * L->img_tiles_sh * 512));
+      }
+    }
+    bool ok = make_kmajor_map(&L->map_w13, L->w13, f8, (int64_t)E * 2 * F, H, 256) &&
+              make_kmajor_map(&L->map_w2, L->w2, f8, (int64_t)E * H, F, 256) &&
+              make_kmajor_map(&L->map_xperm, L->xperm, f8, L->R_max, H, 128) &&
+              make_kmajor_map(&L->map_h, L->hbuf, f8, L->R_max, F, 128);
+    if (Fs) {
+      ok = ok && make_kmajor_map(&L->map_ws13, L->ws13, f8, 2 * Fs, H, 256) &&
+           make_kmajor_map(&L->map_ws2, L->ws2, f8, H, Fs, 256) &&
+           make_kmajor_map(&L->map_hsh, L->hsh, f8, Tm, Fs, 128);
+      if (f8) ok = ok && make_kmajor_map(&L->map_xq, L->xq, true, Tm, H, 128);
+    }
+    if (!ok) return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable?)"));
+  }
   C_TRY(cudaDeviceSynchronize());
 #undef C_TRY
 #undef S_TRY
@@ -337,16 +411,67 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   const void *xa = x;
   const float *xa_s = nullptr;
   if (L->fp8) {
-    CUDA_TRY(launch_act_quant(x, T, H, L->xq, L->xs, st));
+    CUDA_TRY(launch_act_quant(x, T, H, L->xq, L->xs, L->umma ? L->xq_img : nullptr, L->img_tiles_sh, st));
     xa = L->xq;
     xa_s = L->xs;
     mark(L, ST_QUANT, st);
   }
   CUDA_TRY(launch_gather_rows(xa, xa_s, H, L->act_bytes, L->row_token, L->offs_pad, E, R_bound, L->xperm,
-                              L->xperm_s, st));
+                              L->xperm_s, L->umma ? L->xperm_img : nullptr, L->max_tiles, st));
   mark(L, ST_GATHER, st);
-  // 5. routed experts: GEMM1 + SwiGLU, GEMM2
-  {
+  if (L->umma) {
+    // 5+6. routed experts and the shared expert in one persistent tcgen05 launch per GEMM
+    const bool f8 = L->fp8;
+    const int kdiv = f8 ? 128 : 64;
+    UmmaParams p1{};
+    {
+      UmmaGroup &g = p1.g[0];
+      g.a_map = L->map_xperm; g.b_map = L->map_w13;
+      g.sfa = L->xperm_img; g.sfb = L->w13_img; g.sfb_expert_stride = L->w13_img_stride;
+      g.sfa_tile_stride = L->max_tiles; g.sfb_rb = 2 * F / 128; g.n_total = 2 * F; g.kblocks = H / kdiv;
+      g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
+    }
+    if (Fs > 0) {
+      UmmaGroup &g = p1.g[1];
+      if (f8) {
+        g.a_map = L->map_xq;
+      } else if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) {
+        return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
+      }
+      g.b_map = L->map_ws13;
+      g.sfa = L->xq_img; g.sfb = L->ws13_img; g.sfa_tile_stride = L->img_tiles_sh;
+      g.sfb_rb = 2 * Fs / 128; g.n_total = 2 * Fs; g.kblocks = H / kdiv;
+      g.out = L->hsh; g.ldc = Fs; g.out_sf = L->hsh_img; g.out_sf_tile_stride = L->img_tiles_sh;
+    } else {
+      p1.g[1] = p1.g[0];
+    }
+    p1.tiles = L->tiles; p1.n_tiles = L->n_tiles; p1.nb_r = 2 * F / 256;
+    p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = 2 * Fs / 256;
+    CUDA_TRY(launch_umma_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
+    mark(L, ST_GEMM1, st);
+    UmmaParams p2{};
+    {
+      UmmaGroup &g = p2.g[0];
+      g.a_map = L->map_h; g.b_map = L->map_w2;
+      g.sfa = L->h_img; g.sfb = L->w2_img; g.sfb_expert_stride = L->w2_img_stride;
+      g.sfa_tile_stride = L->max_tiles; g.sfb_rb = H / 128; g.n_total = H; g.kblocks = F / kdiv;
+      g.out = L->yperm; g.ldc = H;
+    }
+    if (Fs > 0) {
+      UmmaGroup &g = p2.g[1];
+      g.a_map = L->map_hsh; g.b_map = L->map_ws2;
+      g.sfa = L->hsh_img; g.sfb = L->ws2_img; g.sfa_tile_stride = L->img_tiles_sh;
+      g.sfb_rb = H / 128; g.n_total = H; g.kblocks = Fs / kdiv;
+      g.out = L->ysh; g.ldc = H;
+    } else {
+      p2.g[1] = p2.g[0];
+    }
+    p2.tiles = L->tiles; p2.n_tiles = L->n_tiles; p2.nb_r = H / 256;
+    p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256;
+    CUDA_TRY(launch_umma_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
+    mark(L, ST_GEMM2, st);
+  } else {
+    // 5. routed experts: GEMM1 + SwiGLU, GEMM2 (CUDA-core path: F32 weights, H % 256 != 0)
     SimtGemmArgs a{};
     a.A = L->xperm; a.As = L->xperm_s; a.lda = H; a.a_fp8 = L->fp8;
     a.B = L->w13; a.Bs = L->w13_s; a.b_stride = (int64_t)2 * F * H; a.bs_stride = (int64_t)(2 * F / 128) * (H / 128);
@@ -363,21 +488,21 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     b.C = L->yperm; b.ldc = H;
     CUDA_TRY(launch_simt_gemm(GEMM_PLAIN, b, 2 * tile_bound, st));
     mark(L, ST_GEMM2, st);
-  }
-  // 6. shared expert on every token
-  if (Fs > 0) {
-    SimtGemmArgs a{};
-    a.A = xa; a.As = xa_s; a.lda = H; a.a_fp8 = L->fp8;
-    a.B = L->ws13; a.Bs = L->ws13_s; a.b_type = btype; a.N = 2 * Fs; a.K = H;
-    a.M = T; a.C = L->hsh; a.Cs = L->hsh_s; a.ldc = Fs; a.out_fp8 = L->fp8;
-    CUDA_TRY(launch_simt_gemm(GEMM_SWIGLU, a, (T + 63) / 64, st));
-    mark(L, ST_SH1, st);
-    SimtGemmArgs b{};
-    b.A = L->hsh; b.As = L->hsh_s; b.lda = Fs; b.a_fp8 = L->fp8;
-    b.B = L->ws2; b.Bs = L->ws2_s; b.b_type = btype; b.N = H; b.K = Fs;
-    b.M = T; b.C = L->ysh; b.ldc = H;
-    CUDA_TRY(launch_simt_gemm(GEMM_PLAIN, b, (T + 63) / 64, st));
-    mark(L, ST_SH2, st);
+    // 6. shared expert on every token
+    if (Fs > 0) {
+      SimtGemmArgs a{};
+      a.A = xa; a.As = xa_s; a.lda = H; a.a_fp8 = L->fp8;
+      a.B = L->ws13; a.Bs = L->ws13_s; a.b_type = btype; a.N = 2 * Fs; a.K = H;
+      a.M = T; a.C = L->hsh; a.Cs = L->hsh_s; a.ldc = Fs; a.out_fp8 = L->fp8;
+      CUDA_TRY(launch_simt_gemm(GEMM_SWIGLU, a, (T + 63) / 64, st));
+      mark(L, ST_SH1, st);
+      SimtGemmArgs b{};
+      b.A = L->hsh; b.As = L->hsh_s; b.lda = Fs; b.a_fp8 = L->fp8;
+      b.B = L->ws2; b.Bs = L->ws2_s; b.b_type = btype; b.N = H; b.K = Fs;
+      b.M = T; b.C = L->ysh; b.ldc = H;
+      CUDA_TRY(launch_simt_gemm(GEMM_PLAIN, b, (T + 63) / 64, st));
+      mark(L, ST_SH2, st);
+    }
   }
   // 7. weighted combine + residual (+ deferral split)
   {

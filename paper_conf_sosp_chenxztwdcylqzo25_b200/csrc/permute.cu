@@ -68,7 +68,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(PermuteArgs a, int n
     a.offs[e] = off;
     a.offs_pad[e] = off_pad;
     for (int m = 0; m < ntile; ++m)
-      a.tiles[tile_off + m] = make_int4(e, off_pad + m * kPadM, off_pad + cnt, 0);
+      a.tiles[tile_off + m] = make_int4(e, off_pad + m * kPadM, off_pad + cnt, tile_off | (ntile << 16));
     if (cnt > 0) a.act_list[act_off] = e;
   }
   if (e == 0) {

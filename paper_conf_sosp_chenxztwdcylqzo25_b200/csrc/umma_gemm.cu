@@ -60,13 +60,6 @@ __device__ __forceinline__ UnitInfo decode_unit(const UmmaParams &p, int u, int 
   return r;
 }
 
-// byte offset of the UE8M0 scale of (row, k-block) in a scale image
-__device__ __forceinline__ size_t sf_image_offset(int row, int kb, int tile_stride) {
-  const int tile = row >> 7, r = row & 127;
-  const int word = (r & 31) * 4 + (r >> 5);
-  return ((size_t)((kb >> 2) * tile_stride + tile) * 128 + word) * 4 + (kb & 3);
-}
-
 template <bool FP8, int EPI>
 __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_constant__ UmmaParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -211,7 +204,7 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
               }
               dst[v] = make_uint4(w[0], w[1], w[2], w[3]);
             }
-            g.out_sf[sf_image_offset(row, ui.nb, g.out_sf_tile_stride)] = (uint8_t)(e + 127);
+            g.out_sf[sf_img_off(row, ui.nb, g.out_sf_tile_stride)] = (uint8_t)(e + 127);
           }
         } else if (live) {
           uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(g.out) + (size_t)row * g.ldc +
