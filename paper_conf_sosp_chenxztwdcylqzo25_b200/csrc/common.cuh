@@ -65,7 +65,7 @@ __device__ __forceinline__ size_t sf_img_off(int64_t row, int kb, int tile_strid
   return ((size_t)((kb >> 2) * (int64_t)tile_stride + tile) * 128 + word) * 4 + (kb & 3);
 }
 
-__device__ __forceinline__ float silu_f(float g) { return g / (1.f + __expf(-g)); }
+__device__ __forceinline__ float silu_f(float g) { return __fdividef(g, 1.f + __expf(-g)); }
 
 __device__ __forceinline__ float warp_max(float v) {
 #pragma unroll
@@ -121,6 +121,7 @@ struct moe_layer {
   int32_t *n_tiles = nullptr;   // [1]
   int32_t *act_list = nullptr;  // [E] active experts (count > 0), ascending
   int32_t *n_active = nullptr;  // [1]
+  int32_t *sched = nullptr;     // [4] work counters of the persistent GEMM launches
   int32_t *row_token = nullptr; // [R_max] token of each padded row (-1 = pad)
   int32_t *pos = nullptr;       // [maxT*k] padded row of (t, j) (local experts only; -1 = remote)
   void *xq = nullptr;           // [maxT, H] e4m3 (FP8 only)
@@ -139,7 +140,8 @@ struct moe_layer {
   uint8_t *xperm_img = nullptr, *h_img = nullptr, *xq_img = nullptr, *hsh_img = nullptr;   // activation images
   int img_tiles_sh = 0;         // ceil(maxT / 128)
   int64_t w13_img_stride = 0, w2_img_stride = 0;
-  CUtensorMap map_xperm, map_h, map_w13, map_w2, map_xq, map_hsh, map_ws13, map_ws2;
+  CUtensorMap map_xperm, map_h, map_w13, map_w2, map_xq, map_hsh, map_ws13, map_ws2, map_gate;
+  bool gemv_ok = false;         // decode weight-streaming path usable for T <= gemv_max_tokens
   int num_sms = 148;
   int64_t workspace_bytes = 0;
   int max_tiles = 0;

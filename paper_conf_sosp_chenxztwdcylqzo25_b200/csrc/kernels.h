@@ -4,6 +4,7 @@
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
+#include <cuda_bf16.h>
 #include <stdint.h>
 
 namespace moe {
@@ -84,6 +85,24 @@ struct CombineArgs {
 };
 cudaError_t launch_combine(const CombineArgs &a, cudaStream_t st);
 
+// ---------------------------------------------------------------- decode GEMV
+struct GemvArgs {
+  int T, H, F, Fs, fp8, has_shared;
+  const int32_t *act_list, *n_active, *counts, *offs_pad, *row_token;
+  const void *x;                 // bf16 [T, H] (BF16 weights)
+  const void *xq; const float *xs;  // e4m3 [T, H] + [T, H/128] (FP8 weights)
+  const void *w13, *w2, *ws13, *ws2;
+  const float *w13_s, *w2_s, *ws13_s, *ws2_s;
+  void *h, *hsh; float *h_s, *hsh_s;
+  __nv_bfloat16 *yperm, *ysh;
+};
+constexpr int kGemvMaxTokens = 8;
+size_t gemv_smem_bytes(int T, int H, int F, int Fs);
+// which = 1: W13 + SwiGLU -> h;  which = 2: W2 -> y rows
+cudaError_t launch_gemv(const GemvArgs &a, int which, int max_slots, cudaStream_t st);
+cudaError_t launch_router_gemv(const void *x, int T, int H, const void *wg, int rows, float *logits,
+                               cudaStream_t st);
+
 // ---------------------------------------------------------------- tcgen05 GEMM
 struct UmmaGroup {              // one operand set: 0 = routed experts, 1 = shared expert
   CUtensorMap a_map;            // A rows, K-major, box 128 B x 128 rows, SW128
@@ -99,6 +118,7 @@ struct UmmaGroup {              // one operand set: 0 = routed experts, 1 = shar
   int64_t ldc;                  // elements
   uint8_t *out_sf;              // FP8 SwiGLU: scale image of h
   int out_sf_tile_stride;
+  int n_valid;                  // LOGITS: output columns < n_valid are written
 };
 struct UmmaParams {
   UmmaGroup g[2];
@@ -107,6 +127,8 @@ struct UmmaParams {
   int nb_r;                     // routed N blocks of 256
   int T_shared;                 // shared-expert rows (0 = none)
   int nb_s;                     // shared N blocks of 256
+  int *sched;                   // device work counter, zero at launch (dynamic scheduler)
+  int debug_mode;               // 0; (MOE_DEBUG_GEMM) 1 = loads only, 2 = no epilogue -- timing experiments
 };
 cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st);
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);

@@ -5,6 +5,7 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
 #include <string>
 #include <vector>
 
@@ -46,7 +47,7 @@ void free_all(moe_layer *L) {
   void *ptrs[] = {L->gate_w, L->gate_bias, L->w13, L->w13_s, L->w2, L->w2_s, L->ws13, L->ws13_s, L->ws2,
                   L->ws2_s, L->logits, L->topk_idx, L->topk_w, L->sgate, L->chunk_cnt, L->chunk_base,
                   L->counts, L->offs, L->offs_pad, L->tiles, L->n_tiles, L->act_list, L->n_active,
-                  L->row_token, L->pos, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
+                  L->row_token, L->pos, L->sched, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
                   L->hsh, L->hsh_s, L->ysh, L->w13_img, L->w2_img, L->ws13_img, L->ws2_img,
                   L->xperm_img, L->h_img, L->xq_img, L->hsh_img};
   for (void *p : ptrs)
@@ -209,7 +210,6 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   L->f32w = cfg->wtype == MOE_W_F32;
   L->act_bytes = L->fp8 ? 1 : 2;
   L->max_tokens = cfg->max_tokens;
-  L->gemv_max_tokens = cfg->gemv_max_tokens > 0 ? cfg->gemv_max_tokens : 0;
   const int H = L->H, F = L->F, Fs = L->Fs, E = L->E, k = L->k;
   const int wes = L->fp8 ? 1 : (L->f32w ? 4 : 2);
   auto cleanup = [&](moe_status s) { free_all(L); delete L; return s; };
@@ -280,6 +280,7 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   C_TRY(dalloc(L, &L->n_tiles, 4, false));
   C_TRY(dalloc(L, &L->act_list, (size_t)E * 4, false));
   C_TRY(dalloc(L, &L->n_active, 4, false));
+  C_TRY(dalloc(L, &L->sched, 16, false));
   C_TRY(dalloc(L, &L->row_token, (size_t)L->R_max * 4, false));
   C_TRY(dalloc(L, &L->pos, (size_t)pairs * 4, false));
   if (L->fp8) {
@@ -300,6 +301,16 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
 
   // ---- tcgen05 path: scale images and tensor maps ----
   C_TRY(cudaDeviceGetAttribute(&L->num_sms, cudaDevAttrMultiProcessorCount, cfg->device));
+  if (!make_kmajor_map(&L->map_gate, L->gate_w, false, L->gate_rows, H, 256))
+    return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for the router weights"));
+  {
+    // decode switch (the L170 analog): weight streaming for T <= gemv_max_tokens
+    int g = cfg->gemv_max_tokens > 0 ? cfg->gemv_max_tokens : 4;
+    g = std::min(g, kGemvMaxTokens);
+    while (g > 0 && gemv_smem_bytes(g, H, F, Fs) > 200 * 1024) --g;
+    L->gemv_max_tokens = L->f32w ? 0 : g;
+    L->gemv_ok = L->gemv_max_tokens > 0;
+  }
   if (L->umma) {
     const bool f8 = L->fp8;
     L->img_tiles_sh = (int)((Tm + 127) / 128);
@@ -372,15 +383,23 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   const int H = L->H, F = L->F, Fs = L->Fs, E = L->E, k = L->k;
   const int btype = L->fp8 ? WT_FP8 : (L->f32w ? WT_F32 : WT_BF16);
 
-  // 1. router logits (bf16 x . bf16 Wg, fp32 accumulate)
-  {
-    SimtGemmArgs a{};
-    a.A = x; a.lda = H; a.a_fp8 = 0;
-    a.B = L->gate_w; a.b_type = WT_BF16; a.N = L->gate_rows; a.K = H;
-    a.M = T; a.C = L->logits; a.ldc = L->gate_rows;
-    CUDA_TRY(launch_simt_gemm(GEMM_LOGITS, a, (T + 63) / 64, st));
-    mark(L, ST_LOGITS, st);
+  const bool decode = L->gemv_ok && T <= L->gemv_max_tokens;
+  CUDA_TRY(cudaMemsetAsync(L->sched, 0, 16, st));
+  // 1. router logits (bf16 x . bf16 Wg, fp32 accumulate; reading R9)
+  if (T <= kGemvMaxTokens) {
+    CUDA_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
+  } else {
+    UmmaParams p{};
+    UmmaGroup &g = p.g[1];
+    if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) return fail(MOE_ERR_CUDA, "tensor map for x failed");
+    g.b_map = L->map_gate;
+    g.n_total = 0; g.kblocks = H / 64; g.out = L->logits; g.ldc = L->gate_rows; g.n_valid = L->gate_rows;
+    p.g[0] = g;
+    p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
+    const int units = ((T + 127) / 128) * p.nb_s;
+    CUDA_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
   }
+  mark(L, ST_LOGITS, st);
   // 2. scores + group-limited top-k + weights
   {
     RouterArgs r{};
@@ -416,10 +435,26 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     xa_s = L->xs;
     mark(L, ST_QUANT, st);
   }
-  CUDA_TRY(launch_gather_rows(xa, xa_s, H, L->act_bytes, L->row_token, L->offs_pad, E, R_bound, L->xperm,
-                              L->xperm_s, L->umma ? L->xperm_img : nullptr, L->max_tiles, st));
-  mark(L, ST_GATHER, st);
-  if (L->umma) {
+  if (!decode) {
+    CUDA_TRY(launch_gather_rows(xa, xa_s, H, L->act_bytes, L->row_token, L->offs_pad, E, R_bound, L->xperm,
+                                L->xperm_s, L->umma ? L->xperm_img : nullptr, L->max_tiles, st));
+    mark(L, ST_GATHER, st);
+  }
+  if (decode) {
+    // 5+6 (decode). weight-streaming GEMVs over the active experts + shared expert
+    GemvArgs g{};
+    g.T = T; g.H = H; g.F = F; g.Fs = Fs; g.fp8 = L->fp8; g.has_shared = Fs > 0;
+    g.act_list = L->act_list; g.n_active = L->n_active; g.counts = L->counts; g.offs_pad = L->offs_pad;
+    g.row_token = L->row_token; g.x = x; g.xq = L->xq; g.xs = L->xs;
+    g.w13 = L->w13; g.w2 = L->w2; g.ws13 = L->ws13; g.ws2 = L->ws2;
+    g.w13_s = L->w13_s; g.w2_s = L->w2_s; g.ws13_s = L->ws13_s; g.ws2_s = L->ws2_s;
+    g.h = L->hbuf; g.hsh = L->hsh; g.h_s = L->h_s; g.hsh_s = L->hsh_s; g.yperm = L->yperm; g.ysh = L->ysh;
+    const int slots = (int)std::min<int64_t>(E, pairs) + (Fs > 0 ? 1 : 0);
+    CUDA_TRY(launch_gemv(g, 1, slots, st));
+    mark(L, ST_GEMM1, st);
+    CUDA_TRY(launch_gemv(g, 2, slots, st));
+    mark(L, ST_GEMM2, st);
+  } else if (L->umma) {
     // 5+6. routed experts and the shared expert in one persistent tcgen05 launch per GEMM
     const bool f8 = L->fp8;
     const int kdiv = f8 ? 128 : 64;
@@ -446,7 +481,9 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
       p1.g[1] = p1.g[0];
     }
     p1.tiles = L->tiles; p1.n_tiles = L->n_tiles; p1.nb_r = 2 * F / 256;
-    p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = 2 * Fs / 256;
+    p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = 2 * Fs / 256; p1.sched = L->sched;
+    static const int dbg_mode = getenv("MOE_DEBUG_GEMM") ? atoi(getenv("MOE_DEBUG_GEMM")) : 0;
+    p1.debug_mode = dbg_mode;
     CUDA_TRY(launch_umma_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
     mark(L, ST_GEMM1, st);
     UmmaParams p2{};
@@ -467,7 +504,8 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
       p2.g[1] = p2.g[0];
     }
     p2.tiles = L->tiles; p2.n_tiles = L->n_tiles; p2.nb_r = H / 256;
-    p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256;
+    p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256; p2.sched = L->sched + 1;
+    p2.debug_mode = dbg_mode;
     CUDA_TRY(launch_umma_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
     mark(L, ST_GEMM2, st);
   } else {

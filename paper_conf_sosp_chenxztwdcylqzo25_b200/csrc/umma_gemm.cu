@@ -14,10 +14,10 @@
 // Work units = (expert m-tile of 128 rows, 256-wide n-block), ordered expert-
 // major then n-block then m-tile so CTAs running concurrently share one weight
 // slab through L2 (the device-side analog of PAPER.md L181's co-scheduling of
-// same-expert tasks).  Roles per CTA (192 threads, one CTA per SM):
+// same-expert tasks).  Roles per CTA (320 threads, one CTA per SM):
 //   warp 0     TMA producer (A/B tiles, FP8 scale images) into a 4-stage ring
 //   warp 1     TMEM allocator + single-thread tcgen05.mma issuer
-//   warps 2-5  epilogue: tcgen05.ld -> registers -> global
+//   warps 2-9  epilogue: tcgen05.ld -> registers (TMEM released) -> math -> global
 #include <cuda.h>
 
 #include "common.cuh"
@@ -27,14 +27,15 @@
 namespace moe {
 using namespace sm100;
 
-constexpr int UG_BM = 128, UG_BN = 256, UG_STAGES = 4, UG_THREADS = 192;
+constexpr int UG_BM = 128, UG_BN = 256, UG_STAGES = 4, UG_THREADS = 320;
 constexpr int UG_A_BYTES = UG_BM * 128;        // 16 KB (128 rows x 128 B)
 constexpr int UG_B_BYTES = UG_BN * 128;        // 32 KB
 constexpr int UG_SFA_BYTES = 512;              // 128 rows x 4 B image
 constexpr int UG_SFB_BYTES = 1024;             // 256 rows x 4 B image
 constexpr uint32_t UG_TMEM_COLS = 512;
 constexpr uint32_t UG_SFA_COL = 256, UG_SFB_COL = 264;
-constexpr size_t UG_SMEM = 1024 + (size_t)UG_STAGES * (UG_A_BYTES + UG_B_BYTES + UG_SFA_BYTES + UG_SFB_BYTES) + 256;
+constexpr int UG_UQ = 4;                       // depth of the in-CTA work-unit queue
+constexpr size_t UG_SMEM = 1024 + (size_t)UG_STAGES * (UG_A_BYTES + UG_B_BYTES + UG_SFA_BYTES + UG_SFB_BYTES) + 512 + 2048;
 
 struct UnitInfo {
   int valid, group, expert, row0, row_end, nb;
@@ -72,7 +73,10 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
   uint64_t *empty = full + UG_STAGES;
   uint64_t *tmem_full = empty + UG_STAGES;
   uint64_t *tmem_empty = tmem_full + 1;
-  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(tmem_empty + 1);
+  uint64_t *uq_full = tmem_empty + 1;
+  uint64_t *uq_empty = uq_full + UG_UQ;
+  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(uq_empty + UG_UQ);
+  int *unit_q = reinterpret_cast<int *>(tmem_base_smem + 4);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int n_routed_units = p.tiles ? (*p.n_tiles) * p.nb_r : 0;
@@ -82,7 +86,8 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
     prefetch_tmap(&p.g[1].a_map); prefetch_tmap(&p.g[1].b_map);
     for (int s = 0; s < UG_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     mbar_init(tmem_full, 1);
-    mbar_init(tmem_empty, 128);
+    mbar_init(tmem_empty, 8);
+    for (int i = 0; i < UG_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], 9); }
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc(tmem_base_smem, UG_TMEM_COLS);
@@ -95,7 +100,16 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
     // ============================ TMA producer ============================
     if (lane == 0) {
       int stage = 0; uint32_t phase = 0;
-      for (int u = blockIdx.x;; u += gridDim.x) {
+      int qs = 0; uint32_t qph = 0;
+      for (;;) {
+        // dynamic tile scheduler (PAPER.md L181 analog): units are claimed in
+        // index order by whichever CTA is free, so CTAs sharing an expert's
+        // weight slab run at the same time and reuse it through L2
+        const int u = atomicAdd(p.sched, 1);
+        mbar_wait(&uq_empty[qs], qph ^ 1);
+        unit_q[qs] = u;
+        mbar_arrive(&uq_full[qs]);
+        if (++qs == UG_UQ) { qs = 0; qph ^= 1; }
         const UnitInfo ui = decode_unit(p, u, n_routed_units);
         if (!ui.valid) break;
         const UmmaGroup &g = p.g[ui.group];
@@ -122,7 +136,13 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
   } else if (warp == 1) {
     // ============================ MMA issuer ============================
     int stage = 0; uint32_t phase = 0; uint32_t acc_phase = 0;
-    for (int u = blockIdx.x;; u += gridDim.x) {
+    int qs = 0; uint32_t qph = 0;
+    for (;;) {
+      mbar_wait(&uq_full[qs], qph);
+      const int u = unit_q[qs];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&uq_empty[qs]);
+      if (++qs == UG_UQ) { qs = 0; qph ^= 1; }
       const UnitInfo ui = decode_unit(p, u, n_routed_units);
       if (!ui.valid) break;
       const int kblocks = p.g[ui.group].kblocks;
@@ -131,7 +151,7 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
       for (int kb = 0; kb < kblocks; ++kb) {
         mbar_wait(&full[stage], phase);
         tc_fence_after();
-        if (lane == 0) {
+        if (lane == 0 && p.debug_mode != 1) {
           const uint32_t a0 = smem_u32(sA + stage * UG_A_BYTES);
           const uint32_t b0 = smem_u32(sB + stage * UG_B_BYTES);
           if (FP8) {
@@ -152,6 +172,9 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
           }
           mma_commit(&empty[stage]);
           if (kb == kblocks - 1) mma_commit(tmem_full);
+        } else if (lane == 0) {            // debug_mode 1: load pipeline only
+          mbar_arrive(&empty[stage]);
+          if (kb == kblocks - 1) mbar_arrive(tmem_full);
         }
         __syncwarp();
         if (++stage == UG_STAGES) { stage = 0; phase ^= 1; }
@@ -160,10 +183,22 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
     }
   } else {
     // ============================ epilogue ============================
+    // 8 warps: two per TMEM lane quadrant, each owning half of the columns.
+    // Each thread pulls its accumulator columns into registers, releases TMEM
+    // at once (so the next unit's MMAs overlap the math), then computes.
+    const int ew = warp - 2;                      // 0..7
     const int q = warp & 3;                       // TMEM lane quadrant of this warp
+    const int half = ew >> 2;                     // column half
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
+    float *red = reinterpret_cast<float *>(unit_q + UG_UQ);   // [2 parity][2 half][128 rows]
     uint32_t acc_phase = 0;
-    for (int u = blockIdx.x;; u += gridDim.x) {
+    int qs = 0; uint32_t qph = 0;
+    for (;;) {
+      mbar_wait(&uq_full[qs], qph);
+      const int u = unit_q[qs];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&uq_empty[qs]);
+      if (++qs == UG_UQ) { qs = 0; qph ^= 1; }
       const UnitInfo ui = decode_unit(p, u, n_routed_units);
       if (!ui.valid) break;
       const UmmaGroup &g = p.g[ui.group];
@@ -171,30 +206,44 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
       tc_fence_after();
       const int row = ui.row0 + q * 32 + lane;
       const bool live = row < ui.row_end;
-      if constexpr (EPI == GEMM_SWIGLU) {
-        float h[128];
-#pragma unroll
-        for (int c = 0; c < 4; ++c) {
-          uint32_t gr[32], ur[32];
-          tmem_ld_32x32b_x32(tmem + lane_base + c * 32, gr);
-          tmem_ld_32x32b_x32(tmem + lane_base + 128 + c * 32, ur);
-          tmem_ld_wait();
-#pragma unroll
-          for (int i = 0; i < 32; ++i) h[c * 32 + i] = silu_f(__uint_as_float(gr[i])) * __uint_as_float(ur[i]);
-        }
+      if (p.debug_mode >= 1) {            // debug: no epilogue work
         tc_fence_before();
-        mbar_arrive(tmem_empty);
-        if (FP8) {
-          float amax = 0.f;
+        __syncwarp();
+        if (lane == 0) mbar_arrive(tmem_empty);
+        acc_phase ^= 1;
+        continue;
+      }
+      if constexpr (EPI == GEMM_SWIGLU) {
+        // gate columns [64*half, +64), up columns [128 + 64*half, +64)
+        uint32_t gr[64], ur[64];
+        tmem_ld_32x32b_x32(tmem + lane_base + half * 64, *reinterpret_cast<uint32_t(*)[32]>(gr));
+        tmem_ld_32x32b_x32(tmem + lane_base + half * 64 + 32, *reinterpret_cast<uint32_t(*)[32]>(gr + 32));
+        tmem_ld_32x32b_x32(tmem + lane_base + 128 + half * 64, *reinterpret_cast<uint32_t(*)[32]>(ur));
+        tmem_ld_32x32b_x32(tmem + lane_base + 128 + half * 64 + 32, *reinterpret_cast<uint32_t(*)[32]>(ur + 32));
+        tmem_ld_wait();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(tmem_empty);
+        float h[64];
+        float amax = 0.f;
 #pragma unroll
-          for (int i = 0; i < 128; ++i) amax = fmaxf(amax, fabsf(h[i]));
+        for (int i = 0; i < 64; ++i) {
+          h[i] = silu_f(__uint_as_float(gr[i])) * __uint_as_float(ur[i]);
+          amax = fmaxf(amax, fabsf(h[i]));
+        }
+        const int f0 = ui.nb * 128 + half * 64;
+        if (FP8) {
+          // the 1x128 block of h spans both halves: exchange partial amax
+          float *rb = red + (acc_phase * 2) * 128;
+          rb[half * 128 + q * 32 + lane] = amax;
+          asm volatile("bar.sync 1, 256;" ::: "memory");
+          amax = fmaxf(amax, rb[(half ^ 1) * 128 + q * 32 + lane]);
           const int e = ue8m0_exponent(amax);
           const float inv = exp2i(-e);
           if (live) {
-            uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<uint8_t *>(g.out) + (size_t)row * g.ldc +
-                                                   ui.nb * 128);
+            uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<uint8_t *>(g.out) + (size_t)row * g.ldc + f0);
 #pragma unroll
-            for (int v = 0; v < 8; ++v) {
+            for (int v = 0; v < 4; ++v) {
               uint32_t w[4];
 #pragma unroll
               for (int j = 0; j < 4; ++j) {
@@ -204,13 +253,12 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
               }
               dst[v] = make_uint4(w[0], w[1], w[2], w[3]);
             }
-            g.out_sf[sf_img_off(row, ui.nb, g.out_sf_tile_stride)] = (uint8_t)(e + 127);
+            if (half == 0) g.out_sf[sf_img_off(row, ui.nb, g.out_sf_tile_stride)] = (uint8_t)(e + 127);
           }
         } else if (live) {
-          uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(g.out) + (size_t)row * g.ldc +
-                                                 ui.nb * 128);
+          uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(g.out) + (size_t)row * g.ldc + f0);
 #pragma unroll
-          for (int v = 0; v < 16; ++v) {
+          for (int v = 0; v < 8; ++v) {
             uint32_t w[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
@@ -221,29 +269,38 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
           }
         }
       } else {
-        __nv_bfloat16 *crow = reinterpret_cast<__nv_bfloat16 *>(g.out) + (size_t)row * g.ldc + ui.nb * UG_BN;
-#pragma unroll 1
-        for (int c = 0; c < 8; ++c) {
-          uint32_t r[32];
-          tmem_ld_32x32b_x32(tmem + lane_base + c * 32, r);
-          tmem_ld_wait();
+        // PLAIN (bf16 rows) / LOGITS (fp32 rows): columns [128*half, +128)
+        uint32_t r[128];
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+          tmem_ld_32x32b_x32(tmem + lane_base + half * 128 + c * 32, *reinterpret_cast<uint32_t(*)[32]>(r + 32 * c));
+        tmem_ld_wait();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(tmem_empty);
+        const int n0 = ui.nb * UG_BN + half * 128;
+        if constexpr (EPI == GEMM_LOGITS) {
+          // router logits: fp32 columns n < n_valid (PAPER.md L187 gating network)
           if (live) {
-            uint4 *dst = reinterpret_cast<uint4 *>(crow + c * 32);
+            float *crow = reinterpret_cast<float *>(g.out) + (size_t)row * g.ldc;
 #pragma unroll
-            for (int v = 0; v < 4; ++v) {
-              uint32_t w[4];
+            for (int i = 0; i < 128; ++i)
+              if (n0 + i < g.n_valid) crow[n0 + i] = __uint_as_float(r[i]);
+          }
+        } else if (live) {
+          uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(g.out) + (size_t)row * g.ldc + n0);
 #pragma unroll
-              for (int j = 0; j < 4; ++j) {
-                __nv_bfloat162 b2 = __floats2bfloat162_rn(__uint_as_float(r[v * 8 + 2 * j]),
-                                                          __uint_as_float(r[v * 8 + 2 * j + 1]));
-                w[j] = *reinterpret_cast<uint32_t *>(&b2);
-              }
-              dst[v] = make_uint4(w[0], w[1], w[2], w[3]);
+          for (int v = 0; v < 16; ++v) {
+            uint32_t w[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              __nv_bfloat162 b2 = __floats2bfloat162_rn(__uint_as_float(r[v * 8 + 2 * j]),
+                                                        __uint_as_float(r[v * 8 + 2 * j + 1]));
+              w[j] = *reinterpret_cast<uint32_t *>(&b2);
             }
+            dst[v] = make_uint4(w[0], w[1], w[2], w[3]);
           }
         }
-        tc_fence_before();
-        mbar_arrive(tmem_empty);
       }
       acc_phase ^= 1;
     }
@@ -268,6 +325,7 @@ static cudaError_t launch_one(const UmmaParams &p, int grid, cudaStream_t st) {
 
 cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st) {
   if (grid <= 0) return cudaSuccess;
+  if (epi == GEMM_LOGITS) return launch_one<false, GEMM_LOGITS>(p, grid, st);
   if (fp8) return epi == GEMM_SWIGLU ? launch_one<true, GEMM_SWIGLU>(p, grid, st) : launch_one<true, GEMM_PLAIN>(p, grid, st);
   return epi == GEMM_SWIGLU ? launch_one<false, GEMM_SWIGLU>(p, grid, st) : launch_one<false, GEMM_PLAIN>(p, grid, st);
 }

@@ -80,6 +80,19 @@ def test_small_decode_shapes(lib, name, T):
     assert rel_l2(res["y"], out["y"]) <= TOL[p.wtype]
 
 
+@pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v25_s"])
+@pytest.mark.parametrize("T,gemv", [(4, 4), (8, 8), (8, 0), (6, 1)])
+def test_decode_gemv_vs_gemm_paths(lib, name, T, gemv):
+    """Weight-streaming decode path (T <= gemv_max_tokens) and the tcgen05 path
+    (T above it) both match the oracle (kernel switch by ARI)."""
+    p = SMALL[name]
+    res = _run(lib, p, T, max_tokens=16, gemv=gemv)
+    out, ties, idx, w = _oracle(p, res)
+    g = res["routing"]
+    check_routing(g["topk_idx"], g["topk_w"], idx, w, ties, p.routed_scale, p.norm_topk)
+    assert rel_l2(res["y"], out["y"]) <= TOL[p.wtype]
+
+
 @pytest.mark.parametrize("name", ["v3_s", "qwen2_s"])
 def test_residual_and_deferral(lib, name):
     """Eq. L241 middle case: y = I + S + R^imm + R^def_{k-1}; deferred_out = R^def."""
