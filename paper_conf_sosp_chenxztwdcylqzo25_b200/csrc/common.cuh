@@ -97,7 +97,8 @@ struct moe_layer {
   void *gate_w = nullptr;      // [E_glob (+1 shared gate row), H] bf16
   float *gate_bias = nullptr;  // [E_glob] or null
   int gate_rows = 0;
-  void *w13 = nullptr;         // [E, 2F, H]  rows interleaved per 128: (W1 blk b, W3 blk b)
+  void *w13 = nullptr;         // [E, 2F, H]  rows interleaved per 128: (W1 blk b, W3 blk b);
+                               // tcgen05 path: as 256-row x 128-byte SW128 tiles
   float *w13_s = nullptr;      // [E, 2F/128, H/128]  (same interleave)
   void *w2 = nullptr;          // [E, H, F]
   float *w2_s = nullptr;       // [E, H/128, F/128]
@@ -121,7 +122,7 @@ struct moe_layer {
   int32_t *n_tiles = nullptr;   // [1]
   int32_t *act_list = nullptr;  // [E] active experts (count > 0), ascending
   int32_t *n_active = nullptr;  // [1]
-  int32_t *sched = nullptr;     // [4] work counters of the persistent GEMM launches
+  int32_t *sched = nullptr;     // [8] work counters of the persistent GEMM launches
   int32_t *row_token = nullptr; // [R_max] token of each padded row (-1 = pad)
   int32_t *pos = nullptr;       // [maxT*k] padded row of (t, j) (local experts only; -1 = remote)
   void *xq = nullptr;           // [maxT, H] e4m3 (FP8 only)
@@ -140,7 +141,8 @@ struct moe_layer {
   uint8_t *xperm_img = nullptr, *h_img = nullptr, *xq_img = nullptr, *hsh_img = nullptr;   // activation images
   int img_tiles_sh = 0;         // ceil(maxT / 128)
   int64_t w13_img_stride = 0, w2_img_stride = 0;
-  CUtensorMap map_xperm, map_h, map_w13, map_w2, map_xq, map_hsh, map_ws13, map_ws2, map_gate;
+  CUtensorMap map_xperm, map_h, map_xq, map_hsh, map_gate;   // activation rows (box 128), router rows
+  CUtensorMap dmap_xperm, dmap_h, dmap_xq, dmap_hsh;           // decode: activation rows (box 16)
   bool gemv_ok = false;         // decode weight-streaming path usable for T <= gemv_max_tokens
   int num_sms = 148;
   int64_t workspace_bytes = 0;

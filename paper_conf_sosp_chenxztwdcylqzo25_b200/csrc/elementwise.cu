@@ -90,6 +90,90 @@ cudaError_t launch_gather_rows(const void *src, const float *src_s, int H, int e
   return cudaGetLastError();
 }
 
+// decode: FP8 quantisation + gather fused.  CTA per active expert slot: warp w
+// quantises (or copies) token row w of the expert's segment into x_perm
+// (rows >= count zeroed); the extra last CTA quantises all T tokens into xq for
+// the shared expert.  Scale bytes go straight into the tcgen05 scale images.
+// One warp quantises a row: all loads issued up front (lane l holds 8-element
+// chunks c = 32 i + l), one 1x128 block = 16 lanes -> half-warp amax reduction.
+__device__ __forceinline__ void quant_row_e4m3(const __nv_bfloat16 *__restrict__ src, uint8_t *__restrict__ dst,
+                                               int H, int64_t row, uint8_t *img, int img_stride, float *xs_row,
+                                               int lane) {
+  constexpr int G = 16;                             // chunks per lane per batch (64 registers)
+  const int nc = H / 8;
+  for (int c0 = 0; c0 < nc; c0 += G * 32) {
+  uint4 v[G];
+#pragma unroll
+  for (int i = 0; i < G; ++i) {
+    const int c = c0 + i * 32 + lane;
+    if (c < nc) v[i] = __ldg(reinterpret_cast<const uint4 *>(src) + c);
+  }
+#pragma unroll
+  for (int i = 0; i < G; ++i) {
+    if (c0 + i * 32 >= nc) break;
+    const int c = c0 + i * 32 + lane;
+    float f[8];
+    bf16x8_to_f32(v[i], f);
+    float am = 0.f;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) am = fmaxf(am, fabsf(f[j]));
+#pragma unroll
+    for (int o = 8; o > 0; o >>= 1) am = fmaxf(am, __shfl_xor_sync(0xffffffffu, am, o));
+    const int e = ue8m0_exponent(am);
+    const float inv = exp2i(-e);
+    uint2 q;
+    q.x = (uint32_t)f32_to_e4m3(f[0] * inv) | ((uint32_t)f32_to_e4m3(f[1] * inv) << 8) |
+          ((uint32_t)f32_to_e4m3(f[2] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[3] * inv) << 24);
+    q.y = (uint32_t)f32_to_e4m3(f[4] * inv) | ((uint32_t)f32_to_e4m3(f[5] * inv) << 8) |
+          ((uint32_t)f32_to_e4m3(f[6] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[7] * inv) << 24);
+    if (c < nc) {
+      *reinterpret_cast<uint2 *>(dst + c * 8) = q;
+      if ((lane & 15) == 0) {
+        const int b = c / 16;                       // 128-element block index
+        if (img) img[sf_img_off(row, b, img_stride)] = (uint8_t)(e + 127);
+        if (xs_row) xs_row[b] = exp2i(e);
+      }
+    }
+  }
+  }
+}
+
+__global__ void __launch_bounds__(512) quant_gather_decode_kernel(QuantGatherArgs a) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int H = a.H;
+  const __nv_bfloat16 *x = reinterpret_cast<const __nv_bfloat16 *>(a.x);
+  if ((int)blockIdx.x == a.max_slots) {            // shared expert: all tokens -> xq
+    if (!a.xq) return;
+    for (int t = warp; t < a.T; t += 16)
+      quant_row_e4m3(x + (size_t)t * H, reinterpret_cast<uint8_t *>(a.xq) + (size_t)t * H, H, t, a.xq_img,
+                     a.xq_img_stride, a.xs ? a.xs + (size_t)t * (H / 128) : nullptr, lane);
+    return;
+  }
+  if ((int)blockIdx.x >= *a.n_active) return;
+  const int e = a.act_list[blockIdx.x];
+  const int64_t r = (int64_t)a.offs_pad[e] + warp;
+  const int t = warp < a.counts[e] ? a.row_token[r] : -1;
+  if (a.fp8) {
+    uint8_t *d = reinterpret_cast<uint8_t *>(a.xperm) + r * H;
+    if (t >= 0) {
+      quant_row_e4m3(x + (size_t)t * H, d, H, r, a.xperm_img, a.xperm_img_stride, nullptr, lane);
+    } else {
+      for (int i = lane; i < H / 16; i += 32) reinterpret_cast<uint4 *>(d)[i] = make_uint4(0, 0, 0, 0);
+      for (int b = lane; b < H / 128; b += 32) a.xperm_img[sf_img_off(r, b, a.xperm_img_stride)] = 127;
+    }
+  } else {
+    uint4 *d = reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(a.xperm) + r * H);
+    const uint4 *sp = reinterpret_cast<const uint4 *>(x + (size_t)(t >= 0 ? t : 0) * H);
+    for (int i = lane; i < H / 8; i += 32) d[i] = t >= 0 ? __ldg(sp + i) : make_uint4(0, 0, 0, 0);
+  }
+}
+
+cudaError_t launch_quant_gather_decode(const QuantGatherArgs &a, cudaStream_t st) {
+  if (a.T <= 0) return cudaSuccess;
+  quant_gather_decode_kernel<<<a.max_slots + 1, 512, 0, st>>>(a);
+  return cudaGetLastError();
+}
+
 // ------------------------------------------------------------------ combine
 // y[t]   = residual[t] + g_t * ys[t] + sum_{j < n_imm} w_tj * yperm[pos(t,j)] + deferred_in[t]
 // dout[t] = sum_{j >= n_imm} w_tj * yperm[pos(t,j)]
@@ -105,7 +189,7 @@ __global__ void __launch_bounds__(128) combine_kernel(CombineArgs a) {
   __syncthreads();
   const float g = a.sgate ? a.sgate[t] : 1.f;
   const int nvec = a.H / 8;
-  for (int v = threadIdx.x; v < nvec; v += blockDim.x) {
+  for (int v = blockIdx.y * blockDim.x + threadIdx.x; v < nvec; v += gridDim.y * blockDim.x) {
     float acc[8], dacc[8], tmp[8];
 #pragma unroll
     for (int i = 0; i < 8; ++i) { acc[i] = 0.f; dacc[i] = 0.f; }
@@ -154,7 +238,8 @@ __global__ void __launch_bounds__(128) combine_kernel(CombineArgs a) {
 
 cudaError_t launch_combine(const CombineArgs &a, cudaStream_t st) {
   if (a.T <= 0) return cudaSuccess;
-  combine_kernel<<<a.T, 128, 0, st>>>(a);
+  // one CTA per (token, 1024 channels): enough CTAs to fill the GPU at T = 1
+  combine_kernel<<<dim3(a.T, (a.H / 8 + 127) / 128), 128, 0, st>>>(a);
   return cudaGetLastError();
 }
 

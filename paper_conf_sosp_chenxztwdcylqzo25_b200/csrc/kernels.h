@@ -61,6 +61,18 @@ struct PermuteArgs {
 };
 cudaError_t launch_permute(const PermuteArgs &a, cudaStream_t st);
 
+// decode (T <= 16): router logits + selection + permutation in one launch
+struct RouteSmallArgs {
+  RouterArgs r;
+  PermuteArgs p;
+  const void *x;                // bf16 [T, H]
+  const void *wg;               // bf16 [rows, H]
+  int H, rows;
+  int *done;                    // zero-initialised CTA counter (re-armed by the kernel)
+  int debug;                    // timing experiments only (MOE_DEBUG_ROUTE): 1 skip logits, 2 skip tail
+};
+cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st);
+
 // x bf16 [T, H] -> e4m3 [T, H] + [T, H/128] fp32 power-of-two scales
 // (img != null: also the UE8M0 scale image of the T rows, tile stride img_stride)
 cudaError_t launch_act_quant(const void *x, int T, int H, void *xq, float *xs, uint8_t *img, int img_stride,
@@ -106,7 +118,9 @@ cudaError_t launch_router_gemv(const void *x, int T, int H, const void *wg, int 
 // ---------------------------------------------------------------- tcgen05 GEMM
 struct UmmaGroup {              // one operand set: 0 = routed experts, 1 = shared expert
   CUtensorMap a_map;            // A rows, K-major, box 128 B x 128 rows, SW128
-  CUtensorMap b_map;            // B rows of all experts stacked, box 128 B x 256 rows
+  CUtensorMap b_map;            // B rows via TMA (router logits only; expert weights are tiled)
+  const uint8_t *b_tiles;       // tiled weights: [expert][N/256][K/128B][256 rows x 128 B, SW128]
+  int b_ntiles_n;               // N / 256
   const uint8_t *sfa;           // FP8: A scale image [K/512][tiles][512 B]
   const uint8_t *sfb;           // FP8: B scale image [expert][K/512][N/128][512 B]
   int64_t sfb_expert_stride;    // bytes
@@ -131,6 +145,33 @@ struct UmmaParams {
   int debug_mode;               // 0; (MOE_DEBUG_GEMM) 1 = loads only, 2 = no epilogue -- timing experiments
 };
 cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st);
+// Repack row-major weights [rows, K] (es bytes/elem) into 256-row x 128-byte
+// tiles, 128B-swizzled (the smem image TMA would produce).  interleave_f > 0:
+// rows are W13 [2F, K] and tile rows are ordered (W1 block b, W3 block b) per 128.
+cudaError_t launch_tile_weights(const void *src, void *dst, int nexp, int rows, int kbytes, int interleave_f,
+                                cudaStream_t st);
+
+// decode (swap-AB): a_map = activation rows (box 16), b_map = weight rows (box 128),
+// sfa = activation scale image, sfb = weight scale image (same fields as UmmaGroup)
+struct UmmaDecodeParams {
+  UmmaGroup g[2];               // 0 routed, 1 shared
+  int g_nblk[2];                // 128-row blocks per group (MODE 1: F/128, MODE 2: H/128)
+  int nblk;                     // max of g_nblk
+  int max_slots, has_shared, T;
+  const int32_t *n_active, *act_list, *counts, *offs_pad;
+  int *sched;
+};
+cudaError_t launch_umma_decode(bool fp8, int mode, const UmmaDecodeParams &p, int grid, cudaStream_t st);
+// decode: FP8 quantisation / bf16 copy of the tokens into the first 16 rows of
+// each active expert segment, plus xq for the shared expert (one launch)
+struct QuantGatherArgs {
+  const void *x;                 // bf16 [T, H]
+  int T, H, fp8, max_slots;
+  const int32_t *act_list, *n_active, *counts, *offs_pad, *row_token;
+  void *xperm; uint8_t *xperm_img; int xperm_img_stride;
+  void *xq; float *xs; uint8_t *xq_img; int xq_img_stride;   // shared expert (FP8; xq null = none)
+};
+cudaError_t launch_quant_gather_decode(const QuantGatherArgs &a, cudaStream_t st);
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);
 
 }  // namespace moe

@@ -239,10 +239,14 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   }
   // ---- routed experts ----
   C_TRY(dalloc(L, &L->w13, (size_t)E * 2 * F * H * wes, true));
-  C_TRY(interleave_w13(w->w13, L->w13, E, F, H, wes));
-  C_TRY(dalloc(L, &L->w2, (size_t)E * H * F * wes, true));
-  C_TRY(cudaMemcpy(L->w2, w->w2, (size_t)E * H * F * wes, cudaMemcpyDeviceToDevice));
   L->umma = !L->f32w && (H % 256 == 0);
+  // tcgen05 path: weights repacked into 256-row x 128-byte SW128 tiles (one
+  // contiguous 32 KB read per k-block); CUDA-core path: row-major, W13 interleaved
+  if (L->umma) C_TRY(launch_tile_weights(w->w13, L->w13, E, 2 * F, H * wes, F, 0));
+  else C_TRY(interleave_w13(w->w13, L->w13, E, F, H, wes));
+  C_TRY(dalloc(L, &L->w2, (size_t)E * H * F * wes, true));
+  if (L->umma) C_TRY(launch_tile_weights(w->w2, L->w2, E, H, F * wes, 0, 0));
+  else C_TRY(cudaMemcpy(L->w2, w->w2, (size_t)E * H * F * wes, cudaMemcpyDeviceToDevice));
   std::vector<float> hs13, hs2, hss13, hss2;
   if (L->fp8) {
     if (!L->umma) return cleanup(fail(MOE_ERR_UNSUPPORTED, "FP8 weights need hidden %% 256 == 0"));
@@ -251,9 +255,11 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   }
   if (Fs > 0) {
     C_TRY(dalloc(L, &L->ws13, (size_t)2 * Fs * H * wes, true));
-    C_TRY(interleave_w13(w->ws13, L->ws13, 1, Fs, H, wes));
+    if (L->umma) C_TRY(launch_tile_weights(w->ws13, L->ws13, 1, 2 * Fs, H * wes, Fs, 0));
+    else C_TRY(interleave_w13(w->ws13, L->ws13, 1, Fs, H, wes));
     C_TRY(dalloc(L, &L->ws2, (size_t)H * Fs * wes, true));
-    C_TRY(cudaMemcpy(L->ws2, w->ws2, (size_t)H * Fs * wes, cudaMemcpyDeviceToDevice));
+    if (L->umma) C_TRY(launch_tile_weights(w->ws2, L->ws2, 1, H, Fs * wes, 0, 0));
+    else C_TRY(cudaMemcpy(L->ws2, w->ws2, (size_t)H * Fs * wes, cudaMemcpyDeviceToDevice));
     if (L->fp8) {
       S_TRY(load_scales(w->ws13_scale, &L->ws13_s, L, 1, 2 * Fs, H, true, "ws13_scale", &hss13));
       S_TRY(load_scales(w->ws2_scale, &L->ws2_s, L, 1, H, Fs, false, "ws2_scale", &hss2));
@@ -280,7 +286,7 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   C_TRY(dalloc(L, &L->n_tiles, 4, false));
   C_TRY(dalloc(L, &L->act_list, (size_t)E * 4, false));
   C_TRY(dalloc(L, &L->n_active, 4, false));
-  C_TRY(dalloc(L, &L->sched, 16, false));
+  C_TRY(dalloc(L, &L->sched, 32, false));
   C_TRY(dalloc(L, &L->row_token, (size_t)L->R_max * 4, false));
   C_TRY(dalloc(L, &L->pos, (size_t)pairs * 4, false));
   if (L->fp8) {
@@ -305,9 +311,13 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
     return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for the router weights"));
   {
     // decode switch (the L170 analog): weight streaming for T <= gemv_max_tokens
-    int g = cfg->gemv_max_tokens > 0 ? cfg->gemv_max_tokens : 4;
-    g = std::min(g, kGemvMaxTokens);
-    while (g > 0 && gemv_smem_bytes(g, H, F, Fs) > 200 * 1024) --g;
+    // tensor-core decode (swap-AB, N = 16 tokens) when the tcgen05 path is
+    // available, else the CUDA-core GEMV for up to 8 tokens
+    const bool tc = !L->f32w && (H % 256 == 0);
+    int g = cfg->gemv_max_tokens > 0 ? cfg->gemv_max_tokens : (tc ? 16 : 4);
+    g = std::min(g, tc ? 16 : kGemvMaxTokens);
+    if (!tc)
+      while (g > 0 && gemv_smem_bytes(g, H, F, Fs) > 200 * 1024) --g;
     L->gemv_max_tokens = L->f32w ? 0 : g;
     L->gemv_ok = L->gemv_max_tokens > 0;
   }
@@ -334,15 +344,17 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
         C_TRY(cudaMemset(L->hsh_img, 127, gs * L->img_tiles_sh * 512));
       }
     }
-    bool ok = make_kmajor_map(&L->map_w13, L->w13, f8, (int64_t)E * 2 * F, H, 256) &&
-              make_kmajor_map(&L->map_w2, L->w2, f8, (int64_t)E * H, F, 256) &&
-              make_kmajor_map(&L->map_xperm, L->xperm, f8, L->R_max, H, 128) &&
+    bool ok = make_kmajor_map(&L->map_xperm, L->xperm, f8, L->R_max, H, 128) &&
               make_kmajor_map(&L->map_h, L->hbuf, f8, L->R_max, F, 128);
     if (Fs) {
-      ok = ok && make_kmajor_map(&L->map_ws13, L->ws13, f8, 2 * Fs, H, 256) &&
-           make_kmajor_map(&L->map_ws2, L->ws2, f8, H, Fs, 256) &&
-           make_kmajor_map(&L->map_hsh, L->hsh, f8, Tm, Fs, 128);
+      ok = ok && make_kmajor_map(&L->map_hsh, L->hsh, f8, Tm, Fs, 128);
       if (f8) ok = ok && make_kmajor_map(&L->map_xq, L->xq, true, Tm, H, 128);
+    }
+    ok = ok && make_kmajor_map(&L->dmap_xperm, L->xperm, f8, L->R_max, H, 16) &&
+         make_kmajor_map(&L->dmap_h, L->hbuf, f8, L->R_max, F, 16);
+    if (Fs) {
+      ok = ok && make_kmajor_map(&L->dmap_hsh, L->hsh, f8, Tm, Fs, 16);
+      if (f8) ok = ok && make_kmajor_map(&L->dmap_xq, L->xq, true, Tm, H, 16);
     }
     if (!ok) return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable?)"));
   }
@@ -384,43 +396,50 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   const int btype = L->fp8 ? WT_FP8 : (L->f32w ? WT_F32 : WT_BF16);
 
   const bool decode = L->gemv_ok && T <= L->gemv_max_tokens;
-  CUDA_TRY(cudaMemsetAsync(L->sched, 0, 16, st));
-  // 1. router logits (bf16 x . bf16 Wg, fp32 accumulate; reading R9)
-  if (T <= kGemvMaxTokens) {
-    CUDA_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
+  const bool tc_decode = decode && L->umma;        // T <= 16: fused small-T route + swap-AB kernels
+  CUDA_TRY(cudaMemsetAsync(L->sched, 0, 32, st));
+  RouterArgs r{};
+  r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
+  r.T = T; r.E = L->E_glob; r.k = k; r.n_group = L->cfg.n_group; r.topk_group = L->cfg.topk_group;
+  r.group_score = L->cfg.group_score; r.score_fn = L->cfg.score_fn; r.norm_topk = L->cfg.norm_topk;
+  r.routed_scale = L->cfg.routed_scale; r.shared_gated = L->cfg.shared_gated;
+  r.topk_idx = L->topk_idx; r.topk_w = L->topk_w; r.sgate = L->sgate;
+  PermuteArgs pa{};
+  pa.topk_idx = L->topk_idx; pa.T = T; pa.k = k; pa.E = E; pa.e0 = L->e0;
+  pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
+  pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
+  pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
+  pa.dbg_perm = dbg ? dbg->perm : nullptr;
+  pa.dbg_counts = dbg ? dbg->expert_counts : nullptr;
+  if (tc_decode) {
+    // 1-3 (decode). logits + select + count/scan/assign in one launch
+    RouteSmallArgs rs{};
+    rs.r = r; rs.p = pa; rs.x = x; rs.wg = L->gate_w; rs.H = H; rs.rows = L->gate_rows; rs.done = L->sched + 7;
+    static const int dbg_route = getenv("MOE_DEBUG_ROUTE") ? atoi(getenv("MOE_DEBUG_ROUTE")) : 0;
+    rs.debug = dbg_route;
+    CUDA_TRY(launch_route_small(rs, st));
+    mark(L, ST_PERMUTE, st);
   } else {
-    UmmaParams p{};
-    UmmaGroup &g = p.g[1];
-    if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) return fail(MOE_ERR_CUDA, "tensor map for x failed");
-    g.b_map = L->map_gate;
-    g.n_total = 0; g.kblocks = H / 64; g.out = L->logits; g.ldc = L->gate_rows; g.n_valid = L->gate_rows;
-    p.g[0] = g;
-    p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
-    const int units = ((T + 127) / 128) * p.nb_s;
-    CUDA_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
-  }
-  mark(L, ST_LOGITS, st);
-  // 2. scores + group-limited top-k + weights
-  {
-    RouterArgs r{};
-    r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
-    r.T = T; r.E = L->E_glob; r.k = k; r.n_group = L->cfg.n_group; r.topk_group = L->cfg.topk_group;
-    r.group_score = L->cfg.group_score; r.score_fn = L->cfg.score_fn; r.norm_topk = L->cfg.norm_topk;
-    r.routed_scale = L->cfg.routed_scale; r.shared_gated = L->cfg.shared_gated;
-    r.topk_idx = L->topk_idx; r.topk_w = L->topk_w; r.sgate = L->sgate;
+    // 1. router logits (bf16 x . bf16 Wg, fp32 accumulate; reading R9)
+    if (T <= kGemvMaxTokens) {
+      CUDA_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
+    } else {
+      UmmaParams p{};
+      UmmaGroup &g = p.g[1];
+      if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) return fail(MOE_ERR_CUDA, "tensor map for x failed");
+      g.b_map = L->map_gate;
+      g.n_total = 0; g.kblocks = H / 64; g.out = L->logits; g.ldc = L->gate_rows; g.n_valid = L->gate_rows;
+      p.g[0] = g;
+      p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
+      const int units = ((T + 127) / 128) * p.nb_s;
+      CUDA_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
+    }
+    mark(L, ST_LOGITS, st);
+    // 2. scores + group-limited top-k + weights
     CUDA_TRY(launch_router_select(r, st));
     mark(L, ST_SELECT, st);
-  }
-  // 3. count / scan / permute
-  {
-    PermuteArgs p{};
-    p.topk_idx = L->topk_idx; p.T = T; p.k = k; p.E = E; p.e0 = L->e0;
-    p.chunk_cnt = L->chunk_cnt; p.chunk_base = L->chunk_base; p.counts = L->counts; p.offs = L->offs;
-    p.offs_pad = L->offs_pad; p.tiles = L->tiles; p.n_tiles = L->n_tiles; p.act_list = L->act_list;
-    p.n_active = L->n_active; p.row_token = L->row_token; p.R_max = L->R_max; p.pos = L->pos;
-    p.dbg_perm = dbg ? dbg->perm : nullptr;
-    p.dbg_counts = dbg ? dbg->expert_counts : nullptr;
-    CUDA_TRY(launch_permute(p, st));
+    // 3. count / scan / permute
+    CUDA_TRY(launch_permute(pa, st));
     mark(L, ST_PERMUTE, st);
   }
   const int64_t pairs = (int64_t)T * k;
@@ -429,7 +448,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   // 4. activation quantisation (FP8) and gather into expert order
   const void *xa = x;
   const float *xa_s = nullptr;
-  if (L->fp8) {
+  if (L->fp8 && !tc_decode) {
     CUDA_TRY(launch_act_quant(x, T, H, L->xq, L->xs, L->umma ? L->xq_img : nullptr, L->img_tiles_sh, st));
     xa = L->xq;
     xa_s = L->xs;
@@ -440,8 +459,71 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
                                 L->xperm_s, L->umma ? L->xperm_img : nullptr, L->max_tiles, st));
     mark(L, ST_GATHER, st);
   }
-  if (decode) {
-    // 5+6 (decode). weight-streaming GEMVs over the active experts + shared expert
+  if (decode && L->umma) {
+    // 5+6 (decode). swap-AB tensor-core weight stream over the active experts + shared expert
+    const bool f8 = L->fp8;
+    const int kdiv = f8 ? 128 : 64;
+    const int slots = (int)std::min<int64_t>(E, pairs) + (Fs > 0 ? 1 : 0);
+    QuantGatherArgs qg{};
+    qg.x = x; qg.T = T; qg.H = H; qg.fp8 = f8; qg.max_slots = (int)std::min<int64_t>(E, pairs);
+    qg.act_list = L->act_list; qg.n_active = L->n_active; qg.counts = L->counts; qg.offs_pad = L->offs_pad;
+    qg.row_token = L->row_token; qg.xperm = L->xperm; qg.xperm_img = L->xperm_img; qg.xperm_img_stride = L->max_tiles;
+    if (f8 && Fs > 0) { qg.xq = L->xq; qg.xs = L->xs; qg.xq_img = L->xq_img; qg.xq_img_stride = L->img_tiles_sh; }
+    CUDA_TRY(launch_quant_gather_decode(qg, st));
+    mark(L, ST_GATHER, st);
+    UmmaDecodeParams d1{};
+    {
+      UmmaGroup &g = d1.g[0];
+      g.a_map = L->dmap_xperm; g.b_tiles = (const uint8_t *)L->w13; g.b_ntiles_n = 2 * F / 256;
+      g.sfa = L->xperm_img; g.sfa_tile_stride = L->max_tiles;
+      g.sfb = L->w13_img; g.sfb_expert_stride = L->w13_img_stride; g.sfb_rb = 2 * F / 128;
+      g.n_total = 2 * F; g.kblocks = H / kdiv;
+      g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
+    }
+    if (Fs > 0) {
+      UmmaGroup &g = d1.g[1];
+      if (f8) {
+        g.a_map = L->dmap_xq;
+      } else if (!make_kmajor_map(&g.a_map, x, false, T, H, 16)) {
+        return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
+      }
+      g.b_tiles = (const uint8_t *)L->ws13; g.b_ntiles_n = 2 * Fs / 256;
+      g.sfa = L->xq_img; g.sfa_tile_stride = L->img_tiles_sh;
+      g.sfb = L->ws13_img; g.sfb_rb = 2 * Fs / 128; g.n_total = 0; g.kblocks = H / kdiv;
+      g.out = L->hsh; g.ldc = Fs; g.out_sf = L->hsh_img; g.out_sf_tile_stride = L->img_tiles_sh;
+    } else {
+      d1.g[1] = d1.g[0];
+    }
+    d1.g_nblk[0] = F / 128; d1.g_nblk[1] = Fs / 128; d1.nblk = std::max(F, Fs) / 128;
+    d1.max_slots = slots; d1.has_shared = Fs > 0; d1.T = T;
+    d1.n_active = L->n_active; d1.act_list = L->act_list; d1.counts = L->counts; d1.offs_pad = L->offs_pad;
+    d1.sched = L->sched + 3;
+    CUDA_TRY(launch_umma_decode(f8, 1, d1, std::min(L->num_sms, slots * d1.nblk), st));
+    mark(L, ST_GEMM1, st);
+    UmmaDecodeParams d2 = d1;
+    {
+      UmmaGroup &g = d2.g[0];
+      g.a_map = L->dmap_h; g.b_tiles = (const uint8_t *)L->w2; g.b_ntiles_n = H / 256;
+      g.sfa = L->h_img; g.sfa_tile_stride = L->max_tiles;
+      g.sfb = L->w2_img; g.sfb_expert_stride = L->w2_img_stride; g.sfb_rb = H / 128;
+      g.n_total = H; g.kblocks = F / kdiv;
+      g.out = L->yperm; g.ldc = H; g.out_sf = nullptr;
+    }
+    if (Fs > 0) {
+      UmmaGroup &g = d2.g[1];
+      g.a_map = L->dmap_hsh; g.b_tiles = (const uint8_t *)L->ws2; g.b_ntiles_n = H / 256;
+      g.sfa = L->hsh_img; g.sfa_tile_stride = L->img_tiles_sh;
+      g.sfb = L->ws2_img; g.sfb_rb = H / 128; g.n_total = 0; g.kblocks = Fs / kdiv;
+      g.out = L->ysh; g.ldc = H; g.out_sf = nullptr;
+    } else {
+      d2.g[1] = d2.g[0];
+    }
+    d2.g_nblk[0] = H / 128; d2.g_nblk[1] = H / 128; d2.nblk = H / 128;
+    d2.sched = L->sched + 4;
+    CUDA_TRY(launch_umma_decode(f8, 2, d2, std::min(L->num_sms, slots * d2.nblk), st));
+    mark(L, ST_GEMM2, st);
+  } else if (decode) {
+    // 5+6 (decode, CUDA-core path). weight-streaming GEMVs over the active experts + shared expert
     GemvArgs g{};
     g.T = T; g.H = H; g.F = F; g.Fs = Fs; g.fp8 = L->fp8; g.has_shared = Fs > 0;
     g.act_list = L->act_list; g.n_active = L->n_active; g.counts = L->counts; g.offs_pad = L->offs_pad;
@@ -461,7 +543,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     UmmaParams p1{};
     {
       UmmaGroup &g = p1.g[0];
-      g.a_map = L->map_xperm; g.b_map = L->map_w13;
+      g.a_map = L->map_xperm; g.b_tiles = (const uint8_t *)L->w13; g.b_ntiles_n = 2 * F / 256;
       g.sfa = L->xperm_img; g.sfb = L->w13_img; g.sfb_expert_stride = L->w13_img_stride;
       g.sfa_tile_stride = L->max_tiles; g.sfb_rb = 2 * F / 128; g.n_total = 2 * F; g.kblocks = H / kdiv;
       g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
@@ -473,7 +555,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
       } else if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) {
         return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
       }
-      g.b_map = L->map_ws13;
+      g.b_tiles = (const uint8_t *)L->ws13; g.b_ntiles_n = 2 * Fs / 256;
       g.sfa = L->xq_img; g.sfb = L->ws13_img; g.sfa_tile_stride = L->img_tiles_sh;
       g.sfb_rb = 2 * Fs / 128; g.n_total = 2 * Fs; g.kblocks = H / kdiv;
       g.out = L->hsh; g.ldc = Fs; g.out_sf = L->hsh_img; g.out_sf_tile_stride = L->img_tiles_sh;
@@ -489,14 +571,14 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     UmmaParams p2{};
     {
       UmmaGroup &g = p2.g[0];
-      g.a_map = L->map_h; g.b_map = L->map_w2;
+      g.a_map = L->map_h; g.b_tiles = (const uint8_t *)L->w2; g.b_ntiles_n = H / 256;
       g.sfa = L->h_img; g.sfb = L->w2_img; g.sfb_expert_stride = L->w2_img_stride;
       g.sfa_tile_stride = L->max_tiles; g.sfb_rb = H / 128; g.n_total = H; g.kblocks = F / kdiv;
       g.out = L->yperm; g.ldc = H;
     }
     if (Fs > 0) {
       UmmaGroup &g = p2.g[1];
-      g.a_map = L->map_hsh; g.b_map = L->map_ws2;
+      g.a_map = L->map_hsh; g.b_tiles = (const uint8_t *)L->ws2; g.b_ntiles_n = H / 256;
       g.sfa = L->hsh_img; g.sfb = L->ws2_img; g.sfa_tile_stride = L->img_tiles_sh;
       g.sfb_rb = H / 128; g.n_total = H; g.kblocks = Fs / kdiv;
       g.out = L->ysh; g.ldc = H;

@@ -8,6 +8,9 @@
 //           others excluded;  idx = top_k(sel)  (ties -> lower id, reading R2)
 //   w = s[idx] (/ sum w if norm_topk) * routed_scale
 //   slots written in canonical order: w descending, ties -> lower id (R4)
+#include <algorithm>
+#include <cub/block/block_scan.cuh>
+
 #include "common.cuh"
 #include "kernels.h"
 
@@ -29,42 +32,54 @@ __device__ __forceinline__ void warp_argmax(float &v, int &i) {
   }
 }
 
-__global__ void __launch_bounds__(RT_WARPS * 32)
-router_select_kernel(RouterArgs a) {
-  extern __shared__ float smem[];
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int t = blockIdx.x * RT_WARPS + warp;
-  if (t >= a.T) return;
+// One warp routes token t (scratch s/sel: 2 x E floats of shared memory).
+__device__ void select_token(const RouterArgs &args, int t, float *s, float *sel, int lane) {
+  // copy the arguments into registers: the stores below go through generic
+  // pointers the compiler cannot prove disjoint from the argument struct, and
+  // re-loading the fields in every loop iteration costs ~30x the work
+  struct {
+    int E, k, n_group, topk_group, group_score, score_fn, norm_topk, shared_gated;
+    float routed_scale;
+    const float *bias;
+    int32_t *topk_idx;
+    float *topk_w, *sgate;
+  } a = {args.E, args.k, args.n_group, args.topk_group, args.group_score, args.score_fn, args.norm_topk,
+         args.shared_gated, args.routed_scale, args.bias, args.topk_idx, args.topk_w, args.sgate};
   const int E = a.E;
-  float *s = smem + warp * 2 * E;   // scores
-  float *sel = s + E;               // selection scores
-  const float *lg = a.logits + (int64_t)t * a.ldl;
+  const float *lg = args.logits + (int64_t)t * args.ldl;
 
   // ---- scores ----
+  // (compact rolled loops: this code runs once per token on one warp, so its
+  //  instruction footprint -- cold in the i-cache -- sets the latency)
   if (a.score_fn == MOE_SCORE_SOFTMAX) {
     float m = -INFINITY;
+#pragma unroll 1
     for (int e = lane; e < E; e += 32) m = fmaxf(m, lg[e]);
     m = warp_max(m);
     float sum = 0.f;
+#pragma unroll 1
     for (int e = lane; e < E; e += 32) {
-      float v = expf(lg[e] - m);
+      const float v = expf(lg[e] - m);
       s[e] = v;
       sum += v;
     }
     sum = warp_sum(sum);
+#pragma unroll 1
     for (int e = lane; e < E; e += 32) s[e] = s[e] / sum;
   } else {
+#pragma unroll 1
     for (int e = lane; e < E; e += 32) s[e] = 1.f / (1.f + expf(-lg[e]));
   }
+#pragma unroll 1
   for (int e = lane; e < E; e += 32) sel[e] = s[e] + (a.bias ? a.bias[e] : 0.f);
   __syncwarp();
-
   // ---- group limit ----
   if (a.n_group > 1) {
     const int G = a.n_group, gs = E / G;
     float gscore = -INFINITY;
     if (lane < G) {
       float m1 = -INFINITY, m2 = -INFINITY;
+#pragma unroll 1
       for (int i = 0; i < gs; ++i) {
         float v = sel[lane * gs + i];
         if (v > m1) { m2 = m1; m1 = v; } else if (v > m2) { m2 = v; }
@@ -73,6 +88,7 @@ router_select_kernel(RouterArgs a) {
     }
     bool keep = false;
     float gv = (lane < G) ? gscore : -INFINITY;
+#pragma unroll 1
     for (int r = 0; r < a.topk_group; ++r) {
       float v = (lane < G && !keep) ? gv : -INFINITY;
       int i = (lane < G && !keep) ? lane : 0x7fffffff;
@@ -80,6 +96,7 @@ router_select_kernel(RouterArgs a) {
       if (lane == i) keep = true;
     }
     const unsigned keep_mask = __ballot_sync(0xffffffffu, keep);
+#pragma unroll 1
     for (int e = lane; e < E; e += 32)
       if (!((keep_mask >> (e / gs)) & 1u)) sel[e] = -INFINITY;
     __syncwarp();
@@ -87,11 +104,13 @@ router_select_kernel(RouterArgs a) {
 
   // ---- top-k ----
   int my_id = -1;
+#pragma unroll 1
   for (int j = 0; j < a.k; ++j) {
     float v = -INFINITY;
     int i = 0x7fffffff;
+#pragma unroll 1
     for (int e = lane; e < E; e += 32) {
-      float x = sel[e];
+      const float x = sel[e];
       if (better(x, e, v, i)) { v = x; i = e; }
     }
     warp_argmax(v, i);
@@ -110,6 +129,7 @@ router_select_kernel(RouterArgs a) {
 
   // ---- canonical order: w descending, ties -> lower id ----
   int rank = 0;
+#pragma unroll 1
   for (int i = 0; i < a.k; ++i) {
     float wi = __shfl_sync(0xffffffffu, w, i);
     int ii = __shfl_sync(0xffffffffu, my_id, i);
@@ -120,6 +140,271 @@ router_select_kernel(RouterArgs a) {
     a.topk_w[(int64_t)t * a.k + rank] = w;
   }
   if (a.shared_gated && lane == 0) a.sgate[t] = 1.f / (1.f + expf(-lg[E]));
+}
+
+__global__ void __launch_bounds__(RT_WARPS * 32)
+router_select_kernel(RouterArgs a) {
+  extern __shared__ float smem[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int t = blockIdx.x * RT_WARPS + warp;
+  if (t >= a.T) return;
+  select_token(a, t, smem + warp * 2 * a.E, smem + warp * 2 * a.E + a.E, lane);
+}
+
+// Block-parallel routing of ONE token (decode): every thread owns <= 4 experts;
+// selection by rank (rank(e) = #experts that beat e) instead of k sequential
+// arg-max rounds, so the latency is a few short loops over shared memory.
+// Same rules and tie-breaks as select_token.  Scratch: s[E], sel[E], gsc[32],
+// ids[32], ws[32] in shared memory.
+template <int NT>
+__device__ void select_token_block(const RouterArgs &args, int t, float *s, float *sel, float *gsc, int *ids,
+                                   float *ws) {
+  const int E = args.E, k = args.k, G = args.n_group, TG = args.topk_group;
+  const float *lg = args.logits + (int64_t)t * args.ldl;
+  const float *bias = args.bias;
+  const int tid = threadIdx.x;
+  __shared__ float red[NT / 32];
+  // scores
+  float lv[4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) lv[i] = (tid + NT * i < E) ? lg[tid + NT * i] : -INFINITY;
+  if (args.score_fn == MOE_SCORE_SOFTMAX) {
+    float m = fmaxf(fmaxf(lv[0], lv[1]), fmaxf(lv[2], lv[3]));
+    m = warp_max(m);
+    if ((tid & 31) == 0) red[tid >> 5] = m;
+    __syncthreads();
+    m = red[0];
+#pragma unroll 1
+    for (int w = 1; w < NT / 32; ++w) m = fmaxf(m, red[w]);
+    __syncthreads();
+    float sum = 0.f;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) { lv[i] = (tid + NT * i < E) ? expf(lv[i] - m) : 0.f; sum += lv[i]; }
+    sum = warp_sum(sum);
+    if ((tid & 31) == 0) red[tid >> 5] = sum;
+    __syncthreads();
+    sum = 0.f;
+#pragma unroll 1
+    for (int w = 0; w < NT / 32; ++w) sum += red[w];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) lv[i] = lv[i] / sum;
+  } else {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) lv[i] = 1.f / (1.f + expf(-lv[i]));
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int e = tid + NT * i;
+    if (e < E) { s[e] = lv[i]; sel[e] = lv[i] + (bias ? bias[e] : 0.f); }
+  }
+  __syncthreads();
+  // group limit: thread g scores group g, then ranks it
+  if (G > 1) {
+    const int gs = E / G;
+    if (tid < G) {
+      float m1 = -INFINITY, m2 = -INFINITY;
+#pragma unroll 1
+      for (int i = 0; i < gs; ++i) {
+        const float v = sel[tid * gs + i];
+        if (v > m1) { m2 = m1; m1 = v; } else if (v > m2) { m2 = v; }
+      }
+      gsc[tid] = args.group_score == MOE_GROUP_TOP2_SUM ? m1 + m2 : m1;
+    }
+    __syncthreads();
+    if (tid < G) {
+      int rk = 0;
+#pragma unroll 1
+      for (int g = 0; g < G; ++g) rk += better(gsc[g], g, gsc[tid], tid);
+      ids[tid] = rk < TG;                          // keep flag
+    }
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int e = tid + NT * i;
+      if (e < E && !ids[e / gs]) sel[e] = -INFINITY;
+    }
+    __syncthreads();
+  }
+  // expert rank among the allowed ones; the k best land in ids/ws by rank
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int e = tid + NT * i;
+    if (e < E && sel[e] != -INFINITY) {
+      const float v = sel[e];
+      int rk = 0;
+#pragma unroll 4
+      for (int j = 0; j < E; ++j) rk += better(sel[j], j, v, e);
+      if (rk < k) { ids[rk] = e; ws[rk] = s[e]; }
+    }
+  }
+  __syncthreads();
+  // weights + canonical order (warp 0)
+  if (tid < 32) {
+    const int lane = tid;
+    const int my_id = lane < k ? ids[lane] : 0x7fffffff;
+    float w = lane < k ? ws[lane] : 0.f;
+    if (args.norm_topk) w = w / warp_sum(w);
+    w = w * args.routed_scale;
+    int rank = 0;
+#pragma unroll 1
+    for (int i = 0; i < k; ++i) {
+      const float wi = __shfl_sync(0xffffffffu, w, i);
+      const int ii = __shfl_sync(0xffffffffu, my_id, i);
+      if (lane < k && i != lane && better(wi, ii, w, my_id)) ++rank;
+    }
+    if (lane < k) {
+      args.topk_idx[(int64_t)t * k + rank] = my_id;
+      args.topk_w[(int64_t)t * k + rank] = w;
+    }
+    if (args.shared_gated && lane == 0) args.sgate[t] = 1.f / (1.f + expf(-lg[E]));
+  }
+  __syncthreads();
+}
+
+// ------------------------------------------------------------------ small T (decode)
+// One launch for T <= 16 tokens: every CTA computes the router logits of two
+// router rows (128 threads per row, whole row loaded at once), the last CTA to
+// finish routes the tokens (select_token) and builds the expert-sorted order
+// (counts, offsets, active-expert list, stable positions) -- the launch chain
+// logits -> select -> count/scan/assign collapsed for the latency-bound decode step.
+constexpr int RS_THREADS = 256;
+
+__global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs a) {
+  extern __shared__ float rsm[];
+  const RouterArgs &r = a.r;
+  const int H = a.H, T = r.T;
+  const int half = threadIdx.x >> 7, tid = threadIdx.x & 127;
+  const int row = blockIdx.x * 2 + half;
+  __shared__ float red[2][4][16];
+  __shared__ int is_last;
+  // ---- logits of router rows `row` for all T tokens ----
+  {
+    float acc[16];
+#pragma unroll
+    for (int t = 0; t < 16; ++t) acc[t] = 0.f;
+    if (row < a.rows && !(a.debug & 1)) {
+      const uint4 *wr = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.wg) + (size_t)row * H);
+      const int nv = H / 8;
+      for (int c0 = tid; c0 < nv; c0 += 128 * 8) {
+        uint4 w[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) w[u] = (c0 + u * 128 < nv) ? __ldg(wr + c0 + u * 128) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          const int c = c0 + u * 128;
+          if (c >= nv) break;
+          float wf[8];
+          bf16x8_to_f32(w[u], wf);
+#pragma unroll 4
+          for (int t = 0; t < 16; ++t) {
+            if (t < T) {
+              float xf[8];
+              bf16x8_to_f32(__ldg(reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.x) +
+                                                                  (size_t)t * H) + c), xf);
+#pragma unroll
+              for (int j = 0; j < 8; ++j) acc[t] = fmaf(wf[j], xf[j], acc[t]);
+            }
+          }
+        }
+      }
+    }
+    const int w4 = tid >> 5, lane = threadIdx.x & 31;
+#pragma unroll
+    for (int t = 0; t < 16; ++t) {
+      const float v = warp_sum(acc[t]);
+      if (lane == 0) red[half][w4][t] = v;
+    }
+    __syncthreads();
+    if (row < a.rows && tid < T)
+      const_cast<float *>(r.logits)[(size_t)tid * r.ldl + row] = red[half][0][tid] + red[half][1][tid] + red[half][2][tid] + red[half][3][tid];
+  }
+  // ---- last CTA: route + permute ----
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) is_last = (atomicAdd(a.done, 1) == (int)gridDim.x - 1);
+  __syncthreads();
+  if (!is_last) return;
+  if (a.debug & 2) { if (threadIdx.x == 0) *a.done = 0; return; }
+  __threadfence();
+  {
+    float *s = rsm, *sel = rsm + r.E, *gsc = rsm + 2 * r.E, *ws = gsc + 32;
+    int *ids = reinterpret_cast<int *>(ws + 32);
+#pragma unroll 1
+    for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws);
+  }
+  // counts / offsets / active list over the local experts
+  const PermuteArgs &p = a.p;
+  int *cnt = reinterpret_cast<int *>(rsm);          // reuse scratch: [E] counts, [E] running
+  int *run = cnt + p.E;
+  for (int e = threadIdx.x; e < p.E; e += RS_THREADS) cnt[e] = 0;
+  __syncthreads();
+  for (int q = threadIdx.x; q < T * p.k; q += RS_THREADS) {
+    const int e = p.topk_idx[q] - p.e0;
+    p.pos[q] = -1;
+    if (e >= 0 && e < p.E) atomicAdd(&cnt[e], 1);
+  }
+  __syncthreads();
+  {
+    // one exclusive scan over the experts of a packed triple (count | tiles << 11 |
+    // active << 21): T*k <= 512 rows, <= 1024 tiles and experts -- 4 experts per thread
+    using Scan = cub::BlockScan<int, RS_THREADS>;
+    __shared__ typename Scan::TempStorage tmp;
+    int v[4], o[4], tot;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int e = threadIdx.x * 4 + i;
+      const int c = e < p.E ? cnt[e] : 0;
+      v[i] = c | (((c + kPadM - 1) / kPadM) << 11) | ((c > 0) << 21);
+    }
+    Scan(tmp).ExclusiveSum(v, o, tot);
+    if (threadIdx.x == 0) {
+      p.offs[p.E] = tot & 2047;
+      p.offs_pad[p.E] = ((tot >> 11) & 1023) * kPadM;
+      *p.n_active = tot >> 21;
+      *p.n_tiles = 0;
+      *a.done = 0;                                 // re-arm the CTA counter (graph replay)
+    }
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int e = threadIdx.x * 4 + i;
+      if (e < p.E) {
+        const int c = v[i] & 2047;
+        p.counts[e] = c;
+        if (p.dbg_counts) p.dbg_counts[e] = c;
+        p.offs[e] = o[i] & 2047;
+        p.offs_pad[e] = ((o[i] >> 11) & 1023) * kPadM;
+        run[e] = 0;
+        if (c > 0) p.act_list[o[i] >> 21] = e;
+      }
+    }
+  }
+  __syncthreads();
+  // stable assignment: tokens in order, a token's k experts are distinct
+  for (int t = 0; t < T; ++t) {
+    if (threadIdx.x < p.k) {
+      const int q = t * p.k + threadIdx.x;
+      const int e = p.topk_idx[q] - p.e0;
+      if (e >= 0 && e < p.E) {
+        const int i = run[e]++;
+        const int rw = p.offs_pad[e] + i;
+        p.row_token[rw] = t;
+        p.pos[q] = rw;
+        if (p.dbg_perm) p.dbg_perm[p.offs[e] + i] = t;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st) {
+  if (a.r.T <= 0) return cudaSuccess;
+  const size_t sm = std::max<size_t>((size_t)(RS_THREADS / 32) * 2 * a.r.E * sizeof(float), 2 * a.p.E * sizeof(int));
+  if (sm > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(route_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    if (e != cudaSuccess) return e;
+  }
+  route_small_kernel<<<(a.rows + 1) / 2, RS_THREADS, sm, st>>>(a);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_router_select(const RouterArgs &a, cudaStream_t st) {

@@ -82,8 +82,8 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
   const int n_routed_units = p.tiles ? (*p.n_tiles) * p.nb_r : 0;
 
   if (warp == 0 && lane == 0) {
-    prefetch_tmap(&p.g[0].a_map); prefetch_tmap(&p.g[0].b_map);
-    prefetch_tmap(&p.g[1].a_map); prefetch_tmap(&p.g[1].b_map);
+    prefetch_tmap(&p.g[0].a_map); prefetch_tmap(&p.g[1].a_map);
+    if (EPI == GEMM_LOGITS) prefetch_tmap(&p.g[0].b_map);
     for (int s = 0; s < UG_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     mbar_init(tmem_full, 1);
     mbar_init(tmem_empty, 8);
@@ -121,7 +121,13 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
           mbar_expect_tx(&full[stage], bytes);
           const int kc = kb * (FP8 ? 128 : 64);   // element coordinate along K
           tma_load_2d(sA + stage * UG_A_BYTES, &g.a_map, &full[stage], kc, ui.row0);
-          tma_load_2d(sB + stage * UG_B_BYTES, &g.b_map, &full[stage], kc, brow);
+          if (EPI == GEMM_LOGITS) {
+            tma_load_2d(sB + stage * UG_B_BYTES, &g.b_map, &full[stage], kc, brow);
+          } else {
+            // pre-tiled weights: one contiguous 32 KB read per k-block (L157 load-time layout)
+            const uint8_t *bt = g.b_tiles + (((size_t)ui.expert * g.b_ntiles_n + ui.nb) * g.kblocks + kb) * UG_B_BYTES;
+            bulk_load(sB + stage * UG_B_BYTES, bt, UG_B_BYTES, &full[stage]);
+          }
           if (FP8) {
             const uint8_t *sfa = g.sfa + ((size_t)(kb >> 2) * g.sfa_tile_stride + (ui.row0 >> 7)) * 512;
             const uint8_t *sfb = g.sfb + (size_t)ui.expert * g.sfb_expert_stride +
@@ -328,6 +334,43 @@ cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, c
   if (epi == GEMM_LOGITS) return launch_one<false, GEMM_LOGITS>(p, grid, st);
   if (fp8) return epi == GEMM_SWIGLU ? launch_one<true, GEMM_SWIGLU>(p, grid, st) : launch_one<true, GEMM_PLAIN>(p, grid, st);
   return epi == GEMM_SWIGLU ? launch_one<false, GEMM_SWIGLU>(p, grid, st) : launch_one<false, GEMM_PLAIN>(p, grid, st);
+}
+
+// ------------------------------------------------------------------ weight tiling
+// one thread per 16-byte chunk of the destination
+__global__ void tile_weights_kernel(const uint8_t *__restrict__ src, uint8_t *__restrict__ dst, int nexp, int rows,
+                                    int kbytes, int interleave_f, int es) {
+  const int nt = rows / 256, kbn = kbytes / 128;
+  const int64_t per_exp = (int64_t)rows * kbytes / 16;
+  const int64_t total = per_exp * nexp;
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < total; c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t e = c / per_exp;
+    int64_t rem = c % per_exp;
+    const int64_t tile = rem / (256 * 8);          // 2048 chunks of 16 B per tile
+    const int in = (int)(rem % (256 * 8));
+    const int r = in >> 3, j = in & 7;              // tile row, 16-byte chunk slot (swizzled)
+    const int nb = (int)(tile / kbn), kb = (int)(tile % kbn);
+    const int jsrc = j ^ (r & 7);                    // chunk j of row r holds source chunk j ^ (r % 8)
+    int srow;
+    if (interleave_f > 0) {
+      const int rr = nb * 256 + r;                   // interleaved row
+      const int b = rr >> 8, w = rr & 255;
+      srow = w < 128 ? b * 128 + w : interleave_f + b * 128 + (w - 128);
+    } else {
+      srow = nb * 256 + r;
+    }
+    const uint4 v = *reinterpret_cast<const uint4 *>(src + ((int64_t)e * rows + srow) * kbytes + (int64_t)kb * 128 +
+                                                     jsrc * 16);
+    *reinterpret_cast<uint4 *>(dst + c * 16) = v;
+  }
+  (void)nt; (void)es;
+}
+
+cudaError_t launch_tile_weights(const void *src, void *dst, int nexp, int rows, int kbytes, int interleave_f,
+                                cudaStream_t st) {
+  tile_weights_kernel<<<148 * 8, 256, 0, st>>>(reinterpret_cast<const uint8_t *>(src),
+                                              reinterpret_cast<uint8_t *>(dst), nexp, rows, kbytes, interleave_f, 1);
+  return cudaGetLastError();
 }
 
 // ------------------------------------------------------------------ tensor maps

@@ -69,7 +69,7 @@ def test_small_layer_parity(lib, name):
     assert err <= TOL[p.wtype], f"{name}: rel L2 {err:.3e} > {TOL[p.wtype]}"
 
 
-@pytest.mark.parametrize("name", ["toy", "v3_s", "v2lite_s"])
+@pytest.mark.parametrize("name", ["toy", "v3_s", "v2lite_s", "v2lite_h384"])
 @pytest.mark.parametrize("T", [1, 3, 17])
 def test_small_decode_shapes(lib, name, T):
     p = SMALL[name]
