@@ -67,6 +67,10 @@ __device__ __forceinline__ size_t sf_img_off(int64_t row, int kb, int tile_strid
 
 __device__ __forceinline__ float silu_f(float g) { return __fdividef(g, 1.f + __expf(-g)); }
 
+// PDL: wait for the stream predecessor's results / let the successor launch
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 __device__ __forceinline__ float warp_max(float v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
@@ -76,6 +80,80 @@ __device__ __forceinline__ float warp_sum(float v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
   return v;
+}
+
+// Destinations of one token's activation row in the expert-sorted order.
+struct ScatterDst {
+  int fp8;
+  void *xperm; uint8_t *xperm_img; int xperm_img_stride; float *xperm_s;   // sorted rows (+ scales)
+  void *xq; float *xs; uint8_t *xq_img; int xq_img_stride;                // token-order copy (shared expert)
+};
+
+// The whole CTA (NT threads) moves token t's row: thread = 8-element chunks
+// c = tid + NT i with every load issued up front (H <= 8192); FP8 quantises
+// each 1x128 block once (UE8M0 ceil scale of the amax over 16 consecutive
+// threads, e4m3 RNE satfinite; R10) and stores the codes to each of
+// the token's sorted rows pos[0..k) (< 0 = not local) and to xq; bf16 copies.
+template <int NT>
+__device__ __forceinline__ void scatter_token_row(const __nv_bfloat16 *__restrict__ xrow, int H, int64_t t, int k,
+                                                  const int *pos, const ScatterDst &d) {
+  constexpr int MAXI = 8192 / 8 / NT;
+  const int th = threadIdx.x, lane = th & 31;
+  const int nc = H / 8;
+  uint4 raw[MAXI];
+#pragma unroll
+  for (int i = 0; i < MAXI; ++i) {
+    const int c = th + NT * i;
+    if (c < nc) raw[i] = __ldg(reinterpret_cast<const uint4 *>(xrow) + c);
+  }
+#pragma unroll
+  for (int i = 0; i < MAXI; ++i) {
+    const int c = th + NT * i;
+    if (i * NT >= nc) break;                       // warp-uniform (nc % 32 == 0)
+    if (d.fp8) {
+      float f[8];
+      bf16x8_to_f32(raw[i], f);
+      float am = 0.f;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) am = fmaxf(am, fabsf(f[j]));
+#pragma unroll
+      for (int o = 8; o > 0; o >>= 1) am = fmaxf(am, __shfl_xor_sync(0xffffffffu, am, o));
+      if (c >= nc) continue;
+      const int ex = ue8m0_exponent(am);
+      const float inv = exp2i(-ex);
+      uint2 q;
+      q.x = (uint32_t)f32_to_e4m3(f[0] * inv) | ((uint32_t)f32_to_e4m3(f[1] * inv) << 8) |
+            ((uint32_t)f32_to_e4m3(f[2] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[3] * inv) << 24);
+      q.y = (uint32_t)f32_to_e4m3(f[4] * inv) | ((uint32_t)f32_to_e4m3(f[5] * inv) << 8) |
+            ((uint32_t)f32_to_e4m3(f[6] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[7] * inv) << 24);
+      const int b = c >> 4;                        // 128-element block
+      const bool head = (lane & 15) == 0;
+      if (d.xq) {
+        *reinterpret_cast<uint2 *>(reinterpret_cast<uint8_t *>(d.xq) + t * H + c * 8) = q;
+        if (head) {
+          if (d.xq_img) d.xq_img[sf_img_off(t, b, d.xq_img_stride)] = (uint8_t)(ex + 127);
+          if (d.xs) d.xs[t * (H / 128) + b] = exp2i(ex);
+        }
+      }
+#pragma unroll 1
+      for (int j = 0; j < k; ++j) {
+        const int rw = pos[j];
+        if (rw < 0) continue;
+        *reinterpret_cast<uint2 *>(reinterpret_cast<uint8_t *>(d.xperm) + (int64_t)rw * H + c * 8) = q;
+        if (head) {
+          if (d.xperm_img) d.xperm_img[sf_img_off(rw, b, d.xperm_img_stride)] = (uint8_t)(ex + 127);
+          if (d.xperm_s) d.xperm_s[(int64_t)rw * (H / 128) + b] = exp2i(ex);
+        }
+      }
+    } else if (c < nc) {
+#pragma unroll 1
+      for (int j = 0; j < k; ++j) {
+        const int rw = pos[j];
+        if (rw < 0) continue;
+        reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(d.xperm) + (int64_t)rw * H)[c] = raw[i];
+      }
+    }
+  }
 }
 
 }  // namespace moe

@@ -6,8 +6,30 @@
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <stdint.h>
+#include <utility>
+
+#include "common.cuh"
 
 namespace moe {
+
+// Launch with programmatic dependent launch (PDL): the kernel may start while
+// its stream predecessor is still running and must execute pdl_wait() before
+// touching the predecessor's outputs (CUDA-graph capturable).
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                       Args &&...args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
 
 enum { WT_BF16 = 0, WT_FP8 = 1, WT_F32 = 2 };
 enum { GEMM_LOGITS = 0, GEMM_SWIGLU = 1, GEMM_PLAIN = 2 };
@@ -70,18 +92,18 @@ struct RouteSmallArgs {
   int H, rows;
   int *done;                    // zero-initialised CTA counter (re-armed by the kernel)
   int debug;                    // timing experiments only (MOE_DEBUG_ROUTE): 1 skip logits, 2 skip tail
+  // activations into expert order (null xperm = skip): bf16 copy or e4m3 + scale images
+  int fp8;
+  void *xperm; uint8_t *xperm_img; int xperm_img_stride;
+  void *xq; float *xs; uint8_t *xq_img; int xq_img_stride;   // shared expert (FP8)
 };
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st);
 
-// x bf16 [T, H] -> e4m3 [T, H] + [T, H/128] fp32 power-of-two scales
-// (img != null: also the UE8M0 scale image of the T rows, tile stride img_stride)
-cudaError_t launch_act_quant(const void *x, int T, int H, void *xq, float *xs, uint8_t *img, int img_stride,
-                             cudaStream_t st);
-// rows of src (bf16 or e4m3 + scales) gathered into the padded expert order
-cudaError_t launch_gather_rows(const void *src, const float *src_s, int H, int elem_bytes,
-                               const int32_t *row_token, const int32_t *offs_pad, int E,
-                               int64_t R_bound, void *dst, float *dst_s, uint8_t *dst_img, int img_stride,
-                               cudaStream_t st);
+
+
+// prefill: each token's row (FP8-quantised or copied) into its k sorted rows and xq
+cudaError_t launch_scatter_rows(const void *x, int T, int H, int k, const int32_t *pos, const ScatterDst &d,
+                                cudaStream_t st);
 
 struct CombineArgs {
   int T, H, k, n_imm;
@@ -162,16 +184,7 @@ struct UmmaDecodeParams {
   int *sched;
 };
 cudaError_t launch_umma_decode(bool fp8, int mode, const UmmaDecodeParams &p, int grid, cudaStream_t st);
-// decode: FP8 quantisation / bf16 copy of the tokens into the first 16 rows of
-// each active expert segment, plus xq for the shared expert (one launch)
-struct QuantGatherArgs {
-  const void *x;                 // bf16 [T, H]
-  int T, H, fp8, max_slots;
-  const int32_t *act_list, *n_active, *counts, *offs_pad, *row_token;
-  void *xperm; uint8_t *xperm_img; int xperm_img_stride;
-  void *xq; float *xs; uint8_t *xq_img; int xq_img_stride;   // shared expert (FP8; xq null = none)
-};
-cudaError_t launch_quant_gather_decode(const QuantGatherArgs &a, cudaStream_t st);
+
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);
 
 }  // namespace moe

@@ -304,6 +304,9 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
     C_TRY(dalloc(L, &L->ysh, (size_t)Tm * H * 2, false));
   }
   C_TRY(cudaMemset(L->row_token, 0xff, (size_t)L->R_max * 4));
+  // padding rows of the sorted activations are read by the GEMM tiles but never
+  // written by the scatter: start them at zero (finite) once
+  C_TRY(cudaMemset(L->xperm, 0, (size_t)L->R_max * H * ab));
 
   // ---- tcgen05 path: scale images and tensor maps ----
   C_TRY(cudaDeviceGetAttribute(&L->num_sms, cudaDevAttrMultiProcessorCount, cfg->device));
@@ -366,7 +369,7 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
 }
 
 static const char *kStageNames[moe_layer::kStages] = {
-    "router_logits", "router_select", "permute", "act_quant", "gather", "gemm1_swiglu", "gemm2",
+    "router_logits", "router_select", "permute", "act_quant", "quant_scatter", "gemm1_swiglu", "gemm2",
     "shared_gemm1", "shared_gemm2", "combine"};
 enum { ST_LOGITS = 0, ST_SELECT, ST_PERMUTE, ST_QUANT, ST_GATHER, ST_GEMM1, ST_GEMM2, ST_SH1, ST_SH2, ST_COMBINE };
 
@@ -417,6 +420,8 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     rs.r = r; rs.p = pa; rs.x = x; rs.wg = L->gate_w; rs.H = H; rs.rows = L->gate_rows; rs.done = L->sched + 7;
     static const int dbg_route = getenv("MOE_DEBUG_ROUTE") ? atoi(getenv("MOE_DEBUG_ROUTE")) : 0;
     rs.debug = dbg_route;
+    rs.fp8 = L->fp8; rs.xperm = L->xperm; rs.xperm_img = L->xperm_img; rs.xperm_img_stride = L->max_tiles;
+    if (L->fp8 && Fs > 0) { rs.xq = L->xq; rs.xs = L->xs; rs.xq_img = L->xq_img; rs.xq_img_stride = L->img_tiles_sh; }
     CUDA_TRY(launch_route_small(rs, st));
     mark(L, ST_PERMUTE, st);
   } else {
@@ -448,15 +453,20 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   // 4. activation quantisation (FP8) and gather into expert order
   const void *xa = x;
   const float *xa_s = nullptr;
-  if (L->fp8 && !tc_decode) {
-    CUDA_TRY(launch_act_quant(x, T, H, L->xq, L->xs, L->umma ? L->xq_img : nullptr, L->img_tiles_sh, st));
+  if (L->fp8) {
     xa = L->xq;
     xa_s = L->xs;
-    mark(L, ST_QUANT, st);
   }
-  if (!decode) {
-    CUDA_TRY(launch_gather_rows(xa, xa_s, H, L->act_bytes, L->row_token, L->offs_pad, E, R_bound, L->xperm,
-                                L->xperm_s, L->umma ? L->xperm_img : nullptr, L->max_tiles, st));
+  if (!tc_decode) {
+    // each token's row -> its k sorted rows (+ xq): FP8 quantisation fused with the gather
+    ScatterDst d{};
+    d.fp8 = L->fp8; d.xperm = L->xperm;
+    if (L->fp8) {
+      d.xperm_img = L->umma ? L->xperm_img : nullptr; d.xperm_img_stride = L->max_tiles;
+      d.xperm_s = L->umma ? nullptr : L->xperm_s;
+      d.xq = L->xq; d.xs = L->xs; d.xq_img = L->umma ? L->xq_img : nullptr; d.xq_img_stride = L->img_tiles_sh;
+    }
+    CUDA_TRY(launch_scatter_rows(x, T, H, k, L->pos, d, st));
     mark(L, ST_GATHER, st);
   }
   if (decode && L->umma) {
@@ -464,13 +474,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     const bool f8 = L->fp8;
     const int kdiv = f8 ? 128 : 64;
     const int slots = (int)std::min<int64_t>(E, pairs) + (Fs > 0 ? 1 : 0);
-    QuantGatherArgs qg{};
-    qg.x = x; qg.T = T; qg.H = H; qg.fp8 = f8; qg.max_slots = (int)std::min<int64_t>(E, pairs);
-    qg.act_list = L->act_list; qg.n_active = L->n_active; qg.counts = L->counts; qg.offs_pad = L->offs_pad;
-    qg.row_token = L->row_token; qg.xperm = L->xperm; qg.xperm_img = L->xperm_img; qg.xperm_img_stride = L->max_tiles;
-    if (f8 && Fs > 0) { qg.xq = L->xq; qg.xs = L->xs; qg.xq_img = L->xq_img; qg.xq_img_stride = L->img_tiles_sh; }
-    CUDA_TRY(launch_quant_gather_decode(qg, st));
-    mark(L, ST_GATHER, st);
+    // (activations were quantised into expert order by the route kernel's tail)
     UmmaDecodeParams d1{};
     {
       UmmaGroup &g = d1.g[0];

@@ -277,6 +277,7 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
   const int row = blockIdx.x * 2 + half;
   __shared__ float red[2][4][16];
   __shared__ int is_last;
+  pdl_trigger();
   // ---- logits of router rows `row` for all T tokens ----
   {
     float acc[16];
@@ -392,6 +393,19 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
         if (p.dbg_perm) p.dbg_perm[p.offs[e] + i] = t;
       }
     }
+    __syncthreads();
+  }
+  if (!a.xperm) return;
+  // activations into expert order (replaces the quantise + gather launches)
+  __shared__ int spos[32];
+  ScatterDst d{};
+  d.fp8 = a.fp8; d.xperm = a.xperm; d.xperm_img = a.xperm_img; d.xperm_img_stride = a.xperm_img_stride;
+  d.xq = a.xq; d.xs = a.xs; d.xq_img = a.xq_img; d.xq_img_stride = a.xq_img_stride;
+#pragma unroll 1
+  for (int t = 0; t < T; ++t) {
+    if (threadIdx.x < p.k) spos[threadIdx.x] = p.pos[t * p.k + threadIdx.x];
+    __syncthreads();
+    scatter_token_row<RS_THREADS>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H, H, t, p.k, spos, d);
     __syncthreads();
   }
 }

@@ -83,6 +83,8 @@ __global__ void __launch_bounds__(UD_THREADS, 1) umma_decode_kernel(const __grid
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_base_smem;
+  pdl_trigger();                                // the next kernel may start its prologue
+  pdl_wait();                                   // routing / activations of the predecessor
 
   if (warp == 0) {
     // ============================ producer ============================
@@ -250,8 +252,7 @@ static cudaError_t ud_launch(const UmmaDecodeParams &p, int grid, cudaStream_t s
     if (e != cudaSuccess) return e;
     set = true;
   }
-  k<<<grid, UD_THREADS, UD_SMEM, st>>>(p);
-  return cudaGetLastError();
+  return launch_pdl(k, dim3(grid), dim3(UD_THREADS), UD_SMEM, st, p);
 }
 
 cudaError_t launch_umma_decode(bool fp8, int mode, const UmmaDecodeParams &p, int grid, cudaStream_t st) {
