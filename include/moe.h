@@ -118,7 +118,11 @@ moe_status moe_get_unique_id(void *out128);
 
 /* Validate the config, allocate all workspaces for max_tokens and copy/repack
  * the weights.  Synchronous (returns after the copies are done).  *out is set
- * to NULL on failure.  With ep_size > 1 this is collective over the EP group. */
+ * to NULL on failure.  With ep_size > 1 and a unique id this initialises the
+ * NCCL communicator and is collective over the EP group; with ep_size > 1 and
+ * nccl_unique_id == NULL the layer is one rank of an in-process group
+ * (moe_ep_group_forward).  Expert-parallel forwards synchronise the stream to
+ * learn the received row counts (not CUDA-Graph capturable).                 */
 moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights *w,
                             moe_layer **out);
 
@@ -146,6 +150,20 @@ moe_status moe_layer_forward_deferred(moe_layer *layer, const void *x, const voi
                                       int32_t T, int32_t n_deferred, const void *deferred_in,
                                       void *y, void *deferred_out, moe_routing_out *dbg,
                                       void *stream);
+
+/* Expert parallelism inside ONE process: P layers created
+ * with ep_size = P, ep_rank = r and nccl_unique_id = NULL form a group; this
+ * call runs one forward of every rank -- dispatch of each token row to the
+ * ranks owning its experts, expert FFNs there, return of one partial row per
+ * (token, rank) -- with device copies (peer copies when the layers live on
+ * different GPUs) as the transport.  Arrays are indexed by rank; x[r], y[r],
+ * residual[r], deferred_in[r], deferred_out[r] are rank r's device [T[r], H]
+ * bf16 buffers (residual/deferred arrays may be NULL).  Synchronises the
+ * stream twice (the received row counts size the copies).                    */
+moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void *const *x,
+                                const void *const *residual, const int32_t *T, int32_t n_deferred,
+                                const void *const *deferred_in, void *const *y, void *const *deferred_out,
+                                void *stream);
 
 /* Free every library allocation (and the NCCL communicator).  NULL is a no-op. */
 moe_status moe_layer_destroy(moe_layer *layer);

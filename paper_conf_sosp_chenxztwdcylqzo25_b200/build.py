@@ -12,6 +12,17 @@ CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libmoe_b200.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
+
+def _nccl_dir():
+    """NCCL 2.28 headers + libnccl.so.2 (the torch-bundled nvidia-nccl wheel)."""
+    import importlib.util
+    spec = importlib.util.find_spec("nvidia")
+    for base in (spec.submodule_search_locations if spec else []):
+        d = os.path.join(base, "nccl")
+        if os.path.exists(os.path.join(d, "include", "nccl.h")):
+            return d
+    raise RuntimeError("NCCL headers not found (nvidia.nccl)")
+
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-shared", "-Xcompiler", "-fPIC",
          "--expt-relaxed-constexpr", "-Xptxas", "-warn-spills"]
@@ -34,7 +45,10 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not stale():
         return LIB
     tmp = LIB + ".tmp"
-    cmd = [NVCC, *FLAGS, "-I", os.path.join(HERE, "..", "include"), *sources(), "-o", tmp, "-lcuda"]
+    nccl = _nccl_dir()
+    cmd = [NVCC, *FLAGS, "-I", os.path.join(HERE, "..", "include"), "-I", os.path.join(nccl, "include"),
+           *sources(), "-o", tmp, "-lcuda", "-L", os.path.join(nccl, "lib"), "-l:libnccl.so.2",
+           "-Xlinker", "-rpath=" + os.path.join(nccl, "lib")]
     if verbose:
         print(" ".join(cmd), file=sys.stderr)
     r = subprocess.run(cmd, capture_output=True, text=True)

@@ -223,6 +223,25 @@ struct moe_layer {
   CUtensorMap dmap_xperm, dmap_h, dmap_xq, dmap_hsh;           // decode: activation rows (box 16)
   bool gemv_ok = false;         // decode weight-streaming path usable for T <= gemv_max_tokens
   int num_sms = 148;
+  int max_rows = 0;             // routed rows capacity (ep_size * max_tokens)
+  // ---- expert parallelism (ep_size > 1) ----
+  struct Ep {
+    int P = 1, rank = 0;
+    void *comm = nullptr;       // ncclComm_t (NCCL transport) or null (in-process group)
+    __nv_bfloat16 *send_x = nullptr;   // [P][Tm][H]
+    int32_t *send_idx = nullptr;       // [P][Tm][k]
+    float *send_w = nullptr;           // [P][Tm][k]
+    int32_t *sendpos = nullptr;        // [Tm][P]
+    int32_t *cnt_dev = nullptr;        // [2P] send counts, recv counts
+    int32_t *cnt_host = nullptr;       // pinned [2P]
+    __nv_bfloat16 *recv_x = nullptr;   // [P*Tm][H]
+    __nv_bfloat16 *partial = nullptr;  // [P*Tm][H] expert-side weighted sums (immediate)
+    __nv_bfloat16 *partial_def = nullptr;
+    __nv_bfloat16 *back = nullptr;     // [P][Tm][H] partial sums returned to this rank
+    __nv_bfloat16 *back_def = nullptr;
+    int R = 0;                         // rows received this step
+    int roff[33] = {};                 // receive offsets per source
+  } ep;
   int64_t workspace_bytes = 0;
   int max_tiles = 0;
   // ---- stage timing (moe_layer_profile) ----

@@ -137,6 +137,30 @@ cudaError_t launch_gemv(const GemvArgs &a, int which, int max_slots, cudaStream_
 cudaError_t launch_router_gemv(const void *x, int T, int H, const void *wg, int rows, float *logits,
                                cudaStream_t st);
 
+// ---------------------------------------------------------------- expert parallelism
+struct EpCombineArgs {
+  int T, H, P, Tm;
+  const int32_t *sendpos;        // [T][P]
+  const __nv_bfloat16 *back, *back_def;   // [P][Tm][H]
+  const __nv_bfloat16 *ysh; const float *sgate;
+  const __nv_bfloat16 *residual, *deferred_in;
+  __nv_bfloat16 *y, *deferred_out;
+};
+cudaError_t launch_ep_plan(const int32_t *idx, int T, int k, int E_loc, int P, int32_t *sendpos, int32_t *cnt,
+                           cudaStream_t st);
+cudaError_t launch_ep_pack(const void *x, int T, int H, int k, const int32_t *idx, const float *w, int E_loc, int P,
+                           int Tm, const int32_t *sendpos, void *send_x, int32_t *send_idx, float *send_w,
+                           cudaStream_t st);
+cudaError_t launch_ep_final_combine(const EpCombineArgs &a, cudaStream_t st);
+int ep_nccl_get_unique_id(void *out128);
+int ep_nccl_init(void **comm, int P, int rank, const void *uid128);
+void ep_nccl_destroy(void *comm);
+const char *ep_nccl_error(void *comm);
+int ep_nccl_counts(void *comm, const int32_t *send_cnt, int32_t *recv_cnt, int P, cudaStream_t st);
+int ep_nccl_rows(void *comm, int P, const int32_t *send_cnt, const int64_t *send_off, const int32_t *recv_cnt,
+                 const int64_t *recv_off, int nbuf, const void *const *send, void *const *recv,
+                 const int64_t *row_bytes, cudaStream_t st);
+
 // ---------------------------------------------------------------- tcgen05 GEMM
 struct UmmaGroup {              // one operand set: 0 = routed experts, 1 = shared expert
   CUtensorMap a_map;            // A rows, K-major, box 128 B x 128 rows, SW128

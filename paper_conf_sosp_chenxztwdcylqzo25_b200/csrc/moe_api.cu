@@ -52,6 +52,37 @@ void free_all(moe_layer *L) {
                   L->xperm_img, L->h_img, L->xq_img, L->hsh_img};
   for (void *p : ptrs)
     if (p) cudaFree(p);
+  void *eps[] = {L->ep.send_x, L->ep.send_idx, L->ep.send_w, L->ep.sendpos, L->ep.cnt_dev, L->ep.recv_x,
+                 L->ep.partial, L->ep.partial_def, L->ep.back, L->ep.back_def};
+  for (void *p : eps)
+    if (p) cudaFree(p);
+  if (L->ep.cnt_host) cudaFreeHost(L->ep.cnt_host);
+  ep_nccl_destroy(L->ep.comm);
+  L->ep.comm = nullptr;
+}
+
+// Expert-parallel buffers (+ the NCCL communicator when a unique id is given;
+// without one the layer belongs to an in-process group, moe_ep_group_forward).
+moe_status ep_create(moe_layer *L, const moe_layer_config *cfg) {
+  const int P = cfg->ep_size, H = L->H, k = L->k;
+  const size_t Tm = std::max(1, cfg->max_tokens);
+  L->ep.P = P;
+  L->ep.rank = cfg->ep_rank;
+  const size_t rows = (size_t)P * Tm;
+  CUDA_TRY(dalloc(L, &L->ep.send_x, rows * H * 2, false));
+  CUDA_TRY(dalloc(L, &L->ep.send_idx, rows * k * 4, false));
+  CUDA_TRY(dalloc(L, &L->ep.send_w, rows * k * 4, false));
+  CUDA_TRY(dalloc(L, &L->ep.sendpos, Tm * P * 4, false));
+  CUDA_TRY(dalloc(L, &L->ep.cnt_dev, 2 * P * 4, false));
+  CUDA_TRY(dalloc(L, &L->ep.recv_x, rows * H * 2, false));
+  CUDA_TRY(dalloc(L, &L->ep.partial, rows * H * 2, false));
+  CUDA_TRY(dalloc(L, &L->ep.partial_def, rows * H * 2, false));
+  CUDA_TRY(dalloc(L, &L->ep.back, rows * H * 2, false));
+  CUDA_TRY(dalloc(L, &L->ep.back_def, rows * H * 2, false));
+  CUDA_TRY(cudaMallocHost(reinterpret_cast<void **>(&L->ep.cnt_host), 2 * P * 4));
+  if (cfg->nccl_unique_id && ep_nccl_init(&L->ep.comm, P, cfg->ep_rank, cfg->nccl_unique_id) != 0)
+    return fail(MOE_ERR_NCCL, "ncclCommInitRank(P=%d, rank=%d) failed", P, cfg->ep_rank);
+  return MOE_OK;
 }
 
 bool is_pow2(float v) {
@@ -154,7 +185,9 @@ moe_status validate(const moe_layer_config *c, const moe_layer_weights *w) {
   if (c->group_score != MOE_GROUP_MAX && c->group_score != MOE_GROUP_TOP2_SUM) return fail(MOE_ERR_INVALID_ARG, "group_score");
   if (c->wtype != MOE_W_BF16 && c->wtype != MOE_W_FP8_BLOCK128 && c->wtype != MOE_W_F32) return fail(MOE_ERR_INVALID_ARG, "wtype");
   if (c->max_tokens < 0) return fail(MOE_ERR_INVALID_ARG, "max_tokens");
-  if (c->ep_size != 1) return fail(MOE_ERR_UNSUPPORTED, "ep_size %d: expert parallel build not enabled in this library", c->ep_size);
+  if (c->ep_size < 1 || c->ep_size > 32 || c->n_experts % c->ep_size)
+    return fail(MOE_ERR_INVALID_ARG, "ep_size %d must be in [1, 32] and divide n_experts", c->ep_size);
+  if (c->ep_rank < 0 || c->ep_rank >= c->ep_size) return fail(MOE_ERR_INVALID_ARG, "ep_rank %d", c->ep_rank);
   if (!w->gate_w || !w->w13 || !w->w2) return fail(MOE_ERR_INVALID_ARG, "gate_w / w13 / w2 must be non-null");
   if (c->wtype == MOE_W_FP8_BLOCK128 && (!w->w13_scale || !w->w2_scale))
     return fail(MOE_ERR_INVALID_ARG, "FP8 weights need w13_scale and w2_scale");
@@ -186,7 +219,8 @@ const char *moe_last_error(void) { return g_err.c_str(); }
 
 moe_status moe_get_unique_id(void *out128) {
   if (!out128) return fail(MOE_ERR_INVALID_ARG, "null out");
-  return fail(MOE_ERR_UNSUPPORTED, "expert parallel build not enabled in this library");
+  if (ep_nccl_get_unique_id(out128) != 0) return fail(MOE_ERR_NCCL, "ncclGetUniqueId failed");
+  return MOE_OK;
 }
 
 moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights *w, moe_layer **out) {
@@ -268,12 +302,17 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
 
   // ---- workspace, sized for max_tokens ----
   const int64_t Tm = std::max(1, cfg->max_tokens);
-  const int64_t pairs = Tm * k;
+  // expert-parallel: the expert side processes the rows every rank sends here,
+  // at most ep_size * max_tokens (each rank sends a token to a rank at most once)
+  const int64_t Tr = Tm * cfg->ep_size;
+  L->max_rows = (int)Tr;
+  const int64_t pairs = Tr * k;
   L->R_max = pairs + (int64_t)E * kPadM;
   L->max_tiles = (int)(L->R_max / kPadM);
-  L->nchunk_max = (int)((Tm + kChunkTokens - 1) / kChunkTokens);
+  L->nchunk_max = (int)((Tr + kChunkTokens - 1) / kChunkTokens);
   const int ab = L->act_bytes;
   C_TRY(dalloc(L, &L->logits, (size_t)Tm * L->gate_rows * 4, false));
+  if (cfg->ep_size > 1 || cfg->nccl_unique_id) S_TRY(ep_create(L, cfg));
   C_TRY(dalloc(L, &L->topk_idx, (size_t)pairs * 4, false));
   C_TRY(dalloc(L, &L->topk_w, (size_t)pairs * 4, false));
   C_TRY(dalloc(L, &L->sgate, (size_t)Tm * 4, false));
@@ -379,168 +418,18 @@ static inline void mark(moe_layer *L, int stage, cudaStream_t st) {
   L->ev_hit[stage + 1] = true;
 }
 
-static moe_status forward_impl(moe_layer *L, const void *x, const void *residual, int32_t T, int32_t n_def,
-                               const void *deferred_in, void *y, void *deferred_out, moe_routing_out *dbg,
-                               void *stream) {
-  if (!L) return fail(MOE_ERR_INVALID_ARG, "null layer");
-  if (T < 0) return fail(MOE_ERR_INVALID_ARG, "T = %d < 0", T);
-  if (T > L->max_tokens) return fail(MOE_ERR_CAPACITY, "T = %d > max_tokens = %d", T, L->max_tokens);
-  if (n_def < 0 || n_def > L->k - 1) return fail(MOE_ERR_INVALID_ARG, "n_deferred = %d not in [0, k-1]", n_def);
-  if (T > 0 && (!x || !y)) return fail(MOE_ERR_INVALID_ARG, "x and y must be non-null");
-  if (x && x == y) return fail(MOE_ERR_INVALID_ARG, "y must not alias x");
-  if (T == 0) return MOE_OK;
-  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  if (L->prof) {
-    for (int i = 0; i <= moe_layer::kStages; ++i) L->ev_hit[i] = false;
-    cudaEventRecord(L->ev[0], st);
-    L->ev_hit[0] = true;
-  }
-  const int H = L->H, F = L->F, Fs = L->Fs, E = L->E, k = L->k;
+// Prefill-shaped expert GEMMs: routed experts over the sorted rows described by
+// L->tiles (built by the permutation) and the shared expert over T_shared token
+// rows (FP8: L->xq, quantised by the scatter; BF16: x_shared).
+static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_shared, int T_shared,
+                                   cudaStream_t st) {
+  const int H = L->H, F = L->F, Fs = T_shared > 0 ? L->Fs : 0;
+  const int T = T_shared;
+  const void *x = x_shared;
+  const void *xa = L->fp8 ? L->xq : x_shared;
+  const float *xa_s = L->fp8 ? L->xs : nullptr;
   const int btype = L->fp8 ? WT_FP8 : (L->f32w ? WT_F32 : WT_BF16);
-
-  const bool decode = L->gemv_ok && T <= L->gemv_max_tokens;
-  const bool tc_decode = decode && L->umma;        // T <= 16: fused small-T route + swap-AB kernels
-  CUDA_TRY(cudaMemsetAsync(L->sched, 0, 32, st));
-  RouterArgs r{};
-  r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
-  r.T = T; r.E = L->E_glob; r.k = k; r.n_group = L->cfg.n_group; r.topk_group = L->cfg.topk_group;
-  r.group_score = L->cfg.group_score; r.score_fn = L->cfg.score_fn; r.norm_topk = L->cfg.norm_topk;
-  r.routed_scale = L->cfg.routed_scale; r.shared_gated = L->cfg.shared_gated;
-  r.topk_idx = L->topk_idx; r.topk_w = L->topk_w; r.sgate = L->sgate;
-  PermuteArgs pa{};
-  pa.topk_idx = L->topk_idx; pa.T = T; pa.k = k; pa.E = E; pa.e0 = L->e0;
-  pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
-  pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
-  pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
-  pa.dbg_perm = dbg ? dbg->perm : nullptr;
-  pa.dbg_counts = dbg ? dbg->expert_counts : nullptr;
-  if (tc_decode) {
-    // 1-3 (decode). logits + select + count/scan/assign in one launch
-    RouteSmallArgs rs{};
-    rs.r = r; rs.p = pa; rs.x = x; rs.wg = L->gate_w; rs.H = H; rs.rows = L->gate_rows; rs.done = L->sched + 7;
-    static const int dbg_route = getenv("MOE_DEBUG_ROUTE") ? atoi(getenv("MOE_DEBUG_ROUTE")) : 0;
-    rs.debug = dbg_route;
-    rs.fp8 = L->fp8; rs.xperm = L->xperm; rs.xperm_img = L->xperm_img; rs.xperm_img_stride = L->max_tiles;
-    if (L->fp8 && Fs > 0) { rs.xq = L->xq; rs.xs = L->xs; rs.xq_img = L->xq_img; rs.xq_img_stride = L->img_tiles_sh; }
-    CUDA_TRY(launch_route_small(rs, st));
-    mark(L, ST_PERMUTE, st);
-  } else {
-    // 1. router logits (bf16 x . bf16 Wg, fp32 accumulate; reading R9)
-    if (T <= kGemvMaxTokens) {
-      CUDA_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
-    } else {
-      UmmaParams p{};
-      UmmaGroup &g = p.g[1];
-      if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) return fail(MOE_ERR_CUDA, "tensor map for x failed");
-      g.b_map = L->map_gate;
-      g.n_total = 0; g.kblocks = H / 64; g.out = L->logits; g.ldc = L->gate_rows; g.n_valid = L->gate_rows;
-      p.g[0] = g;
-      p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
-      const int units = ((T + 127) / 128) * p.nb_s;
-      CUDA_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
-    }
-    mark(L, ST_LOGITS, st);
-    // 2. scores + group-limited top-k + weights
-    CUDA_TRY(launch_router_select(r, st));
-    mark(L, ST_SELECT, st);
-    // 3. count / scan / permute
-    CUDA_TRY(launch_permute(pa, st));
-    mark(L, ST_PERMUTE, st);
-  }
-  const int64_t pairs = (int64_t)T * k;
-  const int64_t R_bound = std::min<int64_t>(L->R_max, pairs + (int64_t)std::min<int64_t>(E, pairs) * kPadM);
-  const int tile_bound = (int)(R_bound / kPadM);
-  // 4. activation quantisation (FP8) and gather into expert order
-  const void *xa = x;
-  const float *xa_s = nullptr;
-  if (L->fp8) {
-    xa = L->xq;
-    xa_s = L->xs;
-  }
-  if (!tc_decode) {
-    // each token's row -> its k sorted rows (+ xq): FP8 quantisation fused with the gather
-    ScatterDst d{};
-    d.fp8 = L->fp8; d.xperm = L->xperm;
-    if (L->fp8) {
-      d.xperm_img = L->umma ? L->xperm_img : nullptr; d.xperm_img_stride = L->max_tiles;
-      d.xperm_s = L->umma ? nullptr : L->xperm_s;
-      d.xq = L->xq; d.xs = L->xs; d.xq_img = L->umma ? L->xq_img : nullptr; d.xq_img_stride = L->img_tiles_sh;
-    }
-    CUDA_TRY(launch_scatter_rows(x, T, H, k, L->pos, d, st));
-    mark(L, ST_GATHER, st);
-  }
-  if (decode && L->umma) {
-    // 5+6 (decode). swap-AB tensor-core weight stream over the active experts + shared expert
-    const bool f8 = L->fp8;
-    const int kdiv = f8 ? 128 : 64;
-    const int slots = (int)std::min<int64_t>(E, pairs) + (Fs > 0 ? 1 : 0);
-    // (activations were quantised into expert order by the route kernel's tail)
-    UmmaDecodeParams d1{};
-    {
-      UmmaGroup &g = d1.g[0];
-      g.a_map = L->dmap_xperm; g.b_tiles = (const uint8_t *)L->w13; g.b_ntiles_n = 2 * F / 256;
-      g.sfa = L->xperm_img; g.sfa_tile_stride = L->max_tiles;
-      g.sfb = L->w13_img; g.sfb_expert_stride = L->w13_img_stride; g.sfb_rb = 2 * F / 128;
-      g.n_total = 2 * F; g.kblocks = H / kdiv;
-      g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
-    }
-    if (Fs > 0) {
-      UmmaGroup &g = d1.g[1];
-      if (f8) {
-        g.a_map = L->dmap_xq;
-      } else if (!make_kmajor_map(&g.a_map, x, false, T, H, 16)) {
-        return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
-      }
-      g.b_tiles = (const uint8_t *)L->ws13; g.b_ntiles_n = 2 * Fs / 256;
-      g.sfa = L->xq_img; g.sfa_tile_stride = L->img_tiles_sh;
-      g.sfb = L->ws13_img; g.sfb_rb = 2 * Fs / 128; g.n_total = 0; g.kblocks = H / kdiv;
-      g.out = L->hsh; g.ldc = Fs; g.out_sf = L->hsh_img; g.out_sf_tile_stride = L->img_tiles_sh;
-    } else {
-      d1.g[1] = d1.g[0];
-    }
-    d1.g_nblk[0] = F / 128; d1.g_nblk[1] = Fs / 128; d1.nblk = std::max(F, Fs) / 128;
-    d1.max_slots = slots; d1.has_shared = Fs > 0; d1.T = T;
-    d1.n_active = L->n_active; d1.act_list = L->act_list; d1.counts = L->counts; d1.offs_pad = L->offs_pad;
-    d1.sched = L->sched + 3;
-    CUDA_TRY(launch_umma_decode(f8, 1, d1, std::min(L->num_sms, slots * d1.nblk), st));
-    mark(L, ST_GEMM1, st);
-    UmmaDecodeParams d2 = d1;
-    {
-      UmmaGroup &g = d2.g[0];
-      g.a_map = L->dmap_h; g.b_tiles = (const uint8_t *)L->w2; g.b_ntiles_n = H / 256;
-      g.sfa = L->h_img; g.sfa_tile_stride = L->max_tiles;
-      g.sfb = L->w2_img; g.sfb_expert_stride = L->w2_img_stride; g.sfb_rb = H / 128;
-      g.n_total = H; g.kblocks = F / kdiv;
-      g.out = L->yperm; g.ldc = H; g.out_sf = nullptr;
-    }
-    if (Fs > 0) {
-      UmmaGroup &g = d2.g[1];
-      g.a_map = L->dmap_hsh; g.b_tiles = (const uint8_t *)L->ws2; g.b_ntiles_n = H / 256;
-      g.sfa = L->hsh_img; g.sfa_tile_stride = L->img_tiles_sh;
-      g.sfb = L->ws2_img; g.sfb_rb = H / 128; g.n_total = 0; g.kblocks = Fs / kdiv;
-      g.out = L->ysh; g.ldc = H; g.out_sf = nullptr;
-    } else {
-      d2.g[1] = d2.g[0];
-    }
-    d2.g_nblk[0] = H / 128; d2.g_nblk[1] = H / 128; d2.nblk = H / 128;
-    d2.sched = L->sched + 4;
-    CUDA_TRY(launch_umma_decode(f8, 2, d2, std::min(L->num_sms, slots * d2.nblk), st));
-    mark(L, ST_GEMM2, st);
-  } else if (decode) {
-    // 5+6 (decode, CUDA-core path). weight-streaming GEMVs over the active experts + shared expert
-    GemvArgs g{};
-    g.T = T; g.H = H; g.F = F; g.Fs = Fs; g.fp8 = L->fp8; g.has_shared = Fs > 0;
-    g.act_list = L->act_list; g.n_active = L->n_active; g.counts = L->counts; g.offs_pad = L->offs_pad;
-    g.row_token = L->row_token; g.x = x; g.xq = L->xq; g.xs = L->xs;
-    g.w13 = L->w13; g.w2 = L->w2; g.ws13 = L->ws13; g.ws2 = L->ws2;
-    g.w13_s = L->w13_s; g.w2_s = L->w2_s; g.ws13_s = L->ws13_s; g.ws2_s = L->ws2_s;
-    g.h = L->hbuf; g.hsh = L->hsh; g.h_s = L->h_s; g.hsh_s = L->hsh_s; g.yperm = L->yperm; g.ysh = L->ysh;
-    const int slots = (int)std::min<int64_t>(E, pairs) + (Fs > 0 ? 1 : 0);
-    CUDA_TRY(launch_gemv(g, 1, slots, st));
-    mark(L, ST_GEMM1, st);
-    CUDA_TRY(launch_gemv(g, 2, slots, st));
-    mark(L, ST_GEMM2, st);
-  } else if (L->umma) {
+  if (L->umma) {
     // 5+6. routed experts and the shared expert in one persistent tcgen05 launch per GEMM
     const bool f8 = L->fp8;
     const int kdiv = f8 ? 128 : 64;
@@ -628,6 +517,326 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
       mark(L, ST_SH2, st);
     }
   }
+  return MOE_OK;
+}
+
+
+// ======================================================================
+// Expert parallelism: rank r owns experts [e0, e0 + E_loc).
+//   A  route own tokens, plan + pack one row per (token, destination rank)
+//   -- exchange counts, rows + (masked expert ids, weights) --
+//   C  expert side: permute the received rows by local expert, FP8-quantise,
+//      grouped GEMMs (+ the shared expert on the own tokens), weighted partial
+//      sums per received row (immediate / deferred)
+//   -- return the partial rows to their origin --
+//   D  origin: y = residual + shared + sum of partials (+ deferred_in)
+// ======================================================================
+static moe_status run_router_full(moe_layer *L, const void *x, int T, cudaStream_t st) {
+  if (T <= 0) return MOE_OK;
+  const int H = L->H;
+  if (T <= kGemvMaxTokens) {
+    CUDA_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
+  } else {
+    UmmaParams p{};
+    UmmaGroup &g = p.g[1];
+    if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) return fail(MOE_ERR_CUDA, "tensor map for x failed");
+    g.b_map = L->map_gate;
+    g.n_total = 0; g.kblocks = H / 64; g.out = L->logits; g.ldc = L->gate_rows; g.n_valid = L->gate_rows;
+    p.g[0] = g;
+    p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
+    const int units = ((T + 127) / 128) * p.nb_s;
+    CUDA_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
+  }
+  RouterArgs r{};
+  r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
+  r.T = T; r.E = L->E_glob; r.k = L->k; r.n_group = L->cfg.n_group; r.topk_group = L->cfg.topk_group;
+  r.group_score = L->cfg.group_score; r.score_fn = L->cfg.score_fn; r.norm_topk = L->cfg.norm_topk;
+  r.routed_scale = L->cfg.routed_scale; r.shared_gated = L->cfg.shared_gated;
+  r.topk_idx = L->topk_idx; r.topk_w = L->topk_w; r.sgate = L->sgate;
+  CUDA_TRY(launch_router_select(r, st));
+  return MOE_OK;
+}
+
+static moe_status ep_phase_a(moe_layer *L, const void *x, int T, cudaStream_t st) {
+  CUDA_TRY(cudaMemsetAsync(L->sched, 0, 32, st));
+  moe_status s = run_router_full(L, x, T, st);
+  if (s != MOE_OK) return s;
+  const int P = L->ep.P, Tm = std::max(1, L->max_tokens);
+  CUDA_TRY(launch_ep_plan(L->topk_idx, T, L->k, L->E, P, L->ep.sendpos, L->ep.cnt_dev, st));
+  CUDA_TRY(launch_ep_pack(x, T, L->H, L->k, L->topk_idx, L->topk_w, L->E, P, Tm, L->ep.sendpos, L->ep.send_x,
+                          L->ep.send_idx, L->ep.send_w, st));
+  return MOE_OK;
+}
+
+// send counts (cnt_dev[0:P]) and received counts (cnt_dev[P:2P]) -> host
+static moe_status ep_counts_to_host(moe_layer *L, cudaStream_t st) {
+  const int P = L->ep.P;
+  CUDA_TRY(cudaMemcpyAsync(L->ep.cnt_host, L->ep.cnt_dev, 2 * P * 4, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(cudaStreamSynchronize(st));
+  int off = 0;
+  for (int p = 0; p < P; ++p) {
+    L->ep.roff[p] = off;
+    off += L->ep.cnt_host[P + p];
+  }
+  L->ep.roff[P] = off;
+  L->ep.R = off;
+  if (off > L->max_rows) return fail(MOE_ERR_CAPACITY, "received %d rows > %d", off, L->max_rows);
+  return MOE_OK;
+}
+
+static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_def, bool want_def,
+                             cudaStream_t st) {
+  const int R = L->ep.R, k = L->k, H = L->H, Fs = L->Fs, E = L->E;
+  // routing of the received rows (global ids, -1 = not ours) is in topk_idx/topk_w
+  PermuteArgs pa{};
+  pa.topk_idx = L->topk_idx; pa.T = R; pa.k = k; pa.E = E; pa.e0 = L->e0;
+  pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
+  pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
+  pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
+  if (R > 0) {
+    CUDA_TRY(launch_permute(pa, st));
+  } else {
+    CUDA_TRY(cudaMemsetAsync(L->n_tiles, 0, 4, st));
+  }
+  ScatterDst d{};
+  d.fp8 = L->fp8; d.xperm = L->xperm;
+  if (L->fp8) {
+    d.xperm_img = L->umma ? L->xperm_img : nullptr; d.xperm_img_stride = L->max_tiles;
+    d.xperm_s = L->umma ? nullptr : L->xperm_s;
+  }
+  CUDA_TRY(launch_scatter_rows(L->ep.recv_x, R, H, k, L->pos, d, st));
+  if (Fs > 0 && L->fp8 && T_own > 0) {
+    // the shared expert runs on this rank's own tokens: quantise them into xq
+    ScatterDst s{};
+    s.fp8 = 1; s.xq = L->xq; s.xs = L->xs; s.xq_img = L->umma ? L->xq_img : nullptr;
+    s.xq_img_stride = L->img_tiles_sh;
+    CUDA_TRY(launch_scatter_rows(x_own, T_own, H, 0, L->pos, s, st));
+  }
+  const int64_t pairs = (int64_t)R * k;
+  const int64_t R_bound = std::min<int64_t>(L->R_max, pairs + (int64_t)std::min<int64_t>(E, pairs) * kPadM);
+  moe_status gs = run_expert_gemms(L, (int)(R_bound / kPadM), x_own, Fs > 0 ? T_own : 0, st);
+  if (gs != MOE_OK) return gs;
+  if (R > 0) {
+    CombineArgs c{};
+    c.T = R; c.H = H; c.k = k; c.n_imm = want_def ? k - n_def : k;
+    c.pos = L->pos; c.topk_w = L->topk_w; c.yperm = L->yperm;
+    c.y = L->ep.partial; c.deferred_out = want_def ? L->ep.partial_def : nullptr;
+    CUDA_TRY(launch_combine(c, st));
+  }
+  return MOE_OK;
+}
+
+static moe_status ep_phase_d(moe_layer *L, const void *residual, int T, const void *din, void *y, void *dout,
+                             cudaStream_t st) {
+  EpCombineArgs c{};
+  c.T = T; c.H = L->H; c.P = L->ep.P; c.Tm = std::max(1, L->max_tokens);
+  c.sendpos = L->ep.sendpos; c.back = L->ep.back; c.back_def = dout ? L->ep.back_def : nullptr;
+  c.ysh = L->Fs > 0 ? L->ysh : nullptr; c.sgate = L->cfg.shared_gated ? L->sgate : nullptr;
+  c.residual = reinterpret_cast<const __nv_bfloat16 *>(residual);
+  c.deferred_in = reinterpret_cast<const __nv_bfloat16 *>(din);
+  c.y = reinterpret_cast<__nv_bfloat16 *>(y); c.deferred_out = reinterpret_cast<__nv_bfloat16 *>(dout);
+  CUDA_TRY(launch_ep_final_combine(c, st));
+  return MOE_OK;
+}
+
+#define NCCL_TRY(expr)                                                                                 \
+  do {                                                                                                 \
+    if ((expr) != 0) return fail(MOE_ERR_NCCL, "%s failed %s", #expr, ep_nccl_error(L->ep.comm));    \
+  } while (0)
+
+// one rank of an NCCL expert-parallel group (collective over the group)
+static moe_status ep_forward_nccl(moe_layer *L, const void *x, const void *residual, int T, int n_def,
+                                  const void *din, void *y, void *dout, cudaStream_t st) {
+  const int P = L->ep.P, k = L->k, H = L->H;
+  const int64_t Tm = std::max(1, L->max_tokens);
+  moe_status s = ep_phase_a(L, x, T, st);
+  if (s != MOE_OK) return s;
+  NCCL_TRY(ep_nccl_counts(L->ep.comm, L->ep.cnt_dev, L->ep.cnt_dev + P, P, st));
+  if ((s = ep_counts_to_host(L, st)) != MOE_OK) return s;
+  int64_t soff[32], roff[32];
+  for (int p = 0; p < P; ++p) { soff[p] = p * Tm; roff[p] = L->ep.roff[p]; }
+  const int32_t *scnt = L->ep.cnt_host, *rcnt = L->ep.cnt_host + P;
+  {
+    const void *snd[3] = {L->ep.send_x, L->ep.send_idx, L->ep.send_w};
+    void *rcv[3] = {L->ep.recv_x, L->topk_idx, L->topk_w};
+    const int64_t rb[3] = {(int64_t)H * 2, (int64_t)k * 4, (int64_t)k * 4};
+    NCCL_TRY(ep_nccl_rows(L->ep.comm, P, scnt, soff, rcnt, roff, 3, snd, rcv, rb, st));
+  }
+  const bool want_def = dout != nullptr && n_def > 0;
+  if ((s = ep_phase_c(L, x, T, n_def, want_def, st)) != MOE_OK) return s;
+  {
+    const void *snd[2] = {L->ep.partial, L->ep.partial_def};
+    void *rcv[2] = {L->ep.back, L->ep.back_def};
+    const int64_t rb[2] = {(int64_t)H * 2, (int64_t)H * 2};
+    NCCL_TRY(ep_nccl_rows(L->ep.comm, P, rcnt, roff, scnt, soff, want_def ? 2 : 1, snd, rcv, rb, st));
+  }
+  return ep_phase_d(L, residual, T, din, y, want_def ? dout : nullptr, st);
+}
+
+static moe_status forward_impl(moe_layer *L, const void *x, const void *residual, int32_t T, int32_t n_def,
+                               const void *deferred_in, void *y, void *deferred_out, moe_routing_out *dbg,
+                               void *stream) {
+  if (!L) return fail(MOE_ERR_INVALID_ARG, "null layer");
+  if (T < 0) return fail(MOE_ERR_INVALID_ARG, "T = %d < 0", T);
+  if (T > L->max_tokens) return fail(MOE_ERR_CAPACITY, "T = %d > max_tokens = %d", T, L->max_tokens);
+  if (n_def < 0 || n_def > L->k - 1) return fail(MOE_ERR_INVALID_ARG, "n_deferred = %d not in [0, k-1]", n_def);
+  if (T > 0 && (!x || !y)) return fail(MOE_ERR_INVALID_ARG, "x and y must be non-null");
+  if (x && x == y) return fail(MOE_ERR_INVALID_ARG, "y must not alias x");
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  if (L->ep.P > 1 || L->ep.comm) {
+    if (!L->ep.comm)
+      return fail(MOE_ERR_INVALID_ARG, "layer belongs to an in-process EP group: use moe_ep_group_forward");
+    if (dbg) return fail(MOE_ERR_UNSUPPORTED, "routing debug outputs are single-GPU only");
+    return ep_forward_nccl(L, x, residual, T, n_def, deferred_in, y, deferred_out, st);  // T == 0 participates
+  }
+  if (T == 0) return MOE_OK;
+  if (L->prof) {
+    for (int i = 0; i <= moe_layer::kStages; ++i) L->ev_hit[i] = false;
+    cudaEventRecord(L->ev[0], st);
+    L->ev_hit[0] = true;
+  }
+  const int H = L->H, F = L->F, Fs = L->Fs, E = L->E, k = L->k;
+  const bool decode = L->gemv_ok && T <= L->gemv_max_tokens;
+  const bool tc_decode = decode && L->umma;        // T <= 16: fused small-T route + swap-AB kernels
+  CUDA_TRY(cudaMemsetAsync(L->sched, 0, 32, st));
+  RouterArgs r{};
+  r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
+  r.T = T; r.E = L->E_glob; r.k = k; r.n_group = L->cfg.n_group; r.topk_group = L->cfg.topk_group;
+  r.group_score = L->cfg.group_score; r.score_fn = L->cfg.score_fn; r.norm_topk = L->cfg.norm_topk;
+  r.routed_scale = L->cfg.routed_scale; r.shared_gated = L->cfg.shared_gated;
+  r.topk_idx = L->topk_idx; r.topk_w = L->topk_w; r.sgate = L->sgate;
+  PermuteArgs pa{};
+  pa.topk_idx = L->topk_idx; pa.T = T; pa.k = k; pa.E = E; pa.e0 = L->e0;
+  pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
+  pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
+  pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
+  pa.dbg_perm = dbg ? dbg->perm : nullptr;
+  pa.dbg_counts = dbg ? dbg->expert_counts : nullptr;
+  if (tc_decode) {
+    // 1-3 (decode). logits + select + count/scan/assign in one launch
+    RouteSmallArgs rs{};
+    rs.r = r; rs.p = pa; rs.x = x; rs.wg = L->gate_w; rs.H = H; rs.rows = L->gate_rows; rs.done = L->sched + 7;
+    static const int dbg_route = getenv("MOE_DEBUG_ROUTE") ? atoi(getenv("MOE_DEBUG_ROUTE")) : 0;
+    rs.debug = dbg_route;
+    rs.fp8 = L->fp8; rs.xperm = L->xperm; rs.xperm_img = L->xperm_img; rs.xperm_img_stride = L->max_tiles;
+    if (L->fp8 && Fs > 0) { rs.xq = L->xq; rs.xs = L->xs; rs.xq_img = L->xq_img; rs.xq_img_stride = L->img_tiles_sh; }
+    CUDA_TRY(launch_route_small(rs, st));
+    mark(L, ST_PERMUTE, st);
+  } else {
+    // 1. router logits (bf16 x . bf16 Wg, fp32 accumulate; reading R9)
+    if (T <= kGemvMaxTokens) {
+      CUDA_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
+    } else {
+      UmmaParams p{};
+      UmmaGroup &g = p.g[1];
+      if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) return fail(MOE_ERR_CUDA, "tensor map for x failed");
+      g.b_map = L->map_gate;
+      g.n_total = 0; g.kblocks = H / 64; g.out = L->logits; g.ldc = L->gate_rows; g.n_valid = L->gate_rows;
+      p.g[0] = g;
+      p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
+      const int units = ((T + 127) / 128) * p.nb_s;
+      CUDA_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
+    }
+    mark(L, ST_LOGITS, st);
+    // 2. scores + group-limited top-k + weights
+    CUDA_TRY(launch_router_select(r, st));
+    mark(L, ST_SELECT, st);
+    // 3. count / scan / permute
+    CUDA_TRY(launch_permute(pa, st));
+    mark(L, ST_PERMUTE, st);
+  }
+  const int64_t pairs = (int64_t)T * k;
+  const int64_t R_bound = std::min<int64_t>(L->R_max, pairs + (int64_t)std::min<int64_t>(E, pairs) * kPadM);
+  const int tile_bound = (int)(R_bound / kPadM);
+  // 4. activation quantisation (FP8) and gather into expert order
+  if (!tc_decode) {
+    // each token's row -> its k sorted rows (+ xq): FP8 quantisation fused with the gather
+    ScatterDst d{};
+    d.fp8 = L->fp8; d.xperm = L->xperm;
+    if (L->fp8) {
+      d.xperm_img = L->umma ? L->xperm_img : nullptr; d.xperm_img_stride = L->max_tiles;
+      d.xperm_s = L->umma ? nullptr : L->xperm_s;
+      d.xq = L->xq; d.xs = L->xs; d.xq_img = L->umma ? L->xq_img : nullptr; d.xq_img_stride = L->img_tiles_sh;
+    }
+    CUDA_TRY(launch_scatter_rows(x, T, H, k, L->pos, d, st));
+    mark(L, ST_GATHER, st);
+  }
+  if (decode && L->umma) {
+    // 5+6 (decode). swap-AB tensor-core weight stream over the active experts + shared expert
+    const bool f8 = L->fp8;
+    const int kdiv = f8 ? 128 : 64;
+    const int slots = (int)std::min<int64_t>(E, pairs) + (Fs > 0 ? 1 : 0);
+    // (activations were quantised into expert order by the route kernel's tail)
+    UmmaDecodeParams d1{};
+    {
+      UmmaGroup &g = d1.g[0];
+      g.a_map = L->dmap_xperm; g.b_tiles = (const uint8_t *)L->w13; g.b_ntiles_n = 2 * F / 256;
+      g.sfa = L->xperm_img; g.sfa_tile_stride = L->max_tiles;
+      g.sfb = L->w13_img; g.sfb_expert_stride = L->w13_img_stride; g.sfb_rb = 2 * F / 128;
+      g.n_total = 2 * F; g.kblocks = H / kdiv;
+      g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
+    }
+    if (Fs > 0) {
+      UmmaGroup &g = d1.g[1];
+      if (f8) {
+        g.a_map = L->dmap_xq;
+      } else if (!make_kmajor_map(&g.a_map, x, false, T, H, 16)) {
+        return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
+      }
+      g.b_tiles = (const uint8_t *)L->ws13; g.b_ntiles_n = 2 * Fs / 256;
+      g.sfa = L->xq_img; g.sfa_tile_stride = L->img_tiles_sh;
+      g.sfb = L->ws13_img; g.sfb_rb = 2 * Fs / 128; g.n_total = 0; g.kblocks = H / kdiv;
+      g.out = L->hsh; g.ldc = Fs; g.out_sf = L->hsh_img; g.out_sf_tile_stride = L->img_tiles_sh;
+    } else {
+      d1.g[1] = d1.g[0];
+    }
+    d1.g_nblk[0] = F / 128; d1.g_nblk[1] = Fs / 128; d1.nblk = std::max(F, Fs) / 128;
+    d1.max_slots = slots; d1.has_shared = Fs > 0; d1.T = T;
+    d1.n_active = L->n_active; d1.act_list = L->act_list; d1.counts = L->counts; d1.offs_pad = L->offs_pad;
+    d1.sched = L->sched + 3;
+    CUDA_TRY(launch_umma_decode(f8, 1, d1, std::min(L->num_sms, slots * d1.nblk), st));
+    mark(L, ST_GEMM1, st);
+    UmmaDecodeParams d2 = d1;
+    {
+      UmmaGroup &g = d2.g[0];
+      g.a_map = L->dmap_h; g.b_tiles = (const uint8_t *)L->w2; g.b_ntiles_n = H / 256;
+      g.sfa = L->h_img; g.sfa_tile_stride = L->max_tiles;
+      g.sfb = L->w2_img; g.sfb_expert_stride = L->w2_img_stride; g.sfb_rb = H / 128;
+      g.n_total = H; g.kblocks = F / kdiv;
+      g.out = L->yperm; g.ldc = H; g.out_sf = nullptr;
+    }
+    if (Fs > 0) {
+      UmmaGroup &g = d2.g[1];
+      g.a_map = L->dmap_hsh; g.b_tiles = (const uint8_t *)L->ws2; g.b_ntiles_n = H / 256;
+      g.sfa = L->hsh_img; g.sfa_tile_stride = L->img_tiles_sh;
+      g.sfb = L->ws2_img; g.sfb_rb = H / 128; g.n_total = 0; g.kblocks = Fs / kdiv;
+      g.out = L->ysh; g.ldc = H; g.out_sf = nullptr;
+    } else {
+      d2.g[1] = d2.g[0];
+    }
+    d2.g_nblk[0] = H / 128; d2.g_nblk[1] = H / 128; d2.nblk = H / 128;
+    d2.sched = L->sched + 4;
+    CUDA_TRY(launch_umma_decode(f8, 2, d2, std::min(L->num_sms, slots * d2.nblk), st));
+    mark(L, ST_GEMM2, st);
+  } else if (decode) {
+    // 5+6 (decode, CUDA-core path). weight-streaming GEMVs over the active experts + shared expert
+    GemvArgs g{};
+    g.T = T; g.H = H; g.F = F; g.Fs = Fs; g.fp8 = L->fp8; g.has_shared = Fs > 0;
+    g.act_list = L->act_list; g.n_active = L->n_active; g.counts = L->counts; g.offs_pad = L->offs_pad;
+    g.row_token = L->row_token; g.x = x; g.xq = L->xq; g.xs = L->xs;
+    g.w13 = L->w13; g.w2 = L->w2; g.ws13 = L->ws13; g.ws2 = L->ws2;
+    g.w13_s = L->w13_s; g.w2_s = L->w2_s; g.ws13_s = L->ws13_s; g.ws2_s = L->ws2_s;
+    g.h = L->hbuf; g.hsh = L->hsh; g.h_s = L->h_s; g.hsh_s = L->hsh_s; g.yperm = L->yperm; g.ysh = L->ysh;
+    const int slots = (int)std::min<int64_t>(E, pairs) + (Fs > 0 ? 1 : 0);
+    CUDA_TRY(launch_gemv(g, 1, slots, st));
+    mark(L, ST_GEMM1, st);
+    CUDA_TRY(launch_gemv(g, 2, slots, st));
+    mark(L, ST_GEMM2, st);
+  } else {
+    // 5+6. routed experts (sorted rows) + shared expert (all T tokens)
+    moe_status gs = run_expert_gemms(L, tile_bound, x, Fs > 0 ? T : 0, st);
+    if (gs != MOE_OK) return gs;
+  }
   // 7. weighted combine + residual (+ deferral split)
   {
     CombineArgs c{};
@@ -655,6 +864,71 @@ moe_status moe_layer_forward_deferred(moe_layer *L, const void *x, const void *r
                                       int32_t n_deferred, const void *deferred_in, void *y, void *deferred_out,
                                       moe_routing_out *dbg, void *stream) {
   return forward_impl(L, x, residual, T, n_deferred, deferred_in, y, deferred_out, dbg, stream);
+}
+
+moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void *const *x,
+                                const void *const *residual, const int32_t *T, int32_t n_deferred,
+                                const void *const *deferred_in, void *const *y, void *const *deferred_out,
+                                void *stream) {
+  if (!layers || !x || !y || !T || P < 2 || P > 32) return fail(MOE_ERR_INVALID_ARG, "bad group arguments");
+  for (int r = 0; r < P; ++r) {
+    moe_layer *L = layers[r];
+    if (!L || L->ep.P != P || L->ep.rank != r || L->ep.comm)
+      return fail(MOE_ERR_INVALID_ARG, "layer %d is not rank %d of an in-process group of %d", r, r, P);
+    if (T[r] < 0 || T[r] > L->max_tokens) return fail(MOE_ERR_CAPACITY, "T[%d] = %d", r, T[r]);
+    if (n_deferred < 0 || n_deferred > L->k - 1) return fail(MOE_ERR_INVALID_ARG, "n_deferred");
+    if (T[r] > 0 && (!x[r] || !y[r])) return fail(MOE_ERR_INVALID_ARG, "x/y of rank %d", r);
+  }
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  const int64_t Tm = std::max(1, layers[0]->max_tokens);
+  const int H = layers[0]->H, k = layers[0]->k;
+  moe_status s;
+  for (int r = 0; r < P; ++r) {
+    CUDA_TRY(cudaSetDevice(layers[r]->cfg.device));
+    if ((s = ep_phase_a(layers[r], x[r], T[r], st)) != MOE_OK) return s;
+  }
+  // counts: rank d receives cnt_dev[d] of every source
+  for (int d = 0; d < P; ++d)
+    for (int src = 0; src < P; ++src)
+      CUDA_TRY(cudaMemcpyAsync(layers[d]->ep.cnt_dev + P + src, layers[src]->ep.cnt_dev + d, 4, cudaMemcpyDefault, st));
+  for (int r = 0; r < P; ++r)
+    if ((s = ep_counts_to_host(layers[r], st)) != MOE_OK) return s;
+  for (int d = 0; d < P; ++d)
+    for (int src = 0; src < P; ++src) {
+      const int64_t n = layers[src]->ep.cnt_host[d];
+      if (!n) continue;
+      const int64_t ro = layers[d]->ep.roff[src], so = (int64_t)d * Tm;
+      CUDA_TRY(cudaMemcpyAsync(layers[d]->ep.recv_x + ro * H, layers[src]->ep.send_x + so * H, n * H * 2,
+                               cudaMemcpyDefault, st));
+      CUDA_TRY(cudaMemcpyAsync(layers[d]->topk_idx + ro * k, layers[src]->ep.send_idx + so * k, n * k * 4,
+                               cudaMemcpyDefault, st));
+      CUDA_TRY(cudaMemcpyAsync(layers[d]->topk_w + ro * k, layers[src]->ep.send_w + so * k, n * k * 4,
+                               cudaMemcpyDefault, st));
+    }
+  for (int r = 0; r < P; ++r) {
+    CUDA_TRY(cudaSetDevice(layers[r]->cfg.device));
+    const bool want_def = deferred_out && deferred_out[r] && n_deferred > 0;
+    if ((s = ep_phase_c(layers[r], x[r], T[r], n_deferred, want_def, st)) != MOE_OK) return s;
+  }
+  for (int src = 0; src < P; ++src)       // partial rows back to their origin
+    for (int d = 0; d < P; ++d) {
+      const int64_t n = layers[src]->ep.cnt_host[d];
+      if (!n) continue;
+      const int64_t ro = layers[d]->ep.roff[src], so = (int64_t)d * Tm;
+      CUDA_TRY(cudaMemcpyAsync(layers[src]->ep.back + so * H, layers[d]->ep.partial + ro * H, n * H * 2,
+                               cudaMemcpyDefault, st));
+      if (deferred_out && deferred_out[src] && n_deferred > 0)
+        CUDA_TRY(cudaMemcpyAsync(layers[src]->ep.back_def + so * H, layers[d]->ep.partial_def + ro * H, n * H * 2,
+                                 cudaMemcpyDefault, st));
+    }
+  for (int r = 0; r < P; ++r) {
+    CUDA_TRY(cudaSetDevice(layers[r]->cfg.device));
+    const bool want_def = deferred_out && deferred_out[r] && n_deferred > 0;
+    if ((s = ep_phase_d(layers[r], residual ? residual[r] : nullptr, T[r],
+                        deferred_in ? deferred_in[r] : nullptr, y[r], want_def ? deferred_out[r] : nullptr, st)) != MOE_OK)
+      return s;
+  }
+  return MOE_OK;
 }
 
 moe_status moe_layer_profile(moe_layer *L, int32_t enable) {

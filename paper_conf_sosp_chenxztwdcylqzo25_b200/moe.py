@@ -22,7 +22,7 @@ SCORE_SOFTMAX, SCORE_SIGMOID = 0, 1
 GROUP_MAX, GROUP_TOP2_SUM = 0, 1
 W_BF16, W_FP8, W_F32 = 0, 1, 2
 
-EXPORTED = ["moe_get_unique_id", "moe_layer_create", "moe_layer_forward", "moe_layer_forward_deferred",
+EXPORTED = ["moe_ep_group_forward", "moe_get_unique_id", "moe_layer_create", "moe_layer_forward", "moe_layer_forward_deferred",
             "moe_layer_destroy", "moe_status_string", "moe_last_error", "moe_layer_get_info",
             "moe_layer_profile", "moe_layer_stage_times", "moe_stage_name"]
 
@@ -75,6 +75,10 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.moe_status_string.restype = ctypes.c_char_p
     lib.moe_last_error.restype = ctypes.c_char_p
     lib.moe_layer_get_info.argtypes = [vp, ctypes.POINTER(MoEInfo)]
+    lib.moe_ep_group_forward.argtypes = [ctypes.POINTER(vp), i32, ctypes.POINTER(vp), ctypes.POINTER(vp),
+                                         ctypes.POINTER(i32), i32, ctypes.POINTER(vp), ctypes.POINTER(vp),
+                                         ctypes.POINTER(vp), vp]
+    lib.moe_ep_group_forward.restype = i32
     lib.moe_layer_profile.argtypes = [vp, i32]
     lib.moe_layer_stage_times.argtypes = [vp, ctypes.POINTER(ctypes.c_float), i32, ctypes.POINTER(i32)]
     lib.moe_stage_name.argtypes = [i32]
@@ -195,3 +199,53 @@ class MoELayer:
             self.close()
         except Exception:
             pass
+
+
+def slice_experts(weights, rank: int, ep_size: int):
+    """Rank `rank`'s contiguous slice of the routed experts (router and shared
+    expert are replicated) -- the weights a rank passes to moe_layer_create."""
+    import copy
+    E = weights.w13.shape[0]
+    n = E // ep_size
+    w = copy.copy(weights)
+    sl = slice(rank * n, (rank + 1) * n)
+    w.w13 = weights.w13[sl].contiguous()
+    w.w2 = weights.w2[sl].contiguous()
+    if weights.w13_scale is not None:
+        w.w13_scale = weights.w13_scale[sl].contiguous()
+        w.w2_scale = weights.w2_scale[sl].contiguous()
+    return w
+
+
+class MoEGroup:
+    """In-process expert-parallel group (moe_ep_group_forward): P ranks, one
+    MoELayer each, owning E/P experts; devices[r] is rank r's GPU."""
+
+    def __init__(self, preset, weights, ep_size: int, max_tokens: int, devices=None):
+        devices = devices or [0] * ep_size
+        self.P = ep_size
+        self.layers = []
+        for r in range(ep_size):
+            wr = slice_experts(weights, r, ep_size)
+            if devices[r] != weights.w13.device.index:
+                wr = wr.to(f"cuda:{devices[r]}")
+            self.layers.append(MoELayer(preset, wr, max_tokens=max_tokens, device=devices[r], ep_rank=r,
+                                        ep_size=ep_size))
+        self._lib = load_library()
+
+    def forward(self, xs, residuals=None, n_deferred=0, deferred_in=None, want_deferred_out=False, stream=None):
+        P = self.P
+        vp = ctypes.c_void_p
+        arr = lambda ts: (vp * P)(*[None if t is None else _ptr(t) for t in ts]) if ts is not None else None
+        ys = [torch.empty_like(x) for x in xs]
+        douts = [torch.empty_like(x) for x in xs] if want_deferred_out else None
+        T = (ctypes.c_int32 * P)(*[x.shape[0] for x in xs])
+        st = (stream or torch.cuda.current_stream(xs[0].device)).cuda_stream
+        s = self._lib.moe_ep_group_forward((vp * P)(*[l._h.value for l in self.layers]), P, arr(xs), arr(residuals),
+                                           T, n_deferred, arr(deferred_in), arr(ys), arr(douts), st)
+        _check(s, "moe_ep_group_forward")
+        return (ys, douts) if want_deferred_out else ys
+
+    def close(self):
+        for l in self.layers:
+            l.close()

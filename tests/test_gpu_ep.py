@@ -1,0 +1,80 @@
+"""Expert parallelism through the C ABI on one GPU: an in-process group of P
+ranks (moe_ep_group_forward: every transfer of the NCCL path done as device
+copies) and the NCCL transport itself with a 1-rank communicator.  Each rank's
+outputs are checked against the oracle on that rank's tokens."""
+import numpy as np
+import pytest
+import torch
+
+from inputs.presets import SMALL
+from inputs.synthetic import make_tokens, make_weights
+from oracle import moe_oracle as O
+from tests.parity import TOL, oracle_cfg, oracle_weights, rel_l2
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lib():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sosp_chenxztwdcylqzo25_b200 import moe
+    return moe
+
+
+def _oracle_check(p, w_cpu, x, y, residual=None, n_def=0, din=None, dout=None):
+    cfg, W = oracle_cfg(p), oracle_weights(p, w_cpu)
+    x64 = x.to(torch.float64).numpy()
+    if x64.shape[0] == 0:
+        return
+    ties = O.tie_band_tokens(x64, W, cfg, n_deferred=n_def)
+    keep = np.setdiff1d(np.arange(x64.shape[0]), ties)
+    out = O.moe_layer(x64, W, cfg, residual=None if residual is None else residual.to(torch.float64).numpy(),
+                      n_deferred=n_def, deferred_in=None if din is None else din.cpu().to(torch.float64).numpy())
+    assert rel_l2(y.float().cpu().numpy()[keep], out["y"][keep]) <= TOL[p.wtype]
+    if dout is not None:
+        assert rel_l2(dout.float().cpu().numpy()[keep], out["deferred_out"][keep]) <= TOL[p.wtype]
+
+
+@pytest.mark.parametrize("name,P,Ts", [("v3_s", 2, [40, 33]), ("v3_s", 4, [25, 0, 61, 7]),
+                                       ("qwen2_s", 2, [50, 19]), ("v25_s", 4, [30, 30, 30, 30]),
+                                       ("v3_s", 8, [5, 9, 1, 0, 3, 17, 2, 8])])
+def test_ep_group(lib, name, P, Ts):
+    p = SMALL[name]
+    w_cpu = make_weights(p, "cpu")
+    group = lib.MoEGroup(p, w_cpu.to("cuda"), ep_size=P, max_tokens=max(Ts) or 1)
+    xs = [make_tokens(p, t, "cpu", offset=r)[0] for r, t in enumerate(Ts)]
+    ys = group.forward([x.cuda() for x in xs])
+    torch.cuda.synchronize()
+    for x, y in zip(xs, ys):
+        _oracle_check(p, w_cpu, x, y)
+    group.close()
+
+
+def test_ep_group_deferral_and_residual(lib):
+    p = SMALL["v3_s"]
+    P, Ts = 2, [24, 31]
+    w_cpu = make_weights(p, "cpu")
+    group = lib.MoEGroup(p, w_cpu.to("cuda"), ep_size=P, max_tokens=32)
+    xs, rs = zip(*[make_tokens(p, t, "cpu", offset=r) for r, t in enumerate(Ts)])
+    dins = [(torch.randn(t, p.hidden, generator=torch.Generator().manual_seed(r)) * 0.5).to(torch.bfloat16)
+            for r, t in enumerate(Ts)]
+    ys, douts = group.forward([x.cuda() for x in xs], residuals=[r.cuda() for r in rs], n_deferred=3,
+                              deferred_in=[d.cuda() for d in dins], want_deferred_out=True)
+    torch.cuda.synchronize()
+    for x, r, d, y, do in zip(xs, rs, dins, ys, douts):
+        _oracle_check(p, w_cpu, x, y, residual=r, n_def=3, din=d, dout=do)
+    group.close()
+
+
+def test_ep_nccl_single_rank(lib):
+    """The NCCL transport (send/recv to self) with a 1-rank communicator."""
+    p = SMALL["v3_s"]
+    w_cpu = make_weights(p, "cpu")
+    uid = lib.get_unique_id()
+    layer = lib.MoELayer(p, w_cpu.to("cuda"), max_tokens=64, ep_rank=0, ep_size=1, unique_id=uid)
+    x, _ = make_tokens(p, 57, "cpu")
+    y = layer.forward(x.cuda())
+    torch.cuda.synchronize()
+    _oracle_check(p, w_cpu, x, y)
+    layer.close()
