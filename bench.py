@@ -247,7 +247,18 @@ def run_ours(args):
     w = make_weights(p, "cuda")
     x, _ = make_tokens(p, T, "cuda", offset=rank)
     y = torch.empty_like(x)
-    layer = moe.MoELayer(p, w, max_tokens=T, device=local)
+    ep = ws > 1 and not args.replicas
+    if ep:
+        # expert parallelism over NCCL: rank r owns experts [r E/P, (r+1) E/P);
+        # the router and the shared expert are replicated
+        import torch.distributed as dist
+        uid = [moe.get_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        w = moe.slice_experts(w, rank, ws)
+        torch.cuda.empty_cache()
+        layer = moe.MoELayer(p, w, max_tokens=T, device=local, ep_rank=rank, ep_size=ws, unique_id=uid[0])
+    else:
+        layer = moe.MoELayer(p, w, max_tokens=T, device=local)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
     info = layer.info()
 
@@ -255,22 +266,30 @@ def run_ours(args):
     barrier(ws)
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
-        times, stages = timed_steps(layer, [x], y, args.steps, args.warmup, flush)
+        times, stages = timed_steps(layer, [x], y, args.steps, args.warmup, flush, profile=not ep)
     torch.cuda.synchronize()
     barrier(ws)
     ms = max_over_ranks(sum(times) / len(times), ws)
     value = ws * T / (ms * 1e-3)
 
     # routing statistics of this batch (distinct experts hit, for the byte counts)
-    routing = {}
-    layer.forward(x, y=y, routing=routing)
-    counts = routing["expert_counts"].cpu()
-    n_distinct = int((counts > 0).sum())
+    if ep:
+        n_distinct = p.n_experts // ws
+    else:
+        routing = {}
+        layer.forward(x, y=y, routing=routing)
+        counts = routing["expert_counts"].cpu()
+        n_distinct = int((counts > 0).sum())
     alg = algorithmic(p, T, n_distinct)
     fp8 = p.wtype == 1
     tc_peak = (2.0 if fp8 else 1.0) * peaks["bf16_tflops_sustained"]
-    dom = max((k for k in stages if k in alg), key=lambda k: stages[k])
-    ach = alg[dom]["flops"] / (stages[dom] * 1e-3) / 1e12
+    if stages:
+        dom = max((k for k in stages if k in alg), key=lambda k: stages[k])
+        dom_ms = stages[dom]
+    else:                      # expert parallel: whole-step rate of the routed FFN work on this rank
+        dom, dom_ms = "layer_ep", ms
+        alg[dom] = {"flops": alg["gemm1_swiglu"]["flops"] + alg["gemm2"]["flops"]}
+    ach = alg[dom]["flops"] / (dom_ms * 1e-3) / 1e12
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
@@ -288,7 +307,7 @@ def run_ours(args):
     # one CUDA graph), timed with events around the replay; a separate eager
     # pass with stage events gives the per-kernel breakdown.
     decode = None
-    if not args.no_decode:
+    if not args.no_decode and not ep:
         xd, _ = make_tokens(p, args.steps + args.warmup, "cuda", offset=1000 + rank)
         rows = [xd[i:i + 1].contiguous() for i in range(xd.shape[0])]
         yd = torch.empty_like(rows[0])
@@ -330,7 +349,7 @@ def run_ours(args):
 
     # ---------------- e2e through the public API, host buffers ----------------
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and not ep:
         xh = x.cpu().pin_memory()
         yh = torch.empty_like(xh).pin_memory()
         xdev = torch.empty_like(x)
@@ -370,7 +389,8 @@ def run_ours(args):
                 "config": {"workload": f"{p.name}_moe_layer_prefill", "tokens_per_gpu": T, "hidden": p.hidden,
                            "ffn": p.ffn, "experts": p.n_experts, "top_k": p.top_k, "shared_ffn": p.shared_ffn,
                            "weights": "fp8_e4m3_block128_ue8m0" if fp8 else "bf16", "parallelism":
-                           f"replica x{ws}" if ws > 1 else "single", "l2": "flushed before every step (256 MiB write, "
+                           (f"ep{ws} (NCCL all-to-all-v dispatch/combine)" if ep else f"replica x{ws}")
+                           if ws > 1 else "single", "l2": "flushed before every step (256 MiB write, "
                            "outside the timed events); inputs resident in HBM",
                            "distinct_experts_hit": n_distinct},
                 "layer_tflops": layer_tflops,
@@ -396,6 +416,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=20.0)
+    ap.add_argument("--replicas", action="store_true", help="N>1: independent replicas instead of expert parallel")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3

@@ -74,6 +74,7 @@ struct PermuteArgs {
   int32_t *chunk_cnt, *chunk_base;  // [nchunk, E]
   int32_t *counts, *offs, *offs_pad;
   int4 *tiles; int32_t *n_tiles;
+  int4 *pairs; int32_t *n_pairs;   // 2-CTA work list (null = not needed)
   int32_t *act_list; int32_t *n_active;
   int32_t *row_token;       // [R_max]
   int64_t R_max;
@@ -179,6 +180,7 @@ struct UmmaGroup {              // one operand set: 0 = routed experts, 1 = shar
   uint8_t *out_sf;              // FP8 SwiGLU: scale image of h
   int out_sf_tile_stride;
   int n_valid;                  // LOGITS: output columns < n_valid are written
+  CUtensorMap sfa_map, sfb_map; // CTA-pair kernel: scale images as 512-byte rows (box 1 / 2 rows)
 };
 struct UmmaParams {
   UmmaGroup g[2];
@@ -188,6 +190,8 @@ struct UmmaParams {
   int T_shared;                 // shared-expert rows (0 = none)
   int nb_s;                     // shared N blocks of 256
   int *sched;                   // device work counter, zero at launch (dynamic scheduler)
+  const int4 *pairs;            // CTA-pair kernel: routed work list of 256-row tile pairs
+  const int32_t *n_pairs;
   int debug_mode;               // 0; (MOE_DEBUG_GEMM) 1 = loads only, 2 = no epilogue -- timing experiments
 };
 cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st);
@@ -210,5 +214,8 @@ struct UmmaDecodeParams {
 cudaError_t launch_umma_decode(bool fp8, int mode, const UmmaDecodeParams &p, int grid, cudaStream_t st);
 
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);
+bool make_rows_map(CUtensorMap *m, const void *base, bool u32, int64_t rows, int row_elems, int box_rows);
+// grouped GEMM on CTA pairs (cta_group::2); b_map = tiled weights as 128-byte rows
+cudaError_t launch_umma_pair_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st);
 
 }  // namespace moe

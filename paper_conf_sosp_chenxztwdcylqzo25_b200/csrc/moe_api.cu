@@ -47,7 +47,7 @@ void free_all(moe_layer *L) {
   void *ptrs[] = {L->gate_w, L->gate_bias, L->w13, L->w13_s, L->w2, L->w2_s, L->ws13, L->ws13_s, L->ws2,
                   L->ws2_s, L->logits, L->topk_idx, L->topk_w, L->sgate, L->chunk_cnt, L->chunk_base,
                   L->counts, L->offs, L->offs_pad, L->tiles, L->n_tiles, L->act_list, L->n_active,
-                  L->row_token, L->pos, L->sched, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
+                  L->row_token, L->pos, L->sched, L->pairs, L->n_pairs, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
                   L->hsh, L->hsh_s, L->ysh, L->w13_img, L->w2_img, L->ws13_img, L->ws2_img,
                   L->xperm_img, L->h_img, L->xq_img, L->hsh_img};
   for (void *p : ptrs)
@@ -326,6 +326,8 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   C_TRY(dalloc(L, &L->act_list, (size_t)E * 4, false));
   C_TRY(dalloc(L, &L->n_active, 4, false));
   C_TRY(dalloc(L, &L->sched, 32, false));
+  C_TRY(dalloc(L, &L->pairs, (size_t)L->max_tiles * sizeof(int4), false));
+  C_TRY(dalloc(L, &L->n_pairs, 4, false));
   C_TRY(dalloc(L, &L->row_token, (size_t)L->R_max * 4, false));
   C_TRY(dalloc(L, &L->pos, (size_t)pairs * 4, false));
   if (L->fp8) {
@@ -398,6 +400,29 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
       ok = ok && make_kmajor_map(&L->dmap_hsh, L->hsh, f8, Tm, Fs, 16);
       if (f8) ok = ok && make_kmajor_map(&L->dmap_xq, L->xq, true, Tm, H, 16);
     }
+    // CTA-pair GEMM maps (MOE_PAIR=0 disables the pair kernel)
+    {
+      const char *ev = getenv("MOE_PAIR");
+      L->pair = !(ev && ev[0] == '0');
+      const int64_t es = f8 ? 1 : 2;
+      ok = ok && make_rows_map(&L->tmap_w13, L->w13, false, (int64_t)E * 2 * F * H * es / 128, 128, 128) &&
+           make_rows_map(&L->tmap_w2, L->w2, false, (int64_t)E * H * F * es / 128, 128, 128);
+      if (Fs)
+        ok = ok && make_rows_map(&L->tmap_ws13, L->ws13, false, (int64_t)2 * Fs * H * es / 128, 128, 128) &&
+             make_rows_map(&L->tmap_ws2, L->ws2, false, (int64_t)H * Fs * es / 128, 128, 128);
+      if (f8) {
+        const int64_t g1 = (H / 128 + 3) / 4, g2 = (F / 128 + 3) / 4, gs = (Fs / 128 + 3) / 4;
+        ok = ok && make_rows_map(&L->smap_w13, L->w13_img, true, E * g1 * (2 * F / 128), 128, 2) &&
+             make_rows_map(&L->smap_w2, L->w2_img, true, E * g2 * (H / 128), 128, 2) &&
+             make_rows_map(&L->smap_xperm, L->xperm_img, true, g1 * L->max_tiles, 128, 1) &&
+             make_rows_map(&L->smap_h, L->h_img, true, g2 * L->max_tiles, 128, 1) &&
+             make_rows_map(&L->smap_xq, L->xq_img, true, g1 * L->img_tiles_sh, 128, 1);
+        if (Fs)
+          ok = ok && make_rows_map(&L->smap_ws13, L->ws13_img, true, g1 * (2 * Fs / 128), 128, 2) &&
+               make_rows_map(&L->smap_ws2, L->ws2_img, true, gs * (H / 128), 128, 2) &&
+               make_rows_map(&L->smap_hsh, L->hsh_img, true, gs * L->img_tiles_sh, 128, 1);
+      }
+    }
     if (!ok) return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable?)"));
   }
   C_TRY(cudaDeviceSynchronize());
@@ -459,7 +484,16 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = 2 * Fs / 256; p1.sched = L->sched;
     static const int dbg_mode = getenv("MOE_DEBUG_GEMM") ? atoi(getenv("MOE_DEBUG_GEMM")) : 0;
     p1.debug_mode = dbg_mode;
-    CUDA_TRY(launch_umma_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
+    if (L->pair) {
+      // CTA pairs: weights via the tiled-row maps, scale images via 512-byte-row maps
+      p1.g[0].b_map = L->tmap_w13; p1.g[0].sfa_map = L->smap_xperm; p1.g[0].sfb_map = L->smap_w13;
+      if (Fs > 0) { p1.g[1].b_map = L->tmap_ws13; p1.g[1].sfa_map = L->smap_xq; p1.g[1].sfb_map = L->smap_ws13; }
+      else p1.g[1] = p1.g[0];
+      p1.pairs = L->pairs; p1.n_pairs = L->n_pairs;
+      CUDA_TRY(launch_umma_pair_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
+    } else {
+      CUDA_TRY(launch_umma_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
+    }
     mark(L, ST_GEMM1, st);
     UmmaParams p2{};
     {
@@ -481,7 +515,15 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     p2.tiles = L->tiles; p2.n_tiles = L->n_tiles; p2.nb_r = H / 256;
     p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256; p2.sched = L->sched + 1;
     p2.debug_mode = dbg_mode;
-    CUDA_TRY(launch_umma_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
+    if (L->pair) {
+      p2.g[0].b_map = L->tmap_w2; p2.g[0].sfa_map = L->smap_h; p2.g[0].sfb_map = L->smap_w2;
+      if (Fs > 0) { p2.g[1].b_map = L->tmap_ws2; p2.g[1].sfa_map = L->smap_hsh; p2.g[1].sfb_map = L->smap_ws2; }
+      else p2.g[1] = p2.g[0];
+      p2.pairs = L->pairs; p2.n_pairs = L->n_pairs;
+      CUDA_TRY(launch_umma_pair_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
+    } else {
+      CUDA_TRY(launch_umma_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
+    }
     mark(L, ST_GEMM2, st);
   } else {
     // 5. routed experts: GEMM1 + SwiGLU, GEMM2 (CUDA-core path: F32 weights, H % 256 != 0)
@@ -593,10 +635,12 @@ static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_d
   pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
   pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
   pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
+  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs;
   if (R > 0) {
     CUDA_TRY(launch_permute(pa, st));
   } else {
     CUDA_TRY(cudaMemsetAsync(L->n_tiles, 0, 4, st));
+    CUDA_TRY(cudaMemsetAsync(L->n_pairs, 0, 4, st));
   }
   ScatterDst d{};
   d.fp8 = L->fp8; d.xperm = L->xperm;
@@ -710,6 +754,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
   pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
   pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
+  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs;
   pa.dbg_perm = dbg ? dbg->perm : nullptr;
   pa.dbg_counts = dbg ? dbg->expert_counts : nullptr;
   if (tc_decode) {

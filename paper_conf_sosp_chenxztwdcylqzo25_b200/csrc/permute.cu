@@ -62,6 +62,12 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(PermuteArgs a, int n
   Scan(tmp).ExclusiveSum(cnt > 0 ? 1 : 0, act_off, total);
   if (e == 0) *a.n_active = total;
   __syncthreads();
+  // 2-CTA work list: pairs of consecutive 128-row tiles of one expert
+  const int npair = (ntile + 1) / 2;
+  int pair_off;
+  Scan(tmp).ExclusiveSum(npair, pair_off, total);
+  if (e == 0 && a.n_pairs) *a.n_pairs = total;
+  __syncthreads();
   if (e < a.E) {
     a.counts[e] = cnt;
     if (a.dbg_counts) a.dbg_counts[e] = cnt;
@@ -69,6 +75,9 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(PermuteArgs a, int n
     a.offs_pad[e] = off_pad;
     for (int m = 0; m < ntile; ++m)
       a.tiles[tile_off + m] = make_int4(e, off_pad + m * kPadM, off_pad + cnt, tile_off | (ntile << 16));
+    if (a.pairs)
+      for (int m = 0; m < npair; ++m)
+        a.pairs[pair_off + m] = make_int4(e, off_pad + m * 2 * kPadM, off_pad + cnt, pair_off | (npair << 16));
     if (cnt > 0) a.act_list[act_off] = e;
   }
   if (e == 0) {
