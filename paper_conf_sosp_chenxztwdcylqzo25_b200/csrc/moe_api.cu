@@ -400,10 +400,10 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
       ok = ok && make_kmajor_map(&L->dmap_hsh, L->hsh, f8, Tm, Fs, 16);
       if (f8) ok = ok && make_kmajor_map(&L->dmap_xq, L->xq, true, Tm, H, 16);
     }
-    // CTA-pair GEMM maps (MOE_PAIR=0 disables the pair kernel)
+    // CTA-pair GEMM maps (MOE_PAIR=1 enables the pair kernel; off by default, see umma_gemm2.cu)
     {
       const char *ev = getenv("MOE_PAIR");
-      L->pair = !(ev && ev[0] == '0');
+      L->pair = ev && ev[0] == '1';
       const int64_t es = f8 ? 1 : 2;
       ok = ok && make_rows_map(&L->tmap_w13, L->w13, false, (int64_t)E * 2 * F * H * es / 128, 128, 128) &&
            make_rows_map(&L->tmap_w2, L->w2, false, (int64_t)E * H * F * es / 128, 128, 128);
