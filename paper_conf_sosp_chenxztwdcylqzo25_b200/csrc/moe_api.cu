@@ -169,7 +169,8 @@ moe_status build_weight_image(const std::vector<float> &s, int nexp, int rows, i
 
 moe_status validate(const moe_layer_config *c, const moe_layer_weights *w) {
   if (!c || !w) return fail(MOE_ERR_INVALID_ARG, "null config or weights");
-  if (c->hidden <= 0 || c->hidden % 128) return fail(MOE_ERR_UNSUPPORTED, "hidden %d must be a positive multiple of 128", c->hidden);
+  if (c->hidden <= 0 || c->hidden % 128 || c->hidden > 8192)
+    return fail(MOE_ERR_UNSUPPORTED, "hidden %d must be a positive multiple of 128, at most 8192", c->hidden);
   if (c->ffn <= 0 || c->ffn % 128) return fail(MOE_ERR_UNSUPPORTED, "ffn %d must be a positive multiple of 128", c->ffn);
   if (c->shared_ffn < 0 || c->shared_ffn % 128) return fail(MOE_ERR_UNSUPPORTED, "shared_ffn %d must be a multiple of 128", c->shared_ffn);
   if (c->n_experts <= 0 || c->n_experts > 1024) return fail(MOE_ERR_UNSUPPORTED, "n_experts %d not in [1, 1024]", c->n_experts);
@@ -764,7 +765,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     static const int dbg_route = getenv("MOE_DEBUG_ROUTE") ? atoi(getenv("MOE_DEBUG_ROUTE")) : 0;
     rs.debug = dbg_route;
     rs.fp8 = L->fp8; rs.xperm = L->xperm; rs.xperm_img = L->xperm_img; rs.xperm_img_stride = L->max_tiles;
-    if (L->fp8 && Fs > 0) { rs.xq = L->xq; rs.xs = L->xs; rs.xq_img = L->xq_img; rs.xq_img_stride = L->img_tiles_sh; }
+    if (L->fp8) { rs.xq = L->xq; rs.xs = L->xs; rs.xq_img = L->xq_img; rs.xq_img_stride = L->img_tiles_sh; }
     CUDA_TRY(launch_route_small(rs, st));
     mark(L, ST_PERMUTE, st);
   } else {

@@ -201,7 +201,17 @@ __device__ void select_token_block(const RouterArgs &args, int t, float *s, floa
   // group limit: thread g scores group g, then ranks it
   if (G > 1) {
     const int gs = E / G;
-    if (tid < G) {
+    if (gs == 32 && E <= NT) {
+      // one warp per group (DeepSeek-V3: 256 experts / 8 groups): warp reductions
+      const int lane = tid & 31, g = tid >> 5;
+      if (g < G) {
+        const float v = sel[tid];
+        const float m1 = warp_max(v);
+        const int nmax = __popc(__ballot_sync(0xffffffffu, v == m1));
+        const float m2 = nmax >= 2 ? m1 : warp_max(v == m1 ? -INFINITY : v);
+        if (lane == 0) gsc[g] = args.group_score == MOE_GROUP_TOP2_SUM ? m1 + m2 : m1;
+      }
+    } else if (tid < G) {
       float m1 = -INFINITY, m2 = -INFINITY;
 #pragma unroll 1
       for (int i = 0; i < gs; ++i) {
@@ -319,12 +329,52 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
     if (row < a.rows && tid < T)
       const_cast<float *>(r.logits)[(size_t)tid * r.ldl + row] = red[half][0][tid] + red[half][1][tid] + red[half][2][tid] + red[half][3][tid];
   }
+  // ---- FP8: quantise x -> xq (token order) across all CTAs, in parallel with routing ----
+  if (a.fp8 && a.xq) {
+    const int nc = H / 8;                       // 8-element chunks per row; a 1x128 block = 16 chunks
+    const int64_t total = (int64_t)T * nc;
+    const int lane = threadIdx.x & 31;
+    for (int64_t base = ((int64_t)blockIdx.x * RS_THREADS + (threadIdx.x & ~31)); base < total;
+         base += (int64_t)gridDim.x * RS_THREADS) {
+      const int64_t gch = base + lane;
+      const bool ok = gch < total;
+      float f[8];
+      float am = 0.f;
+      if (ok) {
+        const int64_t t = gch / nc, c = gch % nc;
+        bf16x8_to_f32(__ldg(reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + t * H) + c),
+                      f);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) am = fmaxf(am, fabsf(f[j]));
+      }
+#pragma unroll
+      for (int o = 8; o > 0; o >>= 1) am = fmaxf(am, __shfl_xor_sync(0xffffffffu, am, o));
+      if (ok) {
+        const int64_t t = gch / nc, c = gch % nc;
+        const int ex = ue8m0_exponent(am);
+        const float inv = exp2i(-ex);
+        uint2 q;
+        q.x = (uint32_t)f32_to_e4m3(f[0] * inv) | ((uint32_t)f32_to_e4m3(f[1] * inv) << 8) |
+              ((uint32_t)f32_to_e4m3(f[2] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[3] * inv) << 24);
+        q.y = (uint32_t)f32_to_e4m3(f[4] * inv) | ((uint32_t)f32_to_e4m3(f[5] * inv) << 8) |
+              ((uint32_t)f32_to_e4m3(f[6] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[7] * inv) << 24);
+        *reinterpret_cast<uint2 *>(reinterpret_cast<uint8_t *>(a.xq) + t * H + c * 8) = q;
+        if ((lane & 15) == 0) {
+          const int b = (int)(c >> 4);
+          a.xs[t * (H / 128) + b] = exp2i(ex);
+          if (a.xq_img) a.xq_img[sf_img_off(t, b, a.xq_img_stride)] = (uint8_t)(ex + 127);
+        }
+      }
+    }
+  }
+
   // ---- last CTA: route + permute ----
   __threadfence();
   __syncthreads();
   if (threadIdx.x == 0) is_last = (atomicAdd(a.done, 1) == (int)gridDim.x - 1);
   __syncthreads();
   if (!is_last) return;
+  long long ck0 = clock64();
   if (a.debug & 2) { if (threadIdx.x == 0) *a.done = 0; return; }
   __threadfence();
   {
@@ -332,6 +382,9 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
     int *ids = reinterpret_cast<int *>(ws + 32);
 #pragma unroll 1
     for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws);
+  }
+  long long ck1 = clock64();
+  {
   }
   // counts / offsets / active list over the local experts
   const PermuteArgs &p = a.p;
@@ -380,6 +433,7 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
     }
   }
   __syncthreads();
+  long long ck2 = clock64();
   // stable assignment: tokens in order, a token's k experts are distinct
   for (int t = 0; t < T; ++t) {
     if (threadIdx.x < p.k) {
@@ -396,6 +450,7 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
     __syncthreads();
   }
   if (!a.xperm) return;
+  long long ck3 = clock64();
   // activations into expert order (replaces the quantise + gather launches)
   __shared__ int spos[32];
   ScatterDst d{};
@@ -405,9 +460,38 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
   for (int t = 0; t < T; ++t) {
     if (threadIdx.x < p.k) spos[threadIdx.x] = p.pos[t * p.k + threadIdx.x];
     __syncthreads();
-    scatter_token_row<RS_THREADS>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H, H, t, p.k, spos, d);
+    if (a.fp8) {
+      // codes were quantised into xq by all CTAs: copy the row and its scale bytes
+      // every thread loads its chunks (<= 4: H <= 16384) and scale byte once, then stores k times
+      const uint4 *src = reinterpret_cast<const uint4 *>(reinterpret_cast<const uint8_t *>(a.xq) + (size_t)t * H);
+      uint4 v[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int c = threadIdx.x + RS_THREADS * i;
+        if (c < H / 16) v[i] = src[c];
+      }
+      const int b = threadIdx.x;
+      const uint8_t sb = b < H / 128 ? (uint8_t)((__float_as_uint(a.xs[(size_t)t * (H / 128) + b]) >> 23) & 0xFF) : 0;
+#pragma unroll 1
+      for (int j = 0; j < p.k; ++j) {
+        const int rw = spos[j];
+        if (rw < 0) continue;
+        uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<uint8_t *>(a.xperm) + (size_t)rw * H);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int c = threadIdx.x + RS_THREADS * i;
+          if (c < H / 16) dst[c] = v[i];
+        }
+        if (b < H / 128) a.xperm_img[sf_img_off(rw, b, a.xperm_img_stride)] = sb;
+      }
+    } else {
+      scatter_token_row<RS_THREADS>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H, H, t, p.k, spos, d);
+    }
     __syncthreads();
   }
+  if ((a.debug & 4) && threadIdx.x == 0)       // MOE_DEBUG_ROUTE=4: phase cycle counts of the tail
+    printf("route tail cycles: select %lld scan %lld assign %lld rows %lld\n", ck1 - ck0, ck2 - ck1, ck3 - ck2,
+           clock64() - ck3);
 }
 
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st) {

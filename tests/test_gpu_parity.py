@@ -182,3 +182,13 @@ def test_full_size_sampled(lib, name, T):
 
 def test_full_v3_decode_deferral(lib):
     _full(lib, "v3", 1, n_def=3, sample=1)
+
+
+@pytest.mark.parametrize("name", ["v3_s", "qwen2_s"])
+def test_pair_kernel_parity(lib, name, monkeypatch):
+    """The CTA-pair (cta_group::2) grouped GEMM (opt-in, MOE_PAIR=1) matches the oracle."""
+    monkeypatch.setenv("MOE_PAIR", "1")
+    p = SMALL[name]
+    res = _run(lib, p, p.prefill_tokens)
+    out, ties, idx, w = _oracle(p, res)
+    assert rel_l2(res["y"], out["y"]) <= TOL[p.wtype]
