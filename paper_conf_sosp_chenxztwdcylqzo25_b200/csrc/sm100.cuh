@@ -48,6 +48,12 @@ __device__ __forceinline__ void mbar_wait_cluster(uint64_t *bar, uint32_t phase)
       : "memory");
 }
 
+__device__ __forceinline__ int ld_acquire_gpu(const int *p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
 // ------------------------------------------------------------------ TMA / bulk
 __device__ __forceinline__ void prefetch_tmap(const void *map) {
   asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
