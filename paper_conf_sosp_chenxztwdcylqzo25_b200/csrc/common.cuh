@@ -221,11 +221,12 @@ struct moe_layer {
   int64_t w13_img_stride = 0, w2_img_stride = 0;
   CUtensorMap map_xperm, map_h, map_xq, map_hsh, map_gate;   // activation rows (box 128), router rows
   CUtensorMap dmap_xperm, dmap_h, dmap_xq, dmap_hsh;           // decode: activation rows (box 16)
-  // CTA-pair GEMM: tiled weights as 128-byte rows (box 128), scale images as 512-byte rows
+  // swap-AB CTA-pair GEMM (umma_swap.cu): tiled weights as 128-byte rows (box 128),
+  // token rows (box 32), weight scale images (box 1) and token scale images (box 2)
   CUtensorMap tmap_w13, tmap_w2, tmap_ws13, tmap_ws2;
+  CUtensorMap xmap_xperm, xmap_h, xmap_xq, xmap_hsh;
   CUtensorMap smap_w13, smap_w2, smap_ws13, smap_ws2, smap_xperm, smap_h, smap_xq, smap_hsh;
-  bool pair = false;            // use the cta_group::2 kernel for the prefill GEMMs
-  int4 *pairs = nullptr;        // [max_tiles] work list of 2-tile pairs
+  int4 *pairs = nullptr;        // [max_tiles] work list of 256-token tiles (2 x 128-row tiles)
   int32_t *n_pairs = nullptr;
   bool gemv_ok = false;         // decode weight-streaming path usable for T <= gemv_max_tokens
   int num_sms = 148;

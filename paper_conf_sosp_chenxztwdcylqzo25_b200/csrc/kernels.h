@@ -193,6 +193,7 @@ struct UmmaParams {
   const int4 *pairs;            // CTA-pair kernel: routed work list of 256-row tile pairs
   const int32_t *n_pairs;
   int debug_mode;               // 0; (MOE_DEBUG_GEMM) 1 = loads only, 2 = no epilogue -- timing experiments
+  int pf_dist;                  // weight k-blocks prefetched into L2 ahead of the TMA loads (0 = off)
 };
 cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st);
 // Repack row-major weights [rows, K] (es bytes/elem) into 256-row x 128-byte
@@ -215,7 +216,31 @@ cudaError_t launch_umma_decode(bool fp8, int mode, const UmmaDecodeParams &p, in
 
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);
 bool make_rows_map(CUtensorMap *m, const void *base, bool u32, int64_t rows, int row_elems, int box_rows);
-// grouped GEMM on CTA pairs (cta_group::2); b_map = tiled weights as 128-byte rows
-cudaError_t launch_umma_pair_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st);
+// prefill grouped expert GEMM, swap-AB on CTA pairs (umma_swap.cu): weights are
+// the M = 256 operand, an expert's tokens (<= 256, padded to 16) the N operand
+struct SwapGroup {              // one operand set: 0 = routed experts, 1 = shared expert
+  CUtensorMap w_map;            // tiled weights as 128-byte rows, box 128 rows
+  CUtensorMap x_map;            // token rows, K-major SW128, box 32 rows
+  CUtensorMap sfw_map;          // FP8: weight scale images as 512-byte rows, box 1
+  CUtensorMap sfx_map;          // FP8: token scale images as 512-byte rows, box 2
+  int w_nblk;                   // 256-row weight blocks per expert
+  int kblocks;                  // K / 128 bytes
+  int sfw_per_cta;              // 1: an image per 128-row CTA half (W2); 0: per 256-row block (W13)
+  int sfx_tile_stride;          // 128-row tiles per k-group in the token image
+  void *out;                    // h (SWIGLU) or y (PLAIN) rows
+  int64_t ldc;                  // elements
+  uint8_t *out_sf;              // FP8 SWIGLU: scale image of h
+  int out_sf_tile_stride;
+};
+struct SwapParams {
+  SwapGroup g[2];
+  const int4 *tiles;            // routed 256-token tiles (expert, row0, row_end, t0 | nt << 16)
+  const int32_t *n_tiles;
+  int nb_r, nb_s;               // weight blocks per unit group
+  int T_shared;                 // shared-expert tokens (0 = none)
+  int *sched;                   // device work counter, zero at launch
+  int debug_mode;               // 0; (MOE_DEBUG_GEMM) 2 = no epilogue math -- timing experiments
+};
+cudaError_t launch_umma_swap_gemm(bool fp8, int epi, const SwapParams &p, int grid, cudaStream_t st);
 
 }  // namespace moe

@@ -167,6 +167,41 @@ moe_status build_weight_image(const std::vector<float> &s, int nexp, int rows, i
   return MOE_OK;
 }
 
+// W13 scale image for the swap-AB layout (umma_swap.cu / umma_decode.cu): one
+// 512-byte image per (expert, group of 4 k-blocks, 128-column h block nb).  A
+// 128-row CTA half of tile nb holds, per lane quadrant, [gate | up | gate | up]
+// rows of block nb, so TMEM word w (= quadrant) of every lane takes the gate
+// (w even) or up (w odd) block scale.  s = interleaved block scales from
+// load_scales: [(e * 2F/128 + 2 nb (+1 up)) * H/128 + kb].
+moe_status build_w13_swap_image(const std::vector<float> &s, int nexp, int F, int H, uint8_t **dst, moe_layer *L,
+                                int64_t *expert_stride) {
+  const int nbn = F / 128, rb = 2 * nbn, kbn = H / 128, G = (kbn + 3) / 4;
+  const size_t per_exp = (size_t)G * nbn * 512;
+  std::vector<uint8_t> img((size_t)nexp * per_exp);
+  for (int e = 0; e < nexp; ++e)
+    for (int g = 0; g < G; ++g)
+      for (int nb = 0; nb < nbn; ++nb) {
+        uint8_t b[2][4];
+        for (int u = 0; u < 2; ++u)
+          for (int j = 0; j < 4; ++j) {
+            const int kb = 4 * g + j;
+            uint32_t bits = 127u << 23;
+            if (kb < kbn) {
+              const float v = s[((size_t)e * rb + 2 * nb + u) * kbn + kb];
+              memcpy(&bits, &v, 4);
+            }
+            b[u][j] = (uint8_t)((bits >> 23) & 0xFF);
+          }
+        uint8_t *d = img.data() + e * per_exp + ((size_t)g * nbn + nb) * 512;
+        for (int l = 0; l < 32; ++l)
+          for (int w = 0; w < 4; ++w) memcpy(d + 16 * l + 4 * w, b[w & 1], 4);
+      }
+  CUDA_TRY(dalloc(L, dst, img.size(), true));
+  CUDA_TRY(cudaMemcpy(*dst, img.data(), img.size(), cudaMemcpyHostToDevice));
+  *expert_stride = (int64_t)per_exp;
+  return MOE_OK;
+}
+
 moe_status validate(const moe_layer_config *c, const moe_layer_weights *w) {
   if (!c || !w) return fail(MOE_ERR_INVALID_ARG, "null config or weights");
   if (c->hidden <= 0 || c->hidden % 128 || c->hidden > 8192)
@@ -371,10 +406,10 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
     L->img_tiles_sh = (int)((Tm + 127) / 128);
     if (f8) {
       int64_t st;
-      S_TRY(build_weight_image(hs13, E, 2 * F, H, &L->w13_img, L, &st)); L->w13_img_stride = st;
+      S_TRY(build_w13_swap_image(hs13, E, F, H, &L->w13_img, L, &st)); L->w13_img_stride = st;
       S_TRY(build_weight_image(hs2, E, H, F, &L->w2_img, L, &st)); L->w2_img_stride = st;
       if (Fs) {
-        S_TRY(build_weight_image(hss13, 1, 2 * Fs, H, &L->ws13_img, L, &st));
+        S_TRY(build_w13_swap_image(hss13, 1, Fs, H, &L->ws13_img, L, &st));
         S_TRY(build_weight_image(hss2, 1, H, Fs, &L->ws2_img, L, &st));
       }
       const size_t g1 = (H / 128 + 3) / 4, g2 = (F / 128 + 3) / 4, gs = (Fs / 128 + 3) / 4;
@@ -401,27 +436,31 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
       ok = ok && make_kmajor_map(&L->dmap_hsh, L->hsh, f8, Tm, Fs, 16);
       if (f8) ok = ok && make_kmajor_map(&L->dmap_xq, L->xq, true, Tm, H, 16);
     }
-    // CTA-pair GEMM maps (MOE_PAIR=1 enables the pair kernel; off by default, see umma_gemm2.cu)
+    // swap-AB pair GEMM maps: tiled weights as 128-byte rows, token rows (box 32),
+    // scale images as 512-byte rows (weights: box 1 per CTA; tokens: box 2 = 256 rows)
     {
-      const char *ev = getenv("MOE_PAIR");
-      L->pair = ev && ev[0] == '1';
       const int64_t es = f8 ? 1 : 2;
       ok = ok && make_rows_map(&L->tmap_w13, L->w13, false, (int64_t)E * 2 * F * H * es / 128, 128, 128) &&
-           make_rows_map(&L->tmap_w2, L->w2, false, (int64_t)E * H * F * es / 128, 128, 128);
-      if (Fs)
+           make_rows_map(&L->tmap_w2, L->w2, false, (int64_t)E * H * F * es / 128, 128, 128) &&
+           make_kmajor_map(&L->xmap_xperm, L->xperm, f8, L->R_max, H, 32) &&
+           make_kmajor_map(&L->xmap_h, L->hbuf, f8, L->R_max, F, 32);
+      if (Fs) {
         ok = ok && make_rows_map(&L->tmap_ws13, L->ws13, false, (int64_t)2 * Fs * H * es / 128, 128, 128) &&
-             make_rows_map(&L->tmap_ws2, L->ws2, false, (int64_t)H * Fs * es / 128, 128, 128);
+             make_rows_map(&L->tmap_ws2, L->ws2, false, (int64_t)H * Fs * es / 128, 128, 128) &&
+             make_kmajor_map(&L->xmap_hsh, L->hsh, f8, Tm, Fs, 32);
+        if (f8) ok = ok && make_kmajor_map(&L->xmap_xq, L->xq, true, Tm, H, 32);
+      }
       if (f8) {
         const int64_t g1 = (H / 128 + 3) / 4, g2 = (F / 128 + 3) / 4, gs = (Fs / 128 + 3) / 4;
-        ok = ok && make_rows_map(&L->smap_w13, L->w13_img, true, E * g1 * (2 * F / 128), 128, 2) &&
-             make_rows_map(&L->smap_w2, L->w2_img, true, E * g2 * (H / 128), 128, 2) &&
-             make_rows_map(&L->smap_xperm, L->xperm_img, true, g1 * L->max_tiles, 128, 1) &&
-             make_rows_map(&L->smap_h, L->h_img, true, g2 * L->max_tiles, 128, 1) &&
-             make_rows_map(&L->smap_xq, L->xq_img, true, g1 * L->img_tiles_sh, 128, 1);
+        ok = ok && make_rows_map(&L->smap_w13, L->w13_img, true, E * g1 * (F / 128), 128, 1) &&
+             make_rows_map(&L->smap_w2, L->w2_img, true, E * g2 * (H / 128), 128, 1) &&
+             make_rows_map(&L->smap_xperm, L->xperm_img, true, g1 * L->max_tiles, 128, 2) &&
+             make_rows_map(&L->smap_h, L->h_img, true, g2 * L->max_tiles, 128, 2) &&
+             make_rows_map(&L->smap_xq, L->xq_img, true, g1 * L->img_tiles_sh, 128, 2);
         if (Fs)
-          ok = ok && make_rows_map(&L->smap_ws13, L->ws13_img, true, g1 * (2 * Fs / 128), 128, 2) &&
-               make_rows_map(&L->smap_ws2, L->ws2_img, true, gs * (H / 128), 128, 2) &&
-               make_rows_map(&L->smap_hsh, L->hsh_img, true, gs * L->img_tiles_sh, 128, 1);
+          ok = ok && make_rows_map(&L->smap_ws13, L->ws13_img, true, g1 * (Fs / 128), 128, 1) &&
+               make_rows_map(&L->smap_ws2, L->ws2_img, true, gs * (H / 128), 128, 1) &&
+               make_rows_map(&L->smap_hsh, L->hsh_img, true, gs * L->img_tiles_sh, 128, 2);
       }
     }
     if (!ok) return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable?)"));
@@ -456,75 +495,53 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
   const float *xa_s = L->fp8 ? L->xs : nullptr;
   const int btype = L->fp8 ? WT_FP8 : (L->f32w ? WT_F32 : WT_BF16);
   if (L->umma) {
-    // 5+6. routed experts and the shared expert in one persistent tcgen05 launch per GEMM
+    // 5+6. routed experts and the shared expert in one persistent swap-AB CTA-pair
+    // tcgen05 launch per GEMM (umma_swap.cu)
     const bool f8 = L->fp8;
     const int kdiv = f8 ? 128 : 64;
-    UmmaParams p1{};
+    static const int dbg_mode = getenv("MOE_DEBUG_GEMM") ? atoi(getenv("MOE_DEBUG_GEMM")) : 0;
+    SwapParams p1{};
     {
-      UmmaGroup &g = p1.g[0];
-      g.a_map = L->map_xperm; g.b_tiles = (const uint8_t *)L->w13; g.b_ntiles_n = 2 * F / 256;
-      g.sfa = L->xperm_img; g.sfb = L->w13_img; g.sfb_expert_stride = L->w13_img_stride;
-      g.sfa_tile_stride = L->max_tiles; g.sfb_rb = 2 * F / 128; g.n_total = 2 * F; g.kblocks = H / kdiv;
+      SwapGroup &g = p1.g[0];
+      g.w_map = L->tmap_w13; g.x_map = L->xmap_xperm; g.sfw_map = L->smap_w13; g.sfx_map = L->smap_xperm;
+      g.w_nblk = F / 128; g.kblocks = H / kdiv; g.sfw_per_cta = 0; g.sfx_tile_stride = L->max_tiles;
       g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
     }
     if (Fs > 0) {
-      UmmaGroup &g = p1.g[1];
+      SwapGroup &g = p1.g[1];
+      g.w_map = L->tmap_ws13; g.sfw_map = L->smap_ws13; g.sfx_map = L->smap_xq;
       if (f8) {
-        g.a_map = L->map_xq;
-      } else if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) {
+        g.x_map = L->xmap_xq;
+      } else if (!make_kmajor_map(&g.x_map, x, false, T, H, 32)) {
         return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
       }
-      g.b_tiles = (const uint8_t *)L->ws13; g.b_ntiles_n = 2 * Fs / 256;
-      g.sfa = L->xq_img; g.sfb = L->ws13_img; g.sfa_tile_stride = L->img_tiles_sh;
-      g.sfb_rb = 2 * Fs / 128; g.n_total = 2 * Fs; g.kblocks = H / kdiv;
+      g.w_nblk = Fs / 128; g.kblocks = H / kdiv; g.sfw_per_cta = 0; g.sfx_tile_stride = L->img_tiles_sh;
       g.out = L->hsh; g.ldc = Fs; g.out_sf = L->hsh_img; g.out_sf_tile_stride = L->img_tiles_sh;
     } else {
       p1.g[1] = p1.g[0];
     }
-    p1.tiles = L->tiles; p1.n_tiles = L->n_tiles; p1.nb_r = 2 * F / 256;
-    p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = 2 * Fs / 256; p1.sched = L->sched;
-    static const int dbg_mode = getenv("MOE_DEBUG_GEMM") ? atoi(getenv("MOE_DEBUG_GEMM")) : 0;
-    p1.debug_mode = dbg_mode;
-    if (L->pair) {
-      // CTA pairs: weights via the tiled-row maps, scale images via 512-byte-row maps
-      p1.g[0].b_map = L->tmap_w13; p1.g[0].sfa_map = L->smap_xperm; p1.g[0].sfb_map = L->smap_w13;
-      if (Fs > 0) { p1.g[1].b_map = L->tmap_ws13; p1.g[1].sfa_map = L->smap_xq; p1.g[1].sfb_map = L->smap_ws13; }
-      else p1.g[1] = p1.g[0];
-      p1.pairs = L->pairs; p1.n_pairs = L->n_pairs;
-      CUDA_TRY(launch_umma_pair_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
-    } else {
-      CUDA_TRY(launch_umma_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
-    }
+    p1.tiles = L->pairs; p1.n_tiles = L->n_pairs; p1.nb_r = F / 128;
+    p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = Fs / 128; p1.sched = L->sched; p1.debug_mode = dbg_mode;
+    CUDA_TRY(launch_umma_swap_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
     mark(L, ST_GEMM1, st);
-    UmmaParams p2{};
+    SwapParams p2{};
     {
-      UmmaGroup &g = p2.g[0];
-      g.a_map = L->map_h; g.b_tiles = (const uint8_t *)L->w2; g.b_ntiles_n = H / 256;
-      g.sfa = L->h_img; g.sfb = L->w2_img; g.sfb_expert_stride = L->w2_img_stride;
-      g.sfa_tile_stride = L->max_tiles; g.sfb_rb = H / 128; g.n_total = H; g.kblocks = F / kdiv;
+      SwapGroup &g = p2.g[0];
+      g.w_map = L->tmap_w2; g.x_map = L->xmap_h; g.sfw_map = L->smap_w2; g.sfx_map = L->smap_h;
+      g.w_nblk = H / 256; g.kblocks = F / kdiv; g.sfw_per_cta = 1; g.sfx_tile_stride = L->max_tiles;
       g.out = L->yperm; g.ldc = H;
     }
     if (Fs > 0) {
-      UmmaGroup &g = p2.g[1];
-      g.a_map = L->map_hsh; g.b_tiles = (const uint8_t *)L->ws2; g.b_ntiles_n = H / 256;
-      g.sfa = L->hsh_img; g.sfb = L->ws2_img; g.sfa_tile_stride = L->img_tiles_sh;
-      g.sfb_rb = H / 128; g.n_total = H; g.kblocks = Fs / kdiv;
+      SwapGroup &g = p2.g[1];
+      g.w_map = L->tmap_ws2; g.x_map = L->xmap_hsh; g.sfw_map = L->smap_ws2; g.sfx_map = L->smap_hsh;
+      g.w_nblk = H / 256; g.kblocks = Fs / kdiv; g.sfw_per_cta = 1; g.sfx_tile_stride = L->img_tiles_sh;
       g.out = L->ysh; g.ldc = H;
     } else {
       p2.g[1] = p2.g[0];
     }
-    p2.tiles = L->tiles; p2.n_tiles = L->n_tiles; p2.nb_r = H / 256;
-    p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256; p2.sched = L->sched + 1;
-    p2.debug_mode = dbg_mode;
-    if (L->pair) {
-      p2.g[0].b_map = L->tmap_w2; p2.g[0].sfa_map = L->smap_h; p2.g[0].sfb_map = L->smap_w2;
-      if (Fs > 0) { p2.g[1].b_map = L->tmap_ws2; p2.g[1].sfa_map = L->smap_hsh; p2.g[1].sfb_map = L->smap_ws2; }
-      else p2.g[1] = p2.g[0];
-      p2.pairs = L->pairs; p2.n_pairs = L->n_pairs;
-      CUDA_TRY(launch_umma_pair_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
-    } else {
-      CUDA_TRY(launch_umma_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
-    }
+    p2.tiles = L->pairs; p2.n_tiles = L->n_pairs; p2.nb_r = H / 256;
+    p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256; p2.sched = L->sched + 1; p2.debug_mode = dbg_mode;
+    CUDA_TRY(launch_umma_swap_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
     mark(L, ST_GEMM2, st);
   } else {
     // 5. routed experts: GEMM1 + SwiGLU, GEMM2 (CUDA-core path: F32 weights, H % 256 != 0)
@@ -818,7 +835,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
       UmmaGroup &g = d1.g[0];
       g.a_map = L->dmap_xperm; g.b_tiles = (const uint8_t *)L->w13; g.b_ntiles_n = 2 * F / 256;
       g.sfa = L->xperm_img; g.sfa_tile_stride = L->max_tiles;
-      g.sfb = L->w13_img; g.sfb_expert_stride = L->w13_img_stride; g.sfb_rb = 2 * F / 128;
+      g.sfb = L->w13_img; g.sfb_expert_stride = L->w13_img_stride; g.sfb_rb = F / 128;
       g.n_total = 2 * F; g.kblocks = H / kdiv;
       g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
     }
@@ -831,7 +848,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
       }
       g.b_tiles = (const uint8_t *)L->ws13; g.b_ntiles_n = 2 * Fs / 256;
       g.sfa = L->xq_img; g.sfa_tile_stride = L->img_tiles_sh;
-      g.sfb = L->ws13_img; g.sfb_rb = 2 * Fs / 128; g.n_total = 0; g.kblocks = H / kdiv;
+      g.sfb = L->ws13_img; g.sfb_rb = Fs / 128; g.n_total = 0; g.kblocks = H / kdiv;
       g.out = L->hsh; g.ldc = Fs; g.out_sf = L->hsh_img; g.out_sf_tile_stride = L->img_tiles_sh;
     } else {
       d1.g[1] = d1.g[0];

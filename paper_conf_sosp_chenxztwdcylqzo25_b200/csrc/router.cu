@@ -235,16 +235,54 @@ __device__ void select_token_block(const RouterArgs &args, int t, float *s, floa
     }
     __syncthreads();
   }
-  // expert rank among the allowed ones; the k best land in ids/ws by rank
+  // top-k in two warp-level rounds (short loops: this tail runs once, on one SM,
+  // with a cold instruction cache): (1) every warp extracts the k best of its
+  // <= 128 experts by k arg-max rounds; (2) warp 0 merges the NT/32 candidate
+  // lists the same way.  Masked (-inf) experts never qualify.
+  {
+    __shared__ float cv[NT / 32][32];
+    __shared__ int ci[NT / 32][32];
+    const int lane = tid & 31, w = tid >> 5;
+    float v[4];
+    int id[4];
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int e = tid + NT * i;
-    if (e < E && sel[e] != -INFINITY) {
-      const float v = sel[e];
-      int rk = 0;
-#pragma unroll 4
-      for (int j = 0; j < E; ++j) rk += better(sel[j], j, v, e);
-      if (rk < k) { ids[rk] = e; ws[rk] = s[e]; }
+    for (int i = 0; i < 4; ++i) {
+      const int e = tid + NT * i;
+      const float x = e < E ? sel[e] : -INFINITY;
+      v[i] = x; id[i] = x == -INFINITY ? 0x7fffffff : e;
+    }
+#pragma unroll 1
+    for (int r = 0; r < k; ++r) {
+      float bv = v[0]; int bi = id[0];
+#pragma unroll
+      for (int i = 1; i < 4; ++i) if (better(v[i], id[i], bv, bi)) { bv = v[i]; bi = id[i]; }
+      warp_argmax(bv, bi);
+      if (lane == 0) { cv[w][r] = bv; ci[w][r] = bi; }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) if (id[i] == bi) { v[i] = -INFINITY; id[i] = 0x7fffffff; }
+    }
+    __syncthreads();
+    if (w == 0) {
+      // candidates: NT/32 lists of k <= 32 -> <= NT/32 per lane
+      constexpr int NC = NT / 32;
+      float mv[NC]; int mi[NC];
+#pragma unroll
+      for (int i = 0; i < NC; ++i) {
+        const int c = lane + 32 * i;              // candidate index = list * k + rank
+        const bool ok = c < (NT / 32) * k;
+        mv[i] = ok ? cv[c / k][c % k] : -INFINITY;
+        mi[i] = ok ? ci[c / k][c % k] : 0x7fffffff;
+      }
+#pragma unroll 1
+      for (int r = 0; r < k; ++r) {
+        float bv = mv[0]; int bi = mi[0];
+#pragma unroll
+        for (int i = 1; i < NC; ++i) if (better(mv[i], mi[i], bv, bi)) { bv = mv[i]; bi = mi[i]; }
+        warp_argmax(bv, bi);
+        if (lane == 0) { ids[r] = bi; ws[r] = s[bi]; }
+#pragma unroll
+        for (int i = 0; i < NC; ++i) if (mi[i] == bi) { mv[i] = -INFINITY; mi[i] = 0x7fffffff; }
+      }
     }
   }
   __syncthreads();
@@ -382,6 +420,14 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
     int *ids = reinterpret_cast<int *>(ws + 32);
 #pragma unroll 1
     for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws);
+    if (a.debug & 8) {                           // MOE_DEBUG_ROUTE=12: time a second (warm i-cache) pass
+      __syncthreads();
+      const long long w0 = clock64();
+#pragma unroll 1
+      for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws);
+      __syncthreads();
+      if (threadIdx.x == 0) printf("route tail: warm select pass %lld cycles\n", clock64() - w0);
+    }
   }
   long long ck1 = clock64();
   {

@@ -7,9 +7,11 @@
 // tensor cores do the dot products and the kernel is a pure weight stream.
 // (The paper's AVX-512 low-ARI kernel, L170, recast for B200: same memory
 // layout as the prefill GEMM, a different instruction shape.)
-//   MODE 1: unit = (slot, 128 h columns): gate rows [256b, +128) and up rows
-//           [256b+128, +128) of W13 -> two 128x16 accumulators -> SwiGLU ->
-//           h (FP8: 1x128 UE8M0 requant from fp32 + scale image)
+//   MODE 1: unit = (slot, 128 h columns b): the 256-row W13 tile b, whose
+//           128-row halves c hold per lane quadrant [gate | up | gate | up] of
+//           h columns 128b + 64c + [0, 64) -> two 128x16 accumulators; the up
+//           quadrants hand their values to the gate quadrants through shared
+//           memory -> SwiGLU -> h (FP8: 1x128 UE8M0 requant from fp32 + image)
 //   MODE 2: unit = (slot, 128 rows of W2) -> y rows (bf16)
 // Slots: active routed experts (act_list) + the shared expert (last slot).
 #include <cuda.h>
@@ -24,8 +26,10 @@ using namespace sm100;
 constexpr int UD_N = 16, UD_STAGES = 6, UD_THREADS = 192;
 constexpr int UD_A_BYTES = 2 * 128 * 128;     // up to two 128-row weight tiles
 constexpr int UD_B_BYTES = UD_N * 128;        // 16 token rows x 128 B
-constexpr int UD_SFA_BYTES = 1024, UD_SFB_BYTES = 512;
-constexpr size_t UD_SMEM = 1024 + (size_t)UD_STAGES * (UD_A_BYTES + UD_B_BYTES + UD_SFA_BYTES + UD_SFB_BYTES) + 1024;
+constexpr int UD_SFA_BYTES = 512, UD_SFB_BYTES = 512;
+constexpr int UD_XCH_FLOATS = 2 * 2 * UD_N * 32;   // up -> gate exchange [gate warp][acc][token][lane]
+constexpr size_t UD_SMEM = 1024 + (size_t)UD_STAGES * (UD_A_BYTES + UD_B_BYTES + UD_SFA_BYTES + UD_SFB_BYTES) +
+                           UD_XCH_FLOATS * 4 + 1024;
 constexpr uint32_t UD_TMEM_COLS = 128;        // 2 acc stages x 32 cols + scale factors
 constexpr uint32_t UD_SFA_COL = 64, UD_SFB_COL = 72;
 
@@ -69,6 +73,7 @@ __global__ void __launch_bounds__(UD_THREADS, 1) umma_decode_kernel(const __grid
   uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(uq_empty + 4);
   int *unit_q = reinterpret_cast<int *>(tmem_base_smem + 4);
   float *red = reinterpret_cast<float *>(unit_q + 4);   // [4 warps][16 tokens]
+  float *xch = red + 4 * UD_N;                           // MODE 1 up -> gate exchange
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   constexpr int NA = MODE == 1 ? 2 : 1;         // weight tiles per unit
@@ -100,7 +105,7 @@ __global__ void __launch_bounds__(UD_THREADS, 1) umma_decode_kernel(const __grid
         if (++qs == 4) { qs = 0; qph ^= 1; }
         if (!ui.valid) break;
         const UmmaGroup &g = p.g[ui.shared];
-        const uint32_t bytes = NA * 128 * 128 + UD_B_BYTES + (FP8 ? NA * 512 + UD_SFB_BYTES : 0);
+        const uint32_t bytes = NA * 128 * 128 + UD_B_BYTES + (FP8 ? UD_SFA_BYTES + UD_SFB_BYTES : 0);
         for (int kb = 0; kb < g.kblocks; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           mbar_expect_tx(&full[stage], bytes);
@@ -113,10 +118,11 @@ __global__ void __launch_bounds__(UD_THREADS, 1) umma_decode_kernel(const __grid
           bulk_load(sA + stage * UD_A_BYTES, wt, NA * 128 * 128, &full[stage]);
           tma_load_2d(sB + stage * UD_B_BYTES, &g.a_map, &full[stage], kc, ui.row0);
           if (FP8) {
+            // MODE 1: one W13 image per 256-row tile (both halves); MODE 2: per 128-row block
             const uint8_t *sfa = g.sfb + (size_t)ui.expert * g.sfb_expert_stride +
-                                 ((size_t)(kb >> 2) * g.sfb_rb + (MODE == 1 ? ui.blk * 2 : ui.blk)) * 512;
+                                 ((size_t)(kb >> 2) * g.sfb_rb + ui.blk) * 512;
             const uint8_t *sfb = g.sfa + ((size_t)(kb >> 2) * g.sfa_tile_stride + (ui.row0 >> 7)) * 512;
-            bulk_load(sSFA + stage * UD_SFA_BYTES, sfa, NA * 512, &full[stage]);
+            bulk_load(sSFA + stage * UD_SFA_BYTES, sfa, UD_SFA_BYTES, &full[stage]);
             bulk_load(sSFB + stage * UD_SFB_BYTES, sfb, UD_SFB_BYTES, &full[stage]);
           }
           if (++stage == UD_STAGES) { stage = 0; phase ^= 1; }
@@ -147,7 +153,6 @@ __global__ void __launch_bounds__(UD_THREADS, 1) umma_decode_kernel(const __grid
           const uint32_t b0 = smem_u32(sB + stage * UD_B_BYTES);
           if (FP8) {
             tmem_cp_32x128b_x4(tmem + UD_SFA_COL, sf_desc(smem_u32(sSFA + stage * UD_SFA_BYTES)));
-            if (NA == 2) tmem_cp_32x128b_x4(tmem + UD_SFA_COL + 4, sf_desc(smem_u32(sSFA + stage * UD_SFA_BYTES + 512)));
             tmem_cp_32x128b_x4(tmem + UD_SFB_COL, sf_desc(smem_u32(sSFB + stage * UD_SFB_BYTES)));
           }
 #pragma unroll
@@ -159,7 +164,7 @@ __global__ void __launch_bounds__(UD_THREADS, 1) umma_decode_kernel(const __grid
               const uint64_t ad = sw128_kmajor_desc(a0 + t * 128 * 128 + k * 32);
               if (FP8)
                 mma_mxf8(d0 + t * 16, ad, bd, idesc_mxf8(128, UD_N, kb & 3, kb & 3), accum,
-                         tmem + UD_SFA_COL + t * 4, tmem + UD_SFB_COL);
+                         tmem + UD_SFA_COL, tmem + UD_SFB_COL);
               else
                 mma_bf16(d0 + t * 16, ad, bd, idesc_bf16(128, UD_N), accum);
             }
@@ -198,35 +203,61 @@ __global__ void __launch_bounds__(UD_THREADS, 1) umma_decode_kernel(const __grid
       const int n = ui.n;
       const int wr = q * 32 + lane;             // weight row within the 128-row tile
       if (MODE == 1) {
-        float h[UD_N];
-#pragma unroll
-        for (int t = 0; t < UD_N; ++t) h[t] = silu_f(__uint_as_float(r0[t])) * __uint_as_float(r1[t]);
-        const int f = ui.blk * 128 + wr;
-        if (FP8) {
-          // per token: amax over the 128 h values of this block (4 warps)
+        // quadrant q of accumulator c: gate (q even) / up (q odd) rows of h
+        // column 128 blk + 64 c + 32 (q >> 1) + lane
+        const int qg = q >> 1;
+        float *xb = xch + qg * (2 * UD_N * 32);
+        if (q & 1) {
 #pragma unroll
           for (int t = 0; t < UD_N; ++t) {
-            const float m = warp_max(fabsf(h[t]));
-            if (lane == 0) red[q * UD_N + t] = m;
+            xb[t * 32 + lane] = __uint_as_float(r0[t]);
+            xb[(UD_N + t) * 32 + lane] = __uint_as_float(r1[t]);
           }
-          asm volatile("bar.sync 1, 128;" ::: "memory");
+        }
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+        float h0[UD_N], h1[UD_N];
+        if (!(q & 1)) {
 #pragma unroll
           for (int t = 0; t < UD_N; ++t) {
-            if (t < n) {
-              const float am = fmaxf(fmaxf(red[t], red[UD_N + t]), fmaxf(red[2 * UD_N + t], red[3 * UD_N + t]));
-              const int e = ue8m0_exponent(am);
-              const int64_t row = (int64_t)ui.row0 + t;
-              reinterpret_cast<uint8_t *>(g.out)[row * g.ldc + f] = f32_to_e4m3(h[t] * exp2i(-e));
-              if (wr == 0) g.out_sf[sf_img_off(row, ui.blk, g.out_sf_tile_stride)] = (uint8_t)(e + 127);
+            h0[t] = silu_f(__uint_as_float(r0[t])) * xb[t * 32 + lane];
+            h1[t] = silu_f(__uint_as_float(r1[t])) * xb[(UD_N + t) * 32 + lane];
+          }
+        }
+        const int f0 = ui.blk * 128 + qg * 32 + lane;       // accumulator 0; accumulator 1 at + 64
+        if (FP8) {
+          // per token: amax over the 128 h values of this block (2 gate warps x 2 accumulators)
+          if (!(q & 1)) {
+#pragma unroll
+            for (int t = 0; t < UD_N; ++t) {
+              const float m = warp_max(fmaxf(fabsf(h0[t]), fabsf(h1[t])));
+              if (lane == 0) red[qg * UD_N + t] = m;
             }
           }
           asm volatile("bar.sync 1, 128;" ::: "memory");
-        } else {
+          if (!(q & 1)) {
+#pragma unroll
+            for (int t = 0; t < UD_N; ++t) {
+              if (t < n) {
+                const int e = ue8m0_exponent(fmaxf(red[t], red[UD_N + t]));
+                const float inv = exp2i(-e);
+                const int64_t row = (int64_t)ui.row0 + t;
+                uint8_t *o = reinterpret_cast<uint8_t *>(g.out) + row * g.ldc;
+                o[f0] = f32_to_e4m3(h0[t] * inv);
+                o[f0 + 64] = f32_to_e4m3(h1[t] * inv);
+                if (qg == 0 && lane == 0) g.out_sf[sf_img_off(row, ui.blk, g.out_sf_tile_stride)] = (uint8_t)(e + 127);
+              }
+            }
+          }
+        } else if (!(q & 1)) {
 #pragma unroll
           for (int t = 0; t < UD_N; ++t)
-            if (t < n)
-              reinterpret_cast<__nv_bfloat16 *>(g.out)[((int64_t)ui.row0 + t) * g.ldc + f] = __float2bfloat16_rn(h[t]);
+            if (t < n) {
+              __nv_bfloat16 *o = reinterpret_cast<__nv_bfloat16 *>(g.out) + ((int64_t)ui.row0 + t) * g.ldc;
+              o[f0] = __float2bfloat16_rn(h0[t]);
+              o[f0 + 64] = __float2bfloat16_rn(h1[t]);
+            }
         }
+        asm volatile("bar.sync 1, 128;" ::: "memory");   // exchange / red buffers free for the next unit
       } else {
         const int c = ui.blk * 128 + wr;
 #pragma unroll

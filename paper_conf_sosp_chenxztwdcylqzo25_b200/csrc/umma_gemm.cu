@@ -114,8 +114,18 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
         if (!ui.valid) break;
         const UmmaGroup &g = p.g[ui.group];
         const int brow = ui.expert * g.n_total + ui.nb * UG_BN;
+        const uint8_t *btiles = g.b_tiles + ((size_t)ui.expert * g.b_ntiles_n + ui.nb) * g.kblocks * UG_B_BYTES;
+        if (EPI != GEMM_LOGITS)
+          for (int kb = 0; kb < p.pf_dist && kb < g.kblocks; ++kb) bulk_prefetch_l2(btiles + (size_t)kb * UG_B_BYTES, UG_B_BYTES);
         for (int kb = 0; kb < g.kblocks; ++kb) {
+          if (EPI != GEMM_LOGITS && p.pf_dist > 0 && kb + p.pf_dist < g.kblocks)
+            bulk_prefetch_l2(btiles + (size_t)(kb + p.pf_dist) * UG_B_BYTES, UG_B_BYTES);
           mbar_wait(&empty[stage], phase ^ 1);
+          if (p.debug_mode == 3 || p.debug_mode == 4) {   // timing experiment: MMAs on stale smem, no loads
+            mbar_arrive(&full[stage]);
+            if (++stage == UG_STAGES) { stage = 0; phase ^= 1; }
+            continue;
+          }
           uint32_t bytes = UG_A_BYTES + UG_B_BYTES;
           if (FP8) bytes += UG_SFA_BYTES + UG_SFB_BYTES;
           mbar_expect_tx(&full[stage], bytes);
@@ -160,10 +170,16 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
         if (lane == 0 && p.debug_mode != 1) {
           const uint32_t a0 = smem_u32(sA + stage * UG_A_BYTES);
           const uint32_t b0 = smem_u32(sB + stage * UG_B_BYTES);
-          if (FP8) {
-            tmem_cp_32x128b_x4(tmem + UG_SFA_COL, sf_desc(smem_u32(sSFA + stage * UG_SFA_BYTES)));
-            tmem_cp_32x128b_x4(tmem + UG_SFB_COL, sf_desc(smem_u32(sSFB + stage * UG_SFB_BYTES)));
-            tmem_cp_32x128b_x4(tmem + UG_SFB_COL + 4, sf_desc(smem_u32(sSFB + stage * UG_SFB_BYTES + 512)));
+          // a scale image holds 4 k-blocks (one UE8M0 byte each, selected by the
+          // instruction descriptor's sf id): copy it to TMEM once per 4 k-blocks,
+          // alternating between two column sets so the copy never targets
+          // columns the previous group's MMAs still read
+          const uint32_t sf_set = FP8 ? ((kb >> 2) & 1) * 16 : 0;
+          const bool do_cp = FP8 && p.debug_mode != 4 && p.debug_mode != 6 && ((kb & 3) == 0 || p.debug_mode == 7);
+          if (do_cp) {
+            tmem_cp_32x128b_x4(tmem + UG_SFA_COL + sf_set, sf_desc(smem_u32(sSFA + stage * UG_SFA_BYTES)));
+            tmem_cp_32x128b_x4(tmem + UG_SFB_COL + sf_set, sf_desc(smem_u32(sSFB + stage * UG_SFB_BYTES)));
+            tmem_cp_32x128b_x4(tmem + UG_SFB_COL + sf_set + 4, sf_desc(smem_u32(sSFB + stage * UG_SFB_BYTES + 512)));
           }
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
@@ -171,8 +187,8 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
             const uint64_t bd = sw128_kmajor_desc(b0 + k * 32);
             const uint32_t acc = (kb | k) != 0;
             if (FP8)
-              mma_mxf8(tmem, ad, bd, idesc_mxf8(UG_BM, UG_BN, kb & 3, kb & 3), acc, tmem + UG_SFA_COL,
-                       tmem + UG_SFB_COL);
+              mma_mxf8(tmem, ad, bd, idesc_mxf8(UG_BM, UG_BN, kb & 3, kb & 3), acc, tmem + UG_SFA_COL + sf_set,
+                       tmem + UG_SFB_COL + sf_set);
             else
               mma_bf16(tmem, ad, bd, idesc_bf16(UG_BM, UG_BN), acc);
           }
@@ -212,7 +228,7 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
       tc_fence_after();
       const int row = ui.row0 + q * 32 + lane;
       const bool live = row < ui.row_end;
-      if (p.debug_mode >= 1) {            // debug: no epilogue work
+      if (p.debug_mode >= 1 && p.debug_mode <= 5) {   // debug: no epilogue work
         tc_fence_before();
         __syncwarp();
         if (lane == 0) mbar_arrive(tmem_empty);
@@ -331,9 +347,8 @@ static cudaError_t launch_one(const UmmaParams &p, int grid, cudaStream_t st) {
 
 cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st) {
   if (grid <= 0) return cudaSuccess;
-  if (epi == GEMM_LOGITS) return launch_one<false, GEMM_LOGITS>(p, grid, st);
-  if (fp8) return epi == GEMM_SWIGLU ? launch_one<true, GEMM_SWIGLU>(p, grid, st) : launch_one<true, GEMM_PLAIN>(p, grid, st);
-  return epi == GEMM_SWIGLU ? launch_one<false, GEMM_SWIGLU>(p, grid, st) : launch_one<false, GEMM_PLAIN>(p, grid, st);
+  if (epi == GEMM_LOGITS && !fp8) return launch_one<false, GEMM_LOGITS>(p, grid, st);
+  return cudaErrorInvalidValue;   // expert GEMMs run in umma_swap.cu
 }
 
 // ------------------------------------------------------------------ weight tiling
@@ -353,9 +368,12 @@ __global__ void tile_weights_kernel(const uint8_t *__restrict__ src, uint8_t *__
     const int jsrc = j ^ (r & 7);                    // chunk j of row r holds source chunk j ^ (r % 8)
     int srow;
     if (interleave_f > 0) {
-      const int rr = nb * 256 + r;                   // interleaved row
-      const int b = rr >> 8, w = rr & 255;
-      srow = w < 128 ? b * 128 + w : interleave_f + b * 128 + (w - 128);
+      // W13 tile nb = h block nb (128 h columns); 128-row half c holds, per
+      // 32-row lane quadrant q, [gate | up | gate | up] of columns
+      // 128 nb + 64 c + 32 (q >> 1) + i  (umma_swap.cu / umma_decode.cu epilogues)
+      const int c = r >> 7, q = (r >> 5) & 3, i = r & 31;
+      const int f = nb * 128 + c * 64 + (q >> 1) * 32 + i;
+      srow = (q & 1) ? interleave_f + f : f;
     } else {
       srow = nb * 256 + r;
     }
