@@ -29,7 +29,7 @@ cudaError_t launch_scatter_rows(const void *x, int T, int H, int k, const int32_
 // y[t]   = residual[t] + g_t * ys[t] + sum_{j < n_imm} w_tj * yperm[pos(t,j)] + deferred_in[t]
 // dout[t] = sum_{j >= n_imm} w_tj * yperm[pos(t,j)]
 // (PAPER.md L219 / L241; fp32 accumulation, one CTA per token, 8 channels per thread)
-__global__ void __launch_bounds__(128) combine_kernel(CombineArgs a) {
+__global__ void __launch_bounds__(128) combine_kernel(const __grid_constant__ CombineArgs a) {
   const int t = blockIdx.x;
   pdl_wait();
   __shared__ int32_t spos[32];

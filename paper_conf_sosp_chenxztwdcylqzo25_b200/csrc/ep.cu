@@ -75,7 +75,7 @@ __global__ void __launch_bounds__(128) ep_pack_kernel(const __nv_bfloat16 *__res
 // ------------------------------------------------------------------ final combine
 // y[t] = residual + g_t * ys[t] + sum_d back[d][sendpos[t][d]] + deferred_in;
 // deferred_out[t] = sum_d back_def[d][sendpos[t][d]]   (fp32 accumulation)
-__global__ void __launch_bounds__(128) ep_final_combine_kernel(EpCombineArgs a) {
+__global__ void __launch_bounds__(128) ep_final_combine_kernel(const __grid_constant__ EpCombineArgs a) {
   const int t = blockIdx.x;
   const int v = blockIdx.y * blockDim.x + threadIdx.x;
   if (v >= a.H / 8) return;

@@ -52,7 +52,7 @@ __device__ __forceinline__ GvSlot gv_slot(const GemvArgs &a) {
 // CTA = (slot, 256-row block of the interleaved W13 = 128 gate + 128 up rows)
 // -> 128 h values per token.  FP8: h quantised per token over those 128 values.
 template <bool FP8, int NT>
-__global__ void __launch_bounds__(GV_THREADS) gemv13_kernel(GemvArgs a) {
+__global__ void __launch_bounds__(GV_THREADS) gemv13_kernel(const __grid_constant__ GemvArgs a) {
   extern __shared__ __align__(16) uint8_t gsm[];
   const GvSlot s = gv_slot(a);
   if (!s.valid) return;
@@ -181,7 +181,7 @@ __global__ void __launch_bounds__(GV_THREADS) gemv13_kernel(GemvArgs a) {
 // ------------------------------------------------------------------ GEMV2: W2
 // CTA = (slot, 128-row block of W2) -> 128 output channels per token.
 template <bool FP8, int NT>
-__global__ void __launch_bounds__(GV_THREADS) gemv2_kernel(GemvArgs a) {
+__global__ void __launch_bounds__(GV_THREADS) gemv2_kernel(const __grid_constant__ GemvArgs a) {
   extern __shared__ __align__(16) uint8_t gsm[];
   const GvSlot s = gv_slot(a);
   if (!s.valid) return;

@@ -97,6 +97,9 @@ struct RouteSmallArgs {
   int fp8;
   void *xperm; uint8_t *xperm_img; int xperm_img_stride;
   void *xq; float *xs; uint8_t *xq_img; int xq_img_stride;   // shared expert (FP8)
+  // shared-expert weights prefetched into L2 while the router runs (they do
+  // not depend on the routing): [pf[i], pf[i] + pf_bytes[i]), i < 2
+  const void *pf[2]; int64_t pf_bytes[2];
 };
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st);
 
@@ -216,11 +219,13 @@ cudaError_t launch_umma_decode(bool fp8, int mode, const UmmaDecodeParams &p, in
 
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);
 bool make_rows_map(CUtensorMap *m, const void *base, bool u32, int64_t rows, int row_elems, int box_rows);
+bool make_blocks_map(CUtensorMap *m, const void *base, int64_t total_bytes, int row_bytes, int box_rows);
 // prefill grouped expert GEMM, swap-AB on CTA pairs (umma_swap.cu): weights are
 // the M = 256 operand, an expert's tokens (<= 256, padded to 16) the N operand
 struct SwapGroup {              // one operand set: 0 = routed experts, 1 = shared expert
   CUtensorMap w_map;            // tiled weights as 128-byte rows, box 128 rows
-  CUtensorMap x_map;            // token rows, K-major SW128, box 32 rows
+  CUtensorMap x_map;            // token rows, K-major SW128, box 32 rows (ragged tails)
+  CUtensorMap x_map128;         // the same, box 128 rows (full halves)
   CUtensorMap sfw_map;          // FP8: weight scale images as 512-byte rows, box 1
   CUtensorMap sfx_map;          // FP8: token scale images as 512-byte rows, box 2
   int w_nblk;                   // 256-row weight blocks per expert

@@ -440,13 +440,14 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
     // scale images as 512-byte rows (weights: box 1 per CTA; tokens: box 2 = 256 rows)
     {
       const int64_t es = f8 ? 1 : 2;
-      ok = ok && make_rows_map(&L->tmap_w13, L->w13, false, (int64_t)E * 2 * F * H * es / 128, 128, 128) &&
-           make_rows_map(&L->tmap_w2, L->w2, false, (int64_t)E * H * F * es / 128, 128, 128) &&
+      // weights: 2 KB TMA rows (a CTA's 16 KB half tile = 8 rows)
+      ok = ok && make_blocks_map(&L->tmap_w13, L->w13, (int64_t)E * 2 * F * H * es, 2048, 8) &&
+           make_blocks_map(&L->tmap_w2, L->w2, (int64_t)E * H * F * es, 2048, 8) &&
            make_kmajor_map(&L->xmap_xperm, L->xperm, f8, L->R_max, H, 32) &&
            make_kmajor_map(&L->xmap_h, L->hbuf, f8, L->R_max, F, 32);
       if (Fs) {
-        ok = ok && make_rows_map(&L->tmap_ws13, L->ws13, false, (int64_t)2 * Fs * H * es / 128, 128, 128) &&
-             make_rows_map(&L->tmap_ws2, L->ws2, false, (int64_t)H * Fs * es / 128, 128, 128) &&
+        ok = ok && make_blocks_map(&L->tmap_ws13, L->ws13, (int64_t)2 * Fs * H * es, 2048, 8) &&
+             make_blocks_map(&L->tmap_ws2, L->ws2, (int64_t)H * Fs * es, 2048, 8) &&
              make_kmajor_map(&L->xmap_hsh, L->hsh, f8, Tm, Fs, 32);
         if (f8) ok = ok && make_kmajor_map(&L->xmap_xq, L->xq, true, Tm, H, 32);
       }
@@ -503,7 +504,7 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     SwapParams p1{};
     {
       SwapGroup &g = p1.g[0];
-      g.w_map = L->tmap_w13; g.x_map = L->xmap_xperm; g.sfw_map = L->smap_w13; g.sfx_map = L->smap_xperm;
+      g.w_map = L->tmap_w13; g.x_map = L->xmap_xperm; g.x_map128 = L->map_xperm; g.sfw_map = L->smap_w13; g.sfx_map = L->smap_xperm;
       g.w_nblk = F / 128; g.kblocks = H / kdiv; g.sfw_per_cta = 0; g.sfx_tile_stride = L->max_tiles;
       g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
     }
@@ -511,8 +512,8 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
       SwapGroup &g = p1.g[1];
       g.w_map = L->tmap_ws13; g.sfw_map = L->smap_ws13; g.sfx_map = L->smap_xq;
       if (f8) {
-        g.x_map = L->xmap_xq;
-      } else if (!make_kmajor_map(&g.x_map, x, false, T, H, 32)) {
+        g.x_map = L->xmap_xq; g.x_map128 = L->map_xq;
+      } else if (!make_kmajor_map(&g.x_map, x, false, T, H, 32) || !make_kmajor_map(&g.x_map128, x, false, T, H, 128)) {
         return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
       }
       g.w_nblk = Fs / 128; g.kblocks = H / kdiv; g.sfw_per_cta = 0; g.sfx_tile_stride = L->img_tiles_sh;
@@ -527,13 +528,13 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     SwapParams p2{};
     {
       SwapGroup &g = p2.g[0];
-      g.w_map = L->tmap_w2; g.x_map = L->xmap_h; g.sfw_map = L->smap_w2; g.sfx_map = L->smap_h;
+      g.w_map = L->tmap_w2; g.x_map = L->xmap_h; g.x_map128 = L->map_h; g.sfw_map = L->smap_w2; g.sfx_map = L->smap_h;
       g.w_nblk = H / 256; g.kblocks = F / kdiv; g.sfw_per_cta = 1; g.sfx_tile_stride = L->max_tiles;
       g.out = L->yperm; g.ldc = H;
     }
     if (Fs > 0) {
       SwapGroup &g = p2.g[1];
-      g.w_map = L->tmap_ws2; g.x_map = L->xmap_hsh; g.sfw_map = L->smap_ws2; g.sfx_map = L->smap_hsh;
+      g.w_map = L->tmap_ws2; g.x_map = L->xmap_hsh; g.x_map128 = L->map_hsh; g.sfw_map = L->smap_ws2; g.sfx_map = L->smap_hsh;
       g.w_nblk = H / 256; g.kblocks = Fs / kdiv; g.sfw_per_cta = 1; g.sfx_tile_stride = L->img_tiles_sh;
       g.out = L->ysh; g.ldc = H;
     } else {
@@ -783,6 +784,9 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     rs.debug = dbg_route;
     rs.fp8 = L->fp8; rs.xperm = L->xperm; rs.xperm_img = L->xperm_img; rs.xperm_img_stride = L->max_tiles;
     if (L->fp8) { rs.xq = L->xq; rs.xs = L->xs; rs.xq_img = L->xq_img; rs.xq_img_stride = L->img_tiles_sh; }
+    if (Fs > 0 && L->umma && T <= L->gemv_max_tokens) {
+      rs.pf[0] = L->ws13; rs.pf_bytes[0] = (int64_t)2 * Fs * H * (L->fp8 ? 1 : 2);
+    }
     CUDA_TRY(launch_route_small(rs, st));
     mark(L, ST_PERMUTE, st);
   } else {

@@ -16,7 +16,7 @@
 namespace moe {
 
 // (1) per-chunk histogram (order-free, smem atomics) + reset pos to -1
-__global__ void __launch_bounds__(256) chunk_count_kernel(PermuteArgs a) {
+__global__ void __launch_bounds__(256) chunk_count_kernel(const __grid_constant__ PermuteArgs a) {
   extern __shared__ int32_t hist[];
   const int c = blockIdx.x;
   for (int e = threadIdx.x; e < a.E; e += blockDim.x) hist[e] = 0;
@@ -34,7 +34,7 @@ __global__ void __launch_bounds__(256) chunk_count_kernel(PermuteArgs a) {
 
 // (2) single CTA: per-expert totals, chunk bases, padded offsets, tile list
 constexpr int SCAN_THREADS = 1024;
-__global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(PermuteArgs a, int nchunk) {
+__global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(const __grid_constant__ PermuteArgs a, int nchunk) {
   using Scan = cub::BlockScan<int, SCAN_THREADS>;
   __shared__ typename Scan::TempStorage tmp;
   __shared__ int tot[3];
@@ -86,35 +86,43 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(PermuteArgs a, int n
   }
 }
 
-// (3) per chunk, thread per expert: assign rows in token order (stable)
-__global__ void __launch_bounds__(256) assign_kernel(PermuteArgs a) {
-  extern __shared__ int32_t sidx[];
+// (3) per chunk: assign rows in token order (stable).  Each expert gets a
+// bitmask of the chunk's tokens that chose it; an entry's rank among the
+// chunk's rows of its expert is the popcount of the mask below its token.
+constexpr int kMaskWords = kChunkTokens / 32;
+__global__ void __launch_bounds__(256) assign_kernel(const __grid_constant__ PermuteArgs a) {
+  extern __shared__ uint32_t mask[];             // [E][kMaskWords]
   const int c = blockIdx.x;
   const int t0 = c * kChunkTokens;
   const int t1 = min(a.T, t0 + kChunkTokens);
   const int n = (t1 - t0) * a.k;
-  for (int p = threadIdx.x; p < n; p += blockDim.x) sidx[p] = a.topk_idx[(int64_t)t0 * a.k + p];
+  for (int i = threadIdx.x; i < a.E * kMaskWords; i += blockDim.x) mask[i] = 0;
   __syncthreads();
-  for (int e = threadIdx.x; e < a.E; e += blockDim.x) {
-    const int ge = e + a.e0;
-    const int cb = a.chunk_base[(int64_t)c * a.E + e];
-    int r = a.offs_pad[e] + cb;
-    int u = a.offs[e] + cb;
-    for (int p = 0; p < n; ++p) {
-      if (sidx[p] == ge) {
-        const int t = t0 + p / a.k;
-        a.row_token[r] = t;
-        a.pos[(int64_t)t0 * a.k + p] = r;
-        if (a.dbg_perm) a.dbg_perm[u] = t;
-        ++r; ++u;
-      }
-    }
-    // the last chunk with rows of this expert clears the segment's padding
-    if (c == gridDim.x - 1) {
+  for (int p = threadIdx.x; p < n; p += blockDim.x) {
+    const int e = a.topk_idx[(int64_t)t0 * a.k + p] - a.e0;
+    const int tl = p / a.k;
+    if (e >= 0 && e < a.E) atomicOr(&mask[e * kMaskWords + (tl >> 5)], 1u << (tl & 31));
+  }
+  __syncthreads();
+  for (int p = threadIdx.x; p < n; p += blockDim.x) {
+    const int e = a.topk_idx[(int64_t)t0 * a.k + p] - a.e0;
+    if (e < 0 || e >= a.E) continue;
+    const int tl = p / a.k;
+    const uint32_t *m = mask + e * kMaskWords;
+    int rank = __popc(m[tl >> 5] & ((1u << (tl & 31)) - 1u));
+    for (int w = 0; w < (tl >> 5); ++w) rank += __popc(m[w]);
+    const int cb = a.chunk_base[(int64_t)c * a.E + e] + rank;
+    const int r = a.offs_pad[e] + cb;
+    a.row_token[r] = t0 + tl;
+    a.pos[(int64_t)t0 * a.k + p] = r;
+    if (a.dbg_perm) a.dbg_perm[a.offs[e] + cb] = t0 + tl;
+  }
+  // the last chunk clears the padding rows of every expert segment
+  if (c == gridDim.x - 1)
+    for (int e = threadIdx.x; e < a.E; e += blockDim.x) {
       const int end = a.offs_pad[e + 1];
       for (int q = a.offs_pad[e] + a.counts[e]; q < end; ++q) a.row_token[q] = -1;
     }
-  }
 }
 
 cudaError_t launch_permute(const PermuteArgs &a, cudaStream_t st) {
@@ -122,7 +130,7 @@ cudaError_t launch_permute(const PermuteArgs &a, cudaStream_t st) {
   if (nchunk == 0) return cudaSuccess;
   chunk_count_kernel<<<nchunk, 256, a.E * sizeof(int32_t), st>>>(a);
   scan_kernel<<<1, SCAN_THREADS, 0, st>>>(a, nchunk);
-  const size_t sm = (size_t)kChunkTokens * a.k * sizeof(int32_t);
+  const size_t sm = (size_t)a.E * kMaskWords * sizeof(uint32_t);
   if (sm > 48 * 1024) {
     cudaError_t e = cudaFuncSetAttribute(assign_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;

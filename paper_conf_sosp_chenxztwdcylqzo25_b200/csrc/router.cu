@@ -143,7 +143,7 @@ __device__ void select_token(const RouterArgs &args, int t, float *s, float *sel
 }
 
 __global__ void __launch_bounds__(RT_WARPS * 32)
-router_select_kernel(RouterArgs a) {
+router_select_kernel(const __grid_constant__ RouterArgs a) {
   extern __shared__ float smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int t = blockIdx.x * RT_WARPS + warp;
@@ -158,7 +158,8 @@ router_select_kernel(RouterArgs a) {
 // ids[32], ws[32] in shared memory.
 template <int NT>
 __device__ void select_token_block(const RouterArgs &args, int t, float *s, float *sel, float *gsc, int *ids,
-                                   float *ws) {
+                                   float *ws, long long *ck = nullptr) {
+  if (ck && threadIdx.x == 0) ck[0] = clock64();
   const int E = args.E, k = args.k, G = args.n_group, TG = args.topk_group;
   const float *lg = args.logits + (int64_t)t * args.ldl;
   const float *bias = args.bias;
@@ -198,6 +199,7 @@ __device__ void select_token_block(const RouterArgs &args, int t, float *s, floa
     if (e < E) { s[e] = lv[i]; sel[e] = lv[i] + (bias ? bias[e] : 0.f); }
   }
   __syncthreads();
+  if (ck && threadIdx.x == 0) ck[1] = clock64();
   // group limit: thread g scores group g, then ranks it
   if (G > 1) {
     const int gs = E / G;
@@ -234,6 +236,7 @@ __device__ void select_token_block(const RouterArgs &args, int t, float *s, floa
       if (e < E && !ids[e / gs]) sel[e] = -INFINITY;
     }
     __syncthreads();
+    if (ck && threadIdx.x == 0) ck[2] = clock64();
   }
   // top-k in two warp-level rounds (short loops: this tail runs once, on one SM,
   // with a cold instruction cache): (1) every warp extracts the k best of its
@@ -262,6 +265,7 @@ __device__ void select_token_block(const RouterArgs &args, int t, float *s, floa
       for (int i = 0; i < 4; ++i) if (id[i] == bi) { v[i] = -INFINITY; id[i] = 0x7fffffff; }
     }
     __syncthreads();
+    if (ck && threadIdx.x == 0) ck[3] = clock64();
     if (w == 0) {
       // candidates: NT/32 lists of k <= 32 -> <= NT/32 per lane
       constexpr int NC = NT / 32;
@@ -286,6 +290,7 @@ __device__ void select_token_block(const RouterArgs &args, int t, float *s, floa
     }
   }
   __syncthreads();
+  if (ck && threadIdx.x == 0) ck[4] = clock64();
   // weights + canonical order (warp 0)
   if (tid < 32) {
     const int lane = tid;
@@ -307,6 +312,7 @@ __device__ void select_token_block(const RouterArgs &args, int t, float *s, floa
     if (args.shared_gated && lane == 0) args.sgate[t] = 1.f / (1.f + expf(-lg[E]));
   }
   __syncthreads();
+  if (ck && threadIdx.x == 0) ck[5] = clock64();
 }
 
 // ------------------------------------------------------------------ small T (decode)
@@ -317,7 +323,7 @@ __device__ void select_token_block(const RouterArgs &args, int t, float *s, floa
 // logits -> select -> count/scan/assign collapsed for the latency-bound decode step.
 constexpr int RS_THREADS = 256;
 
-__global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs a) {
+__global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_constant__ RouteSmallArgs a) {
   extern __shared__ float rsm[];
   const RouterArgs &r = a.r;
   const int H = a.H, T = r.T;
@@ -326,42 +332,50 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
   __shared__ float red[2][4][16];
   __shared__ int is_last;
   pdl_trigger();
+  // the shared expert's weights do not depend on the routing: pull them into
+  // L2 now (HBM is otherwise idle while the router runs), so the first units
+  // of the decode weight stream hit L2
+  if (threadIdx.x == 0) {
+#pragma unroll 1
+    for (int i = 0; i < 2; ++i) {
+      if (!a.pf[i]) continue;
+      const int64_t per = ((a.pf_bytes[i] + gridDim.x - 1) / gridDim.x + 4095) & ~int64_t(4095);
+      const int64_t b0 = (int64_t)blockIdx.x * per, b1 = b0 + per < a.pf_bytes[i] ? b0 + per : a.pf_bytes[i];
+#pragma unroll 1
+      for (int64_t o = b0; o < b1; o += 32768)
+        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const uint8_t *>(a.pf[i]) + o),
+                     "r"((uint32_t)(b1 - o < 32768 ? b1 - o : 32768))
+                     : "memory");
+    }
+  }
   // ---- logits of router rows `row` for all T tokens ----
+  // (H <= 8192: each thread's <= 8 16-byte chunks of the row are loaded once,
+  //  then a runtime loop over the tokens -- no per-token register arrays)
   {
-    float acc[16];
+    const int w4 = tid >> 5, lane = threadIdx.x & 31;
+    const int nv = H / 8;
+    uint4 w[8];
+    const bool live = row < a.rows && !(a.debug & 1);
+    const uint4 *wr = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.wg) + (size_t)row * H);
 #pragma unroll
-    for (int t = 0; t < 16; ++t) acc[t] = 0.f;
-    if (row < a.rows && !(a.debug & 1)) {
-      const uint4 *wr = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.wg) + (size_t)row * H);
-      const int nv = H / 8;
-      for (int c0 = tid; c0 < nv; c0 += 128 * 8) {
-        uint4 w[8];
+    for (int u = 0; u < 8; ++u) w[u] = (live && tid + u * 128 < nv) ? __ldg(wr + tid + u * 128) : make_uint4(0, 0, 0, 0);
+#pragma unroll 1
+    for (int t = 0; t < T; ++t) {
+      const uint4 *xr = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H);
+      float acc = 0.f;
 #pragma unroll
-        for (int u = 0; u < 8; ++u) w[u] = (c0 + u * 128 < nv) ? __ldg(wr + c0 + u * 128) : make_uint4(0, 0, 0, 0);
-#pragma unroll
-        for (int u = 0; u < 8; ++u) {
-          const int c = c0 + u * 128;
-          if (c >= nv) break;
-          float wf[8];
+      for (int u = 0; u < 8; ++u) {
+        const int c = tid + u * 128;
+        if (c < nv) {
+          float wf[8], xf[8];
           bf16x8_to_f32(w[u], wf);
-#pragma unroll 4
-          for (int t = 0; t < 16; ++t) {
-            if (t < T) {
-              float xf[8];
-              bf16x8_to_f32(__ldg(reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.x) +
-                                                                  (size_t)t * H) + c), xf);
+          bf16x8_to_f32(__ldg(xr + c), xf);
 #pragma unroll
-              for (int j = 0; j < 8; ++j) acc[t] = fmaf(wf[j], xf[j], acc[t]);
-            }
-          }
+          for (int j = 0; j < 8; ++j) acc = fmaf(wf[j], xf[j], acc);
         }
       }
-    }
-    const int w4 = tid >> 5, lane = threadIdx.x & 31;
-#pragma unroll
-    for (int t = 0; t < 16; ++t) {
-      const float v = warp_sum(acc[t]);
-      if (lane == 0) red[half][w4][t] = v;
+      acc = warp_sum(acc);
+      if (lane == 0) red[half][w4][t] = acc;
     }
     __syncthreads();
     if (row < a.rows && tid < T)
@@ -413,20 +427,27 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
   __syncthreads();
   if (!is_last) return;
   long long ck0 = clock64();
+  __shared__ long long cold_ck[8];
   if (a.debug & 2) { if (threadIdx.x == 0) *a.done = 0; return; }
   __threadfence();
   {
     float *s = rsm, *sel = rsm + r.E, *gsc = rsm + 2 * r.E, *ws = gsc + 32;
     int *ids = reinterpret_cast<int *>(ws + 32);
 #pragma unroll 1
-    for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws);
+    for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws, (a.debug & 4) ? cold_ck : nullptr);
     if (a.debug & 8) {                           // MOE_DEBUG_ROUTE=12: time a second (warm i-cache) pass
       __syncthreads();
       const long long w0 = clock64();
+      unsigned long long g0, g1;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g0));
+      __shared__ long long ck[8];
 #pragma unroll 1
-      for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws);
+      for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws, ck);
       __syncthreads();
-      if (threadIdx.x == 0) printf("route tail: warm select pass %lld cycles\n", clock64() - w0);
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g1));
+      if (threadIdx.x == 0)
+        printf("route tail: warm select pass %lld cycles (%llu ns): scores %lld group %lld warp-topk %lld merge %lld weights %lld\n",
+               clock64() - w0, g1 - g0, ck[1] - ck[0], ck[2] - ck[1], ck[3] - ck[2], ck[4] - ck[3], ck[5] - ck[4]);
     }
   }
   long long ck1 = clock64();
@@ -536,7 +557,9 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(RouteSmallArgs 
     __syncthreads();
   }
   if ((a.debug & 4) && threadIdx.x == 0)       // MOE_DEBUG_ROUTE=4: phase cycle counts of the tail
-    printf("route tail cycles: select %lld scan %lld assign %lld rows %lld\n", ck1 - ck0, ck2 - ck1, ck3 - ck2,
+    printf("route tail cycles: select %lld (scores %lld group %lld warp-topk %lld merge %lld weights %lld) scan %lld "
+           "assign %lld rows %lld\n", ck1 - ck0, cold_ck[1] - cold_ck[0], cold_ck[2] - cold_ck[1],
+           cold_ck[3] - cold_ck[2], cold_ck[4] - cold_ck[3], cold_ck[5] - cold_ck[4], ck2 - ck1, ck3 - ck2,
            clock64() - ck3);
 }
 

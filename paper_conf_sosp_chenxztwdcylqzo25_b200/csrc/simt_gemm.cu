@@ -45,7 +45,7 @@ __device__ __forceinline__ void load8_B(const void *B, int btype, int64_t elem_o
 
 template <int MODE>
 __global__ void __launch_bounds__(SG_THREADS)
-simt_gemm_kernel(SimtGemmArgs a) {
+simt_gemm_kernel(const __grid_constant__ SimtGemmArgs a) {
   constexpr int BN = SgCfg<MODE>::BN;
   constexpr int NJ = SgCfg<MODE>::NJ;
   __shared__ __align__(16) float As[SG_BK][SG_BM];

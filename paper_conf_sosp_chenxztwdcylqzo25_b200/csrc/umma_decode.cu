@@ -38,17 +38,20 @@ struct UdUnit {
   int valid, shared, expert, n, row0, blk;
 };
 
+// slot 0 = the shared expert (its weights were prefetched into L2 during
+// routing, so the first units run from L2), then the active routed experts
 __device__ __forceinline__ UdUnit ud_unit(const UmmaDecodeParams &p, int u) {
   UdUnit r{};
   const int slot = u / p.nblk;
   if (slot >= p.max_slots) return r;            // valid = 0
   r.valid = 1;
   r.blk = u % p.nblk;
-  if (slot < *p.n_active) {
-    const int e = p.act_list[slot];
-    r.expert = e; r.n = p.counts[e]; r.row0 = p.offs_pad[e];
-  } else if (p.has_shared && slot == p.max_slots - 1) {
+  const int rs = slot - p.has_shared;           // routed slot index
+  if (rs < 0) {
     r.shared = 1; r.expert = 0; r.n = p.T; r.row0 = 0;
+  } else if (rs < *p.n_active) {
+    const int e = p.act_list[rs];
+    r.expert = e; r.n = p.counts[e]; r.row0 = p.offs_pad[e];
   } else {
     return r;
   }

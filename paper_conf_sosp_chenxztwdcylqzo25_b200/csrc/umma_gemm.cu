@@ -420,6 +420,21 @@ bool make_rows_map(CUtensorMap *m, const void *base, bool u32, int64_t rows, int
   return r == CUDA_SUCCESS;
 }
 
+// contiguous buffer viewed as rows of row_bytes (8-byte elements), box = box_rows
+// whole rows: few, long TMA rows for pre-tiled (already swizzled) operands
+bool make_blocks_map(CUtensorMap *m, const void *base, int64_t total_bytes, int row_bytes, int box_rows) {
+  auto enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)(row_bytes / 8), (cuuint64_t)(total_bytes / row_bytes)};
+  cuuint64_t strides[1] = {(cuuint64_t)row_bytes};
+  cuuint32_t box[2] = {(cuuint32_t)(row_bytes / 8), (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT64, 2, const_cast<void *>(base), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
 // 2-D row-major [rows, cols] K-major operand, box = (128 bytes of K, box_rows), 128B swizzle
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows) {
   auto enc = get_encode();

@@ -45,11 +45,12 @@ constexpr int SW_SFW_BYTES = 512, SW_SFX_BYTES = 1024;
 constexpr int SW_XBOX = 32;                    // token rows per TMA box
 constexpr uint32_t SW_TMEM_COLS = 512;
 constexpr uint32_t SW_SFA_COL = 256, SW_SFB_COL = 264;   // + 16 for the second scale set
-constexpr int SW_XCH = 16;                     // columns per up->gate exchange chunk
+constexpr int SW_XCH = 8;                      // columns per up->gate exchange chunk
 constexpr size_t SW_SMEM = 1024 + (size_t)SW_STAGES * (SW_W_BYTES + SW_X_BYTES + SW_SFW_BYTES + SW_SFX_BYTES) +
                            4 * 32 * SW_XCH * 4 +      // up -> gate exchange
                            2 * 2 * 4 * 128 * 4 +      // amax partials [parity][half][slot][128]
                            2 * 2 * 128 * 4 +          // per-token inverse scales [half][gate warp][128]
+                           4 * 2048 +                 // SWIGLU: per gate warp 32 x 32 transpose tile
                            1024;                      // barriers, unit queue, TMEM base
 
 struct SwapUnit {
@@ -76,11 +77,6 @@ __device__ __forceinline__ SwapUnit swap_unit(const SwapParams &p, int u, int n_
   return r;
 }
 
-__device__ __forceinline__ void st_cluster_v4(uint32_t addr, float a, float b, float c, float d) {
-  asm volatile("st.shared::cluster.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "f"(a), "f"(b), "f"(c), "f"(d)
-               : "memory");
-}
-
 template <bool FP8, int EPI>
 __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_constant__ SwapParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -92,7 +88,10 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
   float *xbuf = reinterpret_cast<float *>(sSFX + SW_STAGES * SW_SFX_BYTES);   // [4 pairs][SW_XCH][32]
   float *am = xbuf + 4 * SW_XCH * 32;                                         // [2][2][4][128]
   float *isc = am + 2 * 2 * 4 * 128;                                          // [2 half][2 gate warp][128]
-  uint64_t *full = reinterpret_cast<uint64_t *>(isc + 2 * 2 * 128);
+  uint8_t *trbuf = reinterpret_cast<uint8_t *>(isc + 2 * 2 * 128);            // [4 gate warps][2 KB]
+  uint64_t *full = reinterpret_cast<uint64_t *>(trbuf + 4 * 2048);
+  // PLAIN reuses xbuf .. trbuf (>= 16 KB) as 8 per-warp 2 KB transpose tiles
+  static_assert(4 * 32 * SW_XCH * 4 + 2 * 2 * 4 * 128 * 4 + 2 * 2 * 128 * 4 + 4 * 2048 >= 8 * 2048, "tr tiles");
   uint64_t *empty = full + SW_STAGES;
   uint64_t *tmem_full = empty + SW_STAGES;
   uint64_t *tmem_empty = tmem_full + 1;
@@ -109,15 +108,15 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
 
   if (warp == 0 && lane == 0) {
     for (int i = 0; i < 2; ++i) {
-      prefetch_tmap(&p.g[i].w_map); prefetch_tmap(&p.g[i].x_map);
+      prefetch_tmap(&p.g[i].w_map); prefetch_tmap(&p.g[i].x_map); prefetch_tmap(&p.g[i].x_map128);
       if (FP8) { prefetch_tmap(&p.g[i].sfw_map); prefetch_tmap(&p.g[i].sfx_map); }
     }
     for (int s = 0; s < SW_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     mbar_init(tmem_full, 1);
     mbar_init(tmem_empty, 16);                   // 8 epilogue warps x 2 CTAs (the leader's copy is used)
     // leader's uq_empty: MMA warp + 8 epilogue warps (leader) + producer + 8 epilogue warps (peer)
-    for (int i = 0; i < SW_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], 18); }
-    for (int i = 0; i < 4; ++i) mbar_init(&am_bar[i], 128);   // 2 gate warps here + 2 in the peer, per lane
+    for (int i = 0; i < SW_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], p.debug_mode >= 4 ? 19 : 18); }
+    for (int i = 0; i < 4; ++i) mbar_init(&am_bar[i], 64);    // 2 gate warps here, per lane (+ peer bytes)
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc_pair(tmem_base_smem, SW_TMEM_COLS);
@@ -126,14 +125,15 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
   tc_fence_after();
   const uint32_t tmem = *tmem_base_smem;
 
+  // unit queue: the leader's producer claims units; the peer receives the id
+  // by st.async (completing on its uq_full); slot releases are plain arrives
   auto next_unit = [&](int &qs, uint32_t &qph) {
-    if (leader) mbar_wait(&uq_full[qs], qph);
-    else mbar_wait_cluster(&uq_full[qs], qph);   // unit id written by the leader (DSMEM)
+    mbar_wait(&uq_full[qs], qph);
     const int u = unit_q[qs];
     __syncwarp();
     if (lane == 0) {
       if (leader) mbar_arrive(&uq_empty[qs]);
-      else mbar_arrive_cluster(map_to_rank(&uq_empty[qs], 0));
+      else mbar_arrive_remote(map_to_rank(&uq_empty[qs], 0));
     }
     if (++qs == SW_UQ) { qs = 0; qph ^= 1; }
     return u;
@@ -150,21 +150,23 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
           u = atomicAdd(p.sched, 1);
           mbar_wait(&uq_empty[qs], qph ^ 1);
           unit_q[qs] = u;
-          st_cluster_u32(map_to_rank(&unit_q[qs], 1), (uint32_t)u);
           mbar_arrive(&uq_full[qs]);
-          mbar_arrive_cluster(map_to_rank(&uq_full[qs], 1));
+          const uint32_t pbar = map_to_rank(&uq_full[qs], 1);
+          mbar_arrive_expect_tx_remote(pbar, 4);
+          st_async_u32(map_to_rank(&unit_q[qs], 1), (uint32_t)u, pbar);
           if (++qs == SW_UQ) { qs = 0; qph ^= 1; }
         } else {
-          mbar_wait_cluster(&uq_full[qs], qph);
+          mbar_wait(&uq_full[qs], qph);
           u = unit_q[qs];
-          mbar_arrive_cluster(map_to_rank(&uq_empty[qs], 0));
+          mbar_arrive_remote(map_to_rank(&uq_empty[qs], 0));
           if (++qs == SW_UQ) { qs = 0; qph ^= 1; }
         }
         const SwapUnit ui = swap_unit(p, u, n_routed_units);
         if (!ui.valid) break;
         const SwapGroup &g = p.g[ui.group];
         const int half_n = ((ui.n + 15) & ~15) >> 1;          // token rows per CTA
-        const int nbox = (half_n + SW_XBOX - 1) / SW_XBOX;
+        const int nbox0 = (half_n + SW_XBOX - 1) / SW_XBOX;
+        const int nbox = nbox0 > 2 ? 4 : nbox0;                // > 64 rows: one 128-row box (4 x 32 rows of bytes)
         const int xrow = ui.row0 + (int)crank * half_n;
         const int64_t wtile = ((int64_t)ui.expert * g.w_nblk + ui.nb) * g.kblocks;
         const int G = (g.kblocks + 3) >> 2;
@@ -176,14 +178,33 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             continue;
           }
           const bool sf = FP8 && (kb & 3) == 0;
+          const int kc = kb * (FP8 ? 128 : 64);
+          if (p.debug_mode >= 4) {                 // timing experiments (loads only, per-CTA 1-SM TMA)
+            const bool dw = p.debug_mode != 5, dx = p.debug_mode != 4;
+            const uint32_t b1 = (dw ? SW_W_BYTES : 0) + (dx ? nbox * (SW_XBOX * 128) : 0);
+            mbar_expect_tx(&full[stage], b1);
+            if (dw) tma_load_2d(sW + stage * SW_W_BYTES, &g.w_map, &full[stage], 0, (int)((wtile + kb) * 16 + crank * 8));
+            if (dx) {
+              if (nbox > 2)
+                tma_load_2d(sX + stage * SW_X_BYTES, &g.x_map128, &full[stage], kc, xrow);
+              else
+                for (int i = 0; i < nbox; ++i)
+                  tma_load_2d(sX + stage * SW_X_BYTES + i * (SW_XBOX * 128), &g.x_map, &full[stage], kc, xrow + i * SW_XBOX);
+            }
+            if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
+            continue;
+          }
           const uint32_t bytes = SW_W_BYTES + nbox * (SW_XBOX * 128) + (sf ? SW_SFW_BYTES + SW_SFX_BYTES : 0);
           if (leader) mbar_expect_tx(&full[stage], 2 * bytes);
-          const int kc = kb * (FP8 ? 128 : 64);
+          // the CTA's 16 KB half of the 256-row tile: 8 rows of 2 KB
           tma_load_2d_pair(sW + stage * SW_W_BYTES, &g.w_map, &full[stage], 0,
-                           (int)((wtile + kb) * 256 + crank * 128));
-          for (int i = 0; i < nbox; ++i)
-            tma_load_2d_pair(sX + stage * SW_X_BYTES + i * (SW_XBOX * 128), &g.x_map, &full[stage], kc,
-                             xrow + i * SW_XBOX);
+                           (int)((wtile + kb) * 16 + crank * 8));
+          if (nbox > 2)                            // one 128-row box (rows past the half are never read)
+            tma_load_2d_pair(sX + stage * SW_X_BYTES, &g.x_map128, &full[stage], kc, xrow);
+          else
+            for (int i = 0; i < nbox; ++i)
+              tma_load_2d_pair(sX + stage * SW_X_BYTES + i * (SW_XBOX * 128), &g.x_map, &full[stage], kc,
+                               xrow + i * SW_XBOX);
           if (sf) {
             const int kg = kb >> 2;
             const int wr = g.sfw_per_cta ? (int)((((int64_t)ui.expert * G + kg) * g.w_nblk + ui.nb) * 2 + crank)
@@ -198,7 +219,25 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
     }
   } else if (warp == 1) {
     // ============================ MMA issuer (pair leader) ============================
-    if (leader) {
+    if (p.debug_mode >= 4) {                     // timing experiments: each CTA drains its own ring
+      int stage = 0; uint32_t phase = 0;
+      int qs = 0; uint32_t qph = 0;
+      for (;;) {
+        const int u = next_unit(qs, qph);
+        const SwapUnit ui = swap_unit(p, u, n_routed_units);
+        if (!ui.valid) break;
+        const int kblocks = p.g[ui.group].kblocks;
+        for (int kb = 0; kb < kblocks; ++kb) {
+          mbar_wait(&full[stage], phase);
+          if (lane == 0) {
+            mbar_arrive(&empty[stage]);
+            if (kb == kblocks - 1) mbar_arrive(tmem_full);
+          }
+          __syncwarp();
+          if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
+        }
+      }
+    } else if (leader) {
       int stage = 0; uint32_t phase = 0; uint32_t acc_phase = 0;
       int qs = 0; uint32_t qph = 0;
       for (;;) {
@@ -277,17 +316,32 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
       __syncwarp();
       if (lane == 0) {
         if (leader) mbar_arrive(tmem_empty);
-        else mbar_arrive_cluster(map_to_rank(tmem_empty, 0));
+        else mbar_arrive_remote(map_to_rank(tmem_empty, 0));
       }
       acc_phase ^= 1;
       const int64_t rbase = (int64_t)ui.row0 + c0;          // token row of this half's column 0
       if (p.debug_mode >= 1) { ++tile_i; continue; }        // timing experiments: no epilogue math
       if constexpr (EPI == GEMM_PLAIN) {
-        const int hrow = ui.nb * 256 + (int)crank * 128 + q * 32 + lane;
-        __nv_bfloat16 *out = reinterpret_cast<__nv_bfloat16 *>(g.out) + hrow;
+        // transpose 32 tokens x 32 H rows per step through a per-warp smem tile,
+        // then 16-byte row stores (token t: 64 contiguous bytes of its y row)
+        const int h0 = ui.nb * 256 + (int)crank * 128 + q * 32;
+        __nv_bfloat16 *tr = reinterpret_cast<__nv_bfloat16 *>(reinterpret_cast<uint8_t *>(xbuf) + ew * 2048);
 #pragma unroll
-        for (int i = 0; i < 128; ++i)
-          if (i < nvalid) out[(rbase + i) * g.ldc] = __float2bfloat16_rn(__uint_as_float(r[i]));
+        for (int c = 0; c < 4; ++c) {
+          if (c < nch) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) tr[j * 32 + lane] = __float2bfloat16_rn(__uint_as_float(r[32 * c + j]));
+            __syncwarp();
+#pragma unroll
+            for (int it = 0; it < 4; ++it) {
+              const int j = it * 8 + (lane >> 2), cc = lane & 3;
+              if (32 * c + j < nvalid)
+                *reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(g.out) + (rbase + 32 * c + j) * g.ldc + h0 +
+                                           cc * 8) = *reinterpret_cast<const uint4 *>(tr + j * 32 + cc * 8);
+            }
+            __syncwarp();
+          }
+        }
       } else {
         // ---- up quadrants (odd q) hand their accumulators to the gate quadrants ----
         const int pi = (q >> 1) + 2 * half;
@@ -316,11 +370,26 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         if (up) { ++tile_i; continue; }
         const int qg = q >> 1;                                // gate warp 0 / 1 of this half
         const int f = ui.nb * 128 + (int)crank * 64 + qg * 32 + lane;
+        const int f0 = f - lane;
+        uint8_t *trw = trbuf + (half * 2 + qg) * 2048;
         if constexpr (!FP8) {
-          __nv_bfloat16 *out = reinterpret_cast<__nv_bfloat16 *>(g.out) + f;
+          __nv_bfloat16 *tr = reinterpret_cast<__nv_bfloat16 *>(trw);
 #pragma unroll
-          for (int i = 0; i < 128; ++i)
-            if (i < nvalid) out[(rbase + i) * g.ldc] = __float2bfloat16_rn(__uint_as_float(r[i]));
+          for (int c = 0; c < 4; ++c) {
+            if (c < nch) {
+#pragma unroll
+              for (int j = 0; j < 32; ++j) tr[j * 32 + lane] = __float2bfloat16_rn(__uint_as_float(r[32 * c + j]));
+              __syncwarp();
+#pragma unroll
+              for (int it = 0; it < 4; ++it) {
+                const int j = it * 8 + (lane >> 2), cc = lane & 3;
+                if (32 * c + j < nvalid)
+                  *reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(g.out) + (rbase + 32 * c + j) * g.ldc + f0 +
+                                             cc * 8) = *reinterpret_cast<const uint4 *>(tr + j * 32 + cc * 8);
+              }
+              __syncwarp();
+            }
+          }
         } else {
           // ---- per-token amax over the 128 h columns of block nb: 32 lanes x
           // 2 gate warps here x 2 in the peer.  Per 32-column chunk c a
@@ -347,12 +416,16 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
           const int par = tile_i & 1;
           const uint32_t ph = (tile_i >> 1) & 1;
           float *amh = am + (par * 2 + half) * 4 * 128;      // [slot][lane][chunk]
+          // local partials by plain stores + arrive (this warp expects its peer
+          // warp's 512 bytes); remote partials by st.async completing on the
+          // peer's barrier
           *reinterpret_cast<float4 *>(amh + qg * 128 + 4 * lane) = make_float4(m4[0], m4[1], m4[2], m4[3]);
-          st_cluster_v4(map_to_rank(amh + (2 + qg) * 128 + 4 * lane, crank ^ 1), m4[0], m4[1], m4[2], m4[3]);
           uint64_t *bar = &am_bar[par * 2 + half];
-          mbar_arrive(bar);
-          mbar_arrive_cluster(map_to_rank(bar, crank ^ 1));
-          mbar_wait_cluster(bar, ph);
+          st_async_v4f32(map_to_rank(amh + (2 + qg) * 128 + 4 * lane, crank ^ 1), m4[0], m4[1], m4[2], m4[3],
+                         map_to_rank(bar, crank ^ 1));
+          if (lane == 0) mbar_expect_tx(bar, 32 * 16);
+          else mbar_arrive(bar);
+          mbar_wait(bar, ph);
           float *sc = isc + (half * 2 + qg) * 128;
           {
             const float4 a0 = *reinterpret_cast<const float4 *>(amh + 4 * lane);
@@ -371,10 +444,24 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             }
           }
           __syncwarp();
-          uint8_t *out = reinterpret_cast<uint8_t *>(g.out) + f;
+          // e4m3 codes: 32 tokens x 32 h columns per step through the smem tile,
+          // then 16-byte stores (token t: 32 contiguous bytes of its h row)
 #pragma unroll
-          for (int i = 0; i < 128; ++i)
-            if (i < nvalid) out[(rbase + i) * g.ldc] = f32_to_e4m3(__uint_as_float(r[i]) * sc[i]);
+          for (int c = 0; c < 4; ++c) {
+            if (c < nch) {
+#pragma unroll
+              for (int j = 0; j < 32; ++j) trw[j * 32 + lane] = f32_to_e4m3(__uint_as_float(r[32 * c + j]) * sc[32 * c + j]);
+              __syncwarp();
+#pragma unroll
+              for (int it = 0; it < 2; ++it) {
+                const int j = it * 16 + (lane >> 1), cc = lane & 1;
+                if (32 * c + j < nvalid)
+                  *reinterpret_cast<uint4 *>(reinterpret_cast<uint8_t *>(g.out) + (rbase + 32 * c + j) * g.ldc + f0 + cc * 16) =
+                      *reinterpret_cast<const uint4 *>(trw + j * 32 + cc * 16);
+              }
+              __syncwarp();
+            }
+          }
         }
       }
       ++tile_i;
