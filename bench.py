@@ -16,7 +16,8 @@ the layer on its own tokens (weak scaling, no data-path collective; DESIGN.md
 §7), value = all ranks' tokens / max-over-ranks time.
 
 Inputs are resident in HBM when the timed region starts; L2 is flushed (a
-256 MiB write, outside the timed events) before every timed step.  Each step is
+256 MiB write, then a 256 MiB read so the dirty lines are written back before
+the events start; all outside the timed events) before every timed step.  Each step is
 timed with CUDA events on the launching stream.  `e2e` re-times the same step
 through the public API with host (pinned) input/output buffers, H2D and D2H
 inside the events.  The oracle (oracle/, a plain fp64 CPU program) is timed on
@@ -205,6 +206,16 @@ def algorithmic(p, T, n_distinct):
     }
 
 
+def flush_l2(flush):
+    """Evict L2 before a timed step: write a 256 MiB buffer (> the 126 MB L2), then
+    read a second one so the dirty zero lines are written back to HBM here, outside
+    the timed events, instead of being evicted (written back) by the timed step."""
+    import torch
+    buf_w, buf_r, sink = flush
+    buf_w.zero_()
+    torch.sum(buf_r, 0, out=sink)
+
+
 def timed_steps(layer, xs, y, steps, warmup, flush, profile=True):
     """Per-step CUDA-event times (ms) and per-stage ms; xs: list of inputs cycled."""
     import torch
@@ -217,7 +228,7 @@ def timed_steps(layer, xs, y, steps, warmup, flush, profile=True):
     times, stages = [], {}
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     for i in range(steps):
-        flush.zero_()
+        flush_l2(flush)
         e0.record(st)
         layer.forward(xs[(warmup + i) % len(xs)], y=y)
         e1.record(st)
@@ -259,7 +270,9 @@ def run_ours(args):
         layer = moe.MoELayer(p, w, max_tokens=T, device=local, ep_rank=rank, ep_size=ws, unique_id=uid[0])
     else:
         layer = moe.MoELayer(p, w, max_tokens=T, device=local)
-    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    flush = (torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda"),
+             torch.zeros(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda"),
+             torch.zeros((), dtype=torch.float32, device="cuda"))
     info = layer.info()
 
     # ---------------- prefill, device-resident inputs ----------------
@@ -269,6 +282,7 @@ def run_ours(args):
         times, stages = timed_steps(layer, [x], y, args.steps, args.warmup, flush, profile=not ep)
     torch.cuda.synchronize()
     barrier(ws)
+    pinfo = layer.info()                 # kernel launches of the last (prefill) forward
     ms = max_over_ranks(sum(times) / len(times), ws)
     value = ws * T / (ms * 1e-3)
 
@@ -301,51 +315,67 @@ def run_ours(args):
                 "stage_ms": {k: round(v, 4) for k, v in stages.items()}}
     layer_tflops = alg["layer_flops"] / (ms * 1e-3) / 1e12
 
-    # ---------------- decode, T = 1 (distinct tokens, L2 flushed) ----------------
-    # The decode step is one CUDA graph replay of the forward (the API is
-    # host-sync-free and capturable; PAPER.md L193 captures the decode step in
-    # one CUDA graph), timed with events around the replay; a separate eager
+    # ---------------- decode, T = 1: a chain of distinct layers ----------------
+    # The decode step is one CUDA graph replay over a stack of `--decode-layers`
+    # distinct layer instances chained like consecutive model layers
+    # (x_{i+1} = y_i = x_i + moe_i(x_i)); weights of the stack (8 x 11.3 GB for V3)
+    # dwarf L2, and L2 is also flushed before every replay (outside the events).
+    # value = replay time / layers.  The API is host-sync-free and capturable
+    # (PAPER.md L193 captures the decode step in one CUDA graph).  A separate eager
     # pass with stage events gives the per-kernel breakdown.
     decode = None
     if not args.no_decode and not ep:
+        nl = max(1, args.decode_layers)
+        dlayers = [layer] + [moe.MoELayer(p, w, max_tokens=16, device=local) for _ in range(nl - 1)]
         xd, _ = make_tokens(p, args.steps + args.warmup, "cuda", offset=1000 + rank)
         rows = [xd[i:i + 1].contiguous() for i in range(xd.shape[0])]
-        yd = torch.empty_like(rows[0])
-        xstatic = torch.empty_like(rows[0])
-        xstatic.copy_(rows[0])
+        bufs = [rows[0].clone(), torch.empty_like(rows[0])]
+
+        def dstep():
+            for i, l in enumerate(dlayers):
+                a_, b_ = bufs[i % 2], bufs[(i + 1) % 2]
+                l.forward(a_, residual=a_, y=b_)
+
         side = torch.cuda.Stream()
         side.wait_stream(torch.cuda.current_stream())
         with torch.cuda.stream(side):
             for _ in range(2):
-                layer.forward(xstatic, y=yd)
+                bufs[0].copy_(rows[0])
+                dstep()
         torch.cuda.current_stream().wait_stream(side)
         graph = torch.cuda.CUDAGraph()
         with torch.cuda.graph(graph):
-            layer.forward(xstatic, y=yd)
+            dstep()
         st = torch.cuda.current_stream()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         for i in range(args.warmup):
-            xstatic.copy_(rows[i])
+            bufs[0].copy_(rows[i])
             graph.replay()
         torch.cuda.synchronize()
         dtimes = []
         for i in range(args.steps):
-            xstatic.copy_(rows[args.warmup + i])
-            flush.zero_()
+            bufs[0].copy_(rows[args.warmup + i])
+            flush_l2(flush)
             e0.record(st)
             graph.replay()
             e1.record(st)
             e1.synchronize()
-            dtimes.append(e0.elapsed_time(e1))
-        _, dstages = timed_steps(layer, rows, yd, min(args.steps, 5), 1, flush)
+            dtimes.append(e0.elapsed_time(e1) / nl)
+        _, dstages = timed_steps(layer, rows, bufs[1], min(args.steps, 5), 1, flush)
+        dinfo = layer.info()
         dus = max_over_ranks(sum(dtimes) / len(dtimes), ws) * 1e3
         algd = algorithmic(p, 1, p.top_k)
-        decode = {"us_per_layer": dus, "tokens": 1, "mode": "cuda_graph_replay",
+        decode = {"us_per_layer": dus, "tokens": 1, "layers_in_graph": nl, "mode": "cuda_graph_replay",
+                  "gpu_launches_per_layer": dinfo.kernels_per_forward_decode,
                   "roofline": {"bound": "hbm", "achieved": algd["layer_bytes"] / (dus * 1e-6) / 1e9,
                                "peak": peaks["hbm_gbs"], "unit": "GB/s",
                                "frac": algd["layer_bytes"] / (dus * 1e-6) / 1e9 / peaks["hbm_gbs"],
                                "bytes": algd["layer_bytes"],
                                "stage_us_eager": {k: round(v * 1e3, 2) for k, v in dstages.items()}}}
+        for l in dlayers[1:]:
+            l.close()
+        del dlayers, graph
+        torch.cuda.empty_cache()
 
     # ---------------- e2e through the public API, host buffers ----------------
     e2e = None
@@ -362,7 +392,7 @@ def run_ours(args):
         torch.cuda.synchronize()
         et = []
         for _ in range(args.steps):
-            flush.zero_()
+            flush_l2(flush)
             e0.record(st)
             xdev.copy_(xh, non_blocking=True)
             layer.forward(xdev, y=y)
@@ -390,12 +420,13 @@ def run_ours(args):
                            "ffn": p.ffn, "experts": p.n_experts, "top_k": p.top_k, "shared_ffn": p.shared_ffn,
                            "weights": "fp8_e4m3_block128_ue8m0" if fp8 else "bf16", "parallelism":
                            (f"ep{ws} (NCCL all-to-all-v dispatch/combine)" if ep else f"replica x{ws}")
-                           if ws > 1 else "single", "l2": "flushed before every step (256 MiB write, "
+                           if ws > 1 else "single", "l2": "flushed before every step (256 MiB write, then 256 MiB read so the dirty lines are written back "
+                           "before the events, "
                            "outside the timed events); inputs resident in HBM",
                            "distinct_experts_hit": n_distinct},
                 "layer_tflops": layer_tflops,
                 "roofline": roofline, "decode": decode, "e2e": e2e, "cpu_baseline": cpu,
-                "gpu_launches": info.kernels_per_forward_prefill * args.steps,
+                "gpu_launches": pinfo.kernels_per_forward_prefill * args.steps,
                 "clocks": clk.summary()}
         print(json.dumps(line), flush=True)
     layer.close()
@@ -413,6 +444,7 @@ def main():
     ap.add_argument("--config", default="v3")
     ap.add_argument("--tokens", type=int, default=0)
     ap.add_argument("--no-decode", action="store_true")
+    ap.add_argument("--decode-layers", type=int, default=8, help="distinct layers chained in the decode graph")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=20.0)

@@ -221,6 +221,10 @@ struct moe_layer {
   int64_t w13_img_stride = 0, w2_img_stride = 0;
   CUtensorMap map_xperm, map_h, map_xq, map_hsh, map_gate;   // activation rows (box 128), router rows
   CUtensorMap dmap_xperm, dmap_h, dmap_xq, dmap_hsh;           // decode: activation rows (box 16)
+  float *dacc = nullptr;        // fused decode: [2][gemv_max_tokens, H] fp32 sums (immediate, deferred), kept zero
+  bool fused_decode = false;
+  int n_launch = 0, launches_prefill = 0, launches_decode = 0;   // kernel launches per forward
+  unsigned long long *trace = nullptr;   // MOE_DEBUG_TRACE timeline buffer (timing experiments)
   // swap-AB CTA-pair GEMM (umma_swap.cu): tiled weights as 128-byte rows (box 128),
   // token rows (box 32), weight scale images (box 1) and token scale images (box 2)
   CUtensorMap tmap_w13, tmap_w2, tmap_ws13, tmap_ws2;

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <stdint.h>
+#include <cstdlib>
 #include <utility>
 
 #include "common.cuh"
@@ -27,7 +28,8 @@ cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t s
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  static const bool no_pdl = getenv("MOE_NO_PDL") && atoi(getenv("MOE_NO_PDL")) == 1;   // A/B experiments
+  cfg.numAttrs = no_pdl ? 0 : 1;
   return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
 }
 
@@ -100,6 +102,8 @@ struct RouteSmallArgs {
   // shared-expert weights prefetched into L2 while the router runs (they do
   // not depend on the routing): [pf[i], pf[i] + pf_bytes[i]), i < 2
   const void *pf[2]; int64_t pf_bytes[2];
+  unsigned long long *trace;     // MOE_DEBUG_TRACE: [0] CTA 0 entry, [1..4] tail start / select / permute / end
+  int minimal;                  // fused decode: active-expert list only (no sorted rows / positions)
 };
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st);
 
@@ -216,6 +220,41 @@ struct UmmaDecodeParams {
   int *sched;
 };
 cudaError_t launch_umma_decode(bool fp8, int mode, const UmmaDecodeParams &p, int grid, cudaStream_t st);
+
+// decode, fused per (slot, 128-column FFN chunk) unit (umma_decode_fused.cu):
+// W13 tile -> SwiGLU (+ FP8 requant) -> h_c in smem -> W2 column block ->
+// weighted fp32 partial sums; decode_finalize writes y / deferred_out
+struct FdGroup {                // 0 routed, 1 shared
+  CUtensorMap x_map;            // token-order activation rows (xq / bf16 x), K-major SW128, box 16 rows
+  const uint8_t *w13;           // tiled W13 [expert][F/128][H/128 B][256 x 128 B]
+  const uint8_t *w13_img;       // FP8: W13 scale image (swap layout) [expert][H/512][F/128][512 B]
+  int64_t w13_img_stride;       // bytes per expert
+  const uint8_t *x_img;         // FP8: activation scale image
+  int x_img_stride;             // 128-row tiles per k-group
+  const uint8_t *w2;            // tiled W2 [expert][H/256][F/128 B][256 x 128 B]
+  const float *w2_s;            // FP8: [expert][H/128][F/128]
+};
+struct FusedDecodeParams {
+  FdGroup g[2];
+  int nch[2];                   // 128-column chunks: F/128, Fs/128
+  int H, T, k, n_imm, has_shared;
+  const int32_t *n_active, *act_list;   // active local experts (ascending)
+  const int32_t *topk_idx; int e0;      // [T, k] global ids (canonical order), first local expert
+  const float *topk_w, *sgate;  // sgate null unless the shared expert is gated (Qwen2)
+  float *acc_imm, *acc_def;     // [T, H] fp32 sums, zero on entry (re-zeroed by decode_finalize)
+  int *sched, *done;            // work counter + exit ticket, zero on entry (re-armed by the kernel)
+  const void *pf[2]; int64_t pf_bytes[2];   // shared-expert weights prefetched into L2 before the PDL wait
+  unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
+};
+cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, cudaStream_t st);
+struct DecodeFinalizeArgs {
+  int T, H, use_def;
+  float *acc_imm, *acc_def;
+  const void *residual, *deferred_in;
+  void *y, *deferred_out;
+  unsigned long long *trace;     // MOE_DEBUG_TRACE: [2000] past the PDL wait, [2001] end (CTA 0)
+};
+cudaError_t launch_decode_finalize(const DecodeFinalizeArgs &a, cudaStream_t st);
 
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);
 bool make_rows_map(CUtensorMap *m, const void *base, bool u32, int64_t rows, int row_elems, int box_rows);

@@ -35,6 +35,14 @@ moe_status fail(moe_status s, const char *fmt, ...) {
                   #expr, cudaGetErrorString(_e), __FILE__, __LINE__);                         \
   } while (0)
 
+// a kernel launch of the forward: checked and counted (moe_layer_info reports the
+// launches of the last prefill / decode forward)
+#define KL_TRY(expr)         \
+  do {                       \
+    CUDA_TRY(expr);          \
+    ++L->n_launch;           \
+  } while (0)
+
 template <class T>
 cudaError_t dalloc(moe_layer *L, T **p, size_t bytes, bool weight) {
   if (bytes == 0) { *p = nullptr; return cudaSuccess; }
@@ -49,7 +57,7 @@ void free_all(moe_layer *L) {
                   L->counts, L->offs, L->offs_pad, L->tiles, L->n_tiles, L->act_list, L->n_active,
                   L->row_token, L->pos, L->sched, L->pairs, L->n_pairs, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
                   L->hsh, L->hsh_s, L->ysh, L->w13_img, L->w2_img, L->ws13_img, L->ws2_img,
-                  L->xperm_img, L->h_img, L->xq_img, L->hsh_img};
+                  L->xperm_img, L->h_img, L->xq_img, L->hsh_img, L->dacc, L->trace};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   void *eps[] = {L->ep.send_x, L->ep.send_idx, L->ep.send_w, L->ep.sendpos, L->ep.cnt_dev, L->ep.recv_x,
@@ -362,6 +370,7 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   C_TRY(dalloc(L, &L->act_list, (size_t)E * 4, false));
   C_TRY(dalloc(L, &L->n_active, 4, false));
   C_TRY(dalloc(L, &L->sched, 32, false));
+  C_TRY(cudaMemset(L->sched, 0, 32));
   C_TRY(dalloc(L, &L->pairs, (size_t)L->max_tiles * sizeof(int4), false));
   C_TRY(dalloc(L, &L->n_pairs, 4, false));
   C_TRY(dalloc(L, &L->row_token, (size_t)L->R_max * 4, false));
@@ -432,10 +441,8 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
     }
     ok = ok && make_kmajor_map(&L->dmap_xperm, L->xperm, f8, L->R_max, H, 16) &&
          make_kmajor_map(&L->dmap_h, L->hbuf, f8, L->R_max, F, 16);
-    if (Fs) {
-      ok = ok && make_kmajor_map(&L->dmap_hsh, L->hsh, f8, Tm, Fs, 16);
-      if (f8) ok = ok && make_kmajor_map(&L->dmap_xq, L->xq, true, Tm, H, 16);
-    }
+    if (Fs) ok = ok && make_kmajor_map(&L->dmap_hsh, L->hsh, f8, Tm, Fs, 16);
+    if (f8) ok = ok && make_kmajor_map(&L->dmap_xq, L->xq, true, Tm, H, 16);   // fused decode + shared expert
     // swap-AB pair GEMM maps: tiled weights as 128-byte rows, token rows (box 32),
     // scale images as 512-byte rows (weights: box 1 per CTA; tokens: box 2 = 256 rows)
     {
@@ -465,6 +472,18 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
       }
     }
     if (!ok) return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable?)"));
+    // fused decode (umma_decode_fused.cu) unless MOE_DECODE_CHAIN=1 selects the two-launch chain
+    if (getenv("MOE_DEBUG_TRACE")) {               // timing experiments: device timeline buffer
+      C_TRY(dalloc(L, &L->trace, 4096 * 8, false));
+      C_TRY(cudaMemset(L->trace, 0, 4096 * 8));
+    }
+    const char *chain = getenv("MOE_DECODE_CHAIN");
+    L->fused_decode = L->gemv_ok && !(chain && atoi(chain) == 1);
+    if (L->fused_decode) {
+      const size_t n = (size_t)2 * L->gemv_max_tokens * H * 4;
+      C_TRY(dalloc(L, &L->dacc, n, false));
+      C_TRY(cudaMemset(L->dacc, 0, n));
+    }
   }
   C_TRY(cudaDeviceSynchronize());
 #undef C_TRY
@@ -523,7 +542,7 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     }
     p1.tiles = L->pairs; p1.n_tiles = L->n_pairs; p1.nb_r = F / 128;
     p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = Fs / 128; p1.sched = L->sched; p1.debug_mode = dbg_mode;
-    CUDA_TRY(launch_umma_swap_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
+    KL_TRY(launch_umma_swap_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
     mark(L, ST_GEMM1, st);
     SwapParams p2{};
     {
@@ -542,7 +561,7 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     }
     p2.tiles = L->pairs; p2.n_tiles = L->n_pairs; p2.nb_r = H / 256;
     p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256; p2.sched = L->sched + 1; p2.debug_mode = dbg_mode;
-    CUDA_TRY(launch_umma_swap_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
+    KL_TRY(launch_umma_swap_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
     mark(L, ST_GEMM2, st);
   } else {
     // 5. routed experts: GEMM1 + SwiGLU, GEMM2 (CUDA-core path: F32 weights, H % 256 != 0)
@@ -552,7 +571,7 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     a.b_type = btype; a.N = 2 * F; a.K = H;
     a.tiles = L->tiles; a.n_tiles = L->n_tiles;
     a.C = L->hbuf; a.Cs = L->h_s; a.ldc = F; a.out_fp8 = L->fp8;
-    CUDA_TRY(launch_simt_gemm(GEMM_SWIGLU, a, 2 * tile_bound, st));
+    KL_TRY(launch_simt_gemm(GEMM_SWIGLU, a, 2 * tile_bound, st));
     mark(L, ST_GEMM1, st);
     SimtGemmArgs b{};
     b.A = L->hbuf; b.As = L->h_s; b.lda = F; b.a_fp8 = L->fp8;
@@ -560,7 +579,7 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     b.b_type = btype; b.N = H; b.K = F;
     b.tiles = L->tiles; b.n_tiles = L->n_tiles;
     b.C = L->yperm; b.ldc = H;
-    CUDA_TRY(launch_simt_gemm(GEMM_PLAIN, b, 2 * tile_bound, st));
+    KL_TRY(launch_simt_gemm(GEMM_PLAIN, b, 2 * tile_bound, st));
     mark(L, ST_GEMM2, st);
     // 6. shared expert on every token
     if (Fs > 0) {
@@ -568,13 +587,13 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
       a.A = xa; a.As = xa_s; a.lda = H; a.a_fp8 = L->fp8;
       a.B = L->ws13; a.Bs = L->ws13_s; a.b_type = btype; a.N = 2 * Fs; a.K = H;
       a.M = T; a.C = L->hsh; a.Cs = L->hsh_s; a.ldc = Fs; a.out_fp8 = L->fp8;
-      CUDA_TRY(launch_simt_gemm(GEMM_SWIGLU, a, (T + 63) / 64, st));
+      KL_TRY(launch_simt_gemm(GEMM_SWIGLU, a, (T + 63) / 64, st));
       mark(L, ST_SH1, st);
       SimtGemmArgs b{};
       b.A = L->hsh; b.As = L->hsh_s; b.lda = Fs; b.a_fp8 = L->fp8;
       b.B = L->ws2; b.Bs = L->ws2_s; b.b_type = btype; b.N = H; b.K = Fs;
       b.M = T; b.C = L->ysh; b.ldc = H;
-      CUDA_TRY(launch_simt_gemm(GEMM_PLAIN, b, (T + 63) / 64, st));
+      KL_TRY(launch_simt_gemm(GEMM_PLAIN, b, (T + 63) / 64, st));
       mark(L, ST_SH2, st);
     }
   }
@@ -596,7 +615,7 @@ static moe_status run_router_full(moe_layer *L, const void *x, int T, cudaStream
   if (T <= 0) return MOE_OK;
   const int H = L->H;
   if (T <= kGemvMaxTokens) {
-    CUDA_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
+    KL_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
   } else {
     UmmaParams p{};
     UmmaGroup &g = p.g[1];
@@ -606,7 +625,7 @@ static moe_status run_router_full(moe_layer *L, const void *x, int T, cudaStream
     p.g[0] = g;
     p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
     const int units = ((T + 127) / 128) * p.nb_s;
-    CUDA_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
+    KL_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
   }
   RouterArgs r{};
   r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
@@ -614,7 +633,7 @@ static moe_status run_router_full(moe_layer *L, const void *x, int T, cudaStream
   r.group_score = L->cfg.group_score; r.score_fn = L->cfg.score_fn; r.norm_topk = L->cfg.norm_topk;
   r.routed_scale = L->cfg.routed_scale; r.shared_gated = L->cfg.shared_gated;
   r.topk_idx = L->topk_idx; r.topk_w = L->topk_w; r.sgate = L->sgate;
-  CUDA_TRY(launch_router_select(r, st));
+  KL_TRY(launch_router_select(r, st));
   return MOE_OK;
 }
 
@@ -623,8 +642,8 @@ static moe_status ep_phase_a(moe_layer *L, const void *x, int T, cudaStream_t st
   moe_status s = run_router_full(L, x, T, st);
   if (s != MOE_OK) return s;
   const int P = L->ep.P, Tm = std::max(1, L->max_tokens);
-  CUDA_TRY(launch_ep_plan(L->topk_idx, T, L->k, L->E, P, L->ep.sendpos, L->ep.cnt_dev, st));
-  CUDA_TRY(launch_ep_pack(x, T, L->H, L->k, L->topk_idx, L->topk_w, L->E, P, Tm, L->ep.sendpos, L->ep.send_x,
+  KL_TRY(launch_ep_plan(L->topk_idx, T, L->k, L->E, P, L->ep.sendpos, L->ep.cnt_dev, st));
+  KL_TRY(launch_ep_pack(x, T, L->H, L->k, L->topk_idx, L->topk_w, L->E, P, Tm, L->ep.sendpos, L->ep.send_x,
                           L->ep.send_idx, L->ep.send_w, st));
   return MOE_OK;
 }
@@ -656,7 +675,8 @@ static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_d
   pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
   pa.pairs = L->pairs; pa.n_pairs = L->n_pairs;
   if (R > 0) {
-    CUDA_TRY(launch_permute(pa, st));
+    KL_TRY(launch_permute(pa, st));
+    L->n_launch += 2;                            // count + scan + assign kernels
   } else {
     CUDA_TRY(cudaMemsetAsync(L->n_tiles, 0, 4, st));
     CUDA_TRY(cudaMemsetAsync(L->n_pairs, 0, 4, st));
@@ -667,13 +687,13 @@ static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_d
     d.xperm_img = L->umma ? L->xperm_img : nullptr; d.xperm_img_stride = L->max_tiles;
     d.xperm_s = L->umma ? nullptr : L->xperm_s;
   }
-  CUDA_TRY(launch_scatter_rows(L->ep.recv_x, R, H, k, L->pos, d, st));
+  KL_TRY(launch_scatter_rows(L->ep.recv_x, R, H, k, L->pos, d, st));
   if (Fs > 0 && L->fp8 && T_own > 0) {
     // the shared expert runs on this rank's own tokens: quantise them into xq
     ScatterDst s{};
     s.fp8 = 1; s.xq = L->xq; s.xs = L->xs; s.xq_img = L->umma ? L->xq_img : nullptr;
     s.xq_img_stride = L->img_tiles_sh;
-    CUDA_TRY(launch_scatter_rows(x_own, T_own, H, 0, L->pos, s, st));
+    KL_TRY(launch_scatter_rows(x_own, T_own, H, 0, L->pos, s, st));
   }
   const int64_t pairs = (int64_t)R * k;
   const int64_t R_bound = std::min<int64_t>(L->R_max, pairs + (int64_t)std::min<int64_t>(E, pairs) * kPadM);
@@ -684,7 +704,7 @@ static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_d
     c.T = R; c.H = H; c.k = k; c.n_imm = want_def ? k - n_def : k;
     c.pos = L->pos; c.topk_w = L->topk_w; c.yperm = L->yperm;
     c.y = L->ep.partial; c.deferred_out = want_def ? L->ep.partial_def : nullptr;
-    CUDA_TRY(launch_combine(c, st));
+    KL_TRY(launch_combine(c, st));
   }
   return MOE_OK;
 }
@@ -698,7 +718,7 @@ static moe_status ep_phase_d(moe_layer *L, const void *residual, int T, const vo
   c.residual = reinterpret_cast<const __nv_bfloat16 *>(residual);
   c.deferred_in = reinterpret_cast<const __nv_bfloat16 *>(din);
   c.y = reinterpret_cast<__nv_bfloat16 *>(y); c.deferred_out = reinterpret_cast<__nv_bfloat16 *>(dout);
-  CUDA_TRY(launch_ep_final_combine(c, st));
+  KL_TRY(launch_ep_final_combine(c, st));
   return MOE_OK;
 }
 
@@ -753,6 +773,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     return ep_forward_nccl(L, x, residual, T, n_def, deferred_in, y, deferred_out, st);  // T == 0 participates
   }
   if (T == 0) return MOE_OK;
+  L->n_launch = 0;
   if (L->prof) {
     for (int i = 0; i <= moe_layer::kStages; ++i) L->ev_hit[i] = false;
     cudaEventRecord(L->ev[0], st);
@@ -760,8 +781,9 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   }
   const int H = L->H, F = L->F, Fs = L->Fs, E = L->E, k = L->k;
   const bool decode = L->gemv_ok && T <= L->gemv_max_tokens;
-  const bool tc_decode = decode && L->umma;        // T <= 16: fused small-T route + swap-AB kernels
-  CUDA_TRY(cudaMemsetAsync(L->sched, 0, 32, st));
+  const bool tc_decode = decode && L->umma && L->E_glob <= 256 && L->E <= 256;  // T <= 16: small-T route + swap-AB kernels
+  const bool fused = tc_decode && L->fused_decode;  // route -> fused W13/W2 stream -> finalize (self-re-arming counters)
+  if (!fused) CUDA_TRY(cudaMemsetAsync(L->sched, 0, 32, st));
   RouterArgs r{};
   r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
   r.T = T; r.E = L->E_glob; r.k = k; r.n_group = L->cfg.n_group; r.topk_group = L->cfg.topk_group;
@@ -782,17 +804,19 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     rs.r = r; rs.p = pa; rs.x = x; rs.wg = L->gate_w; rs.H = H; rs.rows = L->gate_rows; rs.done = L->sched + 7;
     static const int dbg_route = getenv("MOE_DEBUG_ROUTE") ? atoi(getenv("MOE_DEBUG_ROUTE")) : 0;
     rs.debug = dbg_route;
-    rs.fp8 = L->fp8; rs.xperm = L->xperm; rs.xperm_img = L->xperm_img; rs.xperm_img_stride = L->max_tiles;
+    rs.trace = L->trace;
+    rs.fp8 = L->fp8; rs.xperm = fused ? nullptr : L->xperm; rs.xperm_img = L->xperm_img;
+    rs.xperm_img_stride = L->max_tiles; rs.minimal = fused;
     if (L->fp8) { rs.xq = L->xq; rs.xs = L->xs; rs.xq_img = L->xq_img; rs.xq_img_stride = L->img_tiles_sh; }
-    if (Fs > 0 && L->umma && T <= L->gemv_max_tokens) {
+    if (Fs > 0 && L->umma && T <= L->gemv_max_tokens && !fused) {
       rs.pf[0] = L->ws13; rs.pf_bytes[0] = (int64_t)2 * Fs * H * (L->fp8 ? 1 : 2);
     }
-    CUDA_TRY(launch_route_small(rs, st));
+    KL_TRY(launch_route_small(rs, st));
     mark(L, ST_PERMUTE, st);
   } else {
     // 1. router logits (bf16 x . bf16 Wg, fp32 accumulate; reading R9)
     if (T <= kGemvMaxTokens) {
-      CUDA_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
+      KL_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
     } else {
       UmmaParams p{};
       UmmaGroup &g = p.g[1];
@@ -802,14 +826,15 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
       p.g[0] = g;
       p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
       const int units = ((T + 127) / 128) * p.nb_s;
-      CUDA_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
+      KL_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
     }
     mark(L, ST_LOGITS, st);
     // 2. scores + group-limited top-k + weights
-    CUDA_TRY(launch_router_select(r, st));
+    KL_TRY(launch_router_select(r, st));
     mark(L, ST_SELECT, st);
     // 3. count / scan / permute
-    CUDA_TRY(launch_permute(pa, st));
+    KL_TRY(launch_permute(pa, st));
+    L->n_launch += 2;                            // count + scan + assign kernels
     mark(L, ST_PERMUTE, st);
   }
   const int64_t pairs = (int64_t)T * k;
@@ -825,10 +850,64 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
       d.xperm_s = L->umma ? nullptr : L->xperm_s;
       d.xq = L->xq; d.xs = L->xs; d.xq_img = L->umma ? L->xq_img : nullptr; d.xq_img_stride = L->img_tiles_sh;
     }
-    CUDA_TRY(launch_scatter_rows(x, T, H, k, L->pos, d, st));
+    KL_TRY(launch_scatter_rows(x, T, H, k, L->pos, d, st));
     mark(L, ST_GATHER, st);
   }
-  if (decode && L->umma) {
+  if (fused) {
+    // 5+6+7 (decode). one weight stream per (slot, 128-column chunk): W13 -> SwiGLU -> h in smem ->
+    // W2 -> weighted fp32 sums (umma_decode_fused.cu), then residual / deferral / bf16 in finalize
+    const bool f8 = L->fp8;
+    FusedDecodeParams fp{};
+    CUtensorMap xmap;                            // token-order activations, shared by both groups
+    if (f8) {
+      xmap = L->dmap_xq;
+    } else if (!make_kmajor_map(&xmap, x, false, T, H, 16)) {
+      return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
+    }
+    {
+      FdGroup &g = fp.g[0];
+      g.x_map = xmap; g.w13 = (const uint8_t *)L->w13; g.w2 = (const uint8_t *)L->w2;
+      if (f8) {
+        g.w13_img = L->w13_img; g.w13_img_stride = L->w13_img_stride;
+        g.x_img = L->xq_img; g.x_img_stride = L->img_tiles_sh; g.w2_s = L->w2_s;
+      }
+    }
+    if (Fs > 0) {
+      FdGroup &g = fp.g[1];
+      g.x_map = xmap;
+      g.w13 = (const uint8_t *)L->ws13; g.w2 = (const uint8_t *)L->ws2;
+      if (f8) {
+        g.w13_img = L->ws13_img; g.w13_img_stride = 0;
+        g.x_img = L->xq_img; g.x_img_stride = L->img_tiles_sh; g.w2_s = L->ws2_s;
+      }
+      static const int pf_mode = getenv("MOE_DECODE_PF") ? atoi(getenv("MOE_DECODE_PF")) : 0;
+      if (pf_mode == 1) {                        // A/B: shared-expert L2 prefetch during routing
+        fp.pf[0] = L->ws13; fp.pf_bytes[0] = (int64_t)2 * Fs * H * (f8 ? 1 : 2);
+        fp.pf[1] = L->ws2; fp.pf_bytes[1] = (int64_t)H * Fs * (f8 ? 1 : 2);
+      }
+    } else {
+      fp.g[1] = fp.g[0];
+    }
+    fp.nch[0] = F / 128; fp.nch[1] = Fs / 128;
+    fp.H = H; fp.T = T; fp.k = k; fp.n_imm = deferred_out ? k - n_def : k; fp.has_shared = Fs > 0;
+    fp.n_active = L->n_active; fp.act_list = L->act_list;
+    fp.topk_idx = L->topk_idx; fp.e0 = L->e0; fp.topk_w = L->topk_w;
+    fp.sgate = L->cfg.shared_gated ? L->sgate : nullptr;
+    float *acc_imm = L->dacc, *acc_def = L->dacc + (size_t)L->gemv_max_tokens * H;
+    fp.acc_imm = acc_imm; fp.acc_def = acc_def;
+    fp.sched = L->sched + 5; fp.done = L->sched + 6;
+    fp.trace = L->trace;
+    const int units = (Fs > 0 ? Fs / 128 : 0) + (int)std::min<int64_t>(E, pairs) * (F / 128);
+    KL_TRY(launch_umma_decode_fused(f8, fp, std::min(L->num_sms, units), st));
+    mark(L, ST_GEMM1, st);
+    DecodeFinalizeArgs fa{};
+    fa.T = T; fa.H = H; fa.use_def = deferred_out != nullptr && n_def > 0;
+    fa.acc_imm = acc_imm; fa.acc_def = acc_def;
+    fa.residual = residual; fa.deferred_in = deferred_in; fa.y = y; fa.deferred_out = deferred_out;
+    fa.trace = L->trace;
+    KL_TRY(launch_decode_finalize(fa, st));
+    mark(L, ST_COMBINE, st);
+  } else if (decode && L->umma) {
     // 5+6 (decode). swap-AB tensor-core weight stream over the active experts + shared expert
     const bool f8 = L->fp8;
     const int kdiv = f8 ? 128 : 64;
@@ -861,7 +940,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     d1.max_slots = slots; d1.has_shared = Fs > 0; d1.T = T;
     d1.n_active = L->n_active; d1.act_list = L->act_list; d1.counts = L->counts; d1.offs_pad = L->offs_pad;
     d1.sched = L->sched + 3;
-    CUDA_TRY(launch_umma_decode(f8, 1, d1, std::min(L->num_sms, slots * d1.nblk), st));
+    KL_TRY(launch_umma_decode(f8, 1, d1, std::min(L->num_sms, slots * d1.nblk), st));
     mark(L, ST_GEMM1, st);
     UmmaDecodeParams d2 = d1;
     {
@@ -883,7 +962,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     }
     d2.g_nblk[0] = H / 128; d2.g_nblk[1] = H / 128; d2.nblk = H / 128;
     d2.sched = L->sched + 4;
-    CUDA_TRY(launch_umma_decode(f8, 2, d2, std::min(L->num_sms, slots * d2.nblk), st));
+    KL_TRY(launch_umma_decode(f8, 2, d2, std::min(L->num_sms, slots * d2.nblk), st));
     mark(L, ST_GEMM2, st);
   } else if (decode) {
     // 5+6 (decode, CUDA-core path). weight-streaming GEMVs over the active experts + shared expert
@@ -895,9 +974,9 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     g.w13_s = L->w13_s; g.w2_s = L->w2_s; g.ws13_s = L->ws13_s; g.ws2_s = L->ws2_s;
     g.h = L->hbuf; g.hsh = L->hsh; g.h_s = L->h_s; g.hsh_s = L->hsh_s; g.yperm = L->yperm; g.ysh = L->ysh;
     const int slots = (int)std::min<int64_t>(E, pairs) + (Fs > 0 ? 1 : 0);
-    CUDA_TRY(launch_gemv(g, 1, slots, st));
+    KL_TRY(launch_gemv(g, 1, slots, st));
     mark(L, ST_GEMM1, st);
-    CUDA_TRY(launch_gemv(g, 2, slots, st));
+    KL_TRY(launch_gemv(g, 2, slots, st));
     mark(L, ST_GEMM2, st);
   } else {
     // 5+6. routed experts (sorted rows) + shared expert (all T tokens)
@@ -905,15 +984,16 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     if (gs != MOE_OK) return gs;
   }
   // 7. weighted combine + residual (+ deferral split)
-  {
+  if (!fused) {
     CombineArgs c{};
     c.T = T; c.H = H; c.k = k; c.n_imm = deferred_out ? k - n_def : k;
     c.pos = L->pos; c.topk_w = L->topk_w; c.yperm = L->yperm;
     c.ysh = Fs > 0 ? L->ysh : nullptr; c.sgate = L->cfg.shared_gated ? L->sgate : nullptr;
     c.residual = residual; c.deferred_in = deferred_in; c.y = y; c.deferred_out = deferred_out;
-    CUDA_TRY(launch_combine(c, st));
+    KL_TRY(launch_combine(c, st));
     mark(L, ST_COMBINE, st);
   }
+  (decode ? L->launches_decode : L->launches_prefill) = L->n_launch;
   if (dbg) {
     if (dbg->topk_idx)
       CUDA_TRY(cudaMemcpyAsync(dbg->topk_idx, L->topk_idx, pairs * 4, cudaMemcpyDeviceToDevice, st));
@@ -1031,6 +1111,16 @@ const char *moe_stage_name(int32_t i) {
   return (i >= 0 && i < moe_layer::kStages) ? kStageNames[i] : "";
 }
 
+// timing experiments (MOE_DEBUG_TRACE): copy the device timeline buffer (4096 u64) to the host
+moe_status moe_layer_debug_trace(moe_layer *L, void *host, int32_t cap) {
+  if (!L || !host) return fail(MOE_ERR_INVALID_ARG, "null argument");
+  if (!L->trace) return fail(MOE_ERR_UNSUPPORTED, "layer created without MOE_DEBUG_TRACE");
+  CUDA_TRY(cudaDeviceSynchronize());
+  CUDA_TRY(cudaMemcpy(host, L->trace, (size_t)std::min(cap, 4096) * 8, cudaMemcpyDeviceToHost));
+  CUDA_TRY(cudaMemset(L->trace, 0, 4096 * 8));
+  return MOE_OK;
+}
+
 moe_status moe_layer_destroy(moe_layer *L) {
   if (!L) return MOE_OK;
   cudaSetDevice(L->cfg.device);
@@ -1046,8 +1136,8 @@ moe_status moe_layer_get_info(const moe_layer *L, moe_layer_info *info) {
   info->weight_bytes = L->weight_bytes;
   info->workspace_bytes = L->workspace_bytes;
   info->gemv_max_tokens = L->gemv_max_tokens;
-  info->kernels_per_forward_prefill = 9 + (L->fp8 ? 1 : 0) + (L->Fs > 0 ? 2 : 0);
-  info->kernels_per_forward_decode = info->kernels_per_forward_prefill;
+  info->kernels_per_forward_prefill = L->launches_prefill;   // counted by the last forward of each kind
+  info->kernels_per_forward_decode = L->launches_decode;
   info->local_experts = L->E;
   return MOE_OK;
 }

@@ -20,7 +20,7 @@ constexpr int RT_WARPS = 4;
 
 // (v, i) better than (v2, i2): larger value, then smaller index
 __device__ __forceinline__ bool better(float v, int i, float v2, int i2) {
-  return v > v2 || (v == v2 && i < i2);
+  return (v > v2) | ((v == v2) & (i < i2));
 }
 
 __device__ __forceinline__ void warp_argmax(float &v, int &i) {
@@ -151,170 +151,6 @@ router_select_kernel(const __grid_constant__ RouterArgs a) {
   select_token(a, t, smem + warp * 2 * a.E, smem + warp * 2 * a.E + a.E, lane);
 }
 
-// Block-parallel routing of ONE token (decode): every thread owns <= 4 experts;
-// selection by rank (rank(e) = #experts that beat e) instead of k sequential
-// arg-max rounds, so the latency is a few short loops over shared memory.
-// Same rules and tie-breaks as select_token.  Scratch: s[E], sel[E], gsc[32],
-// ids[32], ws[32] in shared memory.
-template <int NT>
-__device__ void select_token_block(const RouterArgs &args, int t, float *s, float *sel, float *gsc, int *ids,
-                                   float *ws, long long *ck = nullptr) {
-  if (ck && threadIdx.x == 0) ck[0] = clock64();
-  const int E = args.E, k = args.k, G = args.n_group, TG = args.topk_group;
-  const float *lg = args.logits + (int64_t)t * args.ldl;
-  const float *bias = args.bias;
-  const int tid = threadIdx.x;
-  __shared__ float red[NT / 32];
-  // scores
-  float lv[4];
-#pragma unroll
-  for (int i = 0; i < 4; ++i) lv[i] = (tid + NT * i < E) ? lg[tid + NT * i] : -INFINITY;
-  if (args.score_fn == MOE_SCORE_SOFTMAX) {
-    float m = fmaxf(fmaxf(lv[0], lv[1]), fmaxf(lv[2], lv[3]));
-    m = warp_max(m);
-    if ((tid & 31) == 0) red[tid >> 5] = m;
-    __syncthreads();
-    m = red[0];
-#pragma unroll 1
-    for (int w = 1; w < NT / 32; ++w) m = fmaxf(m, red[w]);
-    __syncthreads();
-    float sum = 0.f;
-#pragma unroll
-    for (int i = 0; i < 4; ++i) { lv[i] = (tid + NT * i < E) ? expf(lv[i] - m) : 0.f; sum += lv[i]; }
-    sum = warp_sum(sum);
-    if ((tid & 31) == 0) red[tid >> 5] = sum;
-    __syncthreads();
-    sum = 0.f;
-#pragma unroll 1
-    for (int w = 0; w < NT / 32; ++w) sum += red[w];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) lv[i] = lv[i] / sum;
-  } else {
-#pragma unroll
-    for (int i = 0; i < 4; ++i) lv[i] = 1.f / (1.f + expf(-lv[i]));
-  }
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const int e = tid + NT * i;
-    if (e < E) { s[e] = lv[i]; sel[e] = lv[i] + (bias ? bias[e] : 0.f); }
-  }
-  __syncthreads();
-  if (ck && threadIdx.x == 0) ck[1] = clock64();
-  // group limit: thread g scores group g, then ranks it
-  if (G > 1) {
-    const int gs = E / G;
-    if (gs == 32 && E <= NT) {
-      // one warp per group (DeepSeek-V3: 256 experts / 8 groups): warp reductions
-      const int lane = tid & 31, g = tid >> 5;
-      if (g < G) {
-        const float v = sel[tid];
-        const float m1 = warp_max(v);
-        const int nmax = __popc(__ballot_sync(0xffffffffu, v == m1));
-        const float m2 = nmax >= 2 ? m1 : warp_max(v == m1 ? -INFINITY : v);
-        if (lane == 0) gsc[g] = args.group_score == MOE_GROUP_TOP2_SUM ? m1 + m2 : m1;
-      }
-    } else if (tid < G) {
-      float m1 = -INFINITY, m2 = -INFINITY;
-#pragma unroll 1
-      for (int i = 0; i < gs; ++i) {
-        const float v = sel[tid * gs + i];
-        if (v > m1) { m2 = m1; m1 = v; } else if (v > m2) { m2 = v; }
-      }
-      gsc[tid] = args.group_score == MOE_GROUP_TOP2_SUM ? m1 + m2 : m1;
-    }
-    __syncthreads();
-    if (tid < G) {
-      int rk = 0;
-#pragma unroll 1
-      for (int g = 0; g < G; ++g) rk += better(gsc[g], g, gsc[tid], tid);
-      ids[tid] = rk < TG;                          // keep flag
-    }
-    __syncthreads();
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int e = tid + NT * i;
-      if (e < E && !ids[e / gs]) sel[e] = -INFINITY;
-    }
-    __syncthreads();
-    if (ck && threadIdx.x == 0) ck[2] = clock64();
-  }
-  // top-k in two warp-level rounds (short loops: this tail runs once, on one SM,
-  // with a cold instruction cache): (1) every warp extracts the k best of its
-  // <= 128 experts by k arg-max rounds; (2) warp 0 merges the NT/32 candidate
-  // lists the same way.  Masked (-inf) experts never qualify.
-  {
-    __shared__ float cv[NT / 32][32];
-    __shared__ int ci[NT / 32][32];
-    const int lane = tid & 31, w = tid >> 5;
-    float v[4];
-    int id[4];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int e = tid + NT * i;
-      const float x = e < E ? sel[e] : -INFINITY;
-      v[i] = x; id[i] = x == -INFINITY ? 0x7fffffff : e;
-    }
-#pragma unroll 1
-    for (int r = 0; r < k; ++r) {
-      float bv = v[0]; int bi = id[0];
-#pragma unroll
-      for (int i = 1; i < 4; ++i) if (better(v[i], id[i], bv, bi)) { bv = v[i]; bi = id[i]; }
-      warp_argmax(bv, bi);
-      if (lane == 0) { cv[w][r] = bv; ci[w][r] = bi; }
-#pragma unroll
-      for (int i = 0; i < 4; ++i) if (id[i] == bi) { v[i] = -INFINITY; id[i] = 0x7fffffff; }
-    }
-    __syncthreads();
-    if (ck && threadIdx.x == 0) ck[3] = clock64();
-    if (w == 0) {
-      // candidates: NT/32 lists of k <= 32 -> <= NT/32 per lane
-      constexpr int NC = NT / 32;
-      float mv[NC]; int mi[NC];
-#pragma unroll
-      for (int i = 0; i < NC; ++i) {
-        const int c = lane + 32 * i;              // candidate index = list * k + rank
-        const bool ok = c < (NT / 32) * k;
-        mv[i] = ok ? cv[c / k][c % k] : -INFINITY;
-        mi[i] = ok ? ci[c / k][c % k] : 0x7fffffff;
-      }
-#pragma unroll 1
-      for (int r = 0; r < k; ++r) {
-        float bv = mv[0]; int bi = mi[0];
-#pragma unroll
-        for (int i = 1; i < NC; ++i) if (better(mv[i], mi[i], bv, bi)) { bv = mv[i]; bi = mi[i]; }
-        warp_argmax(bv, bi);
-        if (lane == 0) { ids[r] = bi; ws[r] = s[bi]; }
-#pragma unroll
-        for (int i = 0; i < NC; ++i) if (mi[i] == bi) { mv[i] = -INFINITY; mi[i] = 0x7fffffff; }
-      }
-    }
-  }
-  __syncthreads();
-  if (ck && threadIdx.x == 0) ck[4] = clock64();
-  // weights + canonical order (warp 0)
-  if (tid < 32) {
-    const int lane = tid;
-    const int my_id = lane < k ? ids[lane] : 0x7fffffff;
-    float w = lane < k ? ws[lane] : 0.f;
-    if (args.norm_topk) w = w / warp_sum(w);
-    w = w * args.routed_scale;
-    int rank = 0;
-#pragma unroll 1
-    for (int i = 0; i < k; ++i) {
-      const float wi = __shfl_sync(0xffffffffu, w, i);
-      const int ii = __shfl_sync(0xffffffffu, my_id, i);
-      if (lane < k && i != lane && better(wi, ii, w, my_id)) ++rank;
-    }
-    if (lane < k) {
-      args.topk_idx[(int64_t)t * k + rank] = my_id;
-      args.topk_w[(int64_t)t * k + rank] = w;
-    }
-    if (args.shared_gated && lane == 0) args.sgate[t] = 1.f / (1.f + expf(-lg[E]));
-  }
-  __syncthreads();
-  if (ck && threadIdx.x == 0) ck[5] = clock64();
-}
-
 // ------------------------------------------------------------------ small T (decode)
 // One launch for T <= 16 tokens: every CTA computes the router logits of two
 // router rows (128 threads per row, whole row loaded at once), the last CTA to
@@ -322,6 +158,351 @@ __device__ void select_token_block(const RouterArgs &args, int t, float *s, floa
 // (counts, offsets, active-expert list, stable positions) -- the launch chain
 // logits -> select -> count/scan/assign collapsed for the latency-bound decode step.
 constexpr int RS_THREADS = 256;
+__device__ __forceinline__ unsigned long long gtimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+constexpr int RS_MAX_E = 256;      // router experts per lane-major warp layout: 32 lanes x 8
+constexpr int RS_MAX_PAIRS = 512;  // T * k
+
+// One warp routes token t with everything in registers (lane l holds experts
+// 8l .. 8l+7): scores, group limit, k arg-max rounds, weights and the
+// canonical slot order (same rules and tie-breaks as select_token).
+// scratch: E floats of this warp's shared memory.  Writes topk_idx / topk_w /
+// sgate and the canonical ids into ids_s[t * k ..].
+// Control flow is warp-uniform throughout (live only predicates the stores), so the
+// shuffles compile to plain SHFL, not the collective-emulated form.
+#ifdef SELECT_PROFILE
+__device__ long long g_sel_ck[8];
+#define SEL_CK(i) do { if (lane == 0) g_sel_ck[i] = clock64(); } while (0)
+#else
+#define SEL_CK(i) do { } while (0)
+#endif
+// (sel, id) -> 64-bit key, larger = better: order-preserving float bits, then
+// the complemented id (ties -> lower expert id, reading R2)
+__device__ __forceinline__ unsigned long long sel_key(float v, int id) {
+  const uint32_t u = __float_as_uint(v);
+  const uint32_t o = (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+  return ((unsigned long long)o << 32) | (uint32_t)(~(uint32_t)id);
+}
+__device__ __forceinline__ int key_id(unsigned long long key) { return (int)~(uint32_t)key; }
+
+__device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, int *ids_s, int lane, bool live) {
+  const int E = r.E, k = r.k, G = r.n_group;
+  SEL_CK(0);
+  const float *lg = r.logits + (int64_t)t * r.ldl;
+  float *s_sm = scratch;                         // [E] unbiased scores
+  float *sel_sm = scratch + RS_MAX_E;            // [E] selection scores (group pass)
+  float lv[8], bv[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int e = lane * 8 + i;
+    lv[i] = e < E ? lg[e] : -INFINITY;
+    bv[i] = (e < E && r.bias) ? r.bias[e] : 0.f;
+  }
+  float s[8], sel[8];
+  if (r.score_fn == MOE_SCORE_SOFTMAX) {
+    float m = lv[0];
+#pragma unroll
+    for (int i = 1; i < 8; ++i) m = fmaxf(m, lv[i]);
+    m = warp_max(m);
+    float sum = 0.f;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) { s[i] = lane * 8 + i < E ? expf(lv[i] - m) : 0.f; sum += s[i]; }
+    sum = warp_sum(sum);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) s[i] = s[i] / sum;
+  } else {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) s[i] = 1.f / (1.f + expf(-lv[i]));
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int e = lane * 8 + i;
+    sel[i] = e < E ? s[i] + bv[i] : -INFINITY;
+    if (e < E) { s_sm[e] = s[i]; sel_sm[e] = sel[i]; }
+  }
+  __syncwarp();
+  SEL_CK(1);
+  if (G > 1) {
+    // group g = experts [g gs, (g+1) gs): lane g scans it (branch-free top-2)
+    const int gs = E / G;
+    float m1 = -INFINITY, m2 = -INFINITY;
+    if (lane < G) {
+      const float *gp = sel_sm + lane * gs;
+#pragma unroll 8
+      for (int i = 0; i < gs; ++i) {
+        const float v = gp[i];
+        m2 = fmaxf(m2, fminf(m1, v));
+        m1 = fmaxf(m1, v);
+      }
+    }
+    const float gsc = lane < G ? (r.group_score == MOE_GROUP_TOP2_SUM ? m1 + m2 : m1) : -INFINITY;
+    int rk = 0;
+#pragma unroll 8
+    for (int j = 0; j < G; ++j) rk += better(__shfl_sync(0xffffffffu, gsc, j), j, gsc, lane);
+    const unsigned keep = __ballot_sync(0xffffffffu, lane < G && rk < r.topk_group);
+    int g = (lane * 8) / gs, rem = (lane * 8) - g * gs;   // group of expert 8 lane, walked forward
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      sel[i] = (g < 32 && ((keep >> g) & 1u)) ? sel[i] : -INFINITY;
+      ++rem;
+      const bool nx = rem == gs;
+      g += nx;
+      rem = nx ? 0 : rem;
+    }
+  }
+  SEL_CK(2);
+  int my_id = 0;
+  float my_w = 0.f;
+  int rank = 0;
+  if (k <= 8) {
+    // top-k by a sorting network on 64-bit keys: each lane sorts its 8, then five
+    // butterfly steps merge partner lists (bitonic: keep the better of A[i] and
+    // B[7-i], then sort the bitonic 8) -- every lane ends with the token's best 8
+    // in (sel desc, id asc) order.  Branch-free: divergence around the shuffles
+    // makes them collective-emulated (measured ~5x the cycles).
+    unsigned long long key[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) key[i] = sel[i] == -INFINITY ? 0ull : sel_key(sel[i], lane * 8 + i);
+    auto cx = [&](int i, int j) {
+      const unsigned long long a = key[i], b = key[j];
+      key[i] = a > b ? a : b;
+      key[j] = a > b ? b : a;
+    };
+    // Batcher odd-even merge sort of 8 (19 comparators)
+    cx(0, 1); cx(2, 3); cx(4, 5); cx(6, 7);
+    cx(0, 2); cx(1, 3); cx(4, 6); cx(5, 7);
+    cx(1, 2); cx(5, 6);
+    cx(0, 4); cx(1, 5); cx(2, 6); cx(3, 7);
+    cx(2, 4); cx(3, 5);
+    cx(1, 2); cx(3, 4); cx(5, 6);
+    SEL_CK(3);
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      unsigned long long pk[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) pk[i] = __shfl_xor_sync(0xffffffffu, key[i], o);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) key[i] = key[i] > pk[7 - i] ? key[i] : pk[7 - i];
+      cx(0, 4); cx(1, 5); cx(2, 6); cx(3, 7);
+      cx(0, 2); cx(1, 3); cx(4, 6); cx(5, 7);
+      cx(0, 1); cx(2, 3); cx(4, 5); cx(6, 7);
+    }
+    SEL_CK(4);
+    // weights and canonical order, lane-local (every lane holds the list)
+    float sv[8], sum = 0.f;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      sv[i] = i < k ? s_sm[key_id(key[i])] : 0.f;
+      sum += sv[i];
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const float w = (r.norm_topk ? sv[i] / sum : sv[i]) * r.routed_scale;
+      const int id = key_id(key[i]);
+      my_id = i == lane ? id : my_id;
+      my_w = i == lane ? w : my_w;
+      sv[i] = w;
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) rank += (i < k) & (i != lane) & better(sv[i], key_id(key[i]), my_w, my_id);
+  } else {
+    // k > 8: k arg-max rounds; the owner lane retires the winner
+    my_id = 0x7fffffff;
+#pragma unroll 1
+    for (int j = 0; j < k; ++j) {
+      float v = -INFINITY;
+      int id = 0x7fffffff;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const bool b = better(sel[i], lane * 8 + i, v, id) & (sel[i] != -INFINITY);
+        v = b ? sel[i] : v;
+        id = b ? lane * 8 + i : id;
+      }
+      warp_argmax(v, id);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) sel[i] = lane * 8 + i == id ? -INFINITY : sel[i];
+      my_id = lane == j ? id : my_id;
+    }
+    float w = lane < k ? s_sm[my_id] : 0.f;
+    if (r.norm_topk) w = w / warp_sum(w);
+    my_w = w * r.routed_scale;
+#pragma unroll 1
+    for (int i = 0; i < k; ++i) {
+      const float wi = __shfl_sync(0xffffffffu, my_w, i);
+      const int ii = __shfl_sync(0xffffffffu, my_id, i);
+      rank += (i != lane) & better(wi, ii, my_w, my_id);
+    }
+  }
+  if (live && lane < k) {
+    r.topk_idx[(int64_t)t * k + rank] = my_id;
+    r.topk_w[(int64_t)t * k + rank] = my_w;
+    ids_s[t * k + rank] = my_id;
+  }
+  if (live && r.shared_gated && lane == 0) r.sgate[t] = 1.f / (1.f + expf(-lg[E]));
+  SEL_CK(5);
+  __syncwarp();                                  // scratch reuse by the next token of this warp
+}
+
+// The last router CTA: route every token (one warp per token), then the
+// expert-sorted order for T <= 16 tokens -- with at most T <= kPadM rows per
+// expert every active expert's padded segment is one 128-row tile, so its
+// position is (number of active experts below it) x 128, read off a bitmap of
+// the active experts; a pair's row within the segment is the number of
+// earlier tokens that chose the same expert (stable by token).  Finally the
+// token rows (FP8: the codes quantised by all CTAs) are copied to their k rows.
+__device__ void route_small_tail(const RouteSmallArgs &a, float *rsm) {
+  const RouterArgs &r = a.r;
+  const PermuteArgs &p = a.p;
+  const int T = r.T, k = r.k, TK = T * k, H = a.H;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  __shared__ int ids_s[RS_MAX_PAIRS], pos_s[RS_MAX_PAIRS];
+  __shared__ int cnt_s[RS_MAX_E], slot_s[RS_MAX_E], offs_s[RS_MAX_E];
+  __shared__ unsigned bm[RS_MAX_E / 32];
+  long long ck[4];
+  ck[0] = clock64();
+  if (a.trace && tid == 0) a.trace[1] = gtimer_ns();
+  for (int e = tid; e < p.E; e += RS_THREADS) cnt_s[e] = 0;
+  if (tid < RS_MAX_E / 32) bm[tid] = 0u;
+  // uniform trip count; a warp past the last token re-routes token T-1 without storing
+#pragma unroll 1
+  for (int t0 = 0; t0 < T; t0 += RS_THREADS / 32)
+    select_token_regs(r, min(t0 + warp, T - 1), rsm + warp * 2 * RS_MAX_E, ids_s, lane, t0 + warp < T);
+  __syncthreads();
+  ck[1] = clock64();
+  if (a.trace && tid == 0) a.trace[2] = gtimer_ns();
+  if (a.debug & 8) {                             // timing experiment: a second (warm i-cache) select pass
+    const long long w0 = clock64();
+#pragma unroll 1
+    for (int t0 = 0; t0 < T; t0 += RS_THREADS / 32)
+      select_token_regs(r, min(t0 + warp, T - 1), rsm + warp * 2 * RS_MAX_E, ids_s, lane, t0 + warp < T);
+    __syncthreads();
+    if (a.trace && tid == 0) { a.trace[5] = ck[1] - ck[0]; a.trace[6] = clock64() - w0; }
+  }
+  for (int q = tid; q < TK; q += RS_THREADS) {
+    const int e = ids_s[q] - p.e0;
+    if (e >= 0 && e < p.E) {
+      atomicAdd(&cnt_s[e], 1);
+      atomicOr(&bm[e >> 5], 1u << (e & 31));
+    }
+  }
+  __syncthreads();
+  if (a.minimal && !p.dbg_perm && !p.dbg_counts) {
+    // fused decode: the expert kernel reads token-order activations and finds its
+    // tokens in topk_idx, so only the active-expert list is needed (ascending ids)
+    const int e = tid;
+    int below = 0, nact = 0;
+#pragma unroll
+    for (int w = 0; w < RS_MAX_E / 32; ++w) {
+      const int pc = __popc(bm[w]);
+      nact += pc;
+      if (w < (e >> 5)) below += pc;
+    }
+    if (e < p.E && ((bm[e >> 5] >> (e & 31)) & 1u))
+      p.act_list[below + __popc(bm[e >> 5] & ((1u << (e & 31)) - 1u))] = e;
+    if (tid == 0) {
+      *p.n_active = nact;
+      *a.done = 0;                                 // re-arm the CTA counter (graph replay)
+    }
+    if (a.trace && tid == 0) { a.trace[3] = gtimer_ns(); a.trace[4] = a.trace[3]; }
+    return;
+  }
+  {
+    using Scan = cub::BlockScan<int, RS_THREADS>;
+    __shared__ typename Scan::TempStorage tmp;
+    const int e = tid;
+    const int c = e < p.E ? cnt_s[e] : 0;
+    int o, tot;
+    Scan(tmp).ExclusiveSum(c, o, tot);
+    int below = 0, nact = 0;
+#pragma unroll
+    for (int w = 0; w < RS_MAX_E / 32; ++w) {
+      const int pc = __popc(bm[w]);
+      nact += pc;
+      if (w < (e >> 5)) below += pc;
+    }
+    if (e < p.E) {
+      const int slot = below + __popc(bm[e >> 5] & ((1u << (e & 31)) - 1u));
+      p.counts[e] = c;
+      p.offs[e] = o;
+      p.offs_pad[e] = slot * kPadM;
+      if (p.dbg_counts) p.dbg_counts[e] = c;
+      if (c > 0) p.act_list[slot] = e;
+      slot_s[e] = slot;
+      offs_s[e] = o;
+    }
+    if (tid == 0) {
+      p.offs[p.E] = tot;
+      p.offs_pad[p.E] = nact * kPadM;
+      *p.n_active = nact;
+      *p.n_tiles = 0;
+      *a.done = 0;                                 // re-arm the CTA counter (graph replay)
+    }
+  }
+  __syncthreads();
+  for (int q = tid; q < TK; q += RS_THREADS) {
+    const int id = ids_s[q], e = id - p.e0, t = q / k;
+    int rw = -1;
+    if (e >= 0 && e < p.E) {
+      int i = 0;
+#pragma unroll 1
+      for (int q2 = 0; q2 < t * k; ++q2) i += ids_s[q2] == id;
+      rw = slot_s[e] * kPadM + i;
+      p.row_token[rw] = t;
+      if (p.dbg_perm) p.dbg_perm[offs_s[e] + i] = t;
+    }
+    p.pos[q] = rw;
+    pos_s[q] = rw;
+  }
+  __syncthreads();
+  ck[2] = clock64();
+  if (a.trace && tid == 0) a.trace[3] = gtimer_ns();
+  if (a.xperm) {
+    if (a.fp8) {
+      // codes were quantised into xq by all CTAs: every thread loads its chunks
+      // (<= 4: H <= 16384) and scale byte of a token row once, then stores k times
+#pragma unroll 1
+      for (int t = 0; t < T; ++t) {
+        const uint4 *src = reinterpret_cast<const uint4 *>(reinterpret_cast<const uint8_t *>(a.xq) + (size_t)t * H);
+        uint4 v[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int c = tid + RS_THREADS * i;
+          if (c < H / 16) v[i] = src[c];
+        }
+        const int b = tid;
+        const uint8_t sb = b < H / 128 ? (uint8_t)((__float_as_uint(a.xs[(size_t)t * (H / 128) + b]) >> 23) & 0xFF) : 0;
+#pragma unroll 1
+        for (int j = 0; j < k; ++j) {
+          const int rw = pos_s[t * k + j];
+          if (rw < 0) continue;
+          uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<uint8_t *>(a.xperm) + (size_t)rw * H);
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const int c = tid + RS_THREADS * i;
+            if (c < H / 16) dst[c] = v[i];
+          }
+          if (b < H / 128) a.xperm_img[sf_img_off(rw, b, a.xperm_img_stride)] = sb;
+        }
+      }
+    } else {
+      ScatterDst d{};
+      d.fp8 = 0; d.xperm = a.xperm;
+#pragma unroll 1
+      for (int t = 0; t < T; ++t)
+        scatter_token_row<RS_THREADS>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H, H, t, k,
+                                      pos_s + t * k, d);
+    }
+  }
+  ck[3] = clock64();
+  if (a.trace && tid == 0) a.trace[4] = gtimer_ns();
+  if ((a.debug & 4) && tid == 0)                 // MOE_DEBUG_ROUTE=4: phase cycle counts of the tail
+    printf("route tail cycles: select %lld permute %lld rows %lld\n", ck[1] - ck[0], ck[2] - ck[1], ck[3] - ck[2]);
+}
+
+
 
 __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_constant__ RouteSmallArgs a) {
   extern __shared__ float rsm[];
@@ -331,10 +512,22 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   const int row = blockIdx.x * 2 + half;
   __shared__ float red[2][4][16];
   __shared__ int is_last;
+  // router weights first: they do not depend on the predecessor kernel, so with
+  // PDL their HBM latency overlaps the previous layer's tail
+  const int w4 = tid >> 5, lane = threadIdx.x & 31;
+  const int nv = H / 8;
+  uint4 w[8];
+  {
+    const bool live = row < a.rows && !(a.debug & 1);
+    const uint4 *wr = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.wg) + (size_t)row * H);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) w[u] = (live && tid + u * 128 < nv) ? __ldg(wr + tid + u * 128) : make_uint4(0, 0, 0, 0);
+  }
   pdl_trigger();
+  pdl_wait();                                    // x (the previous layer's output) and our workspaces
+  if (a.trace && threadIdx.x == 0 && blockIdx.x == 0) a.trace[0] = gtimer_ns();
   // the shared expert's weights do not depend on the routing: pull them into
-  // L2 now (HBM is otherwise idle while the router runs), so the first units
-  // of the decode weight stream hit L2
+  // L2 now (two-launch decode chain only)
   if (threadIdx.x == 0) {
 #pragma unroll 1
     for (int i = 0; i < 2; ++i) {
@@ -349,16 +542,7 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
     }
   }
   // ---- logits of router rows `row` for all T tokens ----
-  // (H <= 8192: each thread's <= 8 16-byte chunks of the row are loaded once,
-  //  then a runtime loop over the tokens -- no per-token register arrays)
   {
-    const int w4 = tid >> 5, lane = threadIdx.x & 31;
-    const int nv = H / 8;
-    uint4 w[8];
-    const bool live = row < a.rows && !(a.debug & 1);
-    const uint4 *wr = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.wg) + (size_t)row * H);
-#pragma unroll
-    for (int u = 0; u < 8; ++u) w[u] = (live && tid + u * 128 < nv) ? __ldg(wr + tid + u * 128) : make_uint4(0, 0, 0, 0);
 #pragma unroll 1
     for (int t = 0; t < T; ++t) {
       const uint4 *xr = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H);
@@ -421,157 +605,36 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   }
 
   // ---- last CTA: route + permute ----
-  __threadfence();
+  // (one gpu-scope acq_rel fence by the ticket thread after the CTA barrier orders
+  //  every thread's logits / xq stores before the ticket, and the last CTA's reads after)
   __syncthreads();
-  if (threadIdx.x == 0) is_last = (atomicAdd(a.done, 1) == (int)gridDim.x - 1);
+  if (threadIdx.x == 0) {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+    const int tk = atomicAdd(a.done, 1);
+    is_last = tk == (int)gridDim.x - 1;
+    if (is_last) asm volatile("fence.acq_rel.gpu;" ::: "memory");
+  }
   __syncthreads();
   if (!is_last) return;
-  long long ck0 = clock64();
-  __shared__ long long cold_ck[8];
   if (a.debug & 2) { if (threadIdx.x == 0) *a.done = 0; return; }
-  __threadfence();
-  {
-    float *s = rsm, *sel = rsm + r.E, *gsc = rsm + 2 * r.E, *ws = gsc + 32;
-    int *ids = reinterpret_cast<int *>(ws + 32);
-#pragma unroll 1
-    for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws, (a.debug & 4) ? cold_ck : nullptr);
-    if (a.debug & 8) {                           // MOE_DEBUG_ROUTE=12: time a second (warm i-cache) pass
-      __syncthreads();
-      const long long w0 = clock64();
-      unsigned long long g0, g1;
-      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g0));
-      __shared__ long long ck[8];
-#pragma unroll 1
-      for (int t = 0; t < T; ++t) select_token_block<RS_THREADS>(r, t, s, sel, gsc, ids, ws, ck);
-      __syncthreads();
-      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g1));
-      if (threadIdx.x == 0)
-        printf("route tail: warm select pass %lld cycles (%llu ns): scores %lld group %lld warp-topk %lld merge %lld weights %lld\n",
-               clock64() - w0, g1 - g0, ck[1] - ck[0], ck[2] - ck[1], ck[3] - ck[2], ck[4] - ck[3], ck[5] - ck[4]);
-    }
-  }
-  long long ck1 = clock64();
-  {
-  }
-  // counts / offsets / active list over the local experts
-  const PermuteArgs &p = a.p;
-  int *cnt = reinterpret_cast<int *>(rsm);          // reuse scratch: [E] counts, [E] running
-  int *run = cnt + p.E;
-  for (int e = threadIdx.x; e < p.E; e += RS_THREADS) cnt[e] = 0;
-  __syncthreads();
-  for (int q = threadIdx.x; q < T * p.k; q += RS_THREADS) {
-    const int e = p.topk_idx[q] - p.e0;
-    p.pos[q] = -1;
-    if (e >= 0 && e < p.E) atomicAdd(&cnt[e], 1);
-  }
-  __syncthreads();
-  {
-    // one exclusive scan over the experts of a packed triple (count | tiles << 11 |
-    // active << 21): T*k <= 512 rows, <= 1024 tiles and experts -- 4 experts per thread
-    using Scan = cub::BlockScan<int, RS_THREADS>;
-    __shared__ typename Scan::TempStorage tmp;
-    int v[4], o[4], tot;
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int e = threadIdx.x * 4 + i;
-      const int c = e < p.E ? cnt[e] : 0;
-      v[i] = c | (((c + kPadM - 1) / kPadM) << 11) | ((c > 0) << 21);
-    }
-    Scan(tmp).ExclusiveSum(v, o, tot);
-    if (threadIdx.x == 0) {
-      p.offs[p.E] = tot & 2047;
-      p.offs_pad[p.E] = ((tot >> 11) & 1023) * kPadM;
-      *p.n_active = tot >> 21;
-      *p.n_tiles = 0;
-      *a.done = 0;                                 // re-arm the CTA counter (graph replay)
-    }
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int e = threadIdx.x * 4 + i;
-      if (e < p.E) {
-        const int c = v[i] & 2047;
-        p.counts[e] = c;
-        if (p.dbg_counts) p.dbg_counts[e] = c;
-        p.offs[e] = o[i] & 2047;
-        p.offs_pad[e] = ((o[i] >> 11) & 1023) * kPadM;
-        run[e] = 0;
-        if (c > 0) p.act_list[o[i] >> 21] = e;
-      }
-    }
-  }
-  __syncthreads();
-  long long ck2 = clock64();
-  // stable assignment: tokens in order, a token's k experts are distinct
-  for (int t = 0; t < T; ++t) {
-    if (threadIdx.x < p.k) {
-      const int q = t * p.k + threadIdx.x;
-      const int e = p.topk_idx[q] - p.e0;
-      if (e >= 0 && e < p.E) {
-        const int i = run[e]++;
-        const int rw = p.offs_pad[e] + i;
-        p.row_token[rw] = t;
-        p.pos[q] = rw;
-        if (p.dbg_perm) p.dbg_perm[p.offs[e] + i] = t;
-      }
-    }
-    __syncthreads();
-  }
-  if (!a.xperm) return;
-  long long ck3 = clock64();
-  // activations into expert order (replaces the quantise + gather launches)
-  __shared__ int spos[32];
-  ScatterDst d{};
-  d.fp8 = a.fp8; d.xperm = a.xperm; d.xperm_img = a.xperm_img; d.xperm_img_stride = a.xperm_img_stride;
-  d.xq = a.xq; d.xs = a.xs; d.xq_img = a.xq_img; d.xq_img_stride = a.xq_img_stride;
-#pragma unroll 1
-  for (int t = 0; t < T; ++t) {
-    if (threadIdx.x < p.k) spos[threadIdx.x] = p.pos[t * p.k + threadIdx.x];
-    __syncthreads();
-    if (a.fp8) {
-      // codes were quantised into xq by all CTAs: copy the row and its scale bytes
-      // every thread loads its chunks (<= 4: H <= 16384) and scale byte once, then stores k times
-      const uint4 *src = reinterpret_cast<const uint4 *>(reinterpret_cast<const uint8_t *>(a.xq) + (size_t)t * H);
-      uint4 v[4];
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int c = threadIdx.x + RS_THREADS * i;
-        if (c < H / 16) v[i] = src[c];
-      }
-      const int b = threadIdx.x;
-      const uint8_t sb = b < H / 128 ? (uint8_t)((__float_as_uint(a.xs[(size_t)t * (H / 128) + b]) >> 23) & 0xFF) : 0;
-#pragma unroll 1
-      for (int j = 0; j < p.k; ++j) {
-        const int rw = spos[j];
-        if (rw < 0) continue;
-        uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<uint8_t *>(a.xperm) + (size_t)rw * H);
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int c = threadIdx.x + RS_THREADS * i;
-          if (c < H / 16) dst[c] = v[i];
-        }
-        if (b < H / 128) a.xperm_img[sf_img_off(rw, b, a.xperm_img_stride)] = sb;
-      }
-    } else {
-      scatter_token_row<RS_THREADS>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H, H, t, p.k, spos, d);
-    }
-    __syncthreads();
-  }
-  if ((a.debug & 4) && threadIdx.x == 0)       // MOE_DEBUG_ROUTE=4: phase cycle counts of the tail
-    printf("route tail cycles: select %lld (scores %lld group %lld warp-topk %lld merge %lld weights %lld) scan %lld "
-           "assign %lld rows %lld\n", ck1 - ck0, cold_ck[1] - cold_ck[0], cold_ck[2] - cold_ck[1],
-           cold_ck[3] - cold_ck[2], cold_ck[4] - cold_ck[3], cold_ck[5] - cold_ck[4], ck2 - ck1, ck3 - ck2,
-           clock64() - ck3);
+  route_small_tail(a, rsm);
 }
 
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st) {
   if (a.r.T <= 0) return cudaSuccess;
-  const size_t sm = std::max<size_t>((size_t)(RS_THREADS / 32) * 2 * a.r.E * sizeof(float), 2 * a.p.E * sizeof(int));
+  const size_t sm = (size_t)(RS_THREADS / 32) * 2 * RS_MAX_E * sizeof(float);   // per-warp select scratch
+  static bool carve = false;
+  if (!carve) {
+    // max shared-memory carveout: the PDL-launched decode stream kernel (~190 KB
+    // of smem) can then become resident beside the router CTAs
+    cudaFuncSetAttribute(route_small_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    carve = true;
+  }
   if (sm > 48 * 1024) {
     cudaError_t e = cudaFuncSetAttribute(route_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
   }
-  route_small_kernel<<<(a.rows + 1) / 2, RS_THREADS, sm, st>>>(a);
-  return cudaGetLastError();
+  return launch_pdl(route_small_kernel, dim3((a.rows + 1) / 2), dim3(RS_THREADS), sm, st, a);
 }
 
 cudaError_t launch_router_select(const RouterArgs &a, cudaStream_t st) {

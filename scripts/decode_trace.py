@@ -1,0 +1,48 @@
+"""Device timeline of one decode forward (MOE_DEBUG_TRACE=1 set by this script):
+route kernel phases, per-CTA fused-kernel unit phases, finalize (globaltimer ns)."""
+import os, sys, ctypes
+os.environ["MOE_DEBUG_TRACE"] = "1"
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+import torch
+from inputs.presets import PRESETS
+from inputs.synthetic import make_tokens, make_weights
+from paper_conf_sosp_chenxztwdcylqzo25_b200 import moe
+cfg = sys.argv[1] if len(sys.argv) > 1 else "v3"
+T = int(sys.argv[2]) if len(sys.argv) > 2 else 1
+p = PRESETS[cfg]
+w = make_weights(p, "cuda")
+x, _ = make_tokens(p, T, "cuda", offset=5)
+layer = moe.MoELayer(p, w, max_tokens=16)
+lib = layer._lib
+lib.moe_layer_debug_trace.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32]
+buf = np.zeros(4096, dtype=np.uint64)
+y = torch.empty_like(x)
+fw = torch.empty(64 << 20, device="cuda"); fr = torch.zeros(64 << 20, device="cuda"); sink = torch.zeros((), device="cuda")
+for it in range(4):
+    fw.zero_(); torch.sum(fr, 0, out=sink)
+    layer.forward(x, y=y)
+    torch.cuda.synchronize()
+    assert lib.moe_layer_debug_trace(layer._h, buf.ctypes.data, 4096) == 0
+t0 = int(buf[0])
+rel = lambda v: (int(v) - t0) / 1e3
+if buf[6]:
+    print(f"route select cycles: first pass {int(buf[5])}, warm second pass {int(buf[6])}")
+print(f"route: entry 0, tail start {rel(buf[1]):.1f}, select done {rel(buf[2]):.1f}, permute done {rel(buf[3]):.1f}, end {rel(buf[4]):.1f} us")
+cta = buf[8:8 + 8 * 148].reshape(148, 8).astype(np.int64)
+act = cta[cta[:, 5] > 0]
+def st(v):
+    v = np.sort(v); return f"min {v[0]:6.1f} med {v[len(v)//2]:6.1f} max {v[-1]:6.1f}"
+print("fused CTAs with a unit:", len(act))
+for j, name in enumerate(["entry", "past_pdl", "unit", "accA", "h_ready", "unit_end"]):
+    print(f"  {name:9s}", st((act[:, j] - t0) / 1e3))
+print("  phaseA", st((act[:, 3] - act[:, 2]) / 1e3), " epiA", st((act[:, 4] - act[:, 3]) / 1e3),
+      " phaseB", st((act[:, 5] - act[:, 4]) / 1e3))
+sh = act[(act[:, 6] >> 30) == 1]
+if len(sh):
+    print("  shared units end", st((sh[:, 5] - t0) / 1e3))
+order = np.argsort(act[:, 5])[::-1][:8]
+for i in order:
+    u = act[i]
+    print(f"  slowest: sm {u[7]:3d} grp {u[6] >> 30} exp {(u[6] >> 16) & 0x3fff:3d} chunk {u[6] & 0xffff:2d} unit {(u[2]-t0)/1e3:6.1f} accA {(u[3]-t0)/1e3:6.1f} h {(u[4]-t0)/1e3:6.1f} end {(u[5]-t0)/1e3:6.1f}")
+print(f"finalize: past pdl {rel(buf[2000]):.1f}, end {rel(buf[2001]):.1f} us")

@@ -1,0 +1,7 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || exit 1
+timeout 600 python -m pytest tests -m gpu -q -x > gpurun_out/fd12_parity.log 2>&1; echo "rc=$?" >> gpurun_out/fd12_parity.log
+timeout 400 python scripts/decode_ab.py v3 1,4,16 8 > gpurun_out/fd12_ab_L8.log 2>&1
+timeout 200 python scripts/decode_ab.py v3 1 1 > gpurun_out/fd12_ab_L1.log 2>&1
+timeout 200 python scripts/decode_trace.py v3 1 > gpurun_out/fd12_trace.log 2>&1

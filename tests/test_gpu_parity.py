@@ -194,3 +194,43 @@ def test_swap_pair_token_tiles(lib, name, T):
     assert res["routing"]["expert_counts"].max() > 256
     keep = np.setdiff1d(np.arange(T), ties)
     assert rel_l2(res["y"][keep], out["y"][keep]) <= TOL[p.wtype]
+
+
+@pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v2lite_s"])
+@pytest.mark.parametrize("T", [1, 5, 16])
+def test_fused_decode_residual_deferral(lib, name, T):
+    """Fused decode stream (umma_decode_fused.cu): Eq. L241 middle case at decode
+    sizes -- y = I + S + R^imm + R^def_{k-1}, deferred_out = R^def -- vs the oracle,
+    including T = 16 (the N = 16 token operand full)."""
+    p = SMALL[name]
+    n_def = min(3, p.top_k - 1)
+    res = _run(lib, p, T, n_def=n_def, with_deferred_in=True, residual=True, max_tokens=16)
+    out, ties, idx, w = _oracle(p, res, n_def=n_def, residual=True)
+    keep = np.setdiff1d(np.arange(T), ties)
+    assert rel_l2(res["y"][keep], out["y"][keep]) <= TOL[p.wtype]
+    assert rel_l2(res["dout"][keep], out["deferred_out"][keep]) <= TOL[p.wtype]
+
+
+@pytest.mark.parametrize("name", ["v3_s", "qwen2_s"])
+def test_fused_decode_matches_chain_and_repeats(lib, name, monkeypatch):
+    """The fused decode stream and the two-launch chain (MOE_DECODE_CHAIN=1, read at
+    create) agree; repeated fused forwards agree to fp32-atomic rounding (reading R22:
+    the chunk partial sums are added in arrival order)."""
+    p = SMALL[name]
+    T = 7
+    w = make_weights(p, "cpu").to("cuda")
+    x, r = make_tokens(p, T, "cuda", offset=3)
+    fused = lib.MoELayer(p, w, max_tokens=16)
+    monkeypatch.setenv("MOE_DECODE_CHAIN", "1")
+    chain = lib.MoELayer(p, w, max_tokens=16)
+    monkeypatch.delenv("MOE_DECODE_CHAIN")
+    ya = fused.forward(x, residual=r).float()
+    yb = fused.forward(x, residual=r).float()
+    yc = chain.forward(x, residual=r).float()
+    torch.cuda.synchronize()
+    assert rel_l2(ya.cpu().numpy(), yc.cpu().numpy()) <= TOL[p.wtype]
+    # bf16 outputs of two fused runs: at most a rounding step apart
+    d = (ya - yb).abs().max().item()
+    assert d <= 2 ** -6 * max(1.0, ya.abs().max().item()), d
+    fused.close()
+    chain.close()
