@@ -52,7 +52,10 @@ def launches(path, prefix):
     rows = list(csv.reader(io.StringIO("".join(lines))))
     h = rows[0]
     ki, vi, ui = h.index("Kernel Name"), h.index("Metric Value"), h.index("Metric Unit")
-    ours = [(r[ki], float(r[vi]), r[ui]) for r in rows[1:] if len(r) > vi and "moe::" in r[ki]]
+    mine = ("moe::", "umma_", "route_small", "decode_finalize", "combine_kernel", "scatter_rows", "assign_kernel",
+            "scan_kernel", "chunk_count", "router_select", "router_gemv", "tile_weights", "gemv13", "gemv2",
+            "simt_gemm", "ep_plan", "ep_pack", "ep_final")
+    ours = [(r[ki], float(r[vi]), r[ui]) for r in rows[1:] if len(r) > vi and any(m in r[ki] for m in mine)]
     with open(prefix + ".csv", "w") as f:
         f.write("kernel,duration,unit\n")
         for k, v, u in ours:
