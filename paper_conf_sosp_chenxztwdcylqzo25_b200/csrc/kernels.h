@@ -284,6 +284,7 @@ struct SwapParams {
   int T_shared;                 // shared-expert tokens (0 = none)
   int *sched;                   // device work counter, zero at launch
   int debug_mode;               // 0; (MOE_DEBUG_GEMM) 2 = no epilogue math -- timing experiments
+  unsigned long long *trace;     // MOE_DEBUG_TRACE: MMA-warp cycle breakdown per CTA pair (timing experiments)
 };
 cudaError_t launch_umma_swap_gemm(bool fp8, int epi, const SwapParams &p, int grid, cudaStream_t st);
 

@@ -541,7 +541,7 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
       p1.g[1] = p1.g[0];
     }
     p1.tiles = L->pairs; p1.n_tiles = L->n_pairs; p1.nb_r = F / 128;
-    p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = Fs / 128; p1.sched = L->sched; p1.debug_mode = dbg_mode;
+    p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = Fs / 128; p1.sched = L->sched; p1.debug_mode = dbg_mode; p1.trace = L->trace;
     KL_TRY(launch_umma_swap_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
     mark(L, ST_GEMM1, st);
     SwapParams p2{};
@@ -560,7 +560,7 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
       p2.g[1] = p2.g[0];
     }
     p2.tiles = L->pairs; p2.n_tiles = L->n_pairs; p2.nb_r = H / 256;
-    p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256; p2.sched = L->sched + 1; p2.debug_mode = dbg_mode;
+    p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256; p2.sched = L->sched + 1; p2.debug_mode = dbg_mode; p2.trace = L->trace ? L->trace + 2048 : nullptr;
     KL_TRY(launch_umma_swap_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
     mark(L, ST_GEMM2, st);
   } else {

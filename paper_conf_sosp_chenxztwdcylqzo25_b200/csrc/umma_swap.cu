@@ -240,16 +240,24 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
     } else if (leader) {
       int stage = 0; uint32_t phase = 0; uint32_t acc_phase = 0;
       int qs = 0; uint32_t qph = 0;
+      // MOE_DEBUG_TRACE: cycles waiting for a unit / the accumulator / loaded stages, and issuing
+      long long c_unit = 0, c_tmem = 0, c_full = 0, c_issue = 0, n_units = 0, n_flop16 = 0;
+      const bool trc = p.trace != nullptr && lane == 0;
+      long long c0 = trc ? clock64() : 0;
+      const long long c_start = c0;
       for (;;) {
         const int u = next_unit(qs, qph);
         const SwapUnit ui = swap_unit(p, u, n_routed_units);
+        if (trc) { const long long c = clock64(); c_unit += c - c0; c0 = c; }
         if (!ui.valid) break;
         const int kblocks = p.g[ui.group].kblocks;
         const int N = (ui.n + 15) & ~15;
         mbar_wait(tmem_empty, acc_phase ^ 1);
+        if (trc) { const long long c = clock64(); c_tmem += c - c0; c0 = c; ++n_units; n_flop16 += N / 16; }
         tc_fence_after();
         for (int kb = 0; kb < kblocks; ++kb) {
           mbar_wait(&full[stage], phase);
+          if (trc) { const long long c = clock64(); c_full += c - c0; c0 = c; }
           tc_fence_after();
           if (lane == 0 && p.debug_mode == 1) {    // timing experiment: loads only (commit releases the stage)
             mma_commit_pair(&empty[stage]);
@@ -281,9 +289,15 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             if (kb == kblocks - 1) mma_commit_pair(tmem_full);
           }
           __syncwarp();
+          if (trc) { const long long c = clock64(); c_issue += c - c0; c0 = c; }
           if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
         }
         acc_phase ^= 1;
+      }
+      if (trc) {
+        unsigned long long *o = p.trace + 8 * (blockIdx.x >> 1);
+        o[0] = c_unit; o[1] = c_tmem; o[2] = c_full; o[3] = c_issue; o[4] = n_units; o[5] = n_flop16;
+        o[6] = clock64() - c_start;
       }
     }
   } else {
