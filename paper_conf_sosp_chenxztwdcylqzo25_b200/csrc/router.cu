@@ -188,7 +188,8 @@ __device__ __forceinline__ unsigned long long sel_key(float v, int id) {
 }
 __device__ __forceinline__ int key_id(unsigned long long key) { return (int)~(uint32_t)key; }
 
-__device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, int *ids_s, int lane, bool live) {
+__device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, int *ids_s, int lane, bool live,
+                                  const float *bias_pre = nullptr) {
   const int E = r.E, k = r.k, G = r.n_group;
   SEL_CK(0);
   const float *lg = r.logits + (int64_t)t * r.ldl;
@@ -199,7 +200,7 @@ __device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, in
   for (int i = 0; i < 8; ++i) {
     const int e = lane * 8 + i;
     lv[i] = e < E ? lg[e] : -INFINITY;
-    bv[i] = (e < E && r.bias) ? r.bias[e] : 0.f;
+    bv[i] = bias_pre ? bias_pre[i] : ((e < E && r.bias) ? r.bias[e] : 0.f);
   }
   float s[8], sel[8];
   if (r.score_fn == MOE_SCORE_SOFTMAX) {
@@ -279,7 +280,9 @@ __device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, in
     cx(2, 4); cx(3, 5);
     cx(1, 2); cx(3, 4); cx(5, 6);
     SEL_CK(3);
-#pragma unroll
+    // (rolled: this code runs once per token with a cold instruction cache, so its
+    //  footprint, not its instruction count, sets the latency)
+#pragma unroll 1
     for (int o = 1; o < 32; o <<= 1) {
       unsigned long long pk[8];
 #pragma unroll
@@ -353,7 +356,7 @@ __device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, in
 // the active experts; a pair's row within the segment is the number of
 // earlier tokens that chose the same expert (stable by token).  Finally the
 // token rows (FP8: the codes quantised by all CTAs) are copied to their k rows.
-__device__ void route_small_tail(const RouteSmallArgs &a, float *rsm) {
+__device__ void route_small_tail(const RouteSmallArgs &a, float *rsm, const float *bias_pre) {
   const RouterArgs &r = a.r;
   const PermuteArgs &p = a.p;
   const int T = r.T, k = r.k, TK = T * k, H = a.H;
@@ -366,10 +369,12 @@ __device__ void route_small_tail(const RouteSmallArgs &a, float *rsm) {
   if (a.trace && tid == 0) a.trace[1] = gtimer_ns();
   for (int e = tid; e < p.E; e += RS_THREADS) cnt_s[e] = 0;
   if (tid < RS_MAX_E / 32) bm[tid] = 0u;
-  // uniform trip count; a warp past the last token re-routes token T-1 without storing
+  // one warp per token; warps past the last token skip (warp-uniform branch)
 #pragma unroll 1
-  for (int t0 = 0; t0 < T; t0 += RS_THREADS / 32)
-    select_token_regs(r, min(t0 + warp, T - 1), rsm + warp * 2 * RS_MAX_E, ids_s, lane, t0 + warp < T);
+  for (int t0 = 0; t0 < T; t0 += RS_THREADS / 32) {
+    const int t = __shfl_sync(0xffffffffu, t0 + warp, 0);
+    if (t < T) select_token_regs(r, t, rsm + warp * 2 * RS_MAX_E, ids_s, lane, true, bias_pre);
+  }
   __syncthreads();
   ck[1] = clock64();
   if (a.trace && tid == 0) a.trace[2] = gtimer_ns();
@@ -523,6 +528,13 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
 #pragma unroll
     for (int u = 0; u < 8; ++u) w[u] = (live && tid + u * 128 < nv) ? __ldg(wr + tid + u * 128) : make_uint4(0, 0, 0, 0);
   }
+  // the selection bias too (lane l: experts 8l .. 8l+7; used by the last CTA's route)
+  float bpre[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int e = (threadIdx.x & 31) * 8 + i;
+    bpre[i] = (r.bias && e < r.E) ? __ldg(r.bias + e) : 0.f;
+  }
   pdl_trigger();
   pdl_wait();                                    // x (the previous layer's output) and our workspaces
   if (a.trace && threadIdx.x == 0 && blockIdx.x == 0) a.trace[0] = gtimer_ns();
@@ -617,7 +629,7 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   __syncthreads();
   if (!is_last) return;
   if (a.debug & 2) { if (threadIdx.x == 0) *a.done = 0; return; }
-  route_small_tail(a, rsm);
+  route_small_tail(a, rsm, bpre);
 }
 
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st) {

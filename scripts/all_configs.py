@@ -1,0 +1,118 @@
+"""Every BASELINE.json configuration on one B200: prefill tokens/s + TFLOP/s and decode
+us/layer + GB/s (CUDA graph over a chain of distinct layers, L2 flushed), each against the
+measured peaks.  Writes one JSON line per measurement and a markdown table (argv[1])."""
+import json, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+from inputs.presets import PRESETS
+from inputs.synthetic import make_tokens, make_weights
+from paper_conf_sosp_chenxztwdcylqzo25_b200 import moe
+import bench
+
+peaks = bench.load_peaks()
+fw = torch.empty(64 << 20, device="cuda"); fr = torch.zeros(64 << 20, device="cuda"); sink = torch.zeros((), device="cuda")
+flush = (fw, fr, sink)
+rows_out = []
+
+
+def prefill(name, T):
+    p = PRESETS[name]
+    w = make_weights(p, "cuda")
+    x, _ = make_tokens(p, T, "cuda")
+    layer = moe.MoELayer(p, w, max_tokens=T)
+    y = torch.empty_like(x)
+    times, _ = bench.timed_steps(layer, [x], y, 8, 3, flush, profile=False)
+    times.sort()
+    ms = times[len(times) // 2]
+    routing = {}
+    layer.forward(x, y=y, routing=routing)
+    nd = int((routing["expert_counts"] > 0).sum())
+    alg = bench.algorithmic(p, T, nd)
+    fp8 = p.wtype == 1
+    peak_tf = (2 if fp8 else 1) * peaks["bf16_tflops_sustained"]
+    tf = alg["layer_flops"] / (ms * 1e-3) / 1e12
+    gbs = alg["layer_bytes"] / (ms * 1e-3) / 1e9
+    r = {"config": name, "phase": "prefill", "T": T, "ms": ms, "tokens_per_s": T / (ms * 1e-3), "tflops": tf,
+         "tensor_frac": tf / peak_tf, "gbs": gbs, "hbm_frac": gbs / peaks["hbm_gbs"], "distinct_experts": nd,
+         "dtype": "e4m3" if fp8 else ("bf16" if p.wtype == 0 else "f32")}
+    layer.close()
+    del w
+    torch.cuda.empty_cache()
+    return r
+
+
+def decode(name, T, L=4, n_def=0):
+    p = PRESETS[name]
+    w = make_weights(p, "cuda")
+    layers = [moe.MoELayer(p, w, max_tokens=16) for _ in range(L)]
+    del w
+    torch.cuda.empty_cache()
+    xs, _ = make_tokens(p, 16 * T, "cuda", offset=11)
+    rows = [xs[i * T:(i + 1) * T].contiguous() for i in range(16)]
+    bufs = [rows[0].clone(), torch.empty_like(rows[0])]
+    dbufs = [torch.zeros_like(rows[0]), torch.zeros_like(rows[0])]
+
+    def step():
+        for i, l in enumerate(layers):
+            a, b = bufs[i % 2], bufs[(i + 1) % 2]
+            if n_def:
+                din = None if i == 0 else dbufs[(i + 1) % 2]
+                dout = None if i == L - 1 else dbufs[i % 2]
+                l.forward(a, residual=a, y=b, n_deferred=n_def if dout is not None else 0, deferred_in=din,
+                          deferred_out=dout)
+            else:
+                l.forward(a, residual=a, y=b)
+    s = torch.cuda.Stream(); s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        for _ in range(2):
+            bufs[0].copy_(rows[0]); step()
+    torch.cuda.current_stream().wait_stream(s)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        step()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ts = []
+    for i in range(16):
+        bufs[0].copy_(rows[i])
+        bench.flush_l2(flush)
+        e0.record(); g.replay(); e1.record(); e1.synchronize()
+        if i >= 3:
+            ts.append(e0.elapsed_time(e1) * 1e3 / L)
+    ts.sort()
+    us = ts[len(ts) // 2]
+    routing = {}
+    layers[0].forward(rows[0], routing=routing)
+    nd = int((routing["expert_counts"] > 0).sum())
+    alg = bench.algorithmic(p, T, nd)
+    gbs = alg["layer_bytes"] / (us * 1e-6) / 1e9
+    r = {"config": name, "phase": "decode", "T": T, "n_deferred": n_def, "layers_in_graph": L, "us_per_layer": us,
+         "gbs": gbs, "hbm_frac": gbs / peaks["hbm_gbs"], "distinct_experts": nd, "layer_bytes": alg["layer_bytes"]}
+    for l in layers:
+        l.close()
+    torch.cuda.empty_cache()
+    return r
+
+
+plan = [("prefill", "v2lite", 512), ("decode", "v2lite", 1), ("prefill", "qwen2", 2048), ("decode", "qwen2", 1),
+        ("prefill", "v25", 4096), ("decode", "v25", 4), ("prefill", "v3", 8192), ("decode", "v3", 1)]
+for kind, name, T in plan:
+    r = prefill(name, T) if kind == "prefill" else decode(name, T)
+    print(json.dumps(r), flush=True)
+    rows_out.append(r)
+for nd_ in (3, 6):
+    r = decode("v3", 1, n_def=nd_)
+    print(json.dumps(r), flush=True)
+    rows_out.append(r)
+
+with open(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/all_configs.md", "w") as f:
+    f.write("| config | phase | T | time | throughput | roofline |\n|---|---|---|---|---|---|\n")
+    for r in rows_out:
+        if r["phase"] == "prefill":
+            f.write(f"| {r['config']} ({r['dtype']}) | prefill | {r['T']} | {r['ms']:.3f} ms | {r['tokens_per_s']/1e6:.3f} M tok/s, "
+                    f"{r['tflops']:.0f} TFLOP/s | {r['tensor_frac']*100:.1f} % of tensor peak, {r['hbm_frac']*100:.1f} % of HBM "
+                    f"({r['distinct_experts']} experts hit) |\n")
+        else:
+            f.write(f"| {r['config']} | decode{' n_def=%d' % r['n_deferred'] if r['n_deferred'] else ''} | {r['T']} | "
+                    f"{r['us_per_layer']:.1f} us/layer | {r['gbs']:.0f} GB/s | {r['hbm_frac']*100:.1f} % of HBM "
+                    f"({r['distinct_experts']} experts, {r['layer_bytes']/1e6:.1f} MB) |\n")
+print(open(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/all_configs.md").read())

@@ -13,15 +13,33 @@ T = int(sys.argv[2]) if len(sys.argv) > 2 else 1
 p = PRESETS[cfg]
 w = make_weights(p, "cuda")
 x, _ = make_tokens(p, T, "cuda", offset=5)
-layer = moe.MoELayer(p, w, max_tokens=16)
+NL = int(sys.argv[3]) if len(sys.argv) > 3 else 1     # >1: trace the middle layer of a chained graph
+layers = [moe.MoELayer(p, w, max_tokens=16) for _ in range(NL)]
+layer = layers[NL // 2]
 lib = layer._lib
 lib.moe_layer_debug_trace.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32]
 buf = np.zeros(4096, dtype=np.uint64)
 y = torch.empty_like(x)
 fw = torch.empty(64 << 20, device="cuda"); fr = torch.zeros(64 << 20, device="cuda"); sink = torch.zeros((), device="cuda")
+bufs = [x.clone(), torch.empty_like(x)]
+def step():
+    for i, l in enumerate(layers):
+        a, b = bufs[i % 2], bufs[(i + 1) % 2]
+        l.forward(a, residual=a, y=b)
+if NL > 1:
+    s_ = torch.cuda.Stream(); s_.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s_):
+        step(); step()
+    torch.cuda.current_stream().wait_stream(s_)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        step()
 for it in range(4):
     fw.zero_(); torch.sum(fr, 0, out=sink)
-    layer.forward(x, y=y)
+    if NL > 1:
+        bufs[0].copy_(x); g.replay()
+    else:
+        layer.forward(x, y=y)
     torch.cuda.synchronize()
     assert lib.moe_layer_debug_trace(layer._h, buf.ctypes.data, 4096) == 0
 t0 = int(buf[0])

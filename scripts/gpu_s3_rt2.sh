@@ -1,0 +1,7 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || exit 1
+./scripts/micro/select_bench > gpurun_out/rt2_select_micro.txt 2>&1
+timeout 300 python -m pytest tests -m gpu -q -x -k "decode or small" > gpurun_out/rt2_parity.log 2>&1; echo "rc=$?" >> gpurun_out/rt2_parity.log
+timeout 400 python scripts/decode_trace.py v3 1 8 > gpurun_out/rt2_trace_L8.log 2>&1
+timeout 400 python scripts/decode_ab.py v3 1,4 8 > gpurun_out/rt2_ab_L8.log 2>&1
