@@ -381,8 +381,10 @@ __device__ void route_small_tail(const RouteSmallArgs &a, float *rsm, const floa
   if (a.debug & 8) {                             // timing experiment: a second (warm i-cache) select pass
     const long long w0 = clock64();
 #pragma unroll 1
-    for (int t0 = 0; t0 < T; t0 += RS_THREADS / 32)
-      select_token_regs(r, min(t0 + warp, T - 1), rsm + warp * 2 * RS_MAX_E, ids_s, lane, t0 + warp < T);
+    for (int t0 = 0; t0 < T; t0 += RS_THREADS / 32) {
+      const int t = __shfl_sync(0xffffffffu, t0 + warp, 0);
+      if (t < T) select_token_regs(r, t, rsm + warp * 2 * RS_MAX_E, ids_s, lane, true, bias_pre);
+    }
     __syncthreads();
     if (a.trace && tid == 0) { a.trace[5] = ck[1] - ck[0]; a.trace[6] = clock64() - w0; }
   }
