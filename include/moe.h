@@ -133,7 +133,14 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
  *   residual  device [T, H] bf16 or NULL (NULL => no I_k term, reading R7)
  *   y         device [T, H] bf16; may alias residual, must not alias x
  *   T         0 <= T <= max_tokens (T == 0 is legal and launches nothing)
- *   dbg       NULL or routing outputs (see moe_routing_out)                   */
+ *   dbg       NULL or routing outputs (see moe_routing_out)
+ * Kernel choice: T <= gemv_max_tokens (default 16) on the tensor-core path runs
+ * the decode stream (router, fused per-expert-chunk weight stream, finalize);
+ * its expert sums are fp32 atomics, so two calls agree to fp32 rounding, not
+ * bitwise (R22).  Larger T runs the grouped-GEMM path, which is
+ * deterministic.  The kernels use programmatic dependent launch: the first one
+ * may start before the stream's previous kernel ends, but reads nothing the
+ * caller wrote on the stream before its own dependency wait.                 */
 moe_status moe_layer_forward(moe_layer *layer, const void *x, const void *residual, int32_t T,
                              void *y, moe_routing_out *dbg, void *stream);
 
@@ -164,6 +171,13 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
                                 const void *const *residual, const int32_t *T, int32_t n_deferred,
                                 const void *const *deferred_in, void *const *y, void *const *deferred_out,
                                 void *stream);
+
+/* Timing experiments only: a layer created with the environment variable
+ * MOE_DEBUG_TRACE set records globaltimer/clock stamps of its kernels into a
+ * 4096-entry u64 device buffer; this synchronises the device, copies
+ * min(cap, 4096) entries to `host` and clears the buffer.  MOE_ERR_UNSUPPORTED
+ * without MOE_DEBUG_TRACE.  Layout: DESIGN.md §6 / scripts/decode_trace.py.   */
+moe_status moe_layer_debug_trace(moe_layer *layer, void *host, int32_t cap);
 
 /* Free every library allocation (and the NCCL communicator).  NULL is a no-op. */
 moe_status moe_layer_destroy(moe_layer *layer);
