@@ -234,6 +234,13 @@ struct FdGroup {                // 0 routed, 1 shared
   const uint8_t *w2;            // tiled W2 [expert][H/256][F/128 B][256 x 128 B]
   const float *w2_s;            // FP8: [expert][H/128][F/128]
 };
+struct DecodeFinalizeArgs {
+  int T, H, use_def;
+  float *acc_imm, *acc_def;
+  const void *residual, *deferred_in;
+  void *y, *deferred_out;
+  unsigned long long *trace;     // MOE_DEBUG_TRACE: [2000] past the PDL wait, [2001] end (CTA 0)
+};
 struct FusedDecodeParams {
   FdGroup g[2];
   int nch[2];                   // 128-column chunks: F/128, Fs/128
@@ -245,15 +252,11 @@ struct FusedDecodeParams {
   int *sched, *done;            // work counter + exit ticket, zero on entry (re-armed by the kernel)
   const void *pf[2]; int64_t pf_bytes[2];   // shared-expert weights prefetched into L2 before the PDL wait
   unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
+  int early_trigger;            // trigger the finalize launch when the CTA's producer runs out of units
+  int fold_finalize;            // the last CTA runs the finalize (fin) itself (small T)
+  DecodeFinalizeArgs fin;
 };
 cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, cudaStream_t st);
-struct DecodeFinalizeArgs {
-  int T, H, use_def;
-  float *acc_imm, *acc_def;
-  const void *residual, *deferred_in;
-  void *y, *deferred_out;
-  unsigned long long *trace;     // MOE_DEBUG_TRACE: [2000] past the PDL wait, [2001] end (CTA 0)
-};
 cudaError_t launch_decode_finalize(const DecodeFinalizeArgs &a, cudaStream_t st);
 
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);

@@ -897,16 +897,24 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     fp.acc_imm = acc_imm; fp.acc_def = acc_def;
     fp.sched = L->sched + 5; fp.done = L->sched + 6;
     fp.trace = L->trace;
-    const int units = (Fs > 0 ? Fs / 128 : 0) + (int)std::min<int64_t>(E, pairs) * (F / 128);
-    KL_TRY(launch_umma_decode_fused(f8, fp, std::min(L->num_sms, units), st));
-    mark(L, ST_GEMM1, st);
+    static const int late_trig = getenv("MOE_DECODE_LATE_TRIGGER") ? atoi(getenv("MOE_DECODE_LATE_TRIGGER")) : 0;
+    fp.early_trigger = !late_trig;
     DecodeFinalizeArgs fa{};
     fa.T = T; fa.H = H; fa.use_def = deferred_out != nullptr && n_def > 0;
     fa.acc_imm = acc_imm; fa.acc_def = acc_def;
     fa.residual = residual; fa.deferred_in = deferred_in; fa.y = y; fa.deferred_out = deferred_out;
     fa.trace = L->trace;
-    KL_TRY(launch_decode_finalize(fa, st));
-    mark(L, ST_COMBINE, st);
+    // MOE_DECODE_FOLD=1, T <= 2: the fused kernel's last CTA finalizes (no finalize launch)
+    static const int fold_env = getenv("MOE_DECODE_FOLD") ? atoi(getenv("MOE_DECODE_FOLD")) : 0;   // measured slower
+    fp.fold_finalize = fold_env && (int64_t)T * H <= 2 * 8192;
+    fp.fin = fa;
+    const int units = (Fs > 0 ? Fs / 128 : 0) + (int)std::min<int64_t>(E, pairs) * (F / 128);
+    KL_TRY(launch_umma_decode_fused(f8, fp, std::min(L->num_sms, units), st));
+    mark(L, ST_GEMM1, st);
+    if (!fp.fold_finalize) {
+      KL_TRY(launch_decode_finalize(fa, st));
+      mark(L, ST_COMBINE, st);
+    }
   } else if (decode && L->umma) {
     // 5+6 (decode). swap-AB tensor-core weight stream over the active experts + shared expert
     const bool f8 = L->fp8;

@@ -91,6 +91,52 @@ __device__ __forceinline__ FdUnit fd_unit(const FusedDecodeParams &p, int u) {
   return r;
 }
 
+// y = bf16(residual + acc_imm + deferred_in); deferred_out = bf16(acc_def); sums re-zeroed.
+// Elements first, first + stride, ... of the T*H/8 8-element groups.
+__device__ __forceinline__ void decode_finalize_range(const DecodeFinalizeArgs &a, int64_t first, int64_t stride) {
+  const int64_t n8 = (int64_t)a.T * a.H / 8;
+  for (int64_t i = first; i < n8; i += stride) {
+    float4 *s4 = reinterpret_cast<float4 *>(a.acc_imm) + 2 * i;
+    float4 u0 = s4[0], u1 = s4[1];
+    float v[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
+    s4[0] = make_float4(0.f, 0.f, 0.f, 0.f);
+    s4[1] = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (a.residual) {
+      float f[8];
+      bf16x8_to_f32(reinterpret_cast<const uint4 *>(a.residual)[i], f);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) v[j] += f[j];
+    }
+    if (a.deferred_in) {
+      float f[8];
+      bf16x8_to_f32(reinterpret_cast<const uint4 *>(a.deferred_in)[i], f);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) v[j] += f[j];
+    }
+    uint4 o;
+    __nv_bfloat162 *ob = reinterpret_cast<__nv_bfloat162 *>(&o);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) ob[j] = __floats2bfloat162_rn(v[2 * j], v[2 * j + 1]);
+    reinterpret_cast<uint4 *>(a.y)[i] = o;
+    if (a.deferred_out) {
+      float4 d0 = make_float4(0.f, 0.f, 0.f, 0.f), d1 = d0;
+      if (a.use_def) {
+        float4 *d4 = reinterpret_cast<float4 *>(a.acc_def) + 2 * i;
+        d0 = d4[0]; d1 = d4[1];
+        d4[0] = make_float4(0.f, 0.f, 0.f, 0.f);
+        d4[1] = make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+      {
+        uint4 od;
+        __nv_bfloat162 *db = reinterpret_cast<__nv_bfloat162 *>(&od);
+        db[0] = __floats2bfloat162_rn(d0.x, d0.y); db[1] = __floats2bfloat162_rn(d0.z, d0.w);
+        db[2] = __floats2bfloat162_rn(d1.x, d1.y); db[3] = __floats2bfloat162_rn(d1.z, d1.w);
+        reinterpret_cast<uint4 *>(a.deferred_out)[i] = od;
+      }
+    }
+  }
+}
+
 template <bool FP8>
 __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const __grid_constant__ FusedDecodeParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -158,7 +204,12 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         unit_q[qs] = make_int4(ui.expert, ui.row0, ui.n | (ui.chunk << 16), ui.group | (ui.valid << 1));
         mbar_arrive(&uq_full[qs]);
         if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
-        if (!ui.valid) break;
+        if (!ui.valid) {
+          // every load of this CTA is issued: let the finalize kernel launch now, so
+          // its launch latency overlaps the last stages (it waits for our completion)
+          if (p.early_trigger) pdl_trigger();
+          break;
+        }
         const FdGroup &g = p.g[ui.group];
         // ---- phase A: W13 tile `chunk` (256 rows: gate + up of 128 h columns) ----
         const uint32_t bytes_a = FD_A_BYTES + FD_B_BYTES + (FP8 ? 2 * FD_SF_BYTES : 0);
@@ -424,61 +475,30 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   tc_fence_before();
   __syncthreads();
   if (warp == 1) tmem_dealloc(tmem, FD_TMEM_COLS);
+  __shared__ int last_cta;
   if (threadIdx.x == 0) {
     // the last CTA out re-arms the work counter for the next forward (graph replay)
-    if (atomicAdd(p.done, 1) == (int)gridDim.x - 1) {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+    last_cta = atomicAdd(p.done, 1) == (int)gridDim.x - 1;
+    if (last_cta) {
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");
       atomicExch(p.sched, 0);
       atomicExch(p.done, 0);
     }
   }
+  if (p.fold_finalize) {
+    // small T: the last CTA writes y itself (every other CTA's red.adds are ordered
+    // before its ticket) -- no finalize launch, no PDL gap
+    __syncthreads();
+    if (last_cta) decode_finalize_range(p.fin, threadIdx.x, FD_THREADS);
+  }
 }
 
-// y = bf16(residual + acc_imm + deferred_in); deferred_out = bf16(acc_def); sums re-zeroed
 __global__ void decode_finalize_kernel(const __grid_constant__ DecodeFinalizeArgs a) {
   pdl_trigger();                                 // the next layer's router may start loading its weights
   pdl_wait();
   if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) a.trace[2000] = gtimer();
-  const int64_t n8 = (int64_t)a.T * a.H / 8;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += (int64_t)gridDim.x * blockDim.x) {
-    float4 *s4 = reinterpret_cast<float4 *>(a.acc_imm) + 2 * i;
-    float4 u0 = s4[0], u1 = s4[1];
-    float v[8] = {u0.x, u0.y, u0.z, u0.w, u1.x, u1.y, u1.z, u1.w};
-    s4[0] = make_float4(0.f, 0.f, 0.f, 0.f);
-    s4[1] = make_float4(0.f, 0.f, 0.f, 0.f);
-    if (a.residual) {
-      float f[8];
-      bf16x8_to_f32(reinterpret_cast<const uint4 *>(a.residual)[i], f);
-#pragma unroll
-      for (int j = 0; j < 8; ++j) v[j] += f[j];
-    }
-    if (a.deferred_in) {
-      float f[8];
-      bf16x8_to_f32(reinterpret_cast<const uint4 *>(a.deferred_in)[i], f);
-#pragma unroll
-      for (int j = 0; j < 8; ++j) v[j] += f[j];
-    }
-    uint4 o;
-    __nv_bfloat162 *ob = reinterpret_cast<__nv_bfloat162 *>(&o);
-#pragma unroll
-    for (int j = 0; j < 4; ++j) ob[j] = __floats2bfloat162_rn(v[2 * j], v[2 * j + 1]);
-    reinterpret_cast<uint4 *>(a.y)[i] = o;
-    if (a.deferred_out) {
-      float4 d0 = make_float4(0.f, 0.f, 0.f, 0.f), d1 = d0;
-      if (a.use_def) {
-        float4 *d4 = reinterpret_cast<float4 *>(a.acc_def) + 2 * i;
-        d0 = d4[0]; d1 = d4[1];
-        d4[0] = make_float4(0.f, 0.f, 0.f, 0.f);
-        d4[1] = make_float4(0.f, 0.f, 0.f, 0.f);
-      }
-      {
-        uint4 od;
-        __nv_bfloat162 *db = reinterpret_cast<__nv_bfloat162 *>(&od);
-        db[0] = __floats2bfloat162_rn(d0.x, d0.y); db[1] = __floats2bfloat162_rn(d0.z, d0.w);
-        db[2] = __floats2bfloat162_rn(d1.x, d1.y); db[3] = __floats2bfloat162_rn(d1.z, d1.w);
-        reinterpret_cast<uint4 *>(a.deferred_out)[i] = od;
-      }
-    }
-  }
+  decode_finalize_range(a, (int64_t)blockIdx.x * blockDim.x + threadIdx.x, (int64_t)gridDim.x * blockDim.x);
   if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) a.trace[2001] = gtimer();
 }
 
