@@ -342,11 +342,20 @@ __device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, in
   if (live && lane < k) {
     r.topk_idx[(int64_t)t * k + rank] = my_id;
     r.topk_w[(int64_t)t * k + rank] = my_w;
-    ids_s[t * k + rank] = my_id;
+    if (ids_s) ids_s[t * k + rank] = my_id;
   }
   if (live && r.shared_gated && lane == 0) r.sgate[t] = 1.f / (1.f + expf(-lg[E]));
   SEL_CK(5);
   __syncwarp();                                  // scratch reuse by the next token of this warp
+}
+
+// Prefill selection (E <= 256): one warp per token with the register-resident
+// select of the decode router (same rules; ~4x fewer cycles than select_token).
+__global__ void __launch_bounds__(RT_WARPS * 32) router_select_regs_kernel(const __grid_constant__ RouterArgs a) {
+  __shared__ float scratch[RT_WARPS][2 * RS_MAX_E];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int t = __shfl_sync(0xffffffffu, blockIdx.x * RT_WARPS + warp, 0);   // warp-uniform
+  if (t < a.T) select_token_regs(a, t, scratch[warp], nullptr, lane, true);
 }
 
 // The last router CTA: route every token (one warp per token), then the
@@ -658,6 +667,10 @@ cudaError_t launch_router_select(const RouterArgs &a, cudaStream_t st) {
   if (sm > 48 * 1024) {
     cudaError_t e = cudaFuncSetAttribute(router_select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
+  }
+  if (a.E <= RS_MAX_E) {
+    router_select_regs_kernel<<<grid, RT_WARPS * 32, 0, st>>>(a);
+    return cudaGetLastError();
   }
   router_select_kernel<<<grid, RT_WARPS * 32, sm, st>>>(a);
   return cudaGetLastError();
