@@ -175,7 +175,7 @@ def _full(lib, name, T, n_def=0, sample=6):
 
 
 @pytest.mark.parametrize("name,T", [("v3", 1), ("v25", 4), ("v2lite", 1), ("v2lite", 512), ("qwen2", 2048),
-                                    ("v3", 8192)])
+                                    ("v3", 8192), ("qwen2", 1), ("v3", 16)])
 def test_full_size_sampled(lib, name, T):
     _full(lib, name, T, sample=4 if T > 1 else 1)
 
