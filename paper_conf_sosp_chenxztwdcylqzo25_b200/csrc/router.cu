@@ -566,23 +566,36 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   }
   // ---- logits of router rows `row` for all T tokens ----
   {
+    // two tokens per step with all their x loads in flight together (a token at a
+    // time serialised T L2 round trips: ~1.5 us each at T = 4)
 #pragma unroll 1
-    for (int t = 0; t < T; ++t) {
-      const uint4 *xr = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H);
-      float acc = 0.f;
+    for (int t = 0; t < T; t += 2) {
+      const bool two = t + 1 < T;
+      const uint4 *xr0 = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H);
+      const uint4 *xr1 = two ? xr0 + H / 8 : xr0;
+      uint4 xv0[8], xv1[8];
 #pragma unroll
       for (int u = 0; u < 8; ++u) {
         const int c = tid + u * 128;
-        if (c < nv) {
-          float wf[8], xf[8];
-          bf16x8_to_f32(w[u], wf);
-          bf16x8_to_f32(__ldg(xr + c), xf);
-#pragma unroll
-          for (int j = 0; j < 8; ++j) acc = fmaf(wf[j], xf[j], acc);
-        }
+        xv0[u] = c < nv ? __ldg(xr0 + c) : make_uint4(0, 0, 0, 0);
+        xv1[u] = c < nv ? __ldg(xr1 + c) : make_uint4(0, 0, 0, 0);
       }
-      acc = warp_sum(acc);
-      if (lane == 0) red[half][w4][t] = acc;
+      float acc0 = 0.f, acc1 = 0.f;
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        float wf[8], x0[8], x1[8];
+        bf16x8_to_f32(w[u], wf);
+        bf16x8_to_f32(xv0[u], x0);
+        bf16x8_to_f32(xv1[u], x1);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) { acc0 = fmaf(wf[j], x0[j], acc0); acc1 = fmaf(wf[j], x1[j], acc1); }
+      }
+      acc0 = warp_sum(acc0);
+      acc1 = warp_sum(acc1);
+      if (lane == 0) {
+        red[half][w4][t] = acc0;
+        if (two) red[half][w4][t + 1] = acc1;
+      }
     }
     __syncthreads();
     if (row < a.rows && tid < T)
