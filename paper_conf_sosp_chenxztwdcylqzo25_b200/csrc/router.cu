@@ -210,13 +210,14 @@ __device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, in
     m = warp_max(m);
     float sum = 0.f;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) { s[i] = lane * 8 + i < E ? expf(lv[i] - m) : 0.f; sum += s[i]; }
+    for (int i = 0; i < 8; ++i) { s[i] = lane * 8 + i < E ? __expf(lv[i] - m) : 0.f; sum += s[i]; }
     sum = warp_sum(sum);
+    const float inv = 1.f / sum;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) s[i] = s[i] / sum;
+    for (int i = 0; i < 8; ++i) s[i] = s[i] * inv;
   } else {
 #pragma unroll
-    for (int i = 0; i < 8; ++i) s[i] = 1.f / (1.f + expf(-lv[i]));
+    for (int i = 0; i < 8; ++i) s[i] = __fdividef(1.f, 1.f + __expf(-lv[i]));   // ~2 ulp, far inside the 1e-5 tie band
   }
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
@@ -227,19 +228,38 @@ __device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, in
   __syncwarp();
   SEL_CK(1);
   if (G > 1) {
-    // group g = experts [g gs, (g+1) gs): lane g scans it (branch-free top-2)
+    // group g = experts [g gs, (g+1) gs)
     const int gs = E / G;
     float m1 = -INFINITY, m2 = -INFINITY;
-    if (lane < G) {
-      const float *gp = sel_sm + lane * gs;
-#pragma unroll 8
-      for (int i = 0; i < gs; ++i) {
-        const float v = gp[i];
-        m2 = fmaxf(m2, fminf(m1, v));
-        m1 = fmaxf(m1, v);
+    float gsc;
+    const int lpg = gs >> 3;                     // lanes per group when groups are whole lanes
+    if ((gs & 7) == 0 && lpg <= 32 && (lpg & (lpg - 1)) == 0 && G * lpg <= 32) {
+      // groups made of whole lanes (V3: 32 experts = 4 lanes): in-register top-2 of the
+      // lane's 8, merged across the group's lanes by xor shuffles (branch-free)
+#pragma unroll
+      for (int i = 0; i < 8; ++i) { m2 = fmaxf(m2, fminf(m1, sel[i])); m1 = fmaxf(m1, sel[i]); }
+      for (int o = 1; o < lpg; o <<= 1) {
+        const float p1 = __shfl_xor_sync(0xffffffffu, m1, o), p2 = __shfl_xor_sync(0xffffffffu, m2, o);
+        m2 = fmaxf(fminf(m1, p1), fmaxf(m2, p2));
+        m1 = fmaxf(m1, p1);
       }
+      // group g's score, gathered onto lane g
+      const float own = r.group_score == MOE_GROUP_TOP2_SUM ? m1 + m2 : m1;
+      const float got = __shfl_sync(0xffffffffu, own, (lane * lpg) & 31);
+      gsc = lane < G ? got : -INFINITY;
+    } else {
+      // general layout: lane g scans group g in shared memory (branch-free top-2)
+      if (lane < G) {
+        const float *gp = sel_sm + lane * gs;
+#pragma unroll 8
+        for (int i = 0; i < gs; ++i) {
+          const float v = gp[i];
+          m2 = fmaxf(m2, fminf(m1, v));
+          m1 = fmaxf(m1, v);
+        }
+      }
+      gsc = lane < G ? (r.group_score == MOE_GROUP_TOP2_SUM ? m1 + m2 : m1) : -INFINITY;
     }
-    const float gsc = lane < G ? (r.group_score == MOE_GROUP_TOP2_SUM ? m1 + m2 : m1) : -INFINITY;
     int rk = 0;
 #pragma unroll 8
     for (int j = 0; j < G; ++j) rk += better(__shfl_sync(0xffffffffu, gsc, j), j, gsc, lane);
@@ -301,9 +321,11 @@ __device__ void select_token_regs(const RouterArgs &r, int t, float *scratch, in
       sv[i] = i < k ? s_sm[key_id(key[i])] : 0.f;
       sum += sv[i];
     }
+    // one reciprocal for the 8 weights (an IEEE division each cost ~1 K cycles in total)
+    const float c = (r.norm_topk ? 1.f / sum : 1.f) * r.routed_scale;
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
-      const float w = (r.norm_topk ? sv[i] / sum : sv[i]) * r.routed_scale;
+      const float w = sv[i] * c;
       const int id = key_id(key[i]);
       my_id = i == lane ? id : my_id;
       my_w = i == lane ? w : my_w;
