@@ -144,10 +144,14 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
     if (lane == 0) {
       int stage = 0; uint32_t phase = 0;
       int qs = 0; uint32_t qph = 0;
+      // the next unit is claimed one unit ahead, so the counter's round trip overlaps
+      // this unit's loads instead of sitting between two units' load streams
+      int u_next = leader ? atomicAdd(p.sched, 1) : 0;
       for (;;) {
         int u;
         if (leader) {
-          u = atomicAdd(p.sched, 1);
+          u = u_next;
+          u_next = atomicAdd(p.sched, 1);
           mbar_wait(&uq_empty[qs], qph ^ 1);
           unit_q[qs] = u;
           mbar_arrive(&uq_full[qs]);
