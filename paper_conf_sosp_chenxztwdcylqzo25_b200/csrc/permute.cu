@@ -41,10 +41,17 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(const __grid_constan
   const int e = threadIdx.x;   // E <= 1024 (validated at create)
   int cnt = 0;
   if (e < a.E) {
-    for (int c = 0; c < nchunk; ++c) {
-      const int64_t i = (int64_t)c * a.E + e;
-      a.chunk_base[i] = cnt;
-      cnt += a.chunk_cnt[i];
+    // chunk counts loaded 8 at a time (independent loads in flight) before the
+    // running sum -- a load per step serialised nchunk L2 round trips
+    for (int c0 = 0; c0 < nchunk; c0 += 8) {
+      int v[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) v[j] = c0 + j < nchunk ? a.chunk_cnt[(int64_t)(c0 + j) * a.E + e] : 0;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        if (c0 + j < nchunk) a.chunk_base[(int64_t)(c0 + j) * a.E + e] = cnt;
+        cnt += v[j];
+      }
     }
   }
   const int padded = (cnt + kPadM - 1) / kPadM * kPadM;
