@@ -20,10 +20,13 @@
 //            PAPER.md L219-241) -- the k-sum over chunks and the weighted
 //            combine over a token's experts (L187) happen in the same adds.
 // Units are claimed from a device counter (the L181 dynamic task queue): the
-// shared expert's chunks first (its weights do not depend on the routing and
-// were prefetched into L2 by this kernel before it waited on the router), then
-// the active routed experts.  decode_finalize_kernel adds the residual /
-// deferred input, writes bf16 y (and deferred_out) and re-zeroes the sums.
+// shared expert's chunks first, then the active routed experts (ascending id).
+// The kernel is PDL-launched while the router runs; every warp waits for the
+// router's completion before touching routing data or activations (an optional
+// L2 prefetch of the shared expert before that wait, MOE_DECODE_PF=1, measured
+// slower).  The weight stream uses an evict-first L2 policy.
+// decode_finalize_kernel adds the residual / deferred input, writes bf16 y (and
+// deferred_out) and re-zeroes the sums.
 //
 // Summation order across chunks is the order of the atomics (fp32; results
 // are reproducible to fp32 rounding, not bitwise) -- DESIGN.md reading R22.
