@@ -305,9 +305,18 @@ __global__ void __launch_bounds__(UG_THREADS, 1) umma_grouped_gemm(const __grid_
           // router logits: fp32 columns n < n_valid (PAPER.md L187 gating network)
           if (live) {
             float *crow = reinterpret_cast<float *>(g.out) + (size_t)row * g.ldc;
+            if ((g.ldc & 3) == 0 && n0 + 128 <= g.n_valid) {
+              // 16-byte stores (4-byte stores put 32 rows x 4 B in every warp store)
+              float4 *c4 = reinterpret_cast<float4 *>(crow + n0);
 #pragma unroll
-            for (int i = 0; i < 128; ++i)
-              if (n0 + i < g.n_valid) crow[n0 + i] = __uint_as_float(r[i]);
+              for (int i = 0; i < 32; ++i)
+                c4[i] = make_float4(__uint_as_float(r[4 * i]), __uint_as_float(r[4 * i + 1]),
+                                    __uint_as_float(r[4 * i + 2]), __uint_as_float(r[4 * i + 3]));
+            } else {
+#pragma unroll
+              for (int i = 0; i < 128; ++i)
+                if (n0 + i < g.n_valid) crow[n0 + i] = __uint_as_float(r[i]);
+            }
           }
         } else if (live) {
           uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(g.out) + (size_t)row * g.ldc + n0);
