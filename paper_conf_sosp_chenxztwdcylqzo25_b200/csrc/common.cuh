@@ -100,6 +100,7 @@ __device__ __forceinline__ void scatter_token_row(const __nv_bfloat16 *__restric
   constexpr int MAXI = 8192 / 8 / NT;
   const int th = threadIdx.x, lane = th & 31;
   const int nc = H / 8;
+  __shared__ uint8_t exs[8192 / 128];               // FP8: the row's UE8M0 bytes, stored as words below
   uint4 raw[MAXI];
 #pragma unroll
   for (int i = 0; i < MAXI; ++i) {
@@ -128,22 +129,17 @@ __device__ __forceinline__ void scatter_token_row(const __nv_bfloat16 *__restric
             ((uint32_t)f32_to_e4m3(f[6] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[7] * inv) << 24);
       const int b = c >> 4;                        // 128-element block
       const bool head = (lane & 15) == 0;
+      if (head) exs[b] = (uint8_t)(ex + 127);
       if (d.xq) {
         *reinterpret_cast<uint2 *>(reinterpret_cast<uint8_t *>(d.xq) + t * H + c * 8) = q;
-        if (head) {
-          if (d.xq_img) d.xq_img[sf_img_off(t, b, d.xq_img_stride)] = (uint8_t)(ex + 127);
-          if (d.xs) d.xs[t * (H / 128) + b] = exp2i(ex);
-        }
+        if (head && d.xs) d.xs[t * (H / 128) + b] = exp2i(ex);
       }
 #pragma unroll 1
       for (int j = 0; j < k; ++j) {
         const int rw = pos[j];
         if (rw < 0) continue;
         *reinterpret_cast<uint2 *>(reinterpret_cast<uint8_t *>(d.xperm) + (int64_t)rw * H + c * 8) = q;
-        if (head) {
-          if (d.xperm_img) d.xperm_img[sf_img_off(rw, b, d.xperm_img_stride)] = (uint8_t)(ex + 127);
-          if (d.xperm_s) d.xperm_s[(int64_t)rw * (H / 128) + b] = exp2i(ex);
-        }
+        if (head && d.xperm_s) d.xperm_s[(int64_t)rw * (H / 128) + b] = exp2i(ex);
       }
     } else if (c < nc) {
 #pragma unroll 1
@@ -153,6 +149,25 @@ __device__ __forceinline__ void scatter_token_row(const __nv_bfloat16 *__restric
         reinterpret_cast<uint4 *>(reinterpret_cast<__nv_bfloat16 *>(d.xperm) + (int64_t)rw * H)[c] = raw[i];
       }
     }
+  }
+  if (d.fp8 && (d.xq_img || d.xperm_img)) {
+    // scale images: the 4 UE8M0 bytes of k-blocks 4g .. 4g+3 of a row are one
+    // 32-bit word of the image (sf_img_off), so each destination row gets H/512
+    // word stores instead of H/128 scattered byte stores
+    __syncthreads();
+    const int nb = H / 128, ng = (nb + 3) / 4;
+    for (int idx = th; idx < ng * (k + 1); idx += NT) {
+      const int g = idx % ng, dst = idx / ng;      // dst 0: xq (row t), 1..k: the sorted rows
+      uint32_t w = 0;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) w |= (4 * g + j < nb ? (uint32_t)exs[4 * g + j] : 0u) << (8 * j);
+      const int64_t row = dst == 0 ? t : (int64_t)pos[dst - 1];
+      uint8_t *img = dst == 0 ? d.xq_img : d.xperm_img;
+      const int stride = dst == 0 ? d.xq_img_stride : d.xperm_img_stride;
+      if (row < 0 || !img || (dst == 0 && !d.xq)) continue;
+      *reinterpret_cast<uint32_t *>(img + sf_img_off(row, 4 * g, stride)) = w;
+    }
+    __syncthreads();                             // exs is reused by the caller's next token
   }
 }
 
