@@ -372,6 +372,40 @@ def run_ours(args):
                                "frac": algd["layer_bytes"] / (dus * 1e-6) / 1e9 / peaks["hbm_gbs"],
                                "bytes": algd["layer_bytes"],
                                "stage_us_eager": {k: round(v * 1e3, 2) for k, v in dstages.items()}}}
+        # decode TP within every expert: one rank's share of the same
+        # graph-replayed chain at P = 2/4/8 (rank 0's chunks; the per-layer [T, H] all-reduce
+        # over NVLink is not in this single-GPU number)
+        tp = {}
+        if not args.no_decode_tp:
+            for P in (2, 4, 8):
+                if p.ffn // 128 < P or (p.shared_ffn and p.shared_ffn // 128 < P):
+                    continue
+                for l in dlayers:
+                    l.set_decode_tp(0, P)
+                side.wait_stream(torch.cuda.current_stream())
+                with torch.cuda.stream(side):
+                    dstep()
+                torch.cuda.current_stream().wait_stream(side)
+                g2 = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g2):
+                    dstep()
+                for i in range(args.warmup):
+                    g2.replay()
+                torch.cuda.synchronize()
+                tt = []
+                for i in range(args.steps):
+                    bufs[0].copy_(rows[args.warmup + i])
+                    flush_l2(flush)
+                    e0.record(st)
+                    g2.replay()
+                    e1.record(st)
+                    e1.synchronize()
+                    tt.append(e0.elapsed_time(e1) / nl)
+                tp[str(P)] = round(max_over_ranks(sum(tt) / len(tt), ws) * 1e3, 2)
+                del g2
+            for l in dlayers:
+                l.set_decode_tp(0, 1)
+        decode["tp_rank_us_per_layer"] = tp
         for l in dlayers[1:]:
             l.close()
         del dlayers, graph
@@ -488,6 +522,7 @@ def main():
     ap.add_argument("--config", default="v3")
     ap.add_argument("--tokens", type=int, default=0)
     ap.add_argument("--no-decode", action="store_true")
+    ap.add_argument("--no-decode-tp", action="store_true", help="skip the decode-TP per-rank timing")
     ap.add_argument("--decode-layers", type=int, default=8, help="distinct layers chained in the decode graph")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")

@@ -196,6 +196,24 @@ typedef struct {
 } moe_layer_info;
 moe_status moe_layer_get_info(const moe_layer *layer, moe_layer_info *info);
 
+/* Decode tensor parallelism within every expert (the
+ * B200 analog of the paper's NUMA-aware TP, Fig. 8b).
+ * After moe_layer_set_decode_tp(layer, r, P), a decode forward (T <= the
+ * fused stream's limit, moe_layer_info.gemv_max_tokens) streams only the
+ * 128-column FFN chunks c with c % P == r of every active routed expert and
+ * of the shared expert -- W13 rows and W2 columns of the same chunk -- and
+ * writes this rank's PARTIAL output: y_r = bf16(sum over its chunks of the
+ * weighted expert partials), plus residual and deferred_in on rank 0 only
+ * (deferred_out likewise partial).  The caller all-reduces (sums) y_r over the
+ * P ranks; sum_r y_r equals the full layer's y up to the bf16 rounding of each
+ * partial.  Routing is replicated: every rank routes every token itself.
+ * Weights stay fully resident (each rank reads 1/P of the active bytes).
+ * size = 1 restores the normal forward.  Errors: INVALID_ARG (rank not in
+ * [0, size), size > F/128 or > Fs/128), UNSUPPORTED (expert-parallel layer,
+ * or no fused decode stream); a forward with T above the fused limit while
+ * size > 1 returns UNSUPPORTED.  Host-only; no device work.                  */
+moe_status moe_layer_set_decode_tp(moe_layer *layer, int32_t rank, int32_t size);
+
 /* Stage timing (instrumentation for the bench's roofline figures; off by
  * default).  When enabled, forward records a CUDA event after every stage on
  * the forward's stream (adds no synchronisation).  moe_layer_stage_times waits

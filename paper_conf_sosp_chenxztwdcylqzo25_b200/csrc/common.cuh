@@ -238,6 +238,7 @@ struct moe_layer {
   CUtensorMap dmap_xperm, dmap_h, dmap_xq, dmap_hsh;           // decode: activation rows (box 16)
   float *dacc = nullptr;        // fused decode: [2][gemv_max_tokens, H] fp32 sums (immediate, deferred), kept zero
   bool fused_decode = false;
+  int tp_rank = 0, tp_size = 1;   // decode TP (moe_layer_set_decode_tp)
   int n_launch = 0, launches_prefill = 0, launches_decode = 0;   // kernel launches per forward
   unsigned long long *trace = nullptr;   // MOE_DEBUG_TRACE timeline buffer (timing experiments)
   // swap-AB CTA-pair GEMM (umma_swap.cu): tiled weights as 128-byte rows (box 128),

@@ -254,6 +254,7 @@ struct FusedDecodeParams {
   unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
   int early_trigger;            // trigger the finalize launch when the CTA's producer runs out of units
   int fold_finalize;            // the last CTA runs the finalize (fin) itself (small T)
+  int tp_rank, tp_size;         // decode TP: stream chunks c = tp_rank (mod tp_size) only (0, 0/1 = all)
   DecodeFinalizeArgs fin;
 };
 cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, cudaStream_t st);

@@ -783,6 +783,9 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   const bool decode = L->gemv_ok && T <= L->gemv_max_tokens;
   const bool tc_decode = decode && L->umma && L->E_glob <= 256 && L->E <= 256;  // T <= 16: small-T route + swap-AB kernels
   const bool fused = tc_decode && L->fused_decode;  // route -> fused W13/W2 stream -> finalize (self-re-arming counters)
+  if (L->tp_size > 1 && !fused)
+    return fail(MOE_ERR_UNSUPPORTED, "decode TP (tp_size = %d) needs the fused decode stream: T = %d must be <= %d",
+                L->tp_size, T, L->gemv_max_tokens);
   if (!fused) CUDA_TRY(cudaMemsetAsync(L->sched, 0, 32, st));
   RouterArgs r{};
   r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
@@ -903,12 +906,16 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     fa.T = T; fa.H = H; fa.use_def = deferred_out != nullptr && n_def > 0;
     fa.acc_imm = acc_imm; fa.acc_def = acc_def;
     fa.residual = residual; fa.deferred_in = deferred_in; fa.y = y; fa.deferred_out = deferred_out;
+    if (L->tp_size > 1 && L->tp_rank != 0) fa.residual = fa.deferred_in = nullptr;   // added once, by TP rank 0
     fa.trace = L->trace;
     // MOE_DECODE_FOLD=1, T <= 2: the fused kernel's last CTA finalizes (no finalize launch)
     static const int fold_env = getenv("MOE_DECODE_FOLD") ? atoi(getenv("MOE_DECODE_FOLD")) : 0;   // measured slower
     fp.fold_finalize = fold_env && (int64_t)T * H <= 2 * 8192;
     fp.fin = fa;
-    const int units = (Fs > 0 ? Fs / 128 : 0) + (int)std::min<int64_t>(E, pairs) * (F / 128);
+    fp.tp_rank = L->tp_rank; fp.tp_size = L->tp_size;
+    const int tpP = L->tp_size, tpr = L->tp_rank;   // this rank's chunks: c = tpr (mod tpP)
+    const int units = (Fs > 0 ? (Fs / 128 - tpr + tpP - 1) / tpP : 0) +
+                      (int)std::min<int64_t>(E, pairs) * ((F / 128 - tpr + tpP - 1) / tpP);
     KL_TRY(launch_umma_decode_fused(f8, fp, std::min(L->num_sms, units), st));
     mark(L, ST_GEMM1, st);
     if (!fp.fold_finalize) {
@@ -1083,6 +1090,20 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
                         deferred_in ? deferred_in[r] : nullptr, y[r], want_def ? deferred_out[r] : nullptr, st)) != MOE_OK)
       return s;
   }
+  return MOE_OK;
+}
+
+moe_status moe_layer_set_decode_tp(moe_layer *L, int32_t rank, int32_t size) {
+  if (!L) return fail(MOE_ERR_INVALID_ARG, "null layer");
+  if (size < 1 || rank < 0 || rank >= size) return fail(MOE_ERR_INVALID_ARG, "tp rank %d / size %d", rank, size);
+  if (size > 1) {
+    if (L->ep.P > 1 || L->ep.comm) return fail(MOE_ERR_UNSUPPORTED, "decode TP on an expert-parallel layer");
+    if (!L->fused_decode || !L->umma) return fail(MOE_ERR_UNSUPPORTED, "decode TP needs the fused decode stream");
+    if (L->F / 128 < size || (L->Fs > 0 && L->Fs / 128 < size))
+      return fail(MOE_ERR_INVALID_ARG, "tp size %d > 128-column chunks (F/128 = %d, Fs/128 = %d)", size,
+                  L->F / 128, L->Fs / 128);
+  }
+  L->tp_rank = rank; L->tp_size = size;
   return MOE_OK;
 }
 

@@ -78,19 +78,24 @@ struct FdUnit {
 };
 
 __device__ __forceinline__ FdUnit fd_unit(const FusedDecodeParams &p, int u) {
+  // decode TP (moe_layer_set_decode_tp): this rank streams the chunks c = tp_rank + tp_size * j
+  // of every expert (W13 rows and W2 columns of the same 128 FFN columns), so its partial sum
+  // over chunks is its share of every expert's output
+  const int P = p.tp_size > 1 ? p.tp_size : 1, rk = P > 1 ? p.tp_rank : 0;
+  const int nl0 = (p.nch[0] - rk + P - 1) / P, nl1 = (p.nch[1] - rk + P - 1) / P;
   FdUnit r{};
-  const int ns = p.has_shared ? p.nch[1] : 0;
+  const int ns = p.has_shared ? nl1 : 0;
   if (u < ns) {
-    r.valid = 1; r.group = 1; r.expert = 0; r.row0 = 0; r.n = p.T; r.chunk = u;
+    r.valid = 1; r.group = 1; r.expert = 0; r.row0 = 0; r.n = p.T; r.chunk = rk + P * u;
     return r;
   }
   const int v = u - ns;
-  const int slot = v / p.nch[0];
+  const int slot = v / nl0;
   if (slot >= *p.n_active) return r;
   const int e = p.act_list[slot];
   // token-order activations (all T <= 16 tokens are the N = 16 operand; the
   // epilogue keeps the columns of the tokens routed to e)
-  r.valid = 1; r.group = 0; r.expert = e; r.row0 = 0; r.n = p.T; r.chunk = v % p.nch[0];
+  r.valid = 1; r.group = 0; r.expert = e; r.row0 = 0; r.n = p.T; r.chunk = rk + P * (v % nl0);
   return r;
 }
 

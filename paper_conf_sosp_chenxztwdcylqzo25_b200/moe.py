@@ -24,7 +24,7 @@ W_BF16, W_FP8, W_F32 = 0, 1, 2
 
 EXPORTED = ["moe_ep_group_forward", "moe_get_unique_id", "moe_layer_create", "moe_layer_forward", "moe_layer_forward_deferred",
             "moe_layer_destroy", "moe_status_string", "moe_last_error", "moe_layer_get_info",
-            "moe_layer_profile", "moe_layer_stage_times", "moe_stage_name"]
+            "moe_layer_profile", "moe_layer_stage_times", "moe_stage_name", "moe_layer_set_decode_tp"]
 
 
 class MoEConfig(ctypes.Structure):
@@ -80,11 +80,13 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
                                          ctypes.POINTER(vp), vp]
     lib.moe_ep_group_forward.restype = i32
     lib.moe_layer_profile.argtypes = [vp, i32]
+    lib.moe_layer_set_decode_tp.argtypes = [vp, i32, i32]
     lib.moe_layer_stage_times.argtypes = [vp, ctypes.POINTER(ctypes.c_float), i32, ctypes.POINTER(i32)]
     lib.moe_stage_name.argtypes = [i32]
     lib.moe_stage_name.restype = ctypes.c_char_p
     for f in ("moe_get_unique_id", "moe_layer_create", "moe_layer_forward", "moe_layer_forward_deferred",
-              "moe_layer_destroy", "moe_layer_get_info", "moe_layer_profile", "moe_layer_stage_times"):
+              "moe_layer_destroy", "moe_layer_get_info", "moe_layer_profile", "moe_layer_stage_times",
+              "moe_layer_set_decode_tp"):
         getattr(lib, f).restype = i32
     _lib = lib
     return lib
@@ -148,6 +150,11 @@ class MoELayer:
 
     def profile(self, enable: bool = True):
         _check(self._lib.moe_layer_profile(self._h, int(enable)), "moe_layer_profile")
+
+    def set_decode_tp(self, rank: int, size: int):
+        """Decode TP within every expert (include/moe.h moe_layer_set_decode_tp):
+        forwards then return this rank's partial y; the caller sums over ranks."""
+        _check(self._lib.moe_layer_set_decode_tp(self._h, int(rank), int(size)), "moe_layer_set_decode_tp")
 
     def stage_times(self) -> dict:
         """Per-stage ms of the last profiled forward (waits for it)."""
@@ -249,3 +256,13 @@ class MoEGroup:
     def close(self):
         for l in self.layers:
             l.close()
+
+
+def decode_tp_forward(layer: "MoELayer", x: torch.Tensor, residual: Optional[torch.Tensor] = None, group=None):
+    """One decode forward of a layer set up with set_decode_tp(rank, P) on each
+    of P processes: this rank's partial y (its 128-column chunks of every
+    expert), summed over the group with one all-reduce."""
+    import torch.distributed as dist
+    y = layer.forward(x, residual)
+    dist.all_reduce(y, group=group)
+    return y
