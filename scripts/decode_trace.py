@@ -16,6 +16,9 @@ x, _ = make_tokens(p, T, "cuda", offset=5)
 NL = int(sys.argv[3]) if len(sys.argv) > 3 else 1     # >1: trace the middle layer of a chained graph
 layers = [moe.MoELayer(p, w, max_tokens=16) for _ in range(NL)]
 layer = layers[NL // 2]
+TP = int(sys.argv[4]) if len(sys.argv) > 4 else 1     # >1: decode TP, rank 0's share (moe_layer_set_decode_tp)
+for l in layers:
+    l.set_decode_tp(0, TP)
 lib = layer._lib
 lib.moe_layer_debug_trace.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32]
 buf = np.zeros(4096, dtype=np.uint64)
