@@ -293,12 +293,15 @@ def test_decode_tp_errors(lib):
     layer.close()
 
 
-def test_full_v3_decode_tp_matches_whole(lib):
-    """Full DeepSeek-V3 layer (F/128 = Fs/128 = 16 chunks), T = 1 and 4: the P partials
-    sum to the single-GPU forward up to the bf16 rounding of each partial."""
-    p = PRESETS["v3"]
+@pytest.mark.parametrize("name,Ps", [("v3", (2, 4, 8, 16)), ("v25", (5, 8, 12)), ("qwen2", (3, 8, 20))])
+def test_full_decode_tp_matches_whole(lib, name, Ps):
+    """Full-size layers, T = 1 and 4: the P partials sum to the single-GPU forward up
+    to the bf16 rounding of each partial.  V3: F/128 = Fs/128 = 16 chunks; V2.5: 12 routed
+    chunks (P = 5, 8 give ranks 2-3 or 1-2 chunks: ragged); Qwen2 (BF16, gated shared
+    expert): 20 routed and 160 shared chunks."""
+    p = PRESETS[name]
     layer = lib.MoELayer(p, make_weights(p, "cuda"), max_tokens=16)
-    for P in (2, 4, 8, 16):
+    for P in Ps:
         for T in (1, 4):
             x, r = make_tokens(p, T, "cuda", offset=P)
             whole = layer.forward(x, residual=r).float()
