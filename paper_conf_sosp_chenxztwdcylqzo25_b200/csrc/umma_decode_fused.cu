@@ -269,9 +269,12 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         if (lane == 0) {
           const uint32_t a0 = smem_u32(sA + stage * FD_A_BYTES);
           const uint32_t b0 = smem_u32(sB + stage * FD_B_BYTES);
-          if (FP8) {
-            tmem_cp_32x128b_x4(tmem + FD_SFA_COL, sf_desc(smem_u32(sSFA + stage * FD_SF_BYTES)));
-            tmem_cp_32x128b_x4(tmem + FD_SFB_COL, sf_desc(smem_u32(sSFB + stage * FD_SF_BYTES)));
+          // scale images hold 4 k-blocks (scale id kb & 3): copy once per 4 k-blocks, into
+          // alternating column sets so the copy never overwrites scales in-flight MMAs read
+          const uint32_t sfset = (uint32_t)((kb >> 2) & 1) * 4;
+          if (FP8 && (kb & 3) == 0) {
+            tmem_cp_32x128b_x4(tmem + FD_SFA_COL + sfset, sf_desc(smem_u32(sSFA + stage * FD_SF_BYTES)));
+            tmem_cp_32x128b_x4(tmem + FD_SFB_COL + sfset, sf_desc(smem_u32(sSFB + stage * FD_SF_BYTES)));
           }
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
@@ -282,7 +285,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
               const uint64_t ad = sw128_kmajor_desc(a0 + t * 128 * 128 + k * 32);
               if (FP8)
                 mma_mxf8(tmem + FD_ACCA + t * 16, ad, bd, idesc_mxf8(128, FD_N, kb & 3, kb & 3), accum,
-                         tmem + FD_SFA_COL, tmem + FD_SFB_COL);
+                         tmem + FD_SFA_COL + sfset, tmem + FD_SFB_COL + sfset);
               else
                 mma_bf16(tmem + FD_ACCA + t * 16, ad, bd, idesc_bf16(128, FD_N), accum);
             }
