@@ -9,11 +9,14 @@ tokens shaped like the DeepSeek-V3 MoE layer (256 routed experts in 8 groups,
 top-4 groups, top-8, H 7168, F 2048, 1 shared expert, FP8 128x128 block-scaled
 weights; BASELINE.json configs[4]), prefill T = 8192 tokens per GPU.
 
-    python bench.py [--gpus N --steps K --warmup W] [--impl reference]
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--config v3|v25|qwen2|v2lite|all]
 
-N > 1: one process per GPU (torchrun), each rank runs an independent replica of
-the layer on its own tokens (weak scaling, no data-path collective; DESIGN.md
-§7), value = all ranks' tokens / max-over-ranks time.
+N > 1: one process per GPU.  Launched without torchrun, `--gpus N` re-executes
+itself under `torch.distributed.run --nproc-per-node N` (and exits with an
+error if fewer than N GPUs are visible).  Each rank owns E/N experts (expert
+parallelism over NCCL, DESIGN.md §7) and T tokens (weak scaling);
+`--replicas` runs N independent single-GPU layers instead.  value = all ranks'
+tokens / max-over-ranks time.
 
 Inputs are resident in HBM when the timed region starts; L2 is flushed (a
 256 MiB write, then a 256 MiB read so the dirty lines are written back before
@@ -129,21 +132,29 @@ def max_over_ranks(v: float, ws: int) -> float:
 
 
 # --------------------------------------------------------------------- oracle
-def oracle_tokens_per_s(p, w, x_rows, budget_s: float = 25.0):
-    """Time the CPU oracle (as it stands) on a bounded sample of tokens."""
-    import numpy as np
+def oracle_layer_call(p, w, x_rows):
+    """Time ONE full-layer call of the CPU oracle (as it stands: every expert the
+    batch hits is dequantised once in that call) on a bounded batch of tokens.
+    Returns (tokens/s, distinct experts hit, seconds)."""
     import torch
     from oracle import moe_oracle as O
     from tests.parity import oracle_cfg, oracle_weights
     cfg, W = oracle_cfg(p), oracle_weights(p, w)
-    done, t0 = 0, time.perf_counter()
-    for i in range(x_rows.shape[0]):
-        O.moe_layer(x_rows[i:i + 1].cpu().to(torch.float64).numpy(), W, cfg)
-        done += 1
-        if time.perf_counter() - t0 > budget_s:
-            break
+    x64 = x_rows.cpu().to(torch.float64).numpy()
+    t0 = time.perf_counter()
+    out = O.moe_layer(x64, W, cfg)
     dt = time.perf_counter() - t0
-    return done / dt, done, dt
+    return x64.shape[0] / dt, len(set(out["idx"].reshape(-1).tolist())), dt
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 def cpu_cores():
@@ -195,9 +206,11 @@ def algorithmic(p, T, n_distinct):
     H, F, Fs, k, E = p.hidden, p.ffn, p.shared_ffn, p.top_k, p.n_experts
     wb = 1 if p.wtype == 1 else 2
     exp_bytes = 3 * H * F * wb + (3 * (H // 128) * (F // 128) * 4 if p.wtype == 1 else 0)
+    # one launch computes the routed experts AND the shared expert (two operand groups)
     return {
-        "gemm1_swiglu": {"flops": 2.0 * T * k * 2 * F * H, "bytes": n_distinct * 2 * H * F * wb},
-        "gemm2": {"flops": 2.0 * T * k * H * F, "bytes": n_distinct * H * F * wb},
+        "gemm1_swiglu": {"flops": 2.0 * T * k * 2 * F * H + 2.0 * T * 2 * Fs * H,
+                         "bytes": n_distinct * 2 * H * F * wb + 2 * H * Fs * wb},
+        "gemm2": {"flops": 2.0 * T * k * H * F + 2.0 * T * H * Fs, "bytes": n_distinct * H * F * wb + H * Fs * wb},
         "shared_gemm1": {"flops": 2.0 * T * 2 * Fs * H, "bytes": 2 * H * Fs * wb},
         "shared_gemm2": {"flops": 2.0 * T * H * Fs, "bytes": H * Fs * wb},
         "router_logits": {"flops": 2.0 * T * H * E, "bytes": E * H * 2 + T * H * 2},
@@ -296,7 +309,9 @@ def run_ours(args):
         n_distinct = int((counts > 0).sum())
     alg = algorithmic(p, T, n_distinct)
     fp8 = p.wtype == 1
-    tc_peak = (2.0 if fp8 else 1.0) * peaks["bf16_tflops_sustained"]
+    # the prefill step is a few ms: the kernel runs at its burst clock, so the peak is the
+    # burst figure (MEASURED_PEAKS.json bf16_tflops, FP8 = 2x, the nominal dtype ratio)
+    tc_peak = (2.0 if fp8 else 1.0) * peaks["bf16_tflops"]
     if stages:
         dom = max((k for k in stages if k in alg), key=lambda k: stages[k])
         dom_ms = stages[dom]
@@ -308,12 +323,17 @@ def run_ours(args):
     tpath = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tpath):
         traffic = json.load(open(tpath)).get(f"{p.name}:{T}:{dom}")
+    layer_tflops = alg["layer_flops"] / (ms * 1e-3) / 1e12
     roofline = {"bound": "tensor", "kernel": dom, "achieved": ach, "peak": tc_peak, "unit": "TFLOP/s",
                 "frac": ach / tc_peak, "traffic": traffic,
-                "peak_source": f"{peaks['_source']}: bf16_tflops_sustained x {'2 (fp8/bf16 nominal ratio)' if fp8 else '1'}",
-                "algorithmic": f"2*T*k*{'2F*H' if dom == 'gemm1_swiglu' else 'H*F'} flops per launch, T={T}",
+                "peak_source": f"{peaks['_source']}: bf16_tflops (burst) x {'2 (fp8/bf16 nominal ratio)' if fp8 else '1'}",
+                "algorithmic": (f"2*T*(k*{'2F*H' if dom == 'gemm1_swiglu' else 'H*F'} + "
+                                f"{'2Fs*H' if dom == 'gemm1_swiglu' else 'H*Fs'}) flops per launch (routed + shared "
+                                f"expert operand groups), T={T}"),
+                "kernel_ms": dom_ms,
+                "layer": {"achieved": layer_tflops, "frac": layer_tflops / tc_peak,
+                          "flops": alg["layer_flops"], "ms": ms},
                 "stage_ms": {k: round(v, 4) for k, v in stages.items()}}
-    layer_tflops = alg["layer_flops"] / (ms * 1e-3) / 1e12
 
     # ---------------- decode, T = 1: a chain of distinct layers ----------------
     # The decode step is one CUDA graph replay over a stack of `--decode-layers`
@@ -485,10 +505,12 @@ def run_ours(args):
     # ---------------- CPU oracle on a bounded sample (rank 0, N = 1) ----------------
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu:
-        v, n, dt = oracle_tokens_per_s(p, w, x[:64], budget_s=args.cpu_budget)
-        cpu = {"value": v, "unit": "tokens/s", "cores": cpu_cores(), "kind": "oracle",
-               "sample": f"{n} tokens of the same batch, one oracle call per token ({dt:.1f} s, fp64 numpy, "
-                         "experts dequantised per call)"}
+        nt = min(args.cpu_tokens, T)
+        v, nexp, dt = oracle_layer_call(p, w, x[:nt])
+        cpu = {"value": v, "unit": "tokens/s", "cores": cpu_cores(), "cpu_model": cpu_model(), "kind": "oracle",
+               "sample": f"one full-layer oracle call (oracle.moe_layer) on the first {nt} tokens of the same "
+                         f"batch: {nexp} distinct experts, each dequantised once in the call; {dt:.1f} s, fp64 "
+                         "numpy, BLAS threads = the host cores"}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": ws, "steps": args.steps,
@@ -526,15 +548,38 @@ def main():
     ap.add_argument("--decode-layers", type=int, default=8, help="distinct layers chained in the decode graph")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--cpu-budget", type=float, default=20.0)
+    ap.add_argument("--cpu-tokens", type=int, default=16, help="tokens of the cpu_baseline oracle call")
     ap.add_argument("--replicas", action="store_true", help="N>1: independent replicas instead of expert parallel")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3
     if args.impl == "reference":
         run_reference(args)
-    else:
-        run_ours(args)
+        return
+    ws = os.environ.get("WORLD_SIZE")
+    if args.gpus > 1 and ws is None:
+        # one process per GPU: re-execute under torchrun (the driver launches it that way itself)
+        import torch
+        n = torch.cuda.device_count()
+        if n < args.gpus:
+            print(f"bench.py: --gpus {args.gpus} needs {args.gpus} visible GPUs, found {n}", file=sys.stderr)
+            sys.exit(2)
+        import socket
+        with socket.socket() as sk:
+            sk.bind(("127.0.0.1", 0))
+            port = sk.getsockname()[1]
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+        sys.exit(subprocess.call(cmd))
+    if ws is not None and int(ws) != args.gpus:
+        print(f"bench.py: WORLD_SIZE={ws} but --gpus {args.gpus}", file=sys.stderr)
+        sys.exit(2)
+    if args.config == "all":
+        for c in ("v3", "v25", "qwen2", "v2lite"):
+            args.config = c
+            run_ours(args)
+        return
+    run_ours(args)
 
 
 if __name__ == "__main__":

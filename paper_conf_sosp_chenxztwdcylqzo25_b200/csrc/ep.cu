@@ -165,11 +165,13 @@ const char *ep_nccl_error(void *comm) {
 int ep_nccl_counts(void *comm, const int32_t *send_cnt, int32_t *recv_cnt, int P, cudaStream_t st) {
   ncclComm_t c = reinterpret_cast<ncclComm_t>(comm);
   if (ncclGroupStart() != ncclSuccess) return -1;
-  for (int p = 0; p < P; ++p) {
-    if (ncclSend(send_cnt + p, 1, ncclInt32, p, c, st) != ncclSuccess) return -1;
-    if (ncclRecv(recv_cnt + p, 1, ncclInt32, p, c, st) != ncclSuccess) return -1;
+  bool ok = true;                       // the group is always closed, even after a failed call
+  for (int p = 0; p < P && ok; ++p) {
+    ok = ncclSend(send_cnt + p, 1, ncclInt32, p, c, st) == ncclSuccess;
+    ok = ok && ncclRecv(recv_cnt + p, 1, ncclInt32, p, c, st) == ncclSuccess;
   }
-  return ncclGroupEnd() == ncclSuccess ? 0 : -1;
+  const bool closed = ncclGroupEnd() == ncclSuccess;
+  return ok && closed ? 0 : -1;
 }
 
 // all-to-all-v of up to 3 row-major buffers (bytes per row each): send_cnt[p]
@@ -180,14 +182,16 @@ int ep_nccl_rows(void *comm, int P, const int32_t *send_cnt, const int64_t *send
                  const int64_t *row_bytes, cudaStream_t st) {
   ncclComm_t c = reinterpret_cast<ncclComm_t>(comm);
   if (ncclGroupStart() != ncclSuccess) return -1;
-  for (int p = 0; p < P; ++p)
-    for (int b = 0; b < nbuf; ++b) {
+  bool ok = true;                       // the group is always closed, even after a failed call
+  for (int p = 0; p < P && ok; ++p)
+    for (int b = 0; b < nbuf && ok; ++b) {
       const char *sp = reinterpret_cast<const char *>(send[b]) + send_off[p] * row_bytes[b];
       char *rp = reinterpret_cast<char *>(recv[b]) + (int64_t)recv_off[p] * row_bytes[b];
-      if (send_cnt[p] && ncclSend(sp, (size_t)send_cnt[p] * row_bytes[b], ncclUint8, p, c, st) != ncclSuccess) return -1;
-      if (recv_cnt[p] && ncclRecv(rp, (size_t)recv_cnt[p] * row_bytes[b], ncclUint8, p, c, st) != ncclSuccess) return -1;
+      if (send_cnt[p]) ok = ncclSend(sp, (size_t)send_cnt[p] * row_bytes[b], ncclUint8, p, c, st) == ncclSuccess;
+      if (ok && recv_cnt[p]) ok = ncclRecv(rp, (size_t)recv_cnt[p] * row_bytes[b], ncclUint8, p, c, st) == ncclSuccess;
     }
-  return ncclGroupEnd() == ncclSuccess ? 0 : -1;
+  const bool closed = ncclGroupEnd() == ncclSuccess;
+  return ok && closed ? 0 : -1;
 }
 
 }  // namespace moe

@@ -335,7 +335,7 @@ cudaError_t launch_router_gemv(const void *x, int T, int H, const void *wg, int 
 template <class K>
 static cudaError_t set_smem(K kern, size_t bytes) {
   if (bytes <= 48 * 1024) return cudaSuccess;
-  return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  return set_kernel_attr((const void *)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
 }
 
 size_t gemv_smem_bytes(int T, int H, int F, int Fs) {

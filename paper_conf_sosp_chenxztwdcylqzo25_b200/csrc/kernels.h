@@ -13,6 +13,22 @@
 
 namespace moe {
 
+// Timing-experiment knobs (stale-smem / loads-only GEMM modes, router phase
+// skips, PDL off): compiled in only with -DMOE_EXPERIMENTS (build.py,
+// MOE_EXPERIMENTS=1); the default library ignores the environment and every
+// knob reads 0, so no stray variable can change a result.
+#ifdef MOE_EXPERIMENTS
+constexpr bool kExperiments = true;
+#else
+constexpr bool kExperiments = false;
+#endif
+int experiment_knob(const char *env);
+
+// cudaFuncSetAttribute acts on the CURRENT device only: remember the
+// (kernel, device, attribute) triples already set instead of one process-wide
+// flag, so a process that drives several GPUs opts in on each of them.
+cudaError_t set_kernel_attr(const void *kernel, cudaFuncAttribute attr, int value);
+
 // Launch with programmatic dependent launch (PDL): the kernel may start while
 // its stream predecessor is still running and must execute pdl_wait() before
 // touching the predecessor's outputs (CUDA-graph capturable).
@@ -28,7 +44,7 @@ cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t s
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  static const bool no_pdl = getenv("MOE_NO_PDL") && atoi(getenv("MOE_NO_PDL")) == 1;   // A/B experiments
+  static const bool no_pdl = experiment_knob("MOE_NO_PDL") == 1;   // A/B experiments (MOE_EXPERIMENTS only)
   cfg.numAttrs = no_pdl ? 0 : 1;
   return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
 }
@@ -94,16 +110,13 @@ struct RouteSmallArgs {
   const void *wg;               // bf16 [rows, H]
   int H, rows;
   int *done;                    // zero-initialised CTA counter (re-armed by the kernel)
-  int debug;                    // timing experiments only (MOE_DEBUG_ROUTE): 1 skip logits, 2 skip tail
-  // activations into expert order (null xperm = skip): bf16 copy or e4m3 + scale images
+  int debug;                    // timing experiments only (MOE_EXPERIMENTS builds, MOE_DEBUG_ROUTE)
+  // FP8: x quantised in token order (1x128 UE8M0 + e4m3) for the fused decode stream
   int fp8;
-  void *xperm; uint8_t *xperm_img; int xperm_img_stride;
-  void *xq; float *xs; uint8_t *xq_img; int xq_img_stride;   // shared expert (FP8)
-  // shared-expert weights prefetched into L2 while the router runs (they do
-  // not depend on the routing): [pf[i], pf[i] + pf_bytes[i]), i < 2
-  const void *pf[2]; int64_t pf_bytes[2];
+  void *xq; float *xs; uint8_t *xq_img; int xq_img_stride;
   unsigned long long *trace;     // MOE_DEBUG_TRACE: [0] CTA 0 entry, [1..4] tail start / select / permute / end
-  int minimal;                  // fused decode: active-expert list only (no sorted rows / positions)
+  // The tail writes only the active-expert list unless dbg_perm / dbg_counts
+  // ask for the full counts and permutation (parity outputs).
 };
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st);
 
@@ -169,57 +182,24 @@ int ep_nccl_rows(void *comm, int P, const int32_t *send_cnt, const int64_t *send
                  const int64_t *recv_off, int nbuf, const void *const *send, void *const *recv,
                  const int64_t *row_bytes, cudaStream_t st);
 
-// ---------------------------------------------------------------- tcgen05 GEMM
-struct UmmaGroup {              // one operand set: 0 = routed experts, 1 = shared expert
-  CUtensorMap a_map;            // A rows, K-major, box 128 B x 128 rows, SW128
-  CUtensorMap b_map;            // B rows via TMA (router logits only; expert weights are tiled)
-  const uint8_t *b_tiles;       // tiled weights: [expert][N/256][K/128B][256 rows x 128 B, SW128]
-  int b_ntiles_n;               // N / 256
-  const uint8_t *sfa;           // FP8: A scale image [K/512][tiles][512 B]
-  const uint8_t *sfb;           // FP8: B scale image [expert][K/512][N/128][512 B]
-  int64_t sfb_expert_stride;    // bytes
-  int sfa_tile_stride;          // 128-row tiles per k-group in the A image
-  int sfb_rb;                   // N/128
-  int n_total;                  // N (B rows per expert)
-  int kblocks;                  // K / 128 bytes
-  void *out;                    // C rows
-  int64_t ldc;                  // elements
-  uint8_t *out_sf;              // FP8 SwiGLU: scale image of h
-  int out_sf_tile_stride;
-  int n_valid;                  // LOGITS: output columns < n_valid are written
-  CUtensorMap sfa_map, sfb_map; // CTA-pair kernel: scale images as 512-byte rows (box 1 / 2 rows)
+// ---------------------------------------------------------------- tcgen05 router logits
+struct LogitsParams {
+  CUtensorMap a_map;            // x [T, H] bf16, K-major SW128, box 64 x 128 rows
+  CUtensorMap b_map;            // router rows [gate_rows, H] bf16, box 64 x 256 rows
+  int kblocks;                  // H / 64
+  float *out;                   // logits [T, ldc] fp32
+  int64_t ldc;
+  int n_valid;                  // columns < n_valid are written
+  int T;                        // token rows
+  int nb;                       // 256-row blocks of router rows
+  int *sched;                   // device work counter, zero at launch
 };
-struct UmmaParams {
-  UmmaGroup g[2];
-  const int4 *tiles;            // routed tiles (expert, row0, row_end, t0 | nt << 16)
-  const int32_t *n_tiles;
-  int nb_r;                     // routed N blocks of 256
-  int T_shared;                 // shared-expert rows (0 = none)
-  int nb_s;                     // shared N blocks of 256
-  int *sched;                   // device work counter, zero at launch (dynamic scheduler)
-  const int4 *pairs;            // CTA-pair kernel: routed work list of 256-row tile pairs
-  const int32_t *n_pairs;
-  int debug_mode;               // 0; (MOE_DEBUG_GEMM) 1 = loads only, 2 = no epilogue -- timing experiments
-  int pf_dist;                  // weight k-blocks prefetched into L2 ahead of the TMA loads (0 = off)
-};
-cudaError_t launch_umma_gemm(bool fp8, int epi, const UmmaParams &p, int grid, cudaStream_t st);
+cudaError_t launch_umma_logits(const LogitsParams &p, int grid, cudaStream_t st);
 // Repack row-major weights [rows, K] (es bytes/elem) into 256-row x 128-byte
 // tiles, 128B-swizzled (the smem image TMA would produce).  interleave_f > 0:
 // rows are W13 [2F, K] and tile rows are ordered (W1 block b, W3 block b) per 128.
 cudaError_t launch_tile_weights(const void *src, void *dst, int nexp, int rows, int kbytes, int interleave_f,
                                 cudaStream_t st);
-
-// decode (swap-AB): a_map = activation rows (box 16), b_map = weight rows (box 128),
-// sfa = activation scale image, sfb = weight scale image (same fields as UmmaGroup)
-struct UmmaDecodeParams {
-  UmmaGroup g[2];               // 0 routed, 1 shared
-  int g_nblk[2];                // 128-row blocks per group (MODE 1: F/128, MODE 2: H/128)
-  int nblk;                     // max of g_nblk
-  int max_slots, has_shared, T;
-  const int32_t *n_active, *act_list, *counts, *offs_pad;
-  int *sched;
-};
-cudaError_t launch_umma_decode(bool fp8, int mode, const UmmaDecodeParams &p, int grid, cudaStream_t st);
 
 // decode, fused per (slot, 128-column FFN chunk) unit (umma_decode_fused.cu):
 // W13 tile -> SwiGLU (+ FP8 requant) -> h_c in smem -> W2 column block ->
@@ -250,12 +230,8 @@ struct FusedDecodeParams {
   const float *topk_w, *sgate;  // sgate null unless the shared expert is gated (Qwen2)
   float *acc_imm, *acc_def;     // [T, H] fp32 sums, zero on entry (re-zeroed by decode_finalize)
   int *sched, *done;            // work counter + exit ticket, zero on entry (re-armed by the kernel)
-  const void *pf[2]; int64_t pf_bytes[2];   // shared-expert weights prefetched into L2 before the PDL wait
   unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
-  int early_trigger;            // trigger the finalize launch when the CTA's producer runs out of units
-  int fold_finalize;            // the last CTA runs the finalize (fin) itself (small T)
   int tp_rank, tp_size;         // decode TP: stream chunks c = tp_rank (mod tp_size) only (0, 0/1 = all)
-  DecodeFinalizeArgs fin;
 };
 cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, cudaStream_t st);
 cudaError_t launch_decode_finalize(const DecodeFinalizeArgs &a, cudaStream_t st);

@@ -9,12 +9,21 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "common.cuh"
 #include "kernels.h"
 
 using namespace moe;
 
 namespace {
+// NVTX range for the host-side enqueue of a call (nsys / ncu --nvtx); header-only
+// NVTX v3, a no-op unless a tool is attached
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+
 thread_local std::string g_err;
 
 moe_status fail(moe_status s, const char *fmt, ...) {
@@ -268,6 +277,7 @@ moe_status moe_get_unique_id(void *out128) {
 }
 
 moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights *w, moe_layer **out) {
+  NvtxRange nvtx("moe_layer_create");
   if (!out) return fail(MOE_ERR_INVALID_ARG, "null out");
   *out = nullptr;
   moe_status st = validate(cfg, w);
@@ -472,13 +482,11 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
       }
     }
     if (!ok) return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed (driver entry point unavailable?)"));
-    // fused decode (umma_decode_fused.cu) unless MOE_DECODE_CHAIN=1 selects the two-launch chain
     if (getenv("MOE_DEBUG_TRACE")) {               // timing experiments: device timeline buffer
       C_TRY(dalloc(L, &L->trace, 4096 * 8, false));
       C_TRY(cudaMemset(L->trace, 0, 4096 * 8));
     }
-    const char *chain = getenv("MOE_DECODE_CHAIN");
-    L->fused_decode = L->gemv_ok && !(chain && atoi(chain) == 1);
+    L->fused_decode = L->gemv_ok;            // decode (T <= 16): the fused stream of umma_decode_fused.cu
     if (L->fused_decode) {
       const size_t n = (size_t)2 * L->gemv_max_tokens * H * 4;
       C_TRY(dalloc(L, &L->dacc, n, false));
@@ -498,6 +506,7 @@ static const char *kStageNames[moe_layer::kStages] = {
 enum { ST_LOGITS = 0, ST_SELECT, ST_PERMUTE, ST_QUANT, ST_GATHER, ST_GEMM1, ST_GEMM2, ST_SH1, ST_SH2, ST_COMBINE };
 
 static inline void mark(moe_layer *L, int stage, cudaStream_t st) {
+  nvtxMarkA(kStageNames[stage]);
   if (!L->prof) return;
   cudaEventRecord(L->ev[stage + 1], st);
   L->ev_hit[stage + 1] = true;
@@ -519,7 +528,7 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     // tcgen05 launch per GEMM (umma_swap.cu)
     const bool f8 = L->fp8;
     const int kdiv = f8 ? 128 : 64;
-    static const int dbg_mode = getenv("MOE_DEBUG_GEMM") ? atoi(getenv("MOE_DEBUG_GEMM")) : 0;
+    static const int dbg_mode = experiment_knob("MOE_DEBUG_GEMM");   // timing experiments (MOE_EXPERIMENTS builds)
     SwapParams p1{};
     {
       SwapGroup &g = p1.g[0];
@@ -611,21 +620,26 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
 //   -- return the partial rows to their origin --
 //   D  origin: y = residual + shared + sum of partials (+ deferred_in)
 // ======================================================================
+// router logits of T > 8 tokens: tcgen05 BF16 GEMM (umma_gemm.cu), fp32 out (reading R9)
+static moe_status launch_logits(moe_layer *L, const void *x, int T, cudaStream_t st) {
+  LogitsParams p{};
+  if (!make_kmajor_map(&p.a_map, x, false, T, L->H, 128)) return fail(MOE_ERR_CUDA, "tensor map for x failed");
+  p.b_map = L->map_gate;
+  p.kblocks = L->H / 64; p.out = L->logits; p.ldc = L->gate_rows; p.n_valid = L->gate_rows;
+  p.T = T; p.nb = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
+  const int units = ((T + 127) / 128) * p.nb;
+  KL_TRY(launch_umma_logits(p, std::min(units, L->num_sms), st));
+  return MOE_OK;
+}
+
 static moe_status run_router_full(moe_layer *L, const void *x, int T, cudaStream_t st) {
   if (T <= 0) return MOE_OK;
   const int H = L->H;
   if (T <= kGemvMaxTokens) {
     KL_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
   } else {
-    UmmaParams p{};
-    UmmaGroup &g = p.g[1];
-    if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) return fail(MOE_ERR_CUDA, "tensor map for x failed");
-    g.b_map = L->map_gate;
-    g.n_total = 0; g.kblocks = H / 64; g.out = L->logits; g.ldc = L->gate_rows; g.n_valid = L->gate_rows;
-    p.g[0] = g;
-    p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
-    const int units = ((T + 127) / 128) * p.nb_s;
-    KL_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
+    moe_status s = launch_logits(L, x, T, st);
+    if (s != MOE_OK) return s;
   }
   RouterArgs r{};
   r.logits = L->logits; r.ldl = L->gate_rows; r.bias = L->gate_bias;
@@ -760,6 +774,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
                                const void *deferred_in, void *y, void *deferred_out, moe_routing_out *dbg,
                                void *stream) {
   if (!L) return fail(MOE_ERR_INVALID_ARG, "null layer");
+  NvtxRange nvtx(T <= L->gemv_max_tokens ? "moe_layer_forward/decode" : "moe_layer_forward/prefill");
   if (T < 0) return fail(MOE_ERR_INVALID_ARG, "T = %d < 0", T);
   if (T > L->max_tokens) return fail(MOE_ERR_CAPACITY, "T = %d > max_tokens = %d", T, L->max_tokens);
   if (n_def < 0 || n_def > L->k - 1) return fail(MOE_ERR_INVALID_ARG, "n_deferred = %d not in [0, k-1]", n_def);
@@ -805,15 +820,11 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     // 1-3 (decode). logits + select + count/scan/assign in one launch
     RouteSmallArgs rs{};
     rs.r = r; rs.p = pa; rs.x = x; rs.wg = L->gate_w; rs.H = H; rs.rows = L->gate_rows; rs.done = L->sched + 7;
-    static const int dbg_route = getenv("MOE_DEBUG_ROUTE") ? atoi(getenv("MOE_DEBUG_ROUTE")) : 0;
+    static const int dbg_route = experiment_knob("MOE_DEBUG_ROUTE");   // timing experiments (MOE_EXPERIMENTS builds)
     rs.debug = dbg_route;
     rs.trace = L->trace;
-    rs.fp8 = L->fp8; rs.xperm = fused ? nullptr : L->xperm; rs.xperm_img = L->xperm_img;
-    rs.xperm_img_stride = L->max_tiles; rs.minimal = fused;
+    rs.fp8 = L->fp8;
     if (L->fp8) { rs.xq = L->xq; rs.xs = L->xs; rs.xq_img = L->xq_img; rs.xq_img_stride = L->img_tiles_sh; }
-    if (Fs > 0 && L->umma && T <= L->gemv_max_tokens && !fused) {
-      rs.pf[0] = L->ws13; rs.pf_bytes[0] = (int64_t)2 * Fs * H * (L->fp8 ? 1 : 2);
-    }
     KL_TRY(launch_route_small(rs, st));
     mark(L, ST_PERMUTE, st);
   } else {
@@ -821,15 +832,8 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     if (T <= kGemvMaxTokens) {
       KL_TRY(launch_router_gemv(x, T, H, L->gate_w, L->gate_rows, L->logits, st));
     } else {
-      UmmaParams p{};
-      UmmaGroup &g = p.g[1];
-      if (!make_kmajor_map(&g.a_map, x, false, T, H, 128)) return fail(MOE_ERR_CUDA, "tensor map for x failed");
-      g.b_map = L->map_gate;
-      g.n_total = 0; g.kblocks = H / 64; g.out = L->logits; g.ldc = L->gate_rows; g.n_valid = L->gate_rows;
-      p.g[0] = g;
-      p.T_shared = T; p.nb_s = (L->gate_rows + 255) / 256; p.sched = L->sched + 2;
-      const int units = ((T + 127) / 128) * p.nb_s;
-      KL_TRY(launch_umma_gemm(false, GEMM_LOGITS, p, std::min(units, L->num_sms), st));
+      moe_status s = launch_logits(L, x, T, st);
+      if (s != MOE_OK) return s;
     }
     mark(L, ST_LOGITS, st);
     // 2. scores + group-limited top-k + weights
@@ -883,11 +887,6 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
         g.w13_img = L->ws13_img; g.w13_img_stride = 0;
         g.x_img = L->xq_img; g.x_img_stride = L->img_tiles_sh; g.w2_s = L->ws2_s;
       }
-      static const int pf_mode = getenv("MOE_DECODE_PF") ? atoi(getenv("MOE_DECODE_PF")) : 0;
-      if (pf_mode == 1) {                        // A/B: shared-expert L2 prefetch during routing
-        fp.pf[0] = L->ws13; fp.pf_bytes[0] = (int64_t)2 * Fs * H * (f8 ? 1 : 2);
-        fp.pf[1] = L->ws2; fp.pf_bytes[1] = (int64_t)H * Fs * (f8 ? 1 : 2);
-      }
     } else {
       fp.g[1] = fp.g[0];
     }
@@ -900,85 +899,20 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     fp.acc_imm = acc_imm; fp.acc_def = acc_def;
     fp.sched = L->sched + 5; fp.done = L->sched + 6;
     fp.trace = L->trace;
-    static const int late_trig = getenv("MOE_DECODE_LATE_TRIGGER") ? atoi(getenv("MOE_DECODE_LATE_TRIGGER")) : 0;
-    fp.early_trigger = !late_trig;
     DecodeFinalizeArgs fa{};
     fa.T = T; fa.H = H; fa.use_def = deferred_out != nullptr && n_def > 0;
     fa.acc_imm = acc_imm; fa.acc_def = acc_def;
     fa.residual = residual; fa.deferred_in = deferred_in; fa.y = y; fa.deferred_out = deferred_out;
     if (L->tp_size > 1 && L->tp_rank != 0) fa.residual = fa.deferred_in = nullptr;   // added once, by TP rank 0
     fa.trace = L->trace;
-    // MOE_DECODE_FOLD=1, T <= 2: the fused kernel's last CTA finalizes (no finalize launch)
-    static const int fold_env = getenv("MOE_DECODE_FOLD") ? atoi(getenv("MOE_DECODE_FOLD")) : 0;   // measured slower
-    fp.fold_finalize = fold_env && (int64_t)T * H <= 2 * 8192;
-    fp.fin = fa;
     fp.tp_rank = L->tp_rank; fp.tp_size = L->tp_size;
     const int tpP = L->tp_size, tpr = L->tp_rank;   // this rank's chunks: c = tpr (mod tpP)
     const int units = (Fs > 0 ? (Fs / 128 - tpr + tpP - 1) / tpP : 0) +
                       (int)std::min<int64_t>(E, pairs) * ((F / 128 - tpr + tpP - 1) / tpP);
     KL_TRY(launch_umma_decode_fused(f8, fp, std::min(L->num_sms, units), st));
     mark(L, ST_GEMM1, st);
-    if (!fp.fold_finalize) {
-      KL_TRY(launch_decode_finalize(fa, st));
-      mark(L, ST_COMBINE, st);
-    }
-  } else if (decode && L->umma) {
-    // 5+6 (decode). swap-AB tensor-core weight stream over the active experts + shared expert
-    const bool f8 = L->fp8;
-    const int kdiv = f8 ? 128 : 64;
-    const int slots = (int)std::min<int64_t>(E, pairs) + (Fs > 0 ? 1 : 0);
-    // (activations were quantised into expert order by the route kernel's tail)
-    UmmaDecodeParams d1{};
-    {
-      UmmaGroup &g = d1.g[0];
-      g.a_map = L->dmap_xperm; g.b_tiles = (const uint8_t *)L->w13; g.b_ntiles_n = 2 * F / 256;
-      g.sfa = L->xperm_img; g.sfa_tile_stride = L->max_tiles;
-      g.sfb = L->w13_img; g.sfb_expert_stride = L->w13_img_stride; g.sfb_rb = F / 128;
-      g.n_total = 2 * F; g.kblocks = H / kdiv;
-      g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
-    }
-    if (Fs > 0) {
-      UmmaGroup &g = d1.g[1];
-      if (f8) {
-        g.a_map = L->dmap_xq;
-      } else if (!make_kmajor_map(&g.a_map, x, false, T, H, 16)) {
-        return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
-      }
-      g.b_tiles = (const uint8_t *)L->ws13; g.b_ntiles_n = 2 * Fs / 256;
-      g.sfa = L->xq_img; g.sfa_tile_stride = L->img_tiles_sh;
-      g.sfb = L->ws13_img; g.sfb_rb = Fs / 128; g.n_total = 0; g.kblocks = H / kdiv;
-      g.out = L->hsh; g.ldc = Fs; g.out_sf = L->hsh_img; g.out_sf_tile_stride = L->img_tiles_sh;
-    } else {
-      d1.g[1] = d1.g[0];
-    }
-    d1.g_nblk[0] = F / 128; d1.g_nblk[1] = Fs / 128; d1.nblk = std::max(F, Fs) / 128;
-    d1.max_slots = slots; d1.has_shared = Fs > 0; d1.T = T;
-    d1.n_active = L->n_active; d1.act_list = L->act_list; d1.counts = L->counts; d1.offs_pad = L->offs_pad;
-    d1.sched = L->sched + 3;
-    KL_TRY(launch_umma_decode(f8, 1, d1, std::min(L->num_sms, slots * d1.nblk), st));
-    mark(L, ST_GEMM1, st);
-    UmmaDecodeParams d2 = d1;
-    {
-      UmmaGroup &g = d2.g[0];
-      g.a_map = L->dmap_h; g.b_tiles = (const uint8_t *)L->w2; g.b_ntiles_n = H / 256;
-      g.sfa = L->h_img; g.sfa_tile_stride = L->max_tiles;
-      g.sfb = L->w2_img; g.sfb_expert_stride = L->w2_img_stride; g.sfb_rb = H / 128;
-      g.n_total = H; g.kblocks = F / kdiv;
-      g.out = L->yperm; g.ldc = H; g.out_sf = nullptr;
-    }
-    if (Fs > 0) {
-      UmmaGroup &g = d2.g[1];
-      g.a_map = L->dmap_hsh; g.b_tiles = (const uint8_t *)L->ws2; g.b_ntiles_n = H / 256;
-      g.sfa = L->hsh_img; g.sfa_tile_stride = L->img_tiles_sh;
-      g.sfb = L->ws2_img; g.sfb_rb = H / 128; g.n_total = 0; g.kblocks = Fs / kdiv;
-      g.out = L->ysh; g.ldc = H; g.out_sf = nullptr;
-    } else {
-      d2.g[1] = d2.g[0];
-    }
-    d2.g_nblk[0] = H / 128; d2.g_nblk[1] = H / 128; d2.nblk = H / 128;
-    d2.sched = L->sched + 4;
-    KL_TRY(launch_umma_decode(f8, 2, d2, std::min(L->num_sms, slots * d2.nblk), st));
-    mark(L, ST_GEMM2, st);
+    KL_TRY(launch_decode_finalize(fa, st));
+    mark(L, ST_COMBINE, st);
   } else if (decode) {
     // 5+6 (decode, CUDA-core path). weight-streaming GEMVs over the active experts + shared expert
     GemvArgs g{};
@@ -1033,6 +967,7 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
                                 const void *const *deferred_in, void *const *y, void *const *deferred_out,
                                 void *stream) {
   if (!layers || !x || !y || !T || P < 2 || P > 32) return fail(MOE_ERR_INVALID_ARG, "bad group arguments");
+  NvtxRange nvtx("moe_ep_group_forward");
   for (int r = 0; r < P; ++r) {
     moe_layer *L = layers[r];
     if (!L || L->ep.P != P || L->ep.rank != r || L->ep.comm)

@@ -139,7 +139,7 @@ cudaError_t launch_permute(const PermuteArgs &a, cudaStream_t st) {
   scan_kernel<<<1, SCAN_THREADS, 0, st>>>(a, nchunk);
   const size_t sm = (size_t)a.E * kMaskWords * sizeof(uint32_t);
   if (sm > 48 * 1024) {
-    cudaError_t e = cudaFuncSetAttribute(assign_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaError_t e = set_kernel_attr((const void *)assign_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
   }
   assign_kernel<<<nchunk, 256, sm, st>>>(a);

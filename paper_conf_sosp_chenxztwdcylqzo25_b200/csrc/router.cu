@@ -390,9 +390,9 @@ __global__ void __launch_bounds__(RT_WARPS * 32) router_select_regs_kernel(const
 __device__ void route_small_tail(const RouteSmallArgs &a, float *rsm, const float *bias_pre) {
   const RouterArgs &r = a.r;
   const PermuteArgs &p = a.p;
-  const int T = r.T, k = r.k, TK = T * k, H = a.H;
+  const int T = r.T, k = r.k, TK = T * k;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  __shared__ int ids_s[RS_MAX_PAIRS], pos_s[RS_MAX_PAIRS];
+  __shared__ int ids_s[RS_MAX_PAIRS];
   __shared__ int cnt_s[RS_MAX_E], slot_s[RS_MAX_E], offs_s[RS_MAX_E];
   __shared__ unsigned bm[RS_MAX_E / 32];
   long long ck[4];
@@ -409,7 +409,7 @@ __device__ void route_small_tail(const RouteSmallArgs &a, float *rsm, const floa
   __syncthreads();
   ck[1] = clock64();
   if (a.trace && tid == 0) a.trace[2] = gtimer_ns();
-  if (a.debug & 8) {                             // timing experiment: a second (warm i-cache) select pass
+  if (kExperiments && (a.debug & 8)) {                             // timing experiment: a second (warm i-cache) select pass
     const long long w0 = clock64();
 #pragma unroll 1
     for (int t0 = 0; t0 < T; t0 += RS_THREADS / 32) {
@@ -427,7 +427,7 @@ __device__ void route_small_tail(const RouteSmallArgs &a, float *rsm, const floa
     }
   }
   __syncthreads();
-  if (a.minimal && !p.dbg_perm && !p.dbg_counts) {
+  if (!p.dbg_perm && !p.dbg_counts) {
     // fused decode: the expert kernel reads token-order activations and finds its
     // tokens in topk_idx, so only the active-expert list is needed (ascending ids)
     const int e = tid;
@@ -492,51 +492,13 @@ __device__ void route_small_tail(const RouteSmallArgs &a, float *rsm, const floa
       if (p.dbg_perm) p.dbg_perm[offs_s[e] + i] = t;
     }
     p.pos[q] = rw;
-    pos_s[q] = rw;
   }
   __syncthreads();
   ck[2] = clock64();
   if (a.trace && tid == 0) a.trace[3] = gtimer_ns();
-  if (a.xperm) {
-    if (a.fp8) {
-      // codes were quantised into xq by all CTAs: every thread loads its chunks
-      // (<= 4: H <= 16384) and scale byte of a token row once, then stores k times
-#pragma unroll 1
-      for (int t = 0; t < T; ++t) {
-        const uint4 *src = reinterpret_cast<const uint4 *>(reinterpret_cast<const uint8_t *>(a.xq) + (size_t)t * H);
-        uint4 v[4];
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int c = tid + RS_THREADS * i;
-          if (c < H / 16) v[i] = src[c];
-        }
-        const int b = tid;
-        const uint8_t sb = b < H / 128 ? (uint8_t)((__float_as_uint(a.xs[(size_t)t * (H / 128) + b]) >> 23) & 0xFF) : 0;
-#pragma unroll 1
-        for (int j = 0; j < k; ++j) {
-          const int rw = pos_s[t * k + j];
-          if (rw < 0) continue;
-          uint4 *dst = reinterpret_cast<uint4 *>(reinterpret_cast<uint8_t *>(a.xperm) + (size_t)rw * H);
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const int c = tid + RS_THREADS * i;
-            if (c < H / 16) dst[c] = v[i];
-          }
-          if (b < H / 128) a.xperm_img[sf_img_off(rw, b, a.xperm_img_stride)] = sb;
-        }
-      }
-    } else {
-      ScatterDst d{};
-      d.fp8 = 0; d.xperm = a.xperm;
-#pragma unroll 1
-      for (int t = 0; t < T; ++t)
-        scatter_token_row<RS_THREADS>(reinterpret_cast<const __nv_bfloat16 *>(a.x) + (size_t)t * H, H, t, k,
-                                      pos_s + t * k, d);
-    }
-  }
   ck[3] = clock64();
   if (a.trace && tid == 0) a.trace[4] = gtimer_ns();
-  if ((a.debug & 4) && tid == 0)                 // MOE_DEBUG_ROUTE=4: phase cycle counts of the tail
+  if (kExperiments && (a.debug & 4) && tid == 0)                 // MOE_DEBUG_ROUTE=4: phase cycle counts of the tail
     printf("route tail cycles: select %lld permute %lld rows %lld\n", ck[1] - ck[0], ck[2] - ck[1], ck[3] - ck[2]);
 }
 
@@ -556,7 +518,7 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   const int nv = H / 8;
   uint4 w[8];
   {
-    const bool live = row < a.rows && !(a.debug & 1);
+    const bool live = row < a.rows && !(kExperiments && (a.debug & 1));
     const uint4 *wr = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(a.wg) + (size_t)row * H);
 #pragma unroll
     for (int u = 0; u < 8; ++u) w[u] = (live && tid + u * 128 < nv) ? __ldg(wr + tid + u * 128) : make_uint4(0, 0, 0, 0);
@@ -571,21 +533,6 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   pdl_trigger();
   pdl_wait();                                    // x (the previous layer's output) and our workspaces
   if (a.trace && threadIdx.x == 0 && blockIdx.x == 0) a.trace[0] = gtimer_ns();
-  // the shared expert's weights do not depend on the routing: pull them into
-  // L2 now (two-launch decode chain only)
-  if (threadIdx.x == 0) {
-#pragma unroll 1
-    for (int i = 0; i < 2; ++i) {
-      if (!a.pf[i]) continue;
-      const int64_t per = ((a.pf_bytes[i] + gridDim.x - 1) / gridDim.x + 4095) & ~int64_t(4095);
-      const int64_t b0 = (int64_t)blockIdx.x * per, b1 = b0 + per < a.pf_bytes[i] ? b0 + per : a.pf_bytes[i];
-#pragma unroll 1
-      for (int64_t o = b0; o < b1; o += 32768)
-        asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<const uint8_t *>(a.pf[i]) + o),
-                     "r"((uint32_t)(b1 - o < 32768 ? b1 - o : 32768))
-                     : "memory");
-    }
-  }
   // ---- logits of router rows `row` for all T tokens ----
   {
     // two tokens per step with all their x loads in flight together (a token at a
@@ -674,22 +621,19 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   }
   __syncthreads();
   if (!is_last) return;
-  if (a.debug & 2) { if (threadIdx.x == 0) *a.done = 0; return; }
+  if (kExperiments && (a.debug & 2)) { if (threadIdx.x == 0) *a.done = 0; return; }
   route_small_tail(a, rsm, bpre);
 }
 
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st) {
   if (a.r.T <= 0) return cudaSuccess;
   const size_t sm = (size_t)(RS_THREADS / 32) * 2 * RS_MAX_E * sizeof(float);   // per-warp select scratch
-  static bool carve = false;
-  if (!carve) {
-    // max shared-memory carveout: the PDL-launched decode stream kernel (~190 KB
-    // of smem) can then become resident beside the router CTAs
-    cudaFuncSetAttribute(route_small_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-    carve = true;
-  }
+  // max shared-memory carveout: the PDL-launched decode stream kernel (~190 KB
+  // of smem) can then become resident beside the router CTAs
+  cudaError_t e = set_kernel_attr((const void *)route_small_kernel, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  if (e != cudaSuccess) return e;
   if (sm > 48 * 1024) {
-    cudaError_t e = cudaFuncSetAttribute(route_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    e = set_kernel_attr((const void *)route_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
   }
   return launch_pdl(route_small_kernel, dim3((a.rows + 1) / 2), dim3(RS_THREADS), sm, st, a);
@@ -700,7 +644,7 @@ cudaError_t launch_router_select(const RouterArgs &a, cudaStream_t st) {
   const int grid = (a.T + RT_WARPS - 1) / RT_WARPS;
   const size_t sm = (size_t)RT_WARPS * 2 * a.E * sizeof(float);
   if (sm > 48 * 1024) {
-    cudaError_t e = cudaFuncSetAttribute(router_select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+    cudaError_t e = set_kernel_attr((const void *)router_select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
     if (e != cudaSuccess) return e;
   }
   if (a.E <= RS_MAX_E) {

@@ -1,12 +1,10 @@
-// simt_gemm.cu -- CUDA-core tiled GEMM used for the router logits and as the
-// portable grouped expert GEMM (F32 toy weights, and the first correct path).
+// simt_gemm.cu -- CUDA-core tiled grouped expert GEMM: the path for the F32
+// toy weights and hidden sizes that are not a multiple of 256 (the router
+// logits of those layers run in gemv.cu's router_gemv / umma_gemm.cu).
 //
 //   C[m, n] = sum_k A[m, k] * B_e[n, k]        (fp32 accumulate)
 //
 // Modes:
-//   LOGITS : A = x bf16 [T, H], B = router rows bf16 [E(+1), H] -> fp32 logits
-//            (router "gating network"; bf16 products, fp32 sum,
-//            DESIGN.md reading R9)
 //   SWIGLU : A = x_perm / x (bf16 or e4m3 + 1x128 scales), B = W13 of expert e
 //            (rows interleaved per 128: W1 block b then W3 block b), epilogue
 //            h = silu(g) * u  (fused gate+up batch), optional
@@ -143,19 +141,7 @@ simt_gemm_kernel(const __grid_constant__ SimtGemmArgs a) {
   }
 
   // ---- epilogues ----
-  if constexpr (MODE == GEMM_LOGITS) {
-    float *C = reinterpret_cast<float *>(a.C);
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int row = row0 + ty * 4 + i;
-      if (row >= row_end) continue;
-#pragma unroll
-      for (int j = 0; j < NJ; ++j) {
-        const int n = n0 + tx + 16 * j;
-        if (n < a.N) C[(int64_t)row * a.ldc + n] = acc[i][j];
-      }
-    }
-  } else if constexpr (MODE == GEMM_PLAIN) {
+  if constexpr (MODE == GEMM_PLAIN) {
     __nv_bfloat16 *C = reinterpret_cast<__nv_bfloat16 *>(a.C);
 #pragma unroll
     for (int i = 0; i < 4; ++i) {
@@ -202,10 +188,7 @@ simt_gemm_kernel(const __grid_constant__ SimtGemmArgs a) {
 
 cudaError_t launch_simt_gemm(int mode, const SimtGemmArgs &a, int grid_x, cudaStream_t st) {
   if (grid_x <= 0) return cudaSuccess;
-  if (mode == GEMM_LOGITS) {
-    dim3 g(grid_x, (a.N + 127) / 128);
-    simt_gemm_kernel<GEMM_LOGITS><<<g, SG_THREADS, 0, st>>>(a);
-  } else if (mode == GEMM_PLAIN) {
+  if (mode == GEMM_PLAIN) {
     dim3 g(grid_x, (a.N + 127) / 128);
     simt_gemm_kernel<GEMM_PLAIN><<<g, SG_THREADS, 0, st>>>(a);
   } else {

@@ -191,17 +191,6 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   if (warp == 0) {
     // ============================ producer ============================
     if (lane == 0) {
-      // the shared expert's weights do not depend on the routing: pull this
-      // CTA's slice of them into L2 while the router runs
-#pragma unroll 1
-      for (int i = 0; i < 2; ++i) {
-        if (!p.pf[i]) continue;
-        const int64_t per = ((p.pf_bytes[i] + gridDim.x - 1) / gridDim.x + 4095) & ~int64_t(4095);
-        const int64_t b0 = (int64_t)blockIdx.x * per, b1 = b0 + per < p.pf_bytes[i] ? b0 + per : p.pf_bytes[i];
-#pragma unroll 1
-        for (int64_t o = b0; o < b1; o += 32768)
-          bulk_prefetch_l2(reinterpret_cast<const uint8_t *>(p.pf[i]) + o, (uint32_t)(b1 - o < 32768 ? b1 - o : 32768));
-      }
       pdl_wait();                                // routing, xq / xperm of the route kernel
       const uint64_t pol = l2_evict_first_policy();   // weights are read once per forward
       int stage = 0; uint32_t phase = 0, qs = 0, qph = 0;
@@ -215,7 +204,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         if (!ui.valid) {
           // every load of this CTA is issued: let the finalize kernel launch now, so
           // its launch latency overlaps the last stages (it waits for our completion)
-          if (p.early_trigger) pdl_trigger();
+          pdl_trigger();
           break;
         }
         const FdGroup &g = p.g[ui.group];
@@ -497,12 +486,6 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       atomicExch(p.done, 0);
     }
   }
-  if (p.fold_finalize) {
-    // small T: the last CTA writes y itself (every other CTA's red.adds are ordered
-    // before its ticket) -- no finalize launch, no PDL gap
-    __syncthreads();
-    if (last_cta) decode_finalize_range(p.fin, threadIdx.x, FD_THREADS);
-  }
 }
 
 __global__ void decode_finalize_kernel(const __grid_constant__ DecodeFinalizeArgs a) {
@@ -516,12 +499,8 @@ __global__ void decode_finalize_kernel(const __grid_constant__ DecodeFinalizeArg
 template <bool FP8>
 static cudaError_t fd_launch(const FusedDecodeParams &p, int grid, cudaStream_t st) {
   auto k = umma_decode_fused_kernel<FP8>;
-  static bool set = false;
-  if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FD_SMEM);
-    if (e != cudaSuccess) return e;
-    set = true;
-  }
+  cudaError_t e = set_kernel_attr((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FD_SMEM);
+  if (e != cudaSuccess) return e;
   return launch_pdl(k, dim3(grid), dim3(FD_THREADS), FD_SMEM, st, p);
 }
 

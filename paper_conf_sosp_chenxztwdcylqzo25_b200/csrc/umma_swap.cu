@@ -115,7 +115,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
     mbar_init(tmem_full, 1);
     mbar_init(tmem_empty, 16);                   // 8 epilogue warps x 2 CTAs (the leader's copy is used)
     // leader's uq_empty: MMA warp + 8 epilogue warps (leader) + producer + 8 epilogue warps (peer)
-    for (int i = 0; i < SW_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], p.debug_mode >= 4 ? 19 : 18); }
+    for (int i = 0; i < SW_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], (kExperiments && p.debug_mode >= 4) ? 19 : 18); }
     for (int i = 0; i < 4; ++i) mbar_init(&am_bar[i], 64);    // 2 gate warps here, per lane (+ peer bytes)
     fence_barrier_init();
   }
@@ -176,14 +176,14 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         const int G = (g.kblocks + 3) >> 2;
         for (int kb = 0; kb < g.kblocks; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          if (p.debug_mode == 3) {                 // timing experiment: MMAs on stale smem, no loads
+          if (kExperiments && p.debug_mode == 3) {                 // timing experiment: MMAs on stale smem, no loads
             if (leader) mbar_arrive(&full[stage]);
             if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
             continue;
           }
           const bool sf = FP8 && (kb & 3) == 0;
           const int kc = kb * (FP8 ? 128 : 64);
-          if (p.debug_mode >= 4) {                 // timing experiments (loads only, per-CTA 1-SM TMA)
+          if (kExperiments && p.debug_mode >= 4) {                 // timing experiments (loads only, per-CTA 1-SM TMA)
             const bool dw = p.debug_mode != 5, dx = p.debug_mode != 4;
             const uint32_t b1 = (dw ? SW_W_BYTES : 0) + (dx ? nbox * (SW_XBOX * 128) : 0);
             mbar_expect_tx(&full[stage], b1);
@@ -223,7 +223,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
     }
   } else if (warp == 1) {
     // ============================ MMA issuer (pair leader) ============================
-    if (p.debug_mode >= 4) {                     // timing experiments: each CTA drains its own ring
+    if (kExperiments && p.debug_mode >= 4) {                     // timing experiments: each CTA drains its own ring
       int stage = 0; uint32_t phase = 0;
       int qs = 0; uint32_t qph = 0;
       for (;;) {
@@ -263,7 +263,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
           mbar_wait(&full[stage], phase);
           if (trc) { const long long c = clock64(); c_full += c - c0; c0 = c; }
           tc_fence_after();
-          if (lane == 0 && p.debug_mode == 1) {    // timing experiment: loads only (commit releases the stage)
+          if (kExperiments && lane == 0 && p.debug_mode == 1) {    // timing experiment: loads only (commit releases the stage)
             mma_commit_pair(&empty[stage]);
             if (kb == kblocks - 1) mma_commit_pair(tmem_full);
           } else if (lane == 0) {
@@ -338,7 +338,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
       }
       acc_phase ^= 1;
       const int64_t rbase = (int64_t)ui.row0 + c0;          // token row of this half's column 0
-      if (p.debug_mode >= 1) { ++tile_i; continue; }        // timing experiments: no epilogue math
+      if (kExperiments && p.debug_mode >= 1) { ++tile_i; continue; }        // timing experiments: no epilogue math
       if constexpr (EPI == GEMM_PLAIN) {
         // transpose 32 tokens x 32 H rows per step through a per-warp smem tile,
         // then 16-byte row stores (token t: 64 contiguous bytes of its y row)
@@ -493,12 +493,8 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
 template <bool FP8, int EPI>
 static cudaError_t launch_swap(const SwapParams &p, int grid, cudaStream_t st) {
   auto k = umma_swap_gemm<FP8, EPI>;
-  static bool set = false;
-  if (!set) {
-    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SW_SMEM);
-    if (e != cudaSuccess) return e;
-    set = true;
-  }
+  cudaError_t e = set_kernel_attr((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SW_SMEM);
+  if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3(grid & ~1);
   cfg.blockDim = dim3(SW_THREADS);

@@ -356,3 +356,133 @@ def test_deferral_three_layer_chain_matches_eq_L241():
     O3 = O2 + S3 + Rd2 + Ra3
     for got, want in zip(outs_api, [O1, O2, O3]):
         np.testing.assert_allclose(got, want, rtol=1e-11, atol=1e-11)
+
+
+# ---------------------------------------------------------------- FP8 x / h quantisation through the FFN
+def _fp8_selector_ffn(x_row, c=None):
+    """H = F = 128.  W1 routes x[0] = 448 (the block amax, so the x scale is 1)
+    into every gate column: g = 64 (silu(64) == 64 in fp64).  Case c is None:
+    W3 shifts x by one (u_f = x[f+1]) so y_j = e4m3(x[j+1]); case c given:
+    u_f = c_f * x[1] with x[1] = 1 so y_j = e4m3(c_j) (the h quantisation;
+    amax(h) = 64 * 448 gives the h scale 64 exactly).  W2 = I / 64."""
+    H = F = 128
+    w1 = np.zeros((F, H)); w1[:, 0] = 1.0 / 7.0
+    w3 = np.zeros((F, H))
+    if c is None:
+        for f in range(F - 1):
+            w3[f, f + 1] = 1.0
+    else:
+        w3[:len(c), 1] = c
+    w2 = np.eye(H) / 64.0
+    return O.swiglu_ffn(np.array([x_row]), w1, w3, w2, fp8_act=True)[0], \
+        O.swiglu_ffn(np.array([x_row]), w1, w3, w2, fp8_act=False)[0]
+
+
+def test_fp8_x_quantised_inside_swiglu_ffn_off_grid():
+    """Off-grid x through swiglu_ffn(fp8_act=True): every value is rounded to its
+    hand-computed e4m3 neighbour (RNE, scale 1 because amax = 448): 1.07 -> 1.125,
+    1.0625 -> 1.0 (tie to even), -3.3 -> -3.25, 0.013 -> 7 * 2^-9 (subnormal),
+    300 -> 288.  An oracle that skipped the x quantisation returns the raw values."""
+    x = np.zeros(128)
+    x[0] = 448.0
+    x[1:6] = [1.07, 1.0625, -3.3, 0.013, 300.0]
+    yq, y = _fp8_selector_ffn(x)
+    want = [1.125, 1.0, -3.25, 7 * 2.0 ** -9, 288.0]
+    np.testing.assert_allclose(yq[:5], want, rtol=1e-12, atol=0)
+    np.testing.assert_allclose(y[:5], x[1:6], rtol=1e-12)           # unquantised: the raw x
+    assert np.all(np.abs(yq[:5] - y[:5]) > 1e-4)
+    assert np.all(yq[5:] == 0)
+
+
+def test_fp8_h_quantised_inside_swiglu_ffn_off_grid():
+    """x on the grid, h = 64 * c off the grid: y_j = e4m3(c_j) * 64 / 64 with the
+    h scale 64 = 2^ceil(log2(64 * 448 / 448)) (exact power of two keeps its exponent)."""
+    x = np.zeros(128)
+    x[0], x[1] = 448.0, 1.0
+    c = [1.07, 1.0625, -3.3, 0.013, 300.0, 448.0]
+    yq, y = _fp8_selector_ffn(x, c=c)
+    np.testing.assert_allclose(yq[:6], [1.125, 1.0, -3.25, 7 * 2.0 ** -9, 288.0, 448.0], rtol=1e-12, atol=0)
+    np.testing.assert_allclose(y[:6], c, rtol=1e-12)
+    assert np.all(yq[6:] == 0)
+
+
+def test_fp8_quantisation_reaches_moe_layer():
+    """The same selector expert as the only routed expert (E = 1, k = 1, softmax
+    -> w = 1) and as the shared expert: moe_layer(fp8=True) returns 2 x e4m3(x)."""
+    H = 128
+    x = np.zeros((1, H))
+    x[0, 0] = 448.0
+    x[0, 1:6] = [1.07, 1.0625, -3.3, 0.013, 300.0]
+    w1 = np.zeros((H, H)); w1[:, 0] = 1.0 / 7.0
+    w3 = np.zeros((H, H))
+    for f in range(H - 1):
+        w3[f, f + 1] = 1.0
+    w2 = np.eye(H) / 64.0
+    W = O.OracleWeights(np.zeros((1, H)), None, lambda e: (w1, w3, w2), lambda: (w1, w3, w2))
+    cfg = O.OracleConfig(hidden=H, ffn=H, n_experts=1, top_k=1, shared_ffn=H, fp8=True)
+    y = O.moe_layer(x, W, cfg)["y"][0]
+    np.testing.assert_allclose(y[:5], 2 * np.array([1.125, 1.0, -3.25, 7 * 2.0 ** -9, 288.0]), rtol=1e-12)
+
+
+# ---------------------------------------------------------------- tie band (north_star 1e-5)
+def test_gap_at():
+    v = np.array([5.0, 3.0, 2.5, 2.5])
+    assert O.gap_at(v, 1) == 2.0
+    assert O.gap_at(v, 2) == 0.5
+    assert O.gap_at(v, 3) == 0.0
+    assert O.gap_at(v, 0) == math.inf and O.gap_at(v, 4) == math.inf
+
+
+def _tie_layer(s_rows, bias=None, **kw):
+    """Tokens whose sigmoid scores are exactly `s_rows` (Wg = I, x = logit(s))."""
+    s = np.array(s_rows, float)
+    E = s.shape[1]
+    x = np.log(s) - np.log1p(-s)
+    W = O.OracleWeights(np.eye(E), None if bias is None else np.array(bias, float),
+                        lambda e: (np.zeros((1, E)),) * 2 + (np.zeros((E, 1)),))
+    base = dict(hidden=E, ffn=1, n_experts=E, score_fn=O.SCORE_SIGMOID)
+    base.update(kw)
+    return x, W, O.OracleConfig(**base)
+
+
+def test_tie_band_tokens_flags_exactly_the_hand_built_ties():
+    """E = 8 in 4 groups of 2, keep 2 groups (top-2-sum score), k = 3.
+      0: k-boundary sel gap 5e-6 (0.7 vs 0.699995)          -> flagged
+      1: k-boundary gap 2e-5                                 -> not flagged
+      2: group scores 0.9 vs 0.899996 at the topk_group boundary -> flagged
+      3: group gap 1.5e-5                                    -> not flagged
+      4: w[1] - w[2] = 4e-6 at k - n_def = 2 (n_def = 1 only) -> flagged iff n_def = 1
+      5: every gap large                                     -> never flagged"""
+    rows = [
+        [0.9, 0.8, 0.7, 0.699995, 0.1, 0.1, 0.05, 0.05],
+        [0.9, 0.8, 0.7, 0.69998, 0.1, 0.1, 0.05, 0.05],
+        [0.9, 0.8, 0.6, 0.3, 0.5, 0.399996, 0.05, 0.05],
+        [0.9, 0.8, 0.6, 0.3, 0.5, 0.399985, 0.05, 0.05],
+        [0.9, 0.8, 0.799996, 0.2, 0.05, 0.05, 0.01, 0.01],
+        [0.9, 0.5, 0.3, 0.1, 0.2, 0.15, 0.02, 0.01],
+    ]
+    x, W, cfg = _tie_layer(rows, n_group=4, topk_group=2, group_score=O.GROUP_TOP2_SUM, top_k=3)
+    assert list(O.tie_band_tokens(x, W, cfg)) == [0, 2]
+    assert list(O.tie_band_tokens(x, W, cfg, n_deferred=1)) == [0, 2, 4]
+    # the group gap of token 2 is what flags it: with one group the token is clean
+    x1, W1, cfg1 = _tie_layer(rows[2:4], top_k=3)
+    assert list(O.tie_band_tokens(x1, W1, cfg1)) == []
+
+
+def test_tie_band_uses_biased_selection_scores():
+    """The k boundary is measured on sel = s + bias, not on s: a bias of 0.099996
+    on expert 3 puts it 4e-6 below expert 2's 0.7."""
+    rows = [[0.9, 0.8, 0.7, 0.6, 0.1, 0.1, 0.05, 0.05]]
+    x, W, cfg = _tie_layer(rows, bias=[0, 0, 0, 0.099996, 0, 0, 0, 0], top_k=3)
+    assert list(O.tie_band_tokens(x, W, cfg)) == [0]
+    x, W, cfg = _tie_layer(rows, top_k=3)
+    assert list(O.tie_band_tokens(x, W, cfg)) == []
+
+
+def test_tie_band_group_max_rule():
+    """DeepSeek-V2.5 group score = max: groups 2 (0.6) and 3 (0.599996) tie at the
+    topk_group = 2 boundary."""
+    rows = [[0.9, 0.1, 0.6, 0.1, 0.599996, 0.1, 0.05, 0.05],
+            [0.9, 0.1, 0.6, 0.1, 0.59, 0.1, 0.05, 0.05]]
+    x, W, cfg = _tie_layer(rows, n_group=4, topk_group=2, group_score=O.GROUP_MAX, top_k=2)
+    assert list(O.tie_band_tokens(x, W, cfg)) == [0]
