@@ -241,7 +241,9 @@ def test_skewed_routing(lib, name):
     out, ties, idx, w = _oracle(p, res)
     g = res["routing"]
     counts = g["expert_counts"]
-    assert counts.max() >= 3 * counts.mean(), (counts.max(), counts.mean())   # it is skewed
+    # it is skewed: the hottest expert carries well above the mean load (qwen2_s has 16
+    # experts and k = 8, so no expert can exceed 2x the mean there)
+    assert counts.max() >= min(2.5, 0.8 * p.n_experts / p.top_k) * counts.mean(), (counts.max(), counts.mean())
     check_tie_fraction(ties, T)
     check_routing(g["topk_idx"], g["topk_w"], idx, w, ties, p.routed_scale, p.norm_topk)
     check_permutation(counts, g["perm"], idx, p.n_experts)
