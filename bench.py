@@ -341,95 +341,121 @@ def run_ours(args):
     # (x_{i+1} = y_i = x_i + moe_i(x_i)); weights of the stack (8 x 11.3 GB for V3)
     # dwarf L2, and L2 is also flushed before every replay (outside the events).
     # value = replay time / layers.  The API is host-sync-free and capturable
-    # (PAPER.md L193 captures the decode step in one CUDA graph).  A separate eager
-    # pass with stage events gives the per-kernel breakdown.
+    # (PAPER.md L193 captures the decode step in one CUDA graph).  Variants:
+    #   deferral: the same chain with Expert Deferral across layers (moe_layer_forward_chained,
+    #             PAPER.md L241; n_def = 3, the paper's BF16 setting L257; last layer 0)
+    #   tp_rank:  one expert-TP rank's share (its 1/P slice of every expert, P = 2/4/8) --
+    #             the all-reduce of the partials needs the other GPUs and is not in it
+    #   tp_nccl:  N > 1 only: the expert-TP chain over the N GPUs, NCCL fp32 all-reduce inside
     decode = None
-    if not args.no_decode and not ep:
+    if not args.no_decode and (not ep or not args.no_decode_tp_nccl):
         nl = max(1, args.decode_layers)
-        dlayers = [layer] + [moe.MoELayer(p, w, max_tokens=16, device=local) for _ in range(nl - 1)]
         xd, _ = make_tokens(p, args.steps + args.warmup, "cuda", offset=1000 + rank)
         rows = [xd[i:i + 1].contiguous() for i in range(xd.shape[0])]
-        bufs = [rows[0].clone(), torch.empty_like(rows[0])]
-
-        def dstep():
-            for i, l in enumerate(dlayers):
-                a_, b_ = bufs[i % 2], bufs[(i + 1) % 2]
-                l.forward(a_, residual=a_, y=b_)
-
-        side = torch.cuda.Stream()
-        side.wait_stream(torch.cuda.current_stream())
-        with torch.cuda.stream(side):
-            for _ in range(2):
-                bufs[0].copy_(rows[0])
-                dstep()
-        torch.cuda.current_stream().wait_stream(side)
-        graph = torch.cuda.CUDAGraph()
-        with torch.cuda.graph(graph):
-            dstep()
         st = torch.cuda.current_stream()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        for i in range(args.warmup):
-            bufs[0].copy_(rows[i])
-            graph.replay()
-        torch.cuda.synchronize()
-        dtimes = []
-        for i in range(args.steps):
-            bufs[0].copy_(rows[args.warmup + i])
-            flush_l2(flush)
-            e0.record(st)
-            graph.replay()
-            e1.record(st)
-            e1.synchronize()
-            dtimes.append(e0.elapsed_time(e1) / nl)
-        _, dstages = timed_steps(layer, rows, bufs[1], min(args.steps, 5), 1, flush)
-        dinfo = layer.info()
-        dus = max_over_ranks(sum(dtimes) / len(dtimes), ws) * 1e3
+
+        def time_chain(dlayers, n_def=0, chained=False):
+            bufs = [rows[0].clone(), torch.empty_like(rows[0])]
+
+            def dstep():
+                prev = None
+                for i, l in enumerate(dlayers):
+                    a_, b_ = bufs[i % 2], bufs[(i + 1) % 2]
+                    if chained:
+                        nd = n_def if i < len(dlayers) - 1 else 0
+                        l.forward_chained(a_, residual=a_, n_deferred=nd, prev=prev, y=b_)
+                        prev = l
+                    else:
+                        l.forward(a_, residual=a_, y=b_)
+
+            side = torch.cuda.Stream()
+            side.wait_stream(torch.cuda.current_stream())
+            with torch.cuda.stream(side):
+                for _ in range(2):
+                    bufs[0].copy_(rows[0])
+                    dstep()
+            torch.cuda.current_stream().wait_stream(side)
+            graph = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(graph):
+                dstep()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            for i in range(args.warmup):
+                bufs[0].copy_(rows[i])
+                graph.replay()
+            torch.cuda.synchronize()
+            barrier(ws)
+            tt = []
+            for i in range(args.steps):
+                bufs[0].copy_(rows[args.warmup + i])
+                flush_l2(flush)
+                barrier(ws)
+                e0.record(st)
+                graph.replay()
+                e1.record(st)
+                e1.synchronize()
+                tt.append(e0.elapsed_time(e1) / len(dlayers))
+            del graph
+            return max_over_ranks(sum(tt) / len(tt), ws) * 1e3
+
         algd = algorithmic(p, 1, p.top_k)
-        decode = {"us_per_layer": dus, "tokens": 1, "layers_in_graph": nl, "mode": "cuda_graph_replay",
-                  "gpu_launches_per_layer": dinfo.kernels_per_forward_decode,
-                  "roofline": {"bound": "hbm", "achieved": algd["layer_bytes"] / (dus * 1e-6) / 1e9,
-                               "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                               "frac": algd["layer_bytes"] / (dus * 1e-6) / 1e9 / peaks["hbm_gbs"],
-                               "bytes": algd["layer_bytes"],
-                               "stage_us_eager": {k: round(v * 1e3, 2) for k, v in dstages.items()}}}
-        # decode TP within every expert: one rank's share of the same
-        # graph-replayed chain at P = 2/4/8 (rank 0's chunks; the per-layer [T, H] all-reduce
-        # over NVLink is not in this single-GPU number)
-        tp = {}
-        if not args.no_decode_tp:
-            for P in (2, 4, 8):
-                if p.ffn // 128 < P or (p.shared_ffn and p.shared_ffn // 128 < P):
-                    continue
-                for l in dlayers:
-                    l.set_decode_tp(0, P)
-                side.wait_stream(torch.cuda.current_stream())
-                with torch.cuda.stream(side):
-                    dstep()
-                torch.cuda.current_stream().wait_stream(side)
-                g2 = torch.cuda.CUDAGraph()
-                with torch.cuda.graph(g2):
-                    dstep()
-                for i in range(args.warmup):
-                    g2.replay()
-                torch.cuda.synchronize()
-                tt = []
-                for i in range(args.steps):
-                    bufs[0].copy_(rows[args.warmup + i])
-                    flush_l2(flush)
-                    e0.record(st)
-                    g2.replay()
-                    e1.record(st)
-                    e1.synchronize()
-                    tt.append(e0.elapsed_time(e1) / nl)
-                tp[str(P)] = round(max_over_ranks(sum(tt) / len(tt), ws) * 1e3, 2)
-                del g2
-            for l in dlayers:
-                l.set_decode_tp(0, 1)
-        decode["tp_rank_us_per_layer"] = tp
-        for l in dlayers[1:]:
-            l.close()
-        del dlayers, graph
-        torch.cuda.empty_cache()
+        hbm = lambda us: {"bound": "hbm", "achieved": algd["layer_bytes"] / (us * 1e-6) / 1e9,
+                          "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                          "frac": algd["layer_bytes"] / (us * 1e-6) / 1e9 / peaks["hbm_gbs"],
+                          "bytes": algd["layer_bytes"]}
+        if not ep:
+            dlayers = [layer] + [moe.MoELayer(p, w, max_tokens=16, device=local) for _ in range(nl - 1)]
+            dus = time_chain(dlayers)
+            _, dstages = timed_steps(layer, rows, torch.empty_like(rows[0]), min(args.steps, 5), 1, flush)
+            dinfo = layer.info()
+            decode = {"us_per_layer": dus, "tokens": 1, "layers_in_graph": nl, "mode": "cuda_graph_replay",
+                      "gpu_launches_per_layer": dinfo.kernels_per_forward_decode, "roofline": hbm(dus)}
+            decode["roofline"]["stage_us_eager"] = {k: round(v * 1e3, 2) for k, v in dstages.items()}
+            if not args.no_deferral and p.top_k > 3:
+                dd = time_chain(dlayers, n_def=3, chained=True)
+                decode["deferral"] = {"n_deferred": 3, "us_per_layer": dd, "speedup_vs_no_deferral": dus / dd,
+                                      "roofline": hbm(dd),
+                                      "mode": "moe_layer_forward_chained: layer i streams layer i-1's deferred "
+                                              "experts while its own router runs (PAPER.md L241)"}
+            for l in dlayers[1:]:
+                l.close()
+            del dlayers
+            torch.cuda.empty_cache()
+            # expert TP: one rank's share (rank 0's slice of every expert as a layer of its own)
+            tp = {}
+            if not args.no_decode_tp:
+                for P in (2, 4, 8):
+                    if p.ffn // 128 < P or (p.shared_ffn and p.shared_ffn // 128 < P):
+                        continue
+                    ws0 = moe.slice_tp(w, 0, P, p.ffn, p.shared_ffn)
+                    p0 = p.with_(ffn=ws0.w2.shape[2], shared_ffn=ws0.ws2.shape[1] if p.shared_ffn else 0)
+                    tl = [moe.MoELayer(p0, ws0, max_tokens=16, device=local) for _ in range(nl)]
+                    tp[str(P)] = round(time_chain(tl), 2)
+                    for l in tl:
+                        l.close()
+                    del tl, ws0
+                    torch.cuda.empty_cache()
+            decode["tp_rank_us_per_layer"] = tp
+        elif p.ffn // 128 >= ws and (not p.shared_ffn or p.shared_ffn // 128 >= ws):
+            # expert TP over the N GPUs of this run (NCCL all-reduce in the graph)
+            import torch.distributed as dist
+            tl = []
+            try:
+                wr = moe.slice_tp(make_weights(p, "cuda"), rank, ws, p.ffn, p.shared_ffn)
+                for _ in range(nl):
+                    uid = [moe.get_unique_id() if rank == 0 else None]
+                    dist.broadcast_object_list(uid, src=0)
+                    tl.append(moe.MoELayer(p, wr, max_tokens=16, device=local, tp_rank=rank, tp_size=ws,
+                                           unique_id=uid[0]))
+                del wr
+                dus = time_chain(tl)
+                decode = {"tp_nccl_us_per_layer": dus, "tokens": 1, "layers_in_graph": nl, "tp": ws,
+                          "mode": "cuda_graph_replay, expert TP over NCCL (fp32 all-reduce of the partials)",
+                          "roofline": hbm(dus)}
+            except Exception as ex:          # keep the prefill line even if this variant fails
+                decode = {"tp_nccl_error": f"{type(ex).__name__}: {ex}"}
+            for l in tl:
+                l.close()
+            torch.cuda.empty_cache()
 
     # ---------------- e2e through the public API, host buffers ----------------
     # Every step copies its inputs from pinned host memory and reads its output back
@@ -545,6 +571,8 @@ def main():
     ap.add_argument("--tokens", type=int, default=0)
     ap.add_argument("--no-decode", action="store_true")
     ap.add_argument("--no-decode-tp", action="store_true", help="skip the decode-TP per-rank timing")
+    ap.add_argument("--no-deferral", action="store_true", help="skip the chained Expert Deferral decode timing")
+    ap.add_argument("--no-decode-tp-nccl", action="store_true", help="N > 1: skip the decode timing with expert TP over NCCL")
     ap.add_argument("--decode-layers", type=int, default=8, help="distinct layers chained in the decode graph")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")

@@ -75,8 +75,30 @@ typedef struct {
                                 0 => library default (the L170 switch) */
   int32_t device;            /* CUDA device ordinal                                  */
   int32_t ep_rank, ep_size;  /* expert parallel group; ep_size 1 => single GPU       */
-  const void *nccl_unique_id;/* host, 128 bytes (ncclUniqueId) when ep_size > 1      */
+  const void *nccl_unique_id;/* host, 128 bytes (ncclUniqueId) when ep_size > 1 or
+                                tp_size > 1 (the group's communicator)              */
+  int32_t tp_rank, tp_size;  /* tensor parallelism within every expert (decode):
+                                tp_size 1 => off; see "Tensor parallelism" below    */
 } moe_layer_config;
+
+/* Tensor parallelism within every expert (the B200
+ * analog of the paper's NUMA-aware TP, Fig. 8b: "each
+ * socket stores only its slice ... lightweight reduce-scatter").
+ * With tp_size = P > 1 (ep_size must be 1) rank r owns the 128-column FFN
+ * chunks [r*n/P, (r+1)*n/P) of every routed expert (n = ffn/128) and of the
+ * shared expert (n = shared_ffn/128): ffn and shared_ffn in the config are the
+ * FULL sizes, and the weights passed to create are this rank's SLICE only
+ *   w13 [E, 2*F_r, H]: rows 0..F_r-1 = W1 rows of the slice, F_r..2F_r-1 = W3 rows
+ *   w2  [E, H, F_r]:   the slice's W2 columns        (F_r = 128 x chunks of rank r;
+ *   scales [E, 2F_r/128, H/128], [E, H/128, F_r/128]; shared expert alike)
+ * so 1/P of the expert bytes are resident per rank.  Routing is replicated (every
+ * rank routes every token).  A forward computes this rank's fp32 partial of
+ * every token's expert sum; the partials are summed over the P ranks (NCCL
+ * all-reduce in fp32 on the layer's own communicator when nccl_unique_id is
+ * given; moe_tp_group_forward for an in-process group), then every rank adds
+ * residual and deferred_in once and writes the full bf16 y (and deferred_out).
+ * Requires P <= ffn/128 (and <= shared_ffn/128) and the decode path: a forward
+ * with T > moe_layer_info.gemv_max_tokens returns MOE_ERR_UNSUPPORTED.      */
 
 /* Weights: DEVICE pointers, row-major, read at create and copied + repacked into
  * library-owned memory (the paper's load-time repack, L157); the caller may
@@ -172,6 +194,39 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
                                 const void *const *deferred_in, void *const *y, void *const *deferred_out,
                                 void *stream);
 
+/* Expert Deferral chained across consecutive layers (§4.1 Eq. 2;
+ * §8(f) NEXT-2):
+ *   O_k = I_k + S_k(I_k) + R_{k-1}^def(I_{k-1}) + R_k^imm(I_k)
+ * The last n_deferred slots of each token's canonical order (the lowest combine
+ * weights, L215) are NOT computed by this call: the NEXT layer's chained
+ * forward computes them (passing this layer as `prev`) and adds them to its own
+ * output.  `prev` (NULL for the first layer, k = 1 case) is the previous layer's
+ * handle whose last call was a chained forward with n_deferred > 0 on the same T
+ * tokens; its deferred experts stream at the start of this call, before this
+ * layer's router has finished -- the overlap the paper's deferral buys.
+ *   y = residual + S(x) + R^imm(x) + R^def_prev(x_prev)
+ * n_deferred = 0 is the last layer (k = L: all experts immediate).  The caller
+ * keeps the chain on one stream (prev's workspace holds x_prev's quantised copy
+ * and routing until prev's next forward).  Decode path only (T <= gemv_max_tokens,
+ * the paper applies deferral in decode, L245); MOE_ERR_UNSUPPORTED otherwise,
+ * MOE_ERR_INVALID_ARG if prev is this layer, has another shape / dtype / device /
+ * TP split, or its last call was not a chained forward with n_deferred > 0 on T
+ * tokens.                                                                     */
+moe_status moe_layer_forward_chained(moe_layer *layer, const void *x, const void *residual, int32_t T,
+                                     int32_t n_deferred, moe_layer *prev, void *y, void *stream);
+
+/* Tensor parallelism inside ONE process (the test vehicle of the NCCL path on a
+ * single GPU): P layers created with tp_size = P, tp_rank = r and no unique id
+ * form a group; this call runs one forward of every rank (rank r's x[r], same
+ * T tokens on every rank), sums the P fp32 partials on the devices with peer
+ * copies and a reduction kernel (what the NCCL all-reduce does across GPUs), and
+ * writes every rank's full y[r] (and deferred_out[r]).  Arrays indexed by rank;
+ * residual / deferred_in / deferred_out arrays may be NULL.                   */
+moe_status moe_tp_group_forward(moe_layer *const *layers, int32_t P, const void *const *x,
+                                const void *const *residual, int32_t T, int32_t n_deferred,
+                                const void *const *deferred_in, void *const *y, void *const *deferred_out,
+                                void *stream);
+
 /* Timing experiments only: a layer created with the environment variable
  * MOE_DEBUG_TRACE set records globaltimer/clock stamps of its kernels into a
  * 4096-entry u64 device buffer; this synchronises the device, copies
@@ -195,24 +250,6 @@ typedef struct {
   int32_t local_experts;     /* E / ep_size                                         */
 } moe_layer_info;
 moe_status moe_layer_get_info(const moe_layer *layer, moe_layer_info *info);
-
-/* Decode tensor parallelism within every expert (the
- * B200 analog of the paper's NUMA-aware TP, Fig. 8b).
- * After moe_layer_set_decode_tp(layer, r, P), a decode forward (T <= the
- * fused stream's limit, moe_layer_info.gemv_max_tokens) streams only the
- * 128-column FFN chunks c with c % P == r of every active routed expert and
- * of the shared expert -- W13 rows and W2 columns of the same chunk -- and
- * writes this rank's PARTIAL output: y_r = bf16(sum over its chunks of the
- * weighted expert partials), plus residual and deferred_in on rank 0 only
- * (deferred_out likewise partial).  The caller all-reduces (sums) y_r over the
- * P ranks; sum_r y_r equals the full layer's y up to the bf16 rounding of each
- * partial.  Routing is replicated: every rank routes every token itself.
- * Weights stay fully resident (each rank reads 1/P of the active bytes).
- * size = 1 restores the normal forward.  Errors: INVALID_ARG (rank not in
- * [0, size), size > F/128 or > Fs/128), UNSUPPORTED (expert-parallel layer,
- * or no fused decode stream); a forward with T above the fused limit while
- * size > 1 returns UNSUPPORTED.  Host-only; no device work.                  */
-moe_status moe_layer_set_decode_tp(moe_layer *layer, int32_t rank, int32_t size);
 
 /* Stage timing (instrumentation for the bench's roofline figures; off by
  * default).  When enabled, forward records a CUDA event after every stage on

@@ -213,7 +213,7 @@ struct moe_layer {
   int32_t *offs_pad = nullptr;  // [E+1] padded to kPadM
   int4 *tiles = nullptr;        // [max_tiles] (expert, row0, row_end, 0)
   int32_t *n_tiles = nullptr;   // [1]
-  int32_t *act_list = nullptr;  // [E] active experts (count > 0), ascending
+  int32_t *act_list = nullptr;  // [E] active experts (count > 0, any slot), ascending
   int32_t *n_active = nullptr;  // [1]
   int32_t *sched = nullptr;     // [8] work counters of the persistent GEMM launches
   int32_t *row_token = nullptr; // [R_max] token of each padded row (-1 = pad)
@@ -238,7 +238,19 @@ struct moe_layer {
   CUtensorMap dmap_xperm, dmap_h, dmap_xq, dmap_hsh;           // decode: activation rows (box 16)
   float *dacc = nullptr;        // fused decode: [2][gemv_max_tokens, H] fp32 sums (immediate, deferred), kept zero
   bool fused_decode = false;
-  int tp_rank = 0, tp_size = 1;   // decode TP (moe_layer_set_decode_tp)
+  // chained Expert Deferral (moe_layer_forward_chained): expert lists of the
+  // immediate / deferred canonical slots, and what the last chained call left
+  int32_t *imm_list = nullptr, *def_list = nullptr;   // [E] ascending local ids
+  int32_t *n_lists = nullptr;                          // [2] lengths (immediate, deferred)
+  int chain_T = -1, chain_ndef = 0;
+  void *xcopy = nullptr;        // BF16 decode: [gemv_max_tokens, H] copy of x (the stream's operand)
+  CUtensorMap dmap_xc;          // its tensor map (box 16 rows)
+  // tensor parallelism within every expert (config tp_rank / tp_size): this rank's
+  // 128-column chunks [c0, c0 + F/128) of the full ffn (F, Fs are the slice sizes)
+  int tp_rank = 0, tp_size = 1;
+  int F_full = 0, Fs_full = 0;
+  void *tp_comm = nullptr;      // ncclComm_t of the TP group (null: in-process group)
+  bool pending_use_def = false; // in-process TP group: the last partial forward kept deferred sums
   int n_launch = 0, launches_prefill = 0, launches_decode = 0;   // kernel launches per forward
   unsigned long long *trace = nullptr;   // MOE_DEBUG_TRACE timeline buffer (timing experiments)
   // swap-AB CTA-pair GEMM (umma_swap.cu): tiled weights as 128-byte rows (box 128),

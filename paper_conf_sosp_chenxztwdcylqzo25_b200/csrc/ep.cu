@@ -161,6 +161,28 @@ const char *ep_nccl_error(void *comm) {
   return "";
 }
 
+int ep_nccl_allreduce_f32(void *comm, float *buf, size_t n, cudaStream_t st) {
+  return ncclAllReduce(buf, buf, n, ncclFloat32, ncclSum, reinterpret_cast<ncclComm_t>(comm), st) == ncclSuccess ? 0 : -1;
+}
+
+struct SumSrc { const float *p[31]; };
+__global__ void sum_f32_kernel(float *__restrict__ dst, const __grid_constant__ SumSrc src, int nsrc, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    float v = dst[i];
+    for (int j = 0; j < nsrc; ++j) v += src.p[j][i];
+    dst[i] = v;
+  }
+}
+
+cudaError_t launch_sum_f32(float *dst, const float *const *src, int nsrc, int64_t n, cudaStream_t st) {
+  if (n <= 0 || nsrc <= 0) return cudaSuccess;
+  if (nsrc > 31) return cudaErrorInvalidValue;
+  SumSrc s{};
+  for (int j = 0; j < nsrc; ++j) s.p[j] = src[j];
+  sum_f32_kernel<<<(int)std::min<int64_t>((n + 255) / 256, 148 * 4), 256, 0, st>>>(dst, s, nsrc, n);
+  return cudaGetLastError();
+}
+
 // exchange of the P send counts (one int32 to every peer)
 int ep_nccl_counts(void *comm, const int32_t *send_cnt, int32_t *recv_cnt, int P, cudaStream_t st) {
   ncclComm_t c = reinterpret_cast<ncclComm_t>(comm);

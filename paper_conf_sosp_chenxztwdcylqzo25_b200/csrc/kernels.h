@@ -111,12 +111,19 @@ struct RouteSmallArgs {
   int H, rows;
   int *done;                    // zero-initialised CTA counter (re-armed by the kernel)
   int debug;                    // timing experiments only (MOE_EXPERIMENTS builds, MOE_DEBUG_ROUTE)
-  // FP8: x quantised in token order (1x128 UE8M0 + e4m3) for the fused decode stream
+  // FP8: x quantised in token order (1x128 UE8M0 + e4m3) for the fused decode stream;
+  // BF16: x copied into the layer's own buffer (the stream reads it there, so a chained
+  // next layer can still read it after the caller reused its x buffer)
   int fp8;
-  void *xq; float *xs; uint8_t *xq_img; int xq_img_stride;
+  void *xq; float *xs;
+  void *xcopy;
   unsigned long long *trace;     // MOE_DEBUG_TRACE: [0] CTA 0 entry, [1..4] tail start / select / permute / end
-  // The tail writes only the active-expert list unless dbg_perm / dbg_counts
-  // ask for the full counts and permutation (parity outputs).
+  // The tail writes the active-expert list (p.act_list: any slot) and, for chained
+  // Expert Deferral, the experts of the immediate slots [0, n_imm) and of the
+  // deferred slots [n_imm, k) (ascending local ids); the full counts and
+  // permutation only when dbg_perm / dbg_counts ask for them (parity outputs).
+  int n_imm;
+  int32_t *imm_list, *n_imm_list, *def_list, *n_def_list;
 };
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st);
 
@@ -178,6 +185,9 @@ int ep_nccl_init(void **comm, int P, int rank, const void *uid128);
 void ep_nccl_destroy(void *comm);
 const char *ep_nccl_error(void *comm);
 int ep_nccl_counts(void *comm, const int32_t *send_cnt, int32_t *recv_cnt, int P, cudaStream_t st);
+int ep_nccl_allreduce_f32(void *comm, float *buf, size_t n, cudaStream_t st);   // in place, sum
+// dst[i] += sum_j src[j][i], i < n (the in-process TP group's reduction)
+cudaError_t launch_sum_f32(float *dst, const float *const *src, int nsrc, int64_t n, cudaStream_t st);
 int ep_nccl_rows(void *comm, int P, const int32_t *send_cnt, const int64_t *send_off, const int32_t *recv_cnt,
                  const int64_t *recv_off, int nbuf, const void *const *send, void *const *recv,
                  const int64_t *row_bytes, cudaStream_t st);
@@ -204,15 +214,20 @@ cudaError_t launch_tile_weights(const void *src, void *dst, int nexp, int rows, 
 // decode, fused per (slot, 128-column FFN chunk) unit (umma_decode_fused.cu):
 // W13 tile -> SwiGLU (+ FP8 requant) -> h_c in smem -> W2 column block ->
 // weighted fp32 partial sums; decode_finalize writes y / deferred_out
-struct FdGroup {                // 0 routed, 1 shared
+struct FdGroup {                // 0 routed, 1 shared, 2 the previous layer's deferred experts
   CUtensorMap x_map;            // token-order activation rows (xq / bf16 x), K-major SW128, box 16 rows
   const uint8_t *w13;           // tiled W13 [expert][F/128][H/128 B][256 x 128 B]
-  const uint8_t *w13_img;       // FP8: W13 scale image (swap layout) [expert][H/512][F/128][512 B]
-  int64_t w13_img_stride;       // bytes per expert
-  const uint8_t *x_img;         // FP8: activation scale image
-  int x_img_stride;             // 128-row tiles per k-group
+  const float *w13_s;           // FP8: [expert][2F/128][H/128] block scales, rows interleaved per 128 (gate, up)
+  const float *xs;              // FP8: [T][H/128] activation scales (token order)
   const uint8_t *w2;            // tiled W2 [expert][H/256][F/128 B][256 x 128 B]
   const float *w2_s;            // FP8: [expert][H/128][F/128]
+  int nch;                      // 128-column FFN chunks per expert (F/128, Fs/128)
+  // routed groups: expert list (ascending local ids) and the routing that picks the tokens
+  const int32_t *list, *n_list;
+  const int32_t *topk_idx;      // [T, k] global ids, canonical slot order
+  const float *topk_w;          // [T, k]
+  int k, e0;
+  int a0, a1, a2;               // canonical slots [a0, a1) -> acc_imm, [a1, a2) -> acc_def, others skipped
 };
 struct DecodeFinalizeArgs {
   int T, H, use_def;
@@ -222,16 +237,12 @@ struct DecodeFinalizeArgs {
   unsigned long long *trace;     // MOE_DEBUG_TRACE: [2000] past the PDL wait, [2001] end (CTA 0)
 };
 struct FusedDecodeParams {
-  FdGroup g[2];
-  int nch[2];                   // 128-column chunks: F/128, Fs/128
-  int H, T, k, n_imm, has_shared;
-  const int32_t *n_active, *act_list;   // active local experts (ascending)
-  const int32_t *topk_idx; int e0;      // [T, k] global ids (canonical order), first local expert
-  const float *topk_w, *sgate;  // sgate null unless the shared expert is gated (Qwen2)
+  FdGroup g[3];
+  int H, T, has_shared, has_prev;
+  const float *sgate;           // null unless the shared expert is gated (Qwen2)
   float *acc_imm, *acc_def;     // [T, H] fp32 sums, zero on entry (re-zeroed by decode_finalize)
   int *sched, *done;            // work counter + exit ticket, zero on entry (re-armed by the kernel)
   unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
-  int tp_rank, tp_size;         // decode TP: stream chunks c = tp_rank (mod tp_size) only (0, 0/1 = all)
 };
 cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, cudaStream_t st);
 cudaError_t launch_decode_finalize(const DecodeFinalizeArgs &a, cudaStream_t st);

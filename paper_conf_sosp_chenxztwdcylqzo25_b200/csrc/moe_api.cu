@@ -66,7 +66,8 @@ void free_all(moe_layer *L) {
                   L->counts, L->offs, L->offs_pad, L->tiles, L->n_tiles, L->act_list, L->n_active,
                   L->row_token, L->pos, L->sched, L->pairs, L->n_pairs, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
                   L->hsh, L->hsh_s, L->ysh, L->w13_img, L->w2_img, L->ws13_img, L->ws2_img,
-                  L->xperm_img, L->h_img, L->xq_img, L->hsh_img, L->dacc, L->trace};
+                  L->xperm_img, L->h_img, L->xq_img, L->hsh_img, L->dacc, L->trace, L->imm_list, L->def_list,
+                  L->n_lists, L->xcopy};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   void *eps[] = {L->ep.send_x, L->ep.send_idx, L->ep.send_w, L->ep.sendpos, L->ep.cnt_dev, L->ep.recv_x,
@@ -76,6 +77,8 @@ void free_all(moe_layer *L) {
   if (L->ep.cnt_host) cudaFreeHost(L->ep.cnt_host);
   ep_nccl_destroy(L->ep.comm);
   L->ep.comm = nullptr;
+  ep_nccl_destroy(L->tp_comm);
+  L->tp_comm = nullptr;
 }
 
 // Expert-parallel buffers (+ the NCCL communicator when a unique id is given;
@@ -241,6 +244,16 @@ moe_status validate(const moe_layer_config *c, const moe_layer_weights *w) {
   if (c->ep_size < 1 || c->ep_size > 32 || c->n_experts % c->ep_size)
     return fail(MOE_ERR_INVALID_ARG, "ep_size %d must be in [1, 32] and divide n_experts", c->ep_size);
   if (c->ep_rank < 0 || c->ep_rank >= c->ep_size) return fail(MOE_ERR_INVALID_ARG, "ep_rank %d", c->ep_rank);
+  if (c->tp_size < 0 || c->tp_size > 32 || c->tp_rank < 0 || (c->tp_size > 1 && c->tp_rank >= c->tp_size))
+    return fail(MOE_ERR_INVALID_ARG, "tp rank %d / size %d", c->tp_rank, c->tp_size);
+  if (c->tp_size > 1) {
+    if (c->ep_size > 1) return fail(MOE_ERR_UNSUPPORTED, "expert parallelism and expert TP together");
+    if (c->ffn / 128 < c->tp_size || (c->shared_ffn > 0 && c->shared_ffn / 128 < c->tp_size))
+      return fail(MOE_ERR_INVALID_ARG, "tp_size %d > 128-column chunks (ffn/128 = %d, shared_ffn/128 = %d)",
+                  c->tp_size, c->ffn / 128, c->shared_ffn / 128);
+    if (c->wtype == MOE_W_F32 || c->hidden % 256)
+      return fail(MOE_ERR_UNSUPPORTED, "expert TP needs the tensor-core decode stream (bf16/fp8, hidden %% 256 == 0)");
+  }
   if (!w->gate_w || !w->w13 || !w->w2) return fail(MOE_ERR_INVALID_ARG, "gate_w / w13 / w2 must be non-null");
   if (c->wtype == MOE_W_FP8_BLOCK128 && (!w->w13_scale || !w->w2_scale))
     return fail(MOE_ERR_INVALID_ARG, "FP8 weights need w13_scale and w2_scale");
@@ -292,8 +305,19 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   L->e0 = cfg->ep_rank * L->E;
   L->k = cfg->top_k;
   L->H = cfg->hidden;
-  L->F = cfg->ffn;
-  L->Fs = cfg->shared_ffn;
+  L->F_full = cfg->ffn;
+  L->Fs_full = cfg->shared_ffn;
+  L->tp_size = cfg->tp_size > 1 ? cfg->tp_size : 1;
+  L->tp_rank = L->tp_size > 1 ? cfg->tp_rank : 0;
+  {
+    // TP: rank r holds chunks [r n / P, (r+1) n / P) of the n 128-column chunks
+    auto slice = [&](int full) {
+      const int n = full / 128, P = L->tp_size, r = L->tp_rank;
+      return ((r + 1) * n / P - r * n / P) * 128;
+    };
+    L->F = slice(cfg->ffn);
+    L->Fs = cfg->shared_ffn > 0 ? slice(cfg->shared_ffn) : 0;
+  }
   L->fp8 = cfg->wtype == MOE_W_FP8_BLOCK128;
   L->f32w = cfg->wtype == MOE_W_F32;
   L->act_bytes = L->fp8 ? 1 : 2;
@@ -366,7 +390,7 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   L->nchunk_max = (int)((Tr + kChunkTokens - 1) / kChunkTokens);
   const int ab = L->act_bytes;
   C_TRY(dalloc(L, &L->logits, (size_t)Tm * L->gate_rows * 4, false));
-  if (cfg->ep_size > 1 || cfg->nccl_unique_id) S_TRY(ep_create(L, cfg));
+  if (cfg->ep_size > 1 || (cfg->nccl_unique_id && L->tp_size == 1)) S_TRY(ep_create(L, cfg));
   C_TRY(dalloc(L, &L->topk_idx, (size_t)pairs * 4, false));
   C_TRY(dalloc(L, &L->topk_w, (size_t)pairs * 4, false));
   C_TRY(dalloc(L, &L->sgate, (size_t)Tm * 4, false));
@@ -379,6 +403,10 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   C_TRY(dalloc(L, &L->n_tiles, 4, false));
   C_TRY(dalloc(L, &L->act_list, (size_t)E * 4, false));
   C_TRY(dalloc(L, &L->n_active, 4, false));
+  C_TRY(dalloc(L, &L->imm_list, (size_t)E * 4, false));
+  C_TRY(dalloc(L, &L->def_list, (size_t)E * 4, false));
+  C_TRY(dalloc(L, &L->n_lists, 8, false));
+  C_TRY(cudaMemset(L->n_lists, 0, 8));
   C_TRY(dalloc(L, &L->sched, 32, false));
   C_TRY(cudaMemset(L->sched, 0, 32));
   C_TRY(dalloc(L, &L->pairs, (size_t)L->max_tiles * sizeof(int4), false));
@@ -491,7 +519,18 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
       const size_t n = (size_t)2 * L->gemv_max_tokens * H * 4;
       C_TRY(dalloc(L, &L->dacc, n, false));
       C_TRY(cudaMemset(L->dacc, 0, n));
+      if (!f8) {
+        C_TRY(dalloc(L, &L->xcopy, (size_t)L->gemv_max_tokens * H * 2, false));
+        C_TRY(cudaMemset(L->xcopy, 0, (size_t)L->gemv_max_tokens * H * 2));
+        if (!make_kmajor_map(&L->dmap_xc, L->xcopy, false, L->gemv_max_tokens, H, 16))
+          return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for the decode x copy"));
+      }
     }
+  }
+  if (L->tp_size > 1) {
+    if (!L->fused_decode) return cleanup(fail(MOE_ERR_UNSUPPORTED, "expert TP needs the fused decode stream"));
+    if (cfg->nccl_unique_id && ep_nccl_init(&L->tp_comm, L->tp_size, L->tp_rank, cfg->nccl_unique_id) != 0)
+      return cleanup(fail(MOE_ERR_NCCL, "ncclCommInitRank(P=%d, rank=%d) failed (TP)", L->tp_size, L->tp_rank));
   }
   C_TRY(cudaDeviceSynchronize());
 #undef C_TRY
@@ -770,10 +809,27 @@ static moe_status ep_forward_nccl(moe_layer *L, const void *x, const void *resid
   return ep_phase_d(L, residual, T, din, y, want_def ? dout : nullptr, st);
 }
 
-static moe_status forward_impl(moe_layer *L, const void *x, const void *residual, int32_t T, int32_t n_def,
-                               const void *deferred_in, void *y, void *deferred_out, moe_routing_out *dbg,
-                               void *stream) {
+// One forward.  Modes: plain / split deferral (moe_layer_forward[_deferred]:
+// deferred slots -> deferred_out) and chained deferral (moe_layer_forward_chained:
+// deferred slots left for the next layer, `prev`'s deferred slots computed here).
+// skip_finalize: leave the fp32 partial sums in L->dacc (in-process TP group).
+struct FwdArgs {
+  const void *x, *residual;
+  int32_t T, n_def;
+  const void *deferred_in;
+  void *y, *deferred_out;
+  moe_routing_out *dbg;
+  bool chained;
+  moe_layer *prev;
+  bool skip_finalize;
+};
+
+static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
   if (!L) return fail(MOE_ERR_INVALID_ARG, "null layer");
+  const void *x = A.x, *residual = A.residual, *deferred_in = A.deferred_in;
+  void *y = A.y, *deferred_out = A.deferred_out;
+  const int32_t T = A.T, n_def = A.n_def;
+  moe_routing_out *dbg = A.dbg;
   NvtxRange nvtx(T <= L->gemv_max_tokens ? "moe_layer_forward/decode" : "moe_layer_forward/prefill");
   if (T < 0) return fail(MOE_ERR_INVALID_ARG, "T = %d < 0", T);
   if (T > L->max_tokens) return fail(MOE_ERR_CAPACITY, "T = %d > max_tokens = %d", T, L->max_tokens);
@@ -781,6 +837,25 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   if (T > 0 && (!x || !y)) return fail(MOE_ERR_INVALID_ARG, "x and y must be non-null");
   if (x && x == y) return fail(MOE_ERR_INVALID_ARG, "y must not alias x");
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  moe_layer *prev = A.prev;
+  if (A.chained) {
+    if (L->ep.P > 1 || L->ep.comm) return fail(MOE_ERR_UNSUPPORTED, "chained deferral on an expert-parallel layer");
+    if (!(L->fused_decode && T >= 1 && T <= L->gemv_max_tokens && L->E_glob <= 256))
+      return fail(MOE_ERR_UNSUPPORTED, "chained deferral runs on the decode stream: T = %d must be in [1, %d]", T,
+                  L->gemv_max_tokens);
+    if (prev) {
+      if (prev == L) return fail(MOE_ERR_INVALID_ARG, "prev is this layer");
+      if (prev->H != L->H || prev->fp8 != L->fp8 || prev->cfg.device != L->cfg.device ||
+          prev->tp_size != L->tp_size || prev->tp_rank != L->tp_rank || !prev->fused_decode || prev->ep.P > 1)
+        return fail(MOE_ERR_INVALID_ARG, "prev has another shape / dtype / device / TP split");
+      if (prev->chain_T != T || prev->chain_ndef <= 0)
+        return fail(MOE_ERR_INVALID_ARG, "prev's last call was not a chained forward with n_deferred > 0 on %d tokens", T);
+    }
+  } else if (prev) {
+    return fail(MOE_ERR_INVALID_ARG, "prev is for chained forwards only");
+  }
+  if (L->tp_size > 1 && !L->tp_comm && !A.skip_finalize)
+    return fail(MOE_ERR_INVALID_ARG, "layer is a rank of an in-process TP group: use moe_tp_group_forward");
   if (L->ep.P > 1 || L->ep.comm) {
     if (!L->ep.comm)
       return fail(MOE_ERR_INVALID_ARG, "layer belongs to an in-process EP group: use moe_ep_group_forward");
@@ -799,7 +874,7 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
   const bool tc_decode = decode && L->umma && L->E_glob <= 256 && L->E <= 256;  // T <= 16: small-T route + swap-AB kernels
   const bool fused = tc_decode && L->fused_decode;  // route -> fused W13/W2 stream -> finalize (self-re-arming counters)
   if (L->tp_size > 1 && !fused)
-    return fail(MOE_ERR_UNSUPPORTED, "decode TP (tp_size = %d) needs the fused decode stream: T = %d must be <= %d",
+    return fail(MOE_ERR_UNSUPPORTED, "expert TP (tp_size = %d) needs the fused decode stream: T = %d must be <= %d",
                 L->tp_size, T, L->gemv_max_tokens);
   if (!fused) CUDA_TRY(cudaMemsetAsync(L->sched, 0, 32, st));
   RouterArgs r{};
@@ -824,7 +899,10 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     rs.debug = dbg_route;
     rs.trace = L->trace;
     rs.fp8 = L->fp8;
-    if (L->fp8) { rs.xq = L->xq; rs.xs = L->xs; rs.xq_img = L->xq_img; rs.xq_img_stride = L->img_tiles_sh; }
+    if (L->fp8) { rs.xq = L->xq; rs.xs = L->xs; }
+    else rs.xcopy = L->xcopy;
+    rs.n_imm = A.chained ? k - n_def : k;
+    rs.imm_list = L->imm_list; rs.def_list = L->def_list; rs.n_imm_list = L->n_lists; rs.n_def_list = L->n_lists + 1;
     KL_TRY(launch_route_small(rs, st));
     mark(L, ST_PERMUTE, st);
   } else {
@@ -861,56 +939,67 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
     mark(L, ST_GATHER, st);
   }
   if (fused) {
-    // 5+6+7 (decode). one weight stream per (slot, 128-column chunk): W13 -> SwiGLU -> h in smem ->
+    // 5+6+7 (decode). one weight stream per (expert, 128-column chunk): W13 -> SwiGLU -> h in smem ->
     // W2 -> weighted fp32 sums (umma_decode_fused.cu), then residual / deferral / bf16 in finalize
     const bool f8 = L->fp8;
     FusedDecodeParams fp{};
-    CUtensorMap xmap;                            // token-order activations, shared by both groups
-    if (f8) {
-      xmap = L->dmap_xq;
-    } else if (!make_kmajor_map(&xmap, x, false, T, H, 16)) {
-      return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
-    }
-    {
-      FdGroup &g = fp.g[0];
-      g.x_map = xmap; g.w13 = (const uint8_t *)L->w13; g.w2 = (const uint8_t *)L->w2;
-      if (f8) {
-        g.w13_img = L->w13_img; g.w13_img_stride = L->w13_img_stride;
-        g.x_img = L->xq_img; g.x_img_stride = L->img_tiles_sh; g.w2_s = L->w2_s;
-      }
-    }
+    auto routed = [&](FdGroup &g, const moe_layer *S, const int32_t *list, const int32_t *n_list, int a0, int a1,
+                      int a2) {
+      g.x_map = S->fp8 ? S->dmap_xq : S->dmap_xc;
+      g.w13 = (const uint8_t *)S->w13; g.w13_s = S->w13_s; g.xs = S->xs;
+      g.w2 = (const uint8_t *)S->w2; g.w2_s = S->w2_s; g.nch = S->F / 128;
+      g.list = list; g.n_list = n_list; g.topk_idx = S->topk_idx; g.topk_w = S->topk_w; g.k = S->k; g.e0 = S->e0;
+      g.a0 = a0; g.a1 = a1; g.a2 = a2;
+    };
+    const bool want_def = !A.chained && deferred_out != nullptr && n_def > 0;
+    if (A.chained && n_def > 0)      // this layer's deferred slots are the next layer's work (Eq. L241)
+      routed(fp.g[0], L, L->imm_list, L->n_lists, 0, k - n_def, k - n_def);
+    else                             // split deferral: [k - n_def, k) -> deferred_out
+      routed(fp.g[0], L, L->act_list, L->n_active, 0, want_def ? k - n_def : k, k);
     if (Fs > 0) {
       FdGroup &g = fp.g[1];
-      g.x_map = xmap;
-      g.w13 = (const uint8_t *)L->ws13; g.w2 = (const uint8_t *)L->ws2;
-      if (f8) {
-        g.w13_img = L->ws13_img; g.w13_img_stride = 0;
-        g.x_img = L->xq_img; g.x_img_stride = L->img_tiles_sh; g.w2_s = L->ws2_s;
-      }
+      g.x_map = f8 ? L->dmap_xq : L->dmap_xc;
+      g.w13 = (const uint8_t *)L->ws13; g.w13_s = L->ws13_s; g.xs = L->xs;
+      g.w2 = (const uint8_t *)L->ws2; g.w2_s = L->ws2_s; g.nch = Fs / 128;
     } else {
       fp.g[1] = fp.g[0];
     }
-    fp.nch[0] = F / 128; fp.nch[1] = Fs / 128;
-    fp.H = H; fp.T = T; fp.k = k; fp.n_imm = deferred_out ? k - n_def : k; fp.has_shared = Fs > 0;
-    fp.n_active = L->n_active; fp.act_list = L->act_list;
-    fp.topk_idx = L->topk_idx; fp.e0 = L->e0; fp.topk_w = L->topk_w;
+    int prev_units = 0;
+    if (prev) {                      // R^def_{k-1}(I_{k-1}) joins this layer's output (acc_imm)
+      routed(fp.g[2], prev, prev->def_list, prev->n_lists + 1, prev->k - prev->chain_ndef, prev->k, prev->k);
+      prev_units = (int)std::min<int64_t>(prev->E, (int64_t)T * prev->chain_ndef) * (prev->F / 128);
+      prev->chain_T = -1;            // consumed
+    } else {
+      fp.g[2] = fp.g[0];
+    }
+    fp.H = H; fp.T = T; fp.has_shared = Fs > 0; fp.has_prev = prev != nullptr;
     fp.sgate = L->cfg.shared_gated ? L->sgate : nullptr;
     float *acc_imm = L->dacc, *acc_def = L->dacc + (size_t)L->gemv_max_tokens * H;
     fp.acc_imm = acc_imm; fp.acc_def = acc_def;
     fp.sched = L->sched + 5; fp.done = L->sched + 6;
     fp.trace = L->trace;
-    DecodeFinalizeArgs fa{};
-    fa.T = T; fa.H = H; fa.use_def = deferred_out != nullptr && n_def > 0;
-    fa.acc_imm = acc_imm; fa.acc_def = acc_def;
-    fa.residual = residual; fa.deferred_in = deferred_in; fa.y = y; fa.deferred_out = deferred_out;
-    if (L->tp_size > 1 && L->tp_rank != 0) fa.residual = fa.deferred_in = nullptr;   // added once, by TP rank 0
-    fa.trace = L->trace;
-    fp.tp_rank = L->tp_rank; fp.tp_size = L->tp_size;
-    const int tpP = L->tp_size, tpr = L->tp_rank;   // this rank's chunks: c = tpr (mod tpP)
-    const int units = (Fs > 0 ? (Fs / 128 - tpr + tpP - 1) / tpP : 0) +
-                      (int)std::min<int64_t>(E, pairs) * ((F / 128 - tpr + tpP - 1) / tpP);
+    const int units = prev_units + Fs / 128 + (int)std::min<int64_t>(E, pairs) * (F / 128);
     KL_TRY(launch_umma_decode_fused(f8, fp, std::min(L->num_sms, units), st));
     mark(L, ST_GEMM1, st);
+    if (A.chained) { L->chain_T = n_def > 0 ? T : -1; L->chain_ndef = n_def; }
+    else L->chain_T = -1;
+    if (L->tp_size > 1 && L->tp_comm) {
+      // TP: sum the P ranks' fp32 partials (immediate and deferred sums) -- PAPER.md L197
+      if (ep_nccl_allreduce_f32(L->tp_comm, acc_imm, (size_t)T * H, st) != 0 ||
+          (want_def && ep_nccl_allreduce_f32(L->tp_comm, acc_def, (size_t)T * H, st) != 0))
+        return fail(MOE_ERR_NCCL, "ncclAllReduce of the TP partials failed %s", ep_nccl_error(L->tp_comm));
+    }
+    if (A.skip_finalize) {
+      L->pending_use_def = want_def;
+      (decode ? L->launches_decode : L->launches_prefill) = L->n_launch;
+      return MOE_OK;
+    }
+    DecodeFinalizeArgs fa{};
+    fa.T = T; fa.H = H; fa.use_def = want_def;
+    fa.acc_imm = acc_imm; fa.acc_def = acc_def;
+    fa.residual = residual; fa.deferred_in = A.chained ? nullptr : deferred_in; fa.y = y;
+    fa.deferred_out = A.chained ? nullptr : deferred_out;
+    fa.trace = L->trace;
     KL_TRY(launch_decode_finalize(fa, st));
     mark(L, ST_COMBINE, st);
   } else if (decode) {
@@ -953,13 +1042,21 @@ static moe_status forward_impl(moe_layer *L, const void *x, const void *residual
 
 moe_status moe_layer_forward(moe_layer *L, const void *x, const void *residual, int32_t T, void *y,
                              moe_routing_out *dbg, void *stream) {
-  return forward_impl(L, x, residual, T, 0, nullptr, y, nullptr, dbg, stream);
+  FwdArgs a{x, residual, T, 0, nullptr, y, nullptr, dbg, false, nullptr, false};
+  return forward_impl(L, a, stream);
 }
 
 moe_status moe_layer_forward_deferred(moe_layer *L, const void *x, const void *residual, int32_t T,
                                       int32_t n_deferred, const void *deferred_in, void *y, void *deferred_out,
                                       moe_routing_out *dbg, void *stream) {
-  return forward_impl(L, x, residual, T, n_deferred, deferred_in, y, deferred_out, dbg, stream);
+  FwdArgs a{x, residual, T, n_deferred, deferred_in, y, deferred_out, dbg, false, nullptr, false};
+  return forward_impl(L, a, stream);
+}
+
+moe_status moe_layer_forward_chained(moe_layer *L, const void *x, const void *residual, int32_t T,
+                                     int32_t n_deferred, moe_layer *prev, void *y, void *stream) {
+  FwdArgs a{x, residual, T, n_deferred, nullptr, y, nullptr, nullptr, true, prev, false};
+  return forward_impl(L, a, stream);
 }
 
 moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void *const *x,
@@ -976,14 +1073,19 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
     if (n_deferred < 0 || n_deferred > L->k - 1) return fail(MOE_ERR_INVALID_ARG, "n_deferred");
     if (T[r] > 0 && (!x[r] || !y[r])) return fail(MOE_ERR_INVALID_ARG, "x/y of rank %d", r);
   }
+  for (int r = 1; r < P; ++r)
+    if (layers[r]->cfg.device != layers[0]->cfg.device)
+      return fail(MOE_ERR_UNSUPPORTED, "in-process EP group: all ranks on one device (the stream's)");
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   const int64_t Tm = std::max(1, layers[0]->max_tokens);
   const int H = layers[0]->H, k = layers[0]->k;
+  int caller_dev = 0;
+  CUDA_TRY(cudaGetDevice(&caller_dev));
+  struct Restore { int d; ~Restore() { cudaSetDevice(d); } } restore{caller_dev};
+  CUDA_TRY(cudaSetDevice(layers[0]->cfg.device));
   moe_status s;
-  for (int r = 0; r < P; ++r) {
-    CUDA_TRY(cudaSetDevice(layers[r]->cfg.device));
+  for (int r = 0; r < P; ++r)
     if ((s = ep_phase_a(layers[r], x[r], T[r], st)) != MOE_OK) return s;
-  }
   // counts: rank d receives cnt_dev[d] of every source
   for (int d = 0; d < P; ++d)
     for (int src = 0; src < P; ++src)
@@ -1003,7 +1105,6 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
                                cudaMemcpyDefault, st));
     }
   for (int r = 0; r < P; ++r) {
-    CUDA_TRY(cudaSetDevice(layers[r]->cfg.device));
     const bool want_def = deferred_out && deferred_out[r] && n_deferred > 0;
     if ((s = ep_phase_c(layers[r], x[r], T[r], n_deferred, want_def, st)) != MOE_OK) return s;
   }
@@ -1019,7 +1120,6 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
                                  cudaMemcpyDefault, st));
     }
   for (int r = 0; r < P; ++r) {
-    CUDA_TRY(cudaSetDevice(layers[r]->cfg.device));
     const bool want_def = deferred_out && deferred_out[r] && n_deferred > 0;
     if ((s = ep_phase_d(layers[r], residual ? residual[r] : nullptr, T[r],
                         deferred_in ? deferred_in[r] : nullptr, y[r], want_def ? deferred_out[r] : nullptr, st)) != MOE_OK)
@@ -1028,18 +1128,61 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
   return MOE_OK;
 }
 
-moe_status moe_layer_set_decode_tp(moe_layer *L, int32_t rank, int32_t size) {
-  if (!L) return fail(MOE_ERR_INVALID_ARG, "null layer");
-  if (size < 1 || rank < 0 || rank >= size) return fail(MOE_ERR_INVALID_ARG, "tp rank %d / size %d", rank, size);
-  if (size > 1) {
-    if (L->ep.P > 1 || L->ep.comm) return fail(MOE_ERR_UNSUPPORTED, "decode TP on an expert-parallel layer");
-    if (!L->fused_decode || !L->umma) return fail(MOE_ERR_UNSUPPORTED, "decode TP needs the fused decode stream");
-    if (L->F / 128 < size || (L->Fs > 0 && L->Fs / 128 < size))
-      return fail(MOE_ERR_INVALID_ARG, "tp size %d > 128-column chunks (F/128 = %d, Fs/128 = %d)", size,
-                  L->F / 128, L->Fs / 128);
+moe_status moe_tp_group_forward(moe_layer *const *layers, int32_t P, const void *const *x,
+                                const void *const *residual, int32_t T, int32_t n_deferred,
+                                const void *const *deferred_in, void *const *y, void *const *deferred_out,
+                                void *stream) {
+  if (!layers || !x || !y || P < 2 || P > 32) return fail(MOE_ERR_INVALID_ARG, "bad group arguments");
+  NvtxRange nvtx("moe_tp_group_forward");
+  const int dev = layers[0] ? layers[0]->cfg.device : 0;
+  for (int r = 0; r < P; ++r) {
+    const moe_layer *L = layers[r];
+    if (!L || L->tp_size != P || L->tp_rank != r || L->tp_comm)
+      return fail(MOE_ERR_INVALID_ARG, "layer %d is not rank %d of an in-process TP group of %d", r, r, P);
+    if (L->cfg.device != dev) return fail(MOE_ERR_UNSUPPORTED, "in-process TP group: all ranks on one device");
+    if (!x[r] || !y[r]) return fail(MOE_ERR_INVALID_ARG, "x/y of rank %d", r);
   }
-  L->tp_rank = rank; L->tp_size = size;
-  return MOE_OK;
+  if (T <= 0) return T == 0 ? MOE_OK : fail(MOE_ERR_INVALID_ARG, "T = %d", T);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  int caller_dev = 0;
+  CUDA_TRY(cudaGetDevice(&caller_dev));
+  CUDA_TRY(cudaSetDevice(dev));
+  moe_status s = MOE_OK;
+  for (int r = 0; r < P && s == MOE_OK; ++r) {
+    const bool want_def = deferred_out && deferred_out[r] && n_deferred > 0;
+    FwdArgs a{x[r], nullptr, T, n_deferred, nullptr, y[r], want_def ? deferred_out[r] : nullptr, nullptr, false,
+              nullptr, true};
+    s = forward_impl(layers[r], a, stream);
+  }
+  if (s == MOE_OK) {
+    // the all-reduce of the fp32 partials, on one device: sum into rank 0, copy back
+    const int H = layers[0]->H;
+    const bool use_def = layers[0]->pending_use_def;
+    const float *src[32];
+    for (int part = 0; part < (use_def ? 2 : 1) && s == MOE_OK; ++part) {
+      const size_t off = part ? (size_t)layers[0]->gemv_max_tokens * H : 0;
+      for (int r = 0; r < P; ++r) src[r] = layers[r]->dacc + (part ? (size_t)layers[r]->gemv_max_tokens * H : 0);
+      cudaError_t e = launch_sum_f32(layers[0]->dacc + off, src + 1, P - 1, (int64_t)T * H, st);
+      for (int r = 1; r < P && e == cudaSuccess; ++r)
+        e = cudaMemcpyAsync(layers[r]->dacc + (part ? (size_t)layers[r]->gemv_max_tokens * H : 0),
+                            layers[0]->dacc + off, (size_t)T * H * 4, cudaMemcpyDeviceToDevice, st);
+      if (e != cudaSuccess) s = fail(MOE_ERR_CUDA, "TP group reduce: %s", cudaGetErrorString(e));
+    }
+    for (int r = 0; r < P && s == MOE_OK; ++r) {
+      moe_layer *L = layers[r];
+      DecodeFinalizeArgs fa{};
+      fa.T = T; fa.H = H; fa.use_def = use_def;
+      fa.acc_imm = L->dacc; fa.acc_def = L->dacc + (size_t)L->gemv_max_tokens * H;
+      fa.residual = residual ? residual[r] : nullptr;
+      fa.deferred_in = deferred_in ? deferred_in[r] : nullptr;
+      fa.y = y[r];
+      fa.deferred_out = deferred_out ? deferred_out[r] : nullptr;
+      cudaError_t e = launch_decode_finalize(fa, st);
+      if (e != cudaSuccess) s = fail(MOE_ERR_CUDA, "finalize: %s", cudaGetErrorString(e));
+    }
+  }
+  cudaSetDevice(caller_dev);
+  return s;
 }
 
 moe_status moe_layer_profile(moe_layer *L, int32_t enable) {

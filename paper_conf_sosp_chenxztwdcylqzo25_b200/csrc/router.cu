@@ -394,12 +394,12 @@ __device__ void route_small_tail(const RouteSmallArgs &a, float *rsm, const floa
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   __shared__ int ids_s[RS_MAX_PAIRS];
   __shared__ int cnt_s[RS_MAX_E], slot_s[RS_MAX_E], offs_s[RS_MAX_E];
-  __shared__ unsigned bm[RS_MAX_E / 32];
+  __shared__ unsigned bm[RS_MAX_E / 32], bmi[RS_MAX_E / 32], bmd[RS_MAX_E / 32];
   long long ck[4];
   ck[0] = clock64();
   if (a.trace && tid == 0) a.trace[1] = gtimer_ns();
   for (int e = tid; e < p.E; e += RS_THREADS) cnt_s[e] = 0;
-  if (tid < RS_MAX_E / 32) bm[tid] = 0u;
+  if (tid < RS_MAX_E / 32) bm[tid] = bmi[tid] = bmd[tid] = 0u;
   // one warp per token; warps past the last token skip (warp-uniform branch)
 #pragma unroll 1
   for (int t0 = 0; t0 < T; t0 += RS_THREADS / 32) {
@@ -424,9 +424,26 @@ __device__ void route_small_tail(const RouteSmallArgs &a, float *rsm, const floa
     if (e >= 0 && e < p.E) {
       atomicAdd(&cnt_s[e], 1);
       atomicOr(&bm[e >> 5], 1u << (e & 31));
+      atomicOr(q % k < a.n_imm ? &bmi[e >> 5] : &bmd[e >> 5], 1u << (e & 31));
     }
   }
   __syncthreads();
+  if (a.imm_list) {
+    // Expert Deferral (chained forwards): the experts of the immediate and of the
+    // deferred canonical slots, ascending (bitmap + popc, one thread per expert)
+    const int e = tid;
+    int bi = 0, ni = 0, bd = 0, nd = 0;
+#pragma unroll
+    for (int w = 0; w < RS_MAX_E / 32; ++w) {
+      const int pi = __popc(bmi[w]), pd = __popc(bmd[w]);
+      ni += pi; nd += pd;
+      if (w < (e >> 5)) { bi += pi; bd += pd; }
+    }
+    const unsigned below = (1u << (e & 31)) - 1u;
+    if (e < p.E && ((bmi[e >> 5] >> (e & 31)) & 1u)) a.imm_list[bi + __popc(bmi[e >> 5] & below)] = e;
+    if (e < p.E && ((bmd[e >> 5] >> (e & 31)) & 1u)) a.def_list[bd + __popc(bmd[e >> 5] & below)] = e;
+    if (tid == 0) { *a.n_imm_list = ni; *a.n_def_list = nd; }
+  }
   if (!p.dbg_perm && !p.dbg_counts) {
     // fused decode: the expert kernel reads token-order activations and finds its
     // tokens in topk_idx, so only the active-expert list is needed (ascending ids)
@@ -600,13 +617,16 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
         q.y = (uint32_t)f32_to_e4m3(f[4] * inv) | ((uint32_t)f32_to_e4m3(f[5] * inv) << 8) |
               ((uint32_t)f32_to_e4m3(f[6] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[7] * inv) << 24);
         *reinterpret_cast<uint2 *>(reinterpret_cast<uint8_t *>(a.xq) + t * H + c * 8) = q;
-        if ((lane & 15) == 0) {
-          const int b = (int)(c >> 4);
-          a.xs[t * (H / 128) + b] = exp2i(ex);
-          if (a.xq_img) a.xq_img[sf_img_off(t, b, a.xq_img_stride)] = (uint8_t)(ex + 127);
-        }
+        if ((lane & 15) == 0) a.xs[t * (H / 128) + (int)(c >> 4)] = exp2i(ex);
       }
     }
+  }
+
+  // ---- BF16: x into the layer's own token-order buffer (read by the decode stream) ----
+  if (!a.fp8 && a.xcopy) {
+    const int64_t n16 = (int64_t)T * H / 8;
+    for (int64_t i = (int64_t)blockIdx.x * RS_THREADS + threadIdx.x; i < n16; i += (int64_t)gridDim.x * RS_THREADS)
+      reinterpret_cast<uint4 *>(a.xcopy)[i] = __ldg(reinterpret_cast<const uint4 *>(a.x) + i);
   }
 
   // ---- last CTA: route + permute ----

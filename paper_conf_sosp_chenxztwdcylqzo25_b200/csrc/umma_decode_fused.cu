@@ -1,32 +1,40 @@
 // umma_decode_fused.cu -- decode expert FFNs as ONE weight stream per unit.
 //
 // Decode (<= 16 tokens per expert) is HBM-bound: every
-// active expert's W13 and W2 must stream through once.  The two-launch chain
-// (umma_decode.cu: W13 -> h in HBM -> W2) pays a launch drain, a W2 tail wave
-// (9 x 56 row blocks on 148 SMs) and the h round trip.  Here a unit is
-// (slot, 128-column chunk c of the expert's FFN dimension):
+// active expert's W13 and W2 must stream through once.  A unit is (expert,
+// 128-column chunk c of its FFN dimension):
 //   phase A: stream the 256-row W13 tile c (gate + up rows of h columns
 //            128c .. 128c+127, all H) through the swap-AB MMA (weights = the
-//            M = 128 operand, the slot's <= 16 token rows the N = 16 operand),
-//            SwiGLU from fp32 TMEM, FP8: 1x128 UE8M0 requant -- exactly the
-//            128-column block of R10/R11, so the scale is local to the unit --
-//            and write h_c [16 tokens x 128] into shared memory as the B
-//            operand of phase B (SW128 K-major image, no HBM round trip);
+//            M = 128 operand, the <= 16 token rows the N = 16 operand).
+//            FP8: UNSCALED kind::f8f6f4 MMAs, one 128-K k-block per TMEM
+//            accumulator slot of a 4-slot ring; the epilogue folds each slot
+//            into fp32 registers with the k-block's 128x128 weight-block scale
+//            x the token's 1x128 activation scale (the same products and
+//            scales as the block-scaled MMA, summed per k-block -- reading
+//            R23), so the MMA issue rate is the unscaled one (~75 vs ~117
+//            cycles per 128x16x32 MMA, profiles/r01/mma_single_micro.txt).
+//            Then SwiGLU from fp32, FP8: 1x128 UE8M0 requant of h -- exactly
+//            the 128-column block of R10/R11, so the scale is local to the
+//            unit -- written into shared memory as phase B's B operand (SW128
+//            K-major image, no HBM round trip).  BF16: one kind::f16
+//            accumulator over all of K.
 //   phase B: stream W2[:, 128c .. 128c+127] (H/256 tiles of 256 rows x 128 B)
-//            against h_c: one k-block per 128-row M tile, so the MMA is the
-//            unscaled kind::f8f6f4 and the W2 block scale x the h scale are
-//            applied in the epilogue, which adds w_tj * partial into an fp32
-//            [T, H] accumulator (red.global.add; immediate or deferred sum,
-//            PAPER.md L219-241) -- the k-sum over chunks and the weighted
-//            combine over a token's experts (L187) happen in the same adds.
-// Units are claimed from a device counter (the L181 dynamic task queue): the
-// shared expert's chunks first, then the active routed experts (ascending id).
-// The kernel is PDL-launched while the router runs; every warp waits for the
-// router's completion before touching routing data or activations (an optional
-// L2 prefetch of the shared expert before that wait, MOE_DECODE_PF=1, measured
-// slower).  The weight stream uses an evict-first L2 policy.
-// decode_finalize_kernel adds the residual / deferred input, writes bf16 y (and
-// deferred_out) and re-zeroes the sums.
+//            against h_c: one k-block per 128-row M tile, unscaled MMA, the W2
+//            block scale x the h scale x the routing weight applied in the
+//            epilogue, which red.adds into fp32 [T, H] sums (PAPER.md
+//            L219-241) -- the k-sum over chunks and the weighted combine over a
+//            token's experts (L187) happen in the same adds.
+// Operand groups: 0 = this layer's routed experts, 1 = the shared expert,
+// 2 = the PREVIOUS layer's deferred experts (Expert Deferral, PAPER.md L241:
+// R^def_{k-1}(I_{k-1}) joins O_k).  Group-2 units depend only on the previous
+// layer's routing and activations, which are complete when this kernel starts,
+// so they are claimed first and stream while this layer's router is still
+// running; every role waits for the router (griddepcontrol.wait) only when it
+// reaches its first group-0/1 unit.  Units are claimed from a device counter
+// (the L181 dynamic task queue): group 2, then the shared expert's chunks,
+// then the routed experts (ascending id).  The weight stream uses an
+// evict-first L2 policy.  decode_finalize_kernel adds the residual / deferred
+// input, writes bf16 y (and deferred_out) and re-zeroes the sums.
 //
 // Summation order across chunks is the order of the atomics (fp32; results
 // are reproducible to fp32 rounding, not bitwise) -- DESIGN.md reading R22.
@@ -40,16 +48,18 @@
 namespace moe {
 using namespace sm100;
 
-constexpr int FD_N = 16, FD_STAGES = 5, FD_THREADS = 192, FD_UQ = 4, FD_ACCB = 4;
+constexpr int FD_N = 16, FD_STAGES = 5, FD_THREADS = 192, FD_UQ = 4, FD_ACCB = 4, FD_ACCA_SLOTS = 4;
 constexpr int FD_A_BYTES = 256 * 128;          // one 256-row weight tile k-block (two 128-row MMA tiles)
 constexpr int FD_B_BYTES = FD_N * 128;         // 16 token rows x 128 B
-constexpr int FD_SF_BYTES = 512;
 constexpr int FD_H_BYTES = 2 * FD_B_BYTES;     // h_c: FP8 one k-block, BF16 two
-constexpr size_t FD_SMEM = 1024 + (size_t)FD_STAGES * (FD_A_BYTES + FD_B_BYTES + 2 * FD_SF_BYTES) + FD_H_BYTES +
+constexpr int FD_MAX_KB = 64;                  // H <= 8192: FP8 k-blocks of W13
+constexpr size_t FD_SMEM = 1024 + (size_t)FD_STAGES * (FD_A_BYTES + FD_B_BYTES) + FD_H_BYTES +
                            2 * 2 * FD_N * 32 * 4 +     // up -> gate exchange [gate warp][acc][token][lane]
+                           2 * FD_MAX_KB * FD_N * 4 +  // activation scales [this layer | previous layer][kb][token]
                            1024;                       // barriers, queue, amax, scales
 constexpr uint32_t FD_TMEM_COLS = 256;
-constexpr uint32_t FD_ACCA = 0, FD_SFA_COL = 32, FD_SFB_COL = 40, FD_ACCB_COL = 64;   // + 32 per ring slot
+constexpr uint32_t FD_ACCA_COL = 0, FD_ACCB_COL = 128;   // + 32 per ring slot (two 16-column MMA tiles)
+static_assert(FD_ACCA_SLOTS * 32 <= (int)FD_ACCB_COL && FD_ACCB_COL + FD_ACCB * 32 <= FD_TMEM_COLS, "TMEM map");
 
 // instruction descriptor, kind::f8f6f4 (E4M3 x E4M3 -> F32, no block scale), K-major A and B
 __host__ __device__ constexpr uint32_t idesc_f8(int M, int N) {
@@ -72,30 +82,36 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
-// unit -> (valid, group, expert, row0, n tokens, chunk).  valid: 0 = past the end
-struct FdUnit {
-  int valid, group, expert, row0, n, chunk;
-};
+// 128-column chunks of a group this kernel streams
+__device__ __forceinline__ int fd_units_per_expert(const FdGroup &g) { return g.nch; }
 
-__device__ __forceinline__ FdUnit fd_unit(const FusedDecodeParams &p, int u) {
-  // decode TP (moe_layer_set_decode_tp): this rank streams the chunks c = tp_rank + tp_size * j
-  // of every expert (W13 rows and W2 columns of the same 128 FFN columns), so its partial sum
-  // over chunks is its share of every expert's output
-  const int P = p.tp_size > 1 ? p.tp_size : 1, rk = P > 1 ? p.tp_rank : 0;
-  const int nl0 = (p.nch[0] - rk + P - 1) / P, nl1 = (p.nch[1] - rk + P - 1) / P;
+// unit -> (valid, group, expert, chunk).  Group 2 first (no dependency on this
+// layer's router), then the shared expert (group 1), then the routed experts.
+struct FdUnit {
+  int valid, group, expert, chunk;
+};
+__device__ __forceinline__ int fd_prev_units(const FusedDecodeParams &p) {
+  return p.has_prev ? (*p.g[2].n_list) * p.g[2].nch : 0;
+}
+// this layer's units (valid only after griddepcontrol.wait: n_list is the router's)
+__device__ __forceinline__ FdUnit fd_unit(const FusedDecodeParams &p, int u, int n_prev) {
   FdUnit r{};
-  const int ns = p.has_shared ? nl1 : 0;
-  if (u < ns) {
-    r.valid = 1; r.group = 1; r.expert = 0; r.row0 = 0; r.n = p.T; r.chunk = rk + P * u;
+  if (u < n_prev) {
+    const FdGroup &g = p.g[2];
+    r.valid = 1; r.group = 2; r.expert = g.list[u / g.nch]; r.chunk = u % g.nch;
     return r;
   }
-  const int v = u - ns;
-  const int slot = v / nl0;
-  if (slot >= *p.n_active) return r;
-  const int e = p.act_list[slot];
-  // token-order activations (all T <= 16 tokens are the N = 16 operand; the
-  // epilogue keeps the columns of the tokens routed to e)
-  r.valid = 1; r.group = 0; r.expert = e; r.row0 = 0; r.n = p.T; r.chunk = rk + P * (v % nl0);
+  u -= n_prev;
+  const int ns = p.has_shared ? p.g[1].nch : 0;
+  if (u < ns) {
+    r.valid = 1; r.group = 1; r.expert = 0; r.chunk = u;
+    return r;
+  }
+  u -= ns;
+  const FdGroup &g = p.g[0];
+  const int slot = u / g.nch;
+  if (slot >= *g.n_list) return r;
+  r.valid = 1; r.group = 0; r.expert = g.list[slot]; r.chunk = u % g.nch;
   return r;
 }
 
@@ -152,26 +168,26 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   uint8_t *sA = smem;
   uint8_t *sH = sA + FD_STAGES * FD_A_BYTES;                 // 1024-aligned
   uint8_t *sB = sH + FD_H_BYTES;
-  uint8_t *sSFA = sB + FD_STAGES * FD_B_BYTES;
-  uint8_t *sSFB = sSFA + FD_STAGES * FD_SF_BYTES;
-  float *xch = reinterpret_cast<float *>(sSFB + FD_STAGES * FD_SF_BYTES);   // [2][2][16][32]
-  uint64_t *full = reinterpret_cast<uint64_t *>(xch + 2 * 2 * FD_N * 32);
+  float *xch = reinterpret_cast<float *>(sB + FD_STAGES * FD_B_BYTES);   // [2][2][16][32]
+  float *xs_s = xch + 2 * 2 * FD_N * 32;                     // [2: this layer, previous layer][FD_MAX_KB][16]
+  uint64_t *full = reinterpret_cast<uint64_t *>(xs_s + 2 * FD_MAX_KB * FD_N);
   uint64_t *empty = full + FD_STAGES;
-  uint64_t *accA_full = empty + FD_STAGES;
-  uint64_t *h_ready = accA_full + 1;
+  uint64_t *accA_full = empty + FD_STAGES;                   // [FD_ACCA_SLOTS]
+  uint64_t *accA_empty = accA_full + FD_ACCA_SLOTS;          // [FD_ACCA_SLOTS]
+  uint64_t *h_ready = accA_empty + FD_ACCA_SLOTS;
   uint64_t *accB_full = h_ready + 1;                         // [FD_ACCB]
   uint64_t *accB_empty = accB_full + FD_ACCB;                // [FD_ACCB]
   uint64_t *uq_full = accB_empty + FD_ACCB;                  // [FD_UQ]
   uint64_t *uq_empty = uq_full + FD_UQ;                      // [FD_UQ]
   uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(uq_empty + FD_UQ);
-  int4 *unit_q = reinterpret_cast<int4 *>(tmem_base_smem + 4);   // [FD_UQ] (expert, row0, n | chunk << 16, group | valid << 1)
+  int4 *unit_q = reinterpret_cast<int4 *>(tmem_base_smem + 4);   // [FD_UQ] (expert, chunk, group, valid)
   float *amax = reinterpret_cast<float *>(unit_q + FD_UQ);       // [2 gate warps][16]
   float *hsc = amax + 2 * FD_N;                                  // [2 unit parity][16] h scale per token (FP8)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < FD_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-    mbar_init(accA_full, 1);
+    for (int s = 0; s < FD_ACCA_SLOTS; ++s) { mbar_init(&accA_full[s], 1); mbar_init(&accA_empty[s], 4); }
     mbar_init(h_ready, 1);
     for (int s = 0; s < FD_ACCB; ++s) { mbar_init(&accB_full[s], 1); mbar_init(&accB_empty[s], 4); }
     for (int i = 0; i < FD_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], 5); }
@@ -191,14 +207,19 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   if (warp == 0) {
     // ============================ producer ============================
     if (lane == 0) {
-      pdl_wait();                                // routing, xq / xperm of the route kernel
+      const int n_prev = fd_prev_units(p);       // the previous layer's routing is complete
+      bool waited = false;
       const uint64_t pol = l2_evict_first_policy();   // weights are read once per forward
       int stage = 0; uint32_t phase = 0, qs = 0, qph = 0;
       for (;;) {
         const int u = atomicAdd(p.sched, 1);
-        const FdUnit ui = fd_unit(p, u);
+        if (u >= n_prev && !waited) {
+          pdl_wait();                            // this layer's routing and xq (route kernel)
+          waited = true;
+        }
+        const FdUnit ui = fd_unit(p, u, n_prev);
         mbar_wait(&uq_empty[qs], qph ^ 1);
-        unit_q[qs] = make_int4(ui.expert, ui.row0, ui.n | (ui.chunk << 16), ui.group | (ui.valid << 1));
+        unit_q[qs] = make_int4(ui.expert, ui.chunk, ui.group, ui.valid);
         mbar_arrive(&uq_full[qs]);
         if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
         if (!ui.valid) {
@@ -209,24 +230,16 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         }
         const FdGroup &g = p.g[ui.group];
         // ---- phase A: W13 tile `chunk` (256 rows: gate + up of 128 h columns) ----
-        const uint32_t bytes_a = FD_A_BYTES + FD_B_BYTES + (FP8 ? 2 * FD_SF_BYTES : 0);
-        const uint8_t *w13 = g.w13 + ((size_t)ui.expert * p.nch[ui.group] + ui.chunk) * (size_t)KA * FD_A_BYTES;
+        const uint8_t *w13 = g.w13 + ((size_t)ui.expert * g.nch + ui.chunk) * (size_t)KA * FD_A_BYTES;
         for (int kb = 0; kb < KA; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          mbar_expect_tx(&full[stage], bytes_a);
+          mbar_expect_tx(&full[stage], FD_A_BYTES + FD_B_BYTES);
           bulk_load_hint(sA + stage * FD_A_BYTES, w13 + (size_t)kb * FD_A_BYTES, FD_A_BYTES, &full[stage], pol);
-          tma_load_2d(sB + stage * FD_B_BYTES, &g.x_map, &full[stage], kb * KDIV, ui.row0);
-          if (FP8) {
-            const uint8_t *sfa = g.w13_img + (size_t)ui.expert * g.w13_img_stride +
-                                 ((size_t)(kb >> 2) * p.nch[ui.group] + ui.chunk) * 512;
-            const uint8_t *sfb = g.x_img + ((size_t)(kb >> 2) * g.x_img_stride + (ui.row0 >> 7)) * 512;
-            bulk_load(sSFA + stage * FD_SF_BYTES, sfa, FD_SF_BYTES, &full[stage]);
-            bulk_load(sSFB + stage * FD_SF_BYTES, sfb, FD_SF_BYTES, &full[stage]);
-          }
+          tma_load_2d(sB + stage * FD_B_BYTES, &g.x_map, &full[stage], kb * KDIV, 0);
           if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
         }
         // ---- phase B: W2 column block `chunk`, H/256 tiles of 256 rows ----
-        const int KB2 = p.nch[ui.group] * KBC;     // W2 k-blocks per tile row
+        const int KB2 = g.nch * KBC;               // W2 k-blocks per tile row
         const uint8_t *w2 = g.w2 + (size_t)ui.expert * NT * KB2 * FD_A_BYTES;
         for (int n = 0; n < NT; ++n) {
           for (int kk = 0; kk < KBC; ++kk) {
@@ -241,51 +254,49 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     }
   } else if (warp == 1) {
     // ============================ MMA issuer ============================
-    pdl_wait();                                  // sleep in the grid dependency, not on an mbarrier, during routing
+    // (touches only shared memory and TMEM: no griddepcontrol.wait needed)
     int stage = 0; uint32_t phase = 0, qs = 0, qph = 0, hph = 0;
     int ab = 0; uint32_t abph = 0;
+    int as = 0; uint32_t asph = 0;
     for (;;) {
       mbar_wait(&uq_full[qs], qph);
       const int4 uq = unit_q[qs];
       __syncwarp();
       if (lane == 0) mbar_arrive(&uq_empty[qs]);
       if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
-      if (!(uq.w >> 1)) break;
-      // phase A (the accumulator is free: the epilogue read it before h_ready of the previous unit)
+      if (!uq.w) break;
+      // ---- phase A ----
       for (int kb = 0; kb < KA; ++kb) {
+        if (FP8) {                               // this k-block's accumulator slot is free
+          mbar_wait(&accA_empty[as], asph ^ 1);
+          tc_fence_after();
+        }
         mbar_wait(&full[stage], phase);
         tc_fence_after();
         if (lane == 0) {
           const uint32_t a0 = smem_u32(sA + stage * FD_A_BYTES);
           const uint32_t b0 = smem_u32(sB + stage * FD_B_BYTES);
-          // scale images hold 4 k-blocks (scale id kb & 3): copy once per 4 k-blocks, into
-          // alternating column sets so the copy never overwrites scales in-flight MMAs read
-          const uint32_t sfset = (uint32_t)((kb >> 2) & 1) * 4;
-          if (FP8 && (kb & 3) == 0) {
-            tmem_cp_32x128b_x4(tmem + FD_SFA_COL + sfset, sf_desc(smem_u32(sSFA + stage * FD_SF_BYTES)));
-            tmem_cp_32x128b_x4(tmem + FD_SFB_COL + sfset, sf_desc(smem_u32(sSFB + stage * FD_SF_BYTES)));
-          }
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
             const uint64_t bd = sw128_kmajor_desc(b0 + k * 32);
-            const uint32_t accum = (kb | k) != 0;
 #pragma unroll
             for (int t = 0; t < 2; ++t) {
               const uint64_t ad = sw128_kmajor_desc(a0 + t * 128 * 128 + k * 32);
               if (FP8)
-                mma_mxf8(tmem + FD_ACCA + t * 16, ad, bd, idesc_mxf8(128, FD_N, kb & 3, kb & 3), accum,
-                         tmem + FD_SFA_COL + sfset, tmem + FD_SFB_COL + sfset);
-              else
-                mma_bf16(tmem + FD_ACCA + t * 16, ad, bd, idesc_bf16(128, FD_N), accum);
+                mma_f8(tmem + FD_ACCA_COL + as * 32 + t * 16, ad, bd, idesc_f8(128, FD_N), k != 0);
+              else   // the accumulator is free: the epilogue read it before h_ready of the previous unit
+                mma_bf16(tmem + FD_ACCA_COL + t * 16, ad, bd, idesc_bf16(128, FD_N), (kb | k) != 0);
             }
           }
           mma_commit(&empty[stage]);
-          if (kb == KA - 1) mma_commit(accA_full);
+          if (FP8) mma_commit(&accA_full[as]);
+          else if (kb == KA - 1) mma_commit(&accA_full[0]);
         }
         __syncwarp();
         if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
+        if (FP8 && ++as == FD_ACCA_SLOTS) { as = 0; asph ^= 1; }
       }
-      // phase B: B operand = h_c in shared memory
+      // ---- phase B: B operand = h_c in shared memory ----
       mbar_wait(h_ready, hph);
       hph ^= 1;
       tc_fence_after();
@@ -323,10 +334,13 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     // ============================ epilogue (4 warps, lanes = weight rows) ============================
     const int q = warp & 3;
     const int qg = q >> 1;
+    const int et = threadIdx.x - 64;             // 0..127
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
     uint32_t qs = 0, qph = 0, aph = 0;
     int ab = 0; uint32_t abph = 0;
+    int as = 0; uint32_t asph = 0;
     int ui_par = 0;
+    bool waited = false;
     // MOE_DEBUG_TRACE: per-CTA timeline (globaltimer ns) into p.trace[8 + 8 * cta ..] (timing experiments)
     unsigned long long *tr = (p.trace && warp == 2 && lane == 0) ? p.trace + 8 + 8 * blockIdx.x : nullptr;
     if (tr) {
@@ -335,53 +349,108 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
       tr[7] = smid;
     }
-    pdl_wait();
-    if (tr) tr[1] = gtimer();                                  // routing results (tokens, weights) of the route kernel
+    // activation scales [kb][token] of a layer into shared memory (FP8; tokens >= T read 0)
+    auto load_xs = [&](const float *xs, float *dst) {
+      for (int i = et; i < KA * FD_N; i += 128) {
+        const int kb = i / FD_N, t = i % FD_N;
+        dst[i] = t < p.T ? xs[(size_t)t * KA + kb] : 0.f;
+      }
+    };
+    if (FP8 && p.has_prev) load_xs(p.g[2].xs, xs_s + FD_MAX_KB * FD_N);   // previous layer: complete
+    asm volatile("bar.sync 3, 128;" ::: "memory");
     for (;;) {
       mbar_wait(&uq_full[qs], qph);
       const int4 uq = unit_q[qs];
       __syncwarp();
       if (lane == 0) mbar_arrive(&uq_empty[qs]);
       if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
-      if (!(uq.w >> 1)) break;
-      const int group = uq.w & 1, expert = uq.x, row0 = uq.y, n = uq.z & 0xFFFF, chunk = uq.z >> 16;
-      // lane t < n: token t -> destination row of the fp32 sums and its weight (routed:
-      // only if the token chose this expert; canonical slot i >= n_imm -> deferred sum)
+      if (!uq.w) break;
+      const int expert = uq.x, chunk = uq.y, group = uq.z;
+      if (group != 2 && !waited) {
+        pdl_wait();                              // this layer's routing results and activation scales
+        if (tr) tr[1] = gtimer();
+        if (FP8) load_xs(p.g[0].xs, xs_s);
+        asm volatile("bar.sync 3, 128;" ::: "memory");
+        waited = true;
+      }
+      const FdGroup &g = p.g[group];
+      const float *xsg = xs_s + (group == 2 ? FD_MAX_KB * FD_N : 0);
+      // lane t < T: token t -> destination row of the fp32 sums and its weight.
+      // Routed groups: only if the token chose this expert, in a canonical slot of
+      // [a0, a1) (-> acc_imm) or [a1, a2) (-> acc_def); shared: every token.
       float *dst_j = nullptr;
       float w_j = 0.f;
-      if (lane < n) {
-        if (group) {
+      if (lane < p.T) {
+        if (group == 1) {
           dst_j = p.acc_imm + (size_t)lane * p.H;
           w_j = p.sgate ? p.sgate[lane] : 1.f;
         } else {
-          const int ge = expert + p.e0;
+          const int ge = expert + g.e0;
           int hit = -1;
-          for (int i = 0; i < p.k; ++i) hit = (hit < 0 && p.topk_idx[lane * p.k + i] == ge) ? i : hit;
-          if (hit >= 0) {
-            w_j = p.topk_w[lane * p.k + hit];
-            dst_j = (hit < p.n_imm ? p.acc_imm : p.acc_def) + (size_t)lane * p.H;
+          for (int i = 0; i < g.k; ++i) hit = (hit < 0 && g.topk_idx[lane * g.k + i] == ge) ? i : hit;
+          if (hit >= g.a0 && hit < g.a2) {
+            w_j = g.topk_w[lane * g.k + hit];
+            dst_j = (hit < g.a1 ? p.acc_imm : p.acc_def) + (size_t)lane * p.H;
           }
         }
       }
       const unsigned tmask = __ballot_sync(0xffffffffu, dst_j != nullptr);
-      (void)row0;
-      // ---- phase A epilogue: SwiGLU + requant -> h_c (B operand of phase B) ----
+      // ---- phase A epilogue: fp32 gate/up accumulators of this lane's two weight rows ----
       if (tr) { tr[2] = gtimer(); tr[6] = (unsigned long long)(group << 30 | expert << 16 | chunk); }
-      mbar_wait(accA_full, aph);
+      float r0[FD_N], r1[FD_N];
+      if constexpr (FP8) {
+        // 128x128 weight-block scales of this warp's rows (gate or up rows of h block
+        // `chunk`, interleaved per 128 rows: row block 2 chunk + (q & 1)), all k-blocks
+        const float *ws = g.w13_s + ((size_t)expert * 2 * g.nch + 2 * chunk + (q & 1)) * KA;
+        const float swa = lane < KA ? ws[lane] : 0.f, swb = lane + 32 < KA ? ws[lane + 32] : 0.f;
+#pragma unroll
+        for (int t = 0; t < FD_N; ++t) r0[t] = r1[t] = 0.f;
+        for (int kb = 0; kb < KA; ++kb) {
+          mbar_wait(&accA_full[as], asph);
+          tc_fence_after();
+          uint32_t v0[16], v1[16];
+          tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCA_COL + as * 32, v0);
+          tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCA_COL + as * 32 + 16, v1);
+          tmem_ld_wait();
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&accA_empty[as]);
+          if (++as == FD_ACCA_SLOTS) { as = 0; asph ^= 1; }
+          const float sw = __shfl_sync(0xffffffffu, kb < 32 ? swa : swb, kb & 31);
+          const float4 *xs4 = reinterpret_cast<const float4 *>(xsg + kb * FD_N);
+#pragma unroll
+          for (int t4 = 0; t4 < FD_N / 4; ++t4) {
+            const float4 x4 = xs4[t4];
+            const float sx[4] = {x4.x, x4.y, x4.z, x4.w};
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const int t = 4 * t4 + j;
+              const float s = sw * sx[j];
+              r0[t] = fmaf(__uint_as_float(v0[t]), s, r0[t]);
+              r1[t] = fmaf(__uint_as_float(v1[t]), s, r1[t]);
+            }
+          }
+        }
+      } else {
+        mbar_wait(&accA_full[0], aph);
+        aph ^= 1;
+        tc_fence_after();
+        uint32_t v0[16], v1[16];
+        tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCA_COL, v0);
+        tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCA_COL + 16, v1);
+        tmem_ld_wait();
+        tc_fence_before();
+#pragma unroll
+        for (int t = 0; t < FD_N; ++t) { r0[t] = __uint_as_float(v0[t]); r1[t] = __uint_as_float(v1[t]); }
+      }
       if (tr) tr[3] = gtimer();
-      aph ^= 1;
-      tc_fence_after();
-      uint32_t r0[16], r1[16];
-      tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCA, r0);
-      tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCA + 16, r1);
-      tmem_ld_wait();
-      tc_fence_before();
+      // ---- SwiGLU + requant -> h_c (B operand of phase B) ----
       float *xb = xch + qg * (2 * FD_N * 32);
       if (q & 1) {
 #pragma unroll
         for (int t = 0; t < FD_N; ++t) {
-          xb[t * 32 + lane] = __uint_as_float(r0[t]);
-          xb[(FD_N + t) * 32 + lane] = __uint_as_float(r1[t]);
+          xb[t * 32 + lane] = r0[t];
+          xb[(FD_N + t) * 32 + lane] = r1[t];
         }
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
@@ -390,8 +459,8 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         float h0[FD_N], h1[FD_N];
 #pragma unroll
         for (int t = 0; t < FD_N; ++t) {
-          h0[t] = t < n ? silu_f(__uint_as_float(r0[t])) * xb[t * 32 + lane] : 0.f;
-          h1[t] = t < n ? silu_f(__uint_as_float(r1[t])) * xb[(FD_N + t) * 32 + lane] : 0.f;
+          h0[t] = t < p.T ? silu_f(r0[t]) * xb[t * 32 + lane] : 0.f;
+          h1[t] = t < p.T ? silu_f(r1[t]) * xb[(FD_N + t) * 32 + lane] : 0.f;
         }
         if (FP8) {
 #pragma unroll
@@ -425,15 +494,13 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       if (q == 0 && lane == 0) mbar_arrive(h_ready);
       if (tr) tr[4] = gtimer();
       // ---- phase B epilogue: scaled, weighted partial sums of W2 row tiles ----
-      const FdGroup &g = p.g[group];
-      const int nchg = p.nch[group];
       // the unit's W2 block scales (H/128 <= 64 row blocks) into registers up front:
       // a global load per tile would put HBM latency on the epilogue's critical path
       float s2a = 1.f, s2b = 1.f;
       if (FP8) {
-        const float *w2s = g.w2_s + (size_t)expert * (p.H / 128) * nchg + chunk;
-        if (lane < p.H / 128) s2a = w2s[(size_t)lane * nchg];
-        if (lane + 32 < p.H / 128) s2b = w2s[(size_t)(lane + 32) * nchg];
+        const float *w2s = g.w2_s + (size_t)expert * (p.H / 128) * g.nch + chunk;
+        if (lane < p.H / 128) s2a = w2s[(size_t)lane * g.nch];
+        if (lane + 32 < p.H / 128) s2b = w2s[(size_t)(lane + 32) * g.nch];
       }
       for (int nt = 0; nt < NT; ++nt) {
         mbar_wait(&accB_full[ab], abph);
@@ -467,6 +534,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       ui_par ^= 1;
       if (tr) tr[5] = gtimer();
     }
+    if (!waited) pdl_wait();                     // (a CTA that only saw group-2 units: nothing left to read)
   }
   // only now may the finalize kernel launch: its CTAs wait in griddepcontrol.wait, which
   // takes issue slots from a co-resident CTA still streaming (measured: a 2.4 us SwiGLU
@@ -475,12 +543,10 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   tc_fence_before();
   __syncthreads();
   if (warp == 1) tmem_dealloc(tmem, FD_TMEM_COLS);
-  __shared__ int last_cta;
   if (threadIdx.x == 0) {
     // the last CTA out re-arms the work counter for the next forward (graph replay)
     asm volatile("fence.acq_rel.gpu;" ::: "memory");
-    last_cta = atomicAdd(p.done, 1) == (int)gridDim.x - 1;
-    if (last_cta) {
+    if (atomicAdd(p.done, 1) == (int)gridDim.x - 1) {
       asm volatile("fence.acq_rel.gpu;" ::: "memory");
       atomicExch(p.sched, 0);
       atomicExch(p.done, 0);

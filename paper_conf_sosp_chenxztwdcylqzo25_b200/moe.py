@@ -23,8 +23,9 @@ GROUP_MAX, GROUP_TOP2_SUM = 0, 1
 W_BF16, W_FP8, W_F32 = 0, 1, 2
 
 EXPORTED = ["moe_ep_group_forward", "moe_get_unique_id", "moe_layer_create", "moe_layer_forward", "moe_layer_forward_deferred",
-            "moe_layer_destroy", "moe_status_string", "moe_last_error", "moe_layer_get_info",
-            "moe_layer_profile", "moe_layer_stage_times", "moe_stage_name", "moe_layer_set_decode_tp"]
+            "moe_layer_forward_chained", "moe_tp_group_forward", "moe_layer_destroy", "moe_status_string",
+            "moe_last_error", "moe_layer_get_info", "moe_layer_profile", "moe_layer_stage_times", "moe_stage_name",
+            "moe_layer_debug_trace"]
 
 
 class MoEConfig(ctypes.Structure):
@@ -34,7 +35,8 @@ class MoEConfig(ctypes.Structure):
                 ("routed_scale", ctypes.c_float), ("shared_ffn", ctypes.c_int32),
                 ("shared_gated", ctypes.c_int32), ("wtype", ctypes.c_int32), ("max_tokens", ctypes.c_int32),
                 ("gemv_max_tokens", ctypes.c_int32), ("device", ctypes.c_int32), ("ep_rank", ctypes.c_int32),
-                ("ep_size", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p)]
+                ("ep_size", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p), ("tp_rank", ctypes.c_int32),
+                ("tp_size", ctypes.c_int32)]
 
 
 class MoEWeights(ctypes.Structure):
@@ -70,6 +72,10 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.moe_layer_create.argtypes = [ctypes.POINTER(MoEConfig), ctypes.POINTER(MoEWeights), ctypes.POINTER(vp)]
     lib.moe_layer_forward.argtypes = [vp, vp, vp, i32, vp, ctypes.POINTER(MoERouting), vp]
     lib.moe_layer_forward_deferred.argtypes = [vp, vp, vp, i32, i32, vp, vp, vp, ctypes.POINTER(MoERouting), vp]
+    lib.moe_layer_forward_chained.argtypes = [vp, vp, vp, i32, i32, vp, vp, vp]
+    lib.moe_tp_group_forward.argtypes = [ctypes.POINTER(vp), i32, ctypes.POINTER(vp), ctypes.POINTER(vp), i32, i32,
+                                         ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(vp), vp]
+    lib.moe_layer_debug_trace.argtypes = [vp, vp, i32]
     lib.moe_layer_destroy.argtypes = [vp]
     lib.moe_status_string.argtypes = [i32]
     lib.moe_status_string.restype = ctypes.c_char_p
@@ -80,13 +86,12 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
                                          ctypes.POINTER(vp), vp]
     lib.moe_ep_group_forward.restype = i32
     lib.moe_layer_profile.argtypes = [vp, i32]
-    lib.moe_layer_set_decode_tp.argtypes = [vp, i32, i32]
     lib.moe_layer_stage_times.argtypes = [vp, ctypes.POINTER(ctypes.c_float), i32, ctypes.POINTER(i32)]
     lib.moe_stage_name.argtypes = [i32]
     lib.moe_stage_name.restype = ctypes.c_char_p
     for f in ("moe_get_unique_id", "moe_layer_create", "moe_layer_forward", "moe_layer_forward_deferred",
-              "moe_layer_destroy", "moe_layer_get_info", "moe_layer_profile", "moe_layer_stage_times",
-              "moe_layer_set_decode_tp"):
+              "moe_layer_forward_chained", "moe_tp_group_forward", "moe_layer_destroy", "moe_layer_get_info",
+              "moe_layer_profile", "moe_layer_stage_times", "moe_layer_debug_trace"):
         getattr(lib, f).restype = i32
     _lib = lib
     return lib
@@ -122,7 +127,8 @@ class MoELayer:
     """One MoE layer handle (moe_layer_create / _forward / _forward_deferred / _destroy)."""
 
     def __init__(self, preset, weights, max_tokens: int, device: int = 0, gemv_max_tokens: int = 0,
-                 ep_rank: int = 0, ep_size: int = 1, unique_id: Optional[bytes] = None):
+                 ep_rank: int = 0, ep_size: int = 1, unique_id: Optional[bytes] = None, tp_rank: int = 0,
+                 tp_size: int = 1):
         lib = load_library()
         self.p = preset
         self.max_tokens = max_tokens
@@ -135,7 +141,9 @@ class MoELayer:
                         routed_scale=preset.routed_scale, shared_ffn=preset.shared_ffn,
                         shared_gated=int(preset.shared_gated), wtype=preset.wtype, max_tokens=max_tokens,
                         gemv_max_tokens=gemv_max_tokens, device=device, ep_rank=ep_rank, ep_size=ep_size,
-                        nccl_unique_id=ctypes.cast(self._uid, ctypes.c_void_p) if self._uid else None)
+                        nccl_unique_id=ctypes.cast(self._uid, ctypes.c_void_p) if self._uid else None,
+                        tp_rank=tp_rank, tp_size=tp_size)
+        self.tp_size = tp_size
         w = MoEWeights(**{n: _ptr(getattr(weights, n)) for n, _ in MoEWeights._fields_})
         h = ctypes.c_void_p()
         with torch.cuda.device(device):
@@ -150,11 +158,6 @@ class MoELayer:
 
     def profile(self, enable: bool = True):
         _check(self._lib.moe_layer_profile(self._h, int(enable)), "moe_layer_profile")
-
-    def set_decode_tp(self, rank: int, size: int):
-        """Decode TP within every expert (include/moe.h moe_layer_set_decode_tp):
-        forwards then return this rank's partial y; the caller sums over ranks."""
-        _check(self._lib.moe_layer_set_decode_tp(self._h, int(rank), int(size)), "moe_layer_set_decode_tp")
 
     def stage_times(self) -> dict:
         """Per-stage ms of the last profiled forward (waits for it)."""
@@ -196,6 +199,27 @@ class MoELayer:
         _check(s, "moe_layer_forward_deferred")
         return (y, deferred_out) if deferred_out is not None else y
 
+    def forward_chained(self, x: torch.Tensor, residual: Optional[torch.Tensor] = None, n_deferred: int = 0,
+                        prev: Optional["MoELayer"] = None, y: Optional[torch.Tensor] = None,
+                        stream: Optional[torch.cuda.Stream] = None) -> torch.Tensor:
+        """Expert Deferral across layers (include/moe.h moe_layer_forward_chained,
+        PAPER.md L241): this layer's last n_deferred slots are left for the next
+        layer; `prev`'s deferred slots are computed here and added to y."""
+        assert x.dtype == torch.bfloat16 and x.dim() == 2 and x.shape[1] == self.p.hidden
+        if y is None:
+            y = torch.empty_like(x)
+        st = (stream or torch.cuda.current_stream(x.device)).cuda_stream
+        s = self._lib.moe_layer_forward_chained(self._h, _ptr(x), _ptr(residual), x.shape[0], n_deferred,
+                                                prev._h if prev is not None else None, _ptr(y), st)
+        _check(s, "moe_layer_forward_chained")
+        return y
+
+    def debug_trace(self, n: int = 4096):
+        import numpy as np
+        buf = np.zeros(n, dtype=np.uint64)
+        _check(self._lib.moe_layer_debug_trace(self._h, buf.ctypes.data, n), "moe_layer_debug_trace")
+        return buf
+
     def close(self):
         if getattr(self, "_h", None):
             self._lib.moe_layer_destroy(self._h)
@@ -224,12 +248,70 @@ def slice_experts(weights, rank: int, ep_size: int):
     return w
 
 
-class MoEGroup:
-    """In-process expert-parallel group (moe_ep_group_forward): P ranks, one
-    MoELayer each, owning E/P experts; devices[r] is rank r's GPU."""
+def slice_tp(weights, rank: int, tp_size: int, ffn: int, shared_ffn: int):
+    """Rank `rank`'s slice for expert tensor parallelism (include/moe.h "Tensor
+    parallelism"): 128-column chunks [r n / P, (r+1) n / P) of every expert's FFN
+    dimension -- W1 and W3 rows, W2 columns, and their 128x128 block scales."""
+    import copy
 
-    def __init__(self, preset, weights, ep_size: int, max_tokens: int, devices=None):
-        devices = devices or [0] * ep_size
+    def cols(full):
+        n = full // 128
+        return (rank * n // tp_size) * 128, ((rank + 1) * n // tp_size) * 128
+
+    w = copy.copy(weights)
+    c0, c1 = cols(ffn)
+    w.w13 = torch.cat([weights.w13[:, c0:c1], weights.w13[:, ffn + c0:ffn + c1]], dim=1).contiguous()
+    w.w2 = weights.w2[:, :, c0:c1].contiguous()
+    if weights.w13_scale is not None:
+        b0, b1, fb = c0 // 128, c1 // 128, ffn // 128
+        w.w13_scale = torch.cat([weights.w13_scale[:, b0:b1], weights.w13_scale[:, fb + b0:fb + b1]], dim=1).contiguous()
+        w.w2_scale = weights.w2_scale[:, :, b0:b1].contiguous()
+    if shared_ffn and weights.ws13 is not None:
+        s0, s1 = cols(shared_ffn)
+        w.ws13 = torch.cat([weights.ws13[s0:s1], weights.ws13[shared_ffn + s0:shared_ffn + s1]], dim=0).contiguous()
+        w.ws2 = weights.ws2[:, s0:s1].contiguous()
+        if weights.ws13_scale is not None:
+            b0, b1, fb = s0 // 128, s1 // 128, shared_ffn // 128
+            w.ws13_scale = torch.cat([weights.ws13_scale[b0:b1], weights.ws13_scale[fb + b0:fb + b1]],
+                                     dim=0).contiguous()
+            w.ws2_scale = weights.ws2_scale[:, b0:b1].contiguous()
+    return w
+
+
+class TPGroup:
+    """In-process expert-TP group on one GPU (moe_tp_group_forward): P ranks, each
+    holding its 1/P slice of every expert; a forward returns every rank's full y."""
+
+    def __init__(self, preset, weights, tp_size: int, max_tokens: int, device: int = 0):
+        self.P = tp_size
+        self.layers = [MoELayer(preset, slice_tp(weights, r, tp_size, preset.ffn, preset.shared_ffn),
+                                max_tokens=max_tokens, device=device, tp_rank=r, tp_size=tp_size)
+                       for r in range(tp_size)]
+        self._lib = load_library()
+
+    def forward(self, xs, residuals=None, n_deferred=0, deferred_in=None, want_deferred_out=False, stream=None):
+        P = self.P
+        vp = ctypes.c_void_p
+        arr = lambda ts: (vp * P)(*[None if t is None else _ptr(t) for t in ts]) if ts is not None else None
+        ys = [torch.empty_like(x) for x in xs]
+        douts = [torch.empty_like(x) for x in xs] if want_deferred_out else None
+        st = (stream or torch.cuda.current_stream(xs[0].device)).cuda_stream
+        s = self._lib.moe_tp_group_forward((vp * P)(*[l._h.value for l in self.layers]), P, arr(xs), arr(residuals),
+                                           xs[0].shape[0], n_deferred, arr(deferred_in), arr(ys), arr(douts), st)
+        _check(s, "moe_tp_group_forward")
+        return (ys, douts) if want_deferred_out else ys
+
+    def close(self):
+        for l in self.layers:
+            l.close()
+
+
+class MoEGroup:
+    """In-process expert-parallel group on one GPU (moe_ep_group_forward): P ranks,
+    one MoELayer each, owning E/P experts (the NCCL transport runs one process per GPU)."""
+
+    def __init__(self, preset, weights, ep_size: int, max_tokens: int, device: int = 0):
+        devices = [device] * ep_size
         self.P = ep_size
         self.layers = []
         for r in range(ep_size):
@@ -256,13 +338,3 @@ class MoEGroup:
     def close(self):
         for l in self.layers:
             l.close()
-
-
-def decode_tp_forward(layer: "MoELayer", x: torch.Tensor, residual: Optional[torch.Tensor] = None, group=None):
-    """One decode forward of a layer set up with set_decode_tp(rank, P) on each
-    of P processes: this rank's partial y (its 128-column chunks of every
-    expert), summed over the group with one all-reduce."""
-    import torch.distributed as dist
-    y = layer.forward(x, residual)
-    dist.all_reduce(y, group=group)
-    return y

@@ -14,21 +14,27 @@ p = PRESETS[cfg]
 w = make_weights(p, "cuda")
 x, _ = make_tokens(p, T, "cuda", offset=5)
 NL = int(sys.argv[3]) if len(sys.argv) > 3 else 1     # >1: trace the middle layer of a chained graph
+TP = int(sys.argv[4]) if len(sys.argv) > 4 else 1     # >1: expert TP, rank 0's slice as a layer of its own
+NDEF = int(sys.argv[5]) if len(sys.argv) > 5 else 0   # >0: chained Expert Deferral (moe_layer_forward_chained)
+if TP > 1:
+    w = moe.slice_tp(w, 0, TP, p.ffn, p.shared_ffn)
+    p = p.with_(ffn=w.w2.shape[2], shared_ffn=w.ws2.shape[1] if p.shared_ffn else 0)
 layers = [moe.MoELayer(p, w, max_tokens=16) for _ in range(NL)]
 layer = layers[NL // 2]
-TP = int(sys.argv[4]) if len(sys.argv) > 4 else 1     # >1: decode TP, rank 0's share (moe_layer_set_decode_tp)
-for l in layers:
-    l.set_decode_tp(0, TP)
 lib = layer._lib
-lib.moe_layer_debug_trace.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32]
 buf = np.zeros(4096, dtype=np.uint64)
 y = torch.empty_like(x)
 fw = torch.empty(64 << 20, device="cuda"); fr = torch.zeros(64 << 20, device="cuda"); sink = torch.zeros((), device="cuda")
 bufs = [x.clone(), torch.empty_like(x)]
 def step():
+    prev = None
     for i, l in enumerate(layers):
         a, b = bufs[i % 2], bufs[(i + 1) % 2]
-        l.forward(a, residual=a, y=b)
+        if NDEF:
+            l.forward_chained(a, residual=a, n_deferred=NDEF if i < len(layers) - 1 else 0, prev=prev, y=b)
+            prev = l
+        else:
+            l.forward(a, residual=a, y=b)
 if NL > 1:
     s_ = torch.cuda.Stream(); s_.wait_stream(torch.cuda.current_stream())
     with torch.cuda.stream(s_):

@@ -302,77 +302,3 @@ def test_fused_decode_repeats(lib, name):
     assert d <= 2 ** -6 * max(1.0, ya.abs().max().item()), d
     fused.close()
     gemm.close()
-
-
-def _tp_sum(lib, layer, x, r, P, n_def=0, din=None):
-    """Sum of the P decode-TP partial outputs of one layer (moe_layer_set_decode_tp),
-    fp32, i.e. what the all-reduce over P GPUs returns (before its bf16 cast)."""
-    y = d = 0
-    for rk in range(P):
-        layer.set_decode_tp(rk, P)
-        out = layer.forward(x, residual=r, n_deferred=n_def, deferred_in=din, want_deferred_out=n_def > 0)
-        yo, do = out if isinstance(out, tuple) else (out, None)
-        y = y + yo.float()
-        if do is not None:
-            d = d + do.float()
-    layer.set_decode_tp(0, 1)
-    torch.cuda.synchronize()
-    return y, d
-
-
-@pytest.mark.parametrize("name,P", [("v3_s", 2), ("qwen2_s", 2), ("v25_s", 2), ("v2lite_s", 2), ("v2lite_s", 3)])
-@pytest.mark.parametrize("T", [1, 6, 16])
-def test_decode_tp_partials_sum_to_oracle(lib, name, P, T):
-    """Decode TP within every expert:
-    rank r streams the 128-column chunks c = r (mod P) of every expert; the sum of
-    the P partial outputs (residual, deferred_in on rank 0) is the layer's output
-    (Eq. L241 with deferral).  v2lite_s at P = 2 gives ranks 2 and 1 routed chunks
-    (F/128 = 3): a ragged split."""
-    p = SMALL[name]
-    n_def = min(2, p.top_k - 1)
-    w_cpu = make_weights(p, "cpu")
-    x_cpu, r_cpu = make_tokens(p, T, "cpu", offset=11)
-    layer = lib.MoELayer(p, w_cpu.to("cuda"), max_tokens=16)
-    din = (torch.randn(T, p.hidden, generator=torch.Generator().manual_seed(7)) * 0.5).to(torch.bfloat16)
-    routing = {}
-    layer.forward(x_cpu.cuda(), routing=routing)       # this layer's routing, for the oracle's tie band
-    y, d = _tp_sum(lib, layer, x_cpu.cuda(), r_cpu.cuda(), P, n_def=n_def, din=din.cuda())
-    res = dict(w_cpu=w_cpu, x=x_cpu, r=r_cpu, din=din, routing={k: v.cpu().numpy() for k, v in routing.items()})
-    out, ties, idx, w = _oracle(p, res, n_def=n_def, residual=True)
-    keep = np.setdiff1d(np.arange(T), ties)
-    assert rel_l2(y.cpu().numpy()[keep], out["y"][keep]) <= TOL[p.wtype]
-    assert rel_l2(d.cpu().numpy()[keep], out["deferred_out"][keep]) <= TOL[p.wtype]
-    layer.close()
-
-
-def test_decode_tp_errors(lib):
-    p = SMALL["v3_s"]                                 # F/128 = Fs/128 = 2
-    layer = lib.MoELayer(p, make_weights(p, "cpu").to("cuda"), max_tokens=64)
-    for rk, P in [(0, 3), (2, 2), (-1, 2), (0, 0)]:
-        with pytest.raises(lib.MoEError):
-            layer.set_decode_tp(rk, P)
-    layer.set_decode_tp(1, 2)
-    x, r = make_tokens(p, 40, "cuda")                 # above the fused decode limit: refused, not silently whole
-    with pytest.raises(lib.MoEError):
-        layer.forward(x, residual=r)
-    layer.set_decode_tp(0, 1)
-    layer.forward(x, residual=r)
-    torch.cuda.synchronize()
-    layer.close()
-
-
-@pytest.mark.parametrize("name,Ps", [("v3", (2, 4, 8, 16)), ("v25", (5, 8, 12)), ("qwen2", (3, 8, 20))])
-def test_full_decode_tp_matches_whole(lib, name, Ps):
-    """Full-size layers, T = 1 and 4: the P partials sum to the single-GPU forward up
-    to the bf16 rounding of each partial.  V3: F/128 = Fs/128 = 16 chunks; V2.5: 12 routed
-    chunks (P = 5, 8 give ranks 2-3 or 1-2 chunks: ragged); Qwen2 (BF16, gated shared
-    expert): 20 routed and 160 shared chunks."""
-    p = PRESETS[name]
-    layer = lib.MoELayer(p, make_weights(p, "cuda"), max_tokens=16)
-    for P in Ps:
-        for T in (1, 4):
-            x, r = make_tokens(p, T, "cuda", offset=P)
-            whole = layer.forward(x, residual=r).float()
-            y, _ = _tp_sum(lib, layer, x, r, P)
-            assert rel_l2(y.cpu().numpy(), whole.cpu().numpy()) <= TOL[p.wtype], (P, T)
-    layer.close()

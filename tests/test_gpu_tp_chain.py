@@ -1,0 +1,221 @@
+"""GPU parity of the two §8(f) rows built on the fused decode stream, through the C ABI:
+  * expert tensor parallelism (NEXT-1; Fig. 8b): P ranks each
+    holding 1/P of every expert (moe.slice_tp), partials summed in fp32
+    (moe_tp_group_forward, the in-process stand-in of the NCCL all-reduce);
+  * Expert Deferral chained across layers (NEXT-2; Eq. 2):
+    moe_layer_forward_chained, layer k computes layer k-1's deferred experts.
+Both against the fp64 oracle (oracle/) on the same seeded inputs."""
+import numpy as np
+import pytest
+import torch
+
+from inputs.presets import PRESETS, SMALL
+from inputs.synthetic import make_tokens, make_weights
+from oracle import moe_oracle as O
+from tests.parity import (TOL, check_output, check_tie_fraction, merged_routing, oracle_cfg, oracle_weights)
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lib():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_sosp_chenxztwdcylqzo25_b200 import moe
+    return moe
+
+
+def _din(T, H, seed=7):
+    return (torch.randn(T, H, generator=torch.Generator().manual_seed(seed)) * 0.5).to(torch.bfloat16)
+
+
+# ------------------------------------------------------------------ expert TP
+@pytest.mark.parametrize("name,P", [("v3_s", 2), ("qwen2_s", 2), ("v25_s", 2), ("v2lite_s", 2), ("v2lite_s", 3),
+                                    ("v3_m", 4), ("v3_m", 3)])
+@pytest.mark.parametrize("T", [1, 6, 16])
+def test_tp_group_matches_oracle(lib, name, P, T):
+    """Every rank's y (and deferred_out) equals the whole layer's (Eq. L241 middle
+    case: residual + deferred_in, n_def slots deferred).  v2lite_s (F/128 = 3) and
+    v3_m at P = 3 split the chunks raggedly."""
+    p = SMALL[name]
+    n_def = min(2, p.top_k - 1)
+    w_cpu = make_weights(p, "cpu")
+    x_cpu, r_cpu = make_tokens(p, T, "cpu", offset=11)
+    din = _din(T, p.hidden)
+    whole = lib.MoELayer(p, w_cpu.to("cuda"), max_tokens=16)
+    routing = {}
+    whole.forward(x_cpu.cuda(), routing=routing)            # routing, for the oracle's tie band
+    grp = lib.TPGroup(p, w_cpu.to("cuda"), P, max_tokens=16)
+    wb = [l.info().weight_bytes for l in grp.layers]
+    assert max(wb) < whole.info().weight_bytes * (1.0 / P + 0.34), (wb, whole.info().weight_bytes)
+    xs = [x_cpu.cuda()] * P
+    ys, ds = grp.forward(xs, residuals=[r_cpu.cuda()] * P, n_deferred=n_def, deferred_in=[din.cuda()] * P,
+                         want_deferred_out=True)
+    torch.cuda.synchronize()
+    cfg, W = oracle_cfg(p), oracle_weights(p, w_cpu)
+    x64 = x_cpu.to(torch.float64).numpy()
+    ties = O.tie_band_tokens(x64, W, cfg, n_deferred=n_def)
+    idx, wt = merged_routing(x64, W, cfg, routing["topk_idx"].cpu().numpy(), ties)
+    out = O.moe_layer(x64, W, cfg, residual=r_cpu.to(torch.float64).numpy(), n_deferred=n_def,
+                      deferred_in=din.to(torch.float64).numpy(), forced_routing=(idx, wt))
+    keep = np.setdiff1d(np.arange(T), ties)
+    for r in range(P):
+        check_output(f"tp/{name}/P{P}/T{T}/rank{r}/y", ys[r].float().cpu().numpy()[keep], out["y"][keep], TOL[p.wtype])
+        check_output(f"tp/{name}/P{P}/T{T}/rank{r}/deferred_out", ds[r].float().cpu().numpy()[keep],
+                     out["deferred_out"][keep], TOL[p.wtype])
+    # every rank holds the same sum
+    for r in range(1, P):
+        assert torch.equal(ys[r], ys[0])
+    grp.close()
+    whole.close()
+
+
+def test_tp_errors(lib):
+    p = SMALL["v3_s"]                                     # F/128 = Fs/128 = 2
+    w = make_weights(p, "cpu").to("cuda")
+    with pytest.raises(lib.MoEError):                     # more ranks than chunks
+        lib.MoELayer(p, lib.slice_tp(w, 0, 3, p.ffn, p.shared_ffn), max_tokens=16, tp_rank=0, tp_size=3)
+    with pytest.raises(lib.MoEError):                     # rank out of range
+        lib.MoELayer(p, w, max_tokens=16, tp_rank=2, tp_size=2)
+    grp = lib.TPGroup(p, w, 2, max_tokens=64)
+    x, r = make_tokens(p, 40, "cuda")                     # above the decode stream: refused, not silently partial
+    with pytest.raises(lib.MoEError) as e:
+        grp.forward([x, x], residuals=[r, r])
+    assert e.value.status == -2
+    with pytest.raises(lib.MoEError) as e:                # a rank of an in-process group alone: no silent partial
+        grp.layers[0].forward(x[:4].contiguous())
+    assert e.value.status == -1
+    grp.close()
+
+
+@pytest.mark.parametrize("name,Ps", [("v3", (2, 4, 8)), ("v25", (5, 8)), ("qwen2", (3, 8))])
+def test_full_tp_matches_whole(lib, name, Ps):
+    """Full-size layers, T = 1 and 4: the TP group's y equals the single-GPU
+    forward within the north_star tolerance; per-rank weight bytes ~ 1/P.  V2.5
+    (12 routed chunks) at P = 5 / 8 and Qwen2 at P = 3 are ragged splits."""
+    p = PRESETS[name]
+    w = make_weights(p, "cuda")
+    whole = lib.MoELayer(p, w, max_tokens=16)
+    wb_whole = whole.info().weight_bytes
+    for P in Ps:
+        grp = lib.TPGroup(p, w, P, max_tokens=16)
+        assert max(l.info().weight_bytes for l in grp.layers) < wb_whole * (1.0 / P + 0.1)
+        for T in (1, 4):
+            x, r = make_tokens(p, T, "cuda", offset=P)
+            ref = whole.forward(x, residual=r).float()
+            ys = grp.forward([x] * P, residuals=[r] * P)
+            check_output(f"tp_full/{name}/P{P}/T{T}", ys[0].float().cpu().numpy(), ref.cpu().numpy(), TOL[p.wtype])
+        grp.close()
+        torch.cuda.empty_cache()
+    whole.close()
+
+
+# ------------------------------------------------------------------ chained Expert Deferral
+def _chain_oracle(p, ws, xs, rs, n_defs):
+    """Eq. L241 over a chain of layers: O_k = I_k + S_k + R^def_{k-1}(I_{k-1}) + R^imm_k(I_k)
+    with the k = 1 (no deferred_in) and k = L (n_def = 0) cases; layer k's input is the
+    GPU's x_k (so every layer is checked on identical inputs)."""
+    cfg = oracle_cfg(p)
+    outs, din, ties = [], None, set()
+    for k, (w, x, r, nd) in enumerate(zip(ws, xs, rs, n_defs)):
+        W = oracle_weights(p, w)
+        x64 = x.cpu().to(torch.float64).numpy()
+        t = O.tie_band_tokens(x64, W, cfg, n_deferred=nd)
+        ties |= set(t.tolist())
+        o = O.moe_layer(x64, W, cfg, residual=r.cpu().to(torch.float64).numpy(), n_deferred=nd, deferred_in=din)
+        outs.append(o["y"])
+        din = o["deferred_out"]
+    return outs, sorted(ties)
+
+
+@pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v2lite_s", "v3_m", "v25_s"])
+@pytest.mark.parametrize("T", [1, 5, 16])
+def test_chained_deferral_matches_eq_L241(lib, name, T):
+    p = SMALL[name]
+    n_def = min(3, p.top_k - 1)
+    L = 3
+    ws = [make_weights(p, "cpu", seed=4000 + 17 * i) for i in range(L)]
+    layers = [lib.MoELayer(p, w.to("cuda"), max_tokens=16) for w in ws]
+    x0, _ = make_tokens(p, T, "cuda", offset=21)
+    xs, rs, ys = [x0], [], []
+    prev = None
+    for i, l in enumerate(layers):
+        nd = n_def if i < L - 1 else 0                   # k = L: all experts immediate (L215)
+        r = xs[-1]                                      # I_k of Eq. L241
+        y = l.forward_chained(xs[-1], residual=r, n_deferred=nd, prev=prev)
+        rs.append(r)
+        ys.append(y)
+        xs.append(y)
+        prev = l
+    torch.cuda.synchronize()
+    outs, ties = _chain_oracle(p, ws, xs[:L], rs, [n_def] * (L - 1) + [0])
+    check_tie_fraction(ties, T * L)
+    keep = np.setdiff1d(np.arange(T), ties)
+    for i in range(L):
+        # the deferred part only: compare y - residual (the residual would dilute the error)
+        got = ys[i].float().cpu().numpy() - rs[i].float().cpu().numpy()
+        want = outs[i] - rs[i].cpu().to(torch.float64).numpy()
+        check_output(f"chain/{name}/T{T}/layer{i}", got[keep], want[keep], TOL[p.wtype])
+    for l in layers:
+        l.close()
+
+
+def test_chained_without_deferral_is_the_plain_forward(lib):
+    p = SMALL["v3_s"]
+    w = make_weights(p, "cpu").to("cuda")
+    a = lib.MoELayer(p, w, max_tokens=16)
+    x, r = make_tokens(p, 5, "cuda")
+    y1 = a.forward(x, residual=r).float()
+    y2 = a.forward_chained(x, residual=r, n_deferred=0).float()
+    torch.cuda.synchronize()
+    assert (y1 - y2).abs().max().item() <= 2 ** -6 * max(1.0, y1.abs().max().item())
+    a.close()
+
+
+def test_chained_errors(lib):
+    p = SMALL["v3_s"]
+    a = lib.MoELayer(p, make_weights(p, "cpu").to("cuda"), max_tokens=64)
+    b = lib.MoELayer(p, make_weights(p, "cpu", seed=77).to("cuda"), max_tokens=64)
+    x, r = make_tokens(p, 4, "cuda")
+    with pytest.raises(lib.MoEError):                     # b's last call was not a chained deferral
+        a.forward_chained(x, residual=r, n_deferred=2, prev=b)
+    y = b.forward_chained(x, residual=r, n_deferred=2)
+    with pytest.raises(lib.MoEError):                     # prev is this layer
+        b.forward_chained(y, residual=y, n_deferred=2, prev=b)
+    with pytest.raises(lib.MoEError):                     # other T
+        a.forward_chained(y[:3].contiguous(), residual=y[:3].contiguous(), n_deferred=0, prev=b)
+    a.forward_chained(y, residual=y, n_deferred=0, prev=b)
+    with pytest.raises(lib.MoEError):                     # consumed once only
+        a.forward_chained(y, residual=y, n_deferred=0, prev=b)
+    x40, r40 = make_tokens(p, 40, "cuda")
+    with pytest.raises(lib.MoEError) as e:                # prefill-size T: decode path only (L245)
+        a.forward_chained(x40, residual=r40, n_deferred=2)
+    assert e.value.status == -2
+    torch.cuda.synchronize()
+    a.close()
+    b.close()
+
+
+def test_full_v3_chain_decode(lib):
+    """Full DeepSeek-V3 layers (FP8, 256 experts, n_def = 3, BF16 setting L257),
+    a 3-layer chain at T = 1 vs the Eq. L241 oracle chain."""
+    p = PRESETS["v3"]
+    L = 3
+    ws = [make_weights(p, "cuda", seed=5000 + i) for i in range(L)]
+    layers = [lib.MoELayer(p, w, max_tokens=16) for w in ws]
+    x0, _ = make_tokens(p, 1, "cuda", offset=5)
+    xs, ys, prev = [x0], [], None
+    for i, l in enumerate(layers):
+        y = l.forward_chained(xs[-1], residual=xs[-1], n_deferred=3 if i < L - 1 else 0, prev=prev)
+        ys.append(y)
+        xs.append(y)
+        prev = l
+    torch.cuda.synchronize()
+    outs, ties = _chain_oracle(p, ws, xs[:L], xs[:L], [3, 3, 0])
+    assert not ties
+    for i in range(L):
+        got = ys[i].float().cpu().numpy() - xs[i].float().cpu().numpy()
+        want = outs[i] - xs[i].cpu().to(torch.float64).numpy()
+        check_output(f"chain_full/v3/layer{i}", got, want, TOL[p.wtype])
+    for l in layers:
+        l.close()

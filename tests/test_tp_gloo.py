@@ -1,12 +1,16 @@
-"""Multi-process (gloo, world_size 2, CPU) check of the decode tensor-parallel
-decomposition behind moe_layer_set_decode_tp (PAPER.md
-L195-197): rank r evaluates only the FFN column chunks c = r (mod P) of every
-routed and shared expert -- W1/W3 rows and W2 columns of the same chunk, as the
-fused decode stream does -- adds the residual on rank 0 only, and
-`moe.decode_tp_forward` all-reduces the partials.  The sum must equal the
-single-process layer -- the oracle, not the CUDA library."""
+"""Multi-process (gloo, world_size 2, CPU) check of the expert tensor-parallel
+decomposition behind moe_layer_config.tp_rank / tp_size (include/moe.h "Tensor
+parallelism"): rank r holds only the
+128-column FFN chunks [r n / P, (r+1) n / P) of every routed and shared expert
+-- cut by the binding's own `moe.slice_tp`, W1/W3 rows and W2 columns of the
+same chunks; a ragged split here (3 chunks over 2 ranks) -- computes its partial
+expert sums, the partials are summed over the group (the library's NCCL
+all-reduce; gloo here), and every rank then adds the residual and deferred_in
+once.  Every rank's result must equal the single-process layer (PAPER.md L219 /
+L241) -- the oracle, not the CUDA library."""
 import os
 import socket
+from types import SimpleNamespace
 
 import numpy as np
 import torch
@@ -15,41 +19,28 @@ import torch.multiprocessing as mp
 
 from oracle import moe_oracle as O
 
-H, F, E, K, P, CH = 32, 24, 8, 3, 2, 4       # F / CH = 6 chunks; rank 0 takes 0,2,4, rank 1 takes 1,3,5
+H, F, FS, E, K, P, NDEF = 16, 384, 256, 4, 2, 2, 1
 
 
-def _layer(seed=0):
+def _weights(seed=0):
     rng = np.random.default_rng(seed)
-    Ws = [(rng.normal(size=(F, H)) / H ** .5, rng.normal(size=(F, H)) / H ** .5, rng.normal(size=(H, F)) / F ** .5)
-          for _ in range(E)]
-    Sh = (rng.normal(size=(F, H)) / H ** .5, rng.normal(size=(F, H)) / H ** .5, rng.normal(size=(H, F)) / F ** .5)
-    W = O.OracleWeights(rng.normal(size=(E, H)) / H ** .5, None, lambda e: Ws[e], lambda: Sh)
-    cfg = O.OracleConfig(hidden=H, ffn=F, n_experts=E, top_k=K, shared_ffn=F, norm_topk=True)
-    return W, cfg
+    return SimpleNamespace(
+        gate_w=torch.from_numpy(rng.normal(size=(E, H)) / H ** .5),
+        w13=torch.from_numpy(rng.normal(size=(E, 2 * F, H)) / H ** .5), w13_scale=None,
+        w2=torch.from_numpy(rng.normal(size=(E, H, F)) / F ** .5), w2_scale=None,
+        ws13=torch.from_numpy(rng.normal(size=(2 * FS, H)) / H ** .5), ws13_scale=None,
+        ws2=torch.from_numpy(rng.normal(size=(H, FS)) / FS ** .5), ws2_scale=None)
 
 
-class _ChunkLayer:
-    """Stands in for a MoELayer after set_decode_tp(rank, P): forward returns
-    this rank's partial output (its chunks of every expert)."""
+def _oracle_weights(w, f, fs):
+    n = lambda t: t.numpy()
+    return O.OracleWeights(n(w.gate_w), None,
+                           lambda e: (n(w.w13[e, :f]), n(w.w13[e, f:]), n(w.w2[e])),
+                           lambda: (n(w.ws13[:fs]), n(w.ws13[fs:]), n(w.ws2)))
 
-    def __init__(self, W, cfg, rank):
-        self.W, self.cfg, self.rank = W, cfg, rank
-        self.cols = np.concatenate([np.arange(c * CH, (c + 1) * CH) for c in range(F // CH) if c % P == rank])
 
-    def _ffn(self, x, w1, w3, w2):
-        c = self.cols
-        return O.swiglu_ffn(x, w1[c], w3[c], w2[:, c])
-
-    def forward(self, x, residual=None):
-        xn = x.numpy()
-        idx, w, _ = O.route(xn, self.W.gate_w, None, self.cfg)
-        y = self._ffn(xn, *self.W.shared())
-        for t in range(xn.shape[0]):
-            for j in range(K):
-                y[t] += w[t, j] * self._ffn(xn[t:t + 1], *self.W.expert(int(idx[t, j])))[0]
-        if self.rank == 0 and residual is not None:
-            y += residual.numpy()
-        return torch.from_numpy(y)
+def _cfg(f, fs):
+    return O.OracleConfig(hidden=H, ffn=f, n_experts=E, top_k=K, shared_ffn=fs, norm_topk=True)
 
 
 def _worker(rank, port, q):
@@ -57,16 +48,29 @@ def _worker(rank, port, q):
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=P)
     from paper_conf_sosp_chenxztwdcylqzo25_b200 import moe
-    W, cfg = _layer()
-    rng = np.random.default_rng(7)                  # replicated tokens: every rank sees the same batch
-    x, r = rng.normal(size=(5, H)), rng.normal(size=(5, H))
-    y = moe.decode_tp_forward(_ChunkLayer(W, cfg, rank), torch.from_numpy(x), torch.from_numpy(r))
-    ref = O.moe_layer(x, W, cfg, residual=r)["y"]
-    q.put((rank, float(np.abs(y.numpy() - ref).max())))
+    w = _weights()
+    ws = moe.slice_tp(w, rank, P, F, FS)                   # this rank's resident slice
+    f_r, fs_r = ws.w2.shape[2], ws.ws2.shape[1]
+    rng = np.random.default_rng(7)                         # replicated tokens: every rank sees the same batch
+    x, r, din = rng.normal(size=(5, H)), rng.normal(size=(5, H)), rng.normal(size=(5, H))
+    # this rank's partial expert sums (no residual / deferred_in): the slice's FFN under the
+    # FULL layer's routing (routing is replicated; the gate does not depend on the slice)
+    full = _oracle_weights(w, F, FS)
+    idx, wt, _ = O.route(x, full.gate_w, None, _cfg(F, FS))
+    part = O.moe_layer(x, _oracle_weights(ws, f_r, fs_r), _cfg(f_r, fs_r), n_deferred=NDEF,
+                       forced_routing=(idx, wt))
+    y_p = torch.from_numpy(part["y"])
+    d_p = torch.from_numpy(part["deferred_out"])
+    dist.all_reduce(y_p)                                   # the library: ncclAllReduce(fp32, sum)
+    dist.all_reduce(d_p)
+    y = y_p.numpy() + r + din                              # finalize on every rank
+    ref = O.moe_layer(x, full, _cfg(F, FS), residual=r, n_deferred=NDEF, deferred_in=din)
+    err = max(float(np.abs(y - ref["y"]).max()), float(np.abs(d_p.numpy() - ref["deferred_out"]).max()))
+    q.put((rank, (f_r, fs_r, err)))
     dist.destroy_process_group()
 
 
-def test_decode_tp_decomposition_gloo():
+def test_tp_decomposition_gloo():
     with socket.socket() as s:
         s.bind(("127.0.0.1", 0))
         port = s.getsockname()[1]
@@ -78,4 +82,5 @@ def test_decode_tp_decomposition_gloo():
     res = dict(q.get(timeout=120) for _ in range(P))
     for pr in procs:
         pr.join(timeout=60)
-    assert all(v < 1e-12 for v in res.values()), res
+    assert res[0][:2] == (128, 128) and res[1][:2] == (256, 128), res    # ragged 3-chunk split, 1/P resident
+    assert all(v[2] < 1e-12 for v in res.values()), res
