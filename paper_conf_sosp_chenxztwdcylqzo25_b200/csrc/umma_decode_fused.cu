@@ -180,7 +180,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   uint64_t *uq_full = accB_empty + FD_ACCB;                  // [FD_UQ]
   uint64_t *uq_empty = uq_full + FD_UQ;                      // [FD_UQ]
   uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(uq_empty + FD_UQ);
-  int4 *unit_q = reinterpret_cast<int4 *>(tmem_base_smem + 4);   // [FD_UQ] (expert, chunk, group, valid)
+  int4 *unit_q = reinterpret_cast<int4 *>((reinterpret_cast<uintptr_t>(tmem_base_smem + 1) + 15) & ~uintptr_t(15));   // [FD_UQ] (expert, chunk, group, valid)
   float *amax = reinterpret_cast<float *>(unit_q + FD_UQ);       // [2 gate warps][16]
   float *hsc = amax + 2 * FD_N;                                  // [2 unit parity][16] h scale per token (FP8)
 
