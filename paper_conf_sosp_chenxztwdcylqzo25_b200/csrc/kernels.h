@@ -243,6 +243,7 @@ struct FusedDecodeParams {
   float *acc_imm, *acc_def;     // [T, H] fp32 sums, zero on entry (re-zeroed by decode_finalize)
   int *sched, *done;            // work counter + exit ticket, zero on entry (re-armed by the kernel)
   unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
+  int debug;                    // MOE_EXPERIMENTS builds (MOE_DEBUG_FD): 1 no phase-A fold, 2 no phase-A MMAs
 };
 cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, cudaStream_t st);
 cudaError_t launch_decode_finalize(const DecodeFinalizeArgs &a, cudaStream_t st);

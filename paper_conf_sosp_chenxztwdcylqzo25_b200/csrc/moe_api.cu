@@ -978,6 +978,8 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     fp.acc_imm = acc_imm; fp.acc_def = acc_def;
     fp.sched = L->sched + 5; fp.done = L->sched + 6;
     fp.trace = L->trace;
+    static const int dbg_fd = experiment_knob("MOE_DEBUG_FD");   // timing experiments (MOE_EXPERIMENTS builds)
+    fp.debug = dbg_fd;
     const int units = prev_units + Fs / 128 + (int)std::min<int64_t>(E, pairs) * (F / 128);
     KL_TRY(launch_umma_decode_fused(f8, fp, std::min(L->num_sms, units), st));
     mark(L, ST_GEMM1, st);

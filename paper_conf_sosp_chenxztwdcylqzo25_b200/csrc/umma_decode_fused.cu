@@ -267,6 +267,17 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       if (!uq.w) break;
       // ---- phase A ----
       for (int kb = 0; kb < KA; ++kb) {
+        if (kExperiments && (p.debug & 2)) {     // timing experiment: phase-A loads only (no MMAs)
+          mbar_wait(&full[stage], phase);
+          if (lane == 0) {
+            mbar_arrive(&empty[stage]);
+            if (FP8 ? true : kb == KA - 1) mbar_arrive(&accA_full[FP8 ? as : 0]);
+          }
+          __syncwarp();
+          if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
+          if (FP8 && ++as == FD_ACCA_SLOTS) { as = 0; asph ^= 1; }
+          continue;
+        }
         if (FP8) {                               // this k-block's accumulator slot is free
           mbar_wait(&accA_empty[as], asph ^ 1);
           tc_fence_after();
@@ -350,11 +361,18 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       tr[7] = smid;
     }
     // activation scales [kb][token] of a layer into shared memory (FP8; tokens >= T read 0)
+    // (every load issued before the first store: one L2 round trip, not KA*16/128 of them --
+    //  the phase-A MMAs can run only FD_ACCA_SLOTS k-blocks ahead of this warp group)
     auto load_xs = [&](const float *xs, float *dst) {
-      for (int i = et; i < KA * FD_N; i += 128) {
-        const int kb = i / FD_N, t = i % FD_N;
-        dst[i] = t < p.T ? xs[(size_t)t * KA + kb] : 0.f;
+      constexpr int NI = FD_MAX_KB * FD_N / 128;
+      float v[NI];
+#pragma unroll
+      for (int j = 0; j < NI; ++j) {
+        const int i = et + 128 * j, kb = i / FD_N, t = i % FD_N;
+        v[j] = (kb < KA && t < p.T) ? __ldg(xs + (size_t)t * KA + kb) : 0.f;
       }
+#pragma unroll
+      for (int j = 0; j < NI; ++j) dst[et + 128 * j] = v[j];
     };
     if (FP8 && p.has_prev) load_xs(p.g[2].xs, xs_s + FD_MAX_KB * FD_N);   // previous layer: complete
     asm volatile("bar.sync 3, 128;" ::: "memory");
@@ -385,9 +403,14 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
           dst_j = p.acc_imm + (size_t)lane * p.H;
           w_j = p.sgate ? p.sgate[lane] : 1.f;
         } else {
+          // all k ids in flight together (a short-circuit scan would serialise k L2 round trips)
           const int ge = expert + g.e0;
+          int ids[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) ids[i] = i < g.k ? __ldg(g.topk_idx + lane * g.k + i) : -1;
           int hit = -1;
-          for (int i = 0; i < g.k; ++i) hit = (hit < 0 && g.topk_idx[lane * g.k + i] == ge) ? i : hit;
+#pragma unroll
+          for (int i = 31; i >= 0; --i) hit = ids[i] == ge ? i : hit;
           if (hit >= g.a0 && hit < g.a2) {
             w_j = g.topk_w[lane * g.k + hit];
             dst_j = (hit < g.a1 ? p.acc_imm : p.acc_def) + (size_t)lane * p.H;
@@ -408,6 +431,12 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         for (int kb = 0; kb < KA; ++kb) {
           mbar_wait(&accA_full[as], asph);
           tc_fence_after();
+          if (kExperiments && (p.debug & 1)) {   // timing experiment: no per-k-block fold
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&accA_empty[as]);
+            if (++as == FD_ACCA_SLOTS) { as = 0; asph ^= 1; }
+            continue;
+          }
           uint32_t v0[16], v1[16];
           tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCA_COL + as * 32, v0);
           tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCA_COL + as * 32 + 16, v1);

@@ -122,7 +122,8 @@ def _chain_oracle(p, ws, xs, rs, n_defs):
         x64 = x.cpu().to(torch.float64).numpy()
         t = O.tie_band_tokens(x64, W, cfg, n_deferred=nd)
         ties |= set(t.tolist())
-        o = O.moe_layer(x64, W, cfg, residual=r.cpu().to(torch.float64).numpy(), n_deferred=nd, deferred_in=din)
+        o = O.moe_layer(x64, W, cfg, residual=None if r is None else r.cpu().to(torch.float64).numpy(),
+                        n_deferred=nd, deferred_in=din)
         outs.append(o["y"])
         din = o["deferred_out"]
     return outs, sorted(ties)
@@ -131,31 +132,28 @@ def _chain_oracle(p, ws, xs, rs, n_defs):
 @pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v2lite_s", "v3_m", "v25_s"])
 @pytest.mark.parametrize("T", [1, 5, 16])
 def test_chained_deferral_matches_eq_L241(lib, name, T):
+    """A 3-layer chain (k = 1: no deferred input; k = L: n_def = 0) against Eq.
+    L241 evaluated by the oracle.  Each layer gets its own seeded tokens (the
+    chain's data dependence x_{k+1} = O_k is not what is checked here, the
+    deferred term R^def_{k-1}(I_{k-1}) joining O_k is) and residual = NULL
+    (reading R12: a residual would dilute the error)."""
     p = SMALL[name]
     n_def = min(3, p.top_k - 1)
     L = 3
     ws = [make_weights(p, "cpu", seed=4000 + 17 * i) for i in range(L)]
     layers = [lib.MoELayer(p, w.to("cuda"), max_tokens=16) for w in ws]
-    x0, _ = make_tokens(p, T, "cuda", offset=21)
-    xs, rs, ys = [x0], [], []
-    prev = None
+    xs = [make_tokens(p, T, "cuda", offset=21 + i)[0] for i in range(L)]
+    ys, prev = [], None
     for i, l in enumerate(layers):
         nd = n_def if i < L - 1 else 0                   # k = L: all experts immediate (L215)
-        r = xs[-1]                                      # I_k of Eq. L241
-        y = l.forward_chained(xs[-1], residual=r, n_deferred=nd, prev=prev)
-        rs.append(r)
-        ys.append(y)
-        xs.append(y)
+        ys.append(l.forward_chained(xs[i], n_deferred=nd, prev=prev))
         prev = l
     torch.cuda.synchronize()
-    outs, ties = _chain_oracle(p, ws, xs[:L], rs, [n_def] * (L - 1) + [0])
+    outs, ties = _chain_oracle(p, ws, xs, [None] * L, [n_def] * (L - 1) + [0])
     check_tie_fraction(ties, T * L)
     keep = np.setdiff1d(np.arange(T), ties)
     for i in range(L):
-        # the deferred part only: compare y - residual (the residual would dilute the error)
-        got = ys[i].float().cpu().numpy() - rs[i].float().cpu().numpy()
-        want = outs[i] - rs[i].cpu().to(torch.float64).numpy()
-        check_output(f"chain/{name}/T{T}/layer{i}", got[keep], want[keep], TOL[p.wtype])
+        check_output(f"chain/{name}/T{T}/layer{i}", ys[i].float().cpu().numpy()[keep], outs[i][keep], TOL[p.wtype])
     for l in layers:
         l.close()
 
@@ -198,24 +196,22 @@ def test_chained_errors(lib):
 
 def test_full_v3_chain_decode(lib):
     """Full DeepSeek-V3 layers (FP8, 256 experts, n_def = 3, BF16 setting L257),
-    a 3-layer chain at T = 1 vs the Eq. L241 oracle chain."""
+    a 3-layer chain at T = 1 and 4 vs the Eq. L241 oracle chain."""
     p = PRESETS["v3"]
     L = 3
     ws = [make_weights(p, "cuda", seed=5000 + i) for i in range(L)]
     layers = [lib.MoELayer(p, w, max_tokens=16) for w in ws]
-    x0, _ = make_tokens(p, 1, "cuda", offset=5)
-    xs, ys, prev = [x0], [], None
-    for i, l in enumerate(layers):
-        y = l.forward_chained(xs[-1], residual=xs[-1], n_deferred=3 if i < L - 1 else 0, prev=prev)
-        ys.append(y)
-        xs.append(y)
-        prev = l
-    torch.cuda.synchronize()
-    outs, ties = _chain_oracle(p, ws, xs[:L], xs[:L], [3, 3, 0])
-    assert not ties
-    for i in range(L):
-        got = ys[i].float().cpu().numpy() - xs[i].float().cpu().numpy()
-        want = outs[i] - xs[i].cpu().to(torch.float64).numpy()
-        check_output(f"chain_full/v3/layer{i}", got, want, TOL[p.wtype])
+    for T in (1, 4):
+        xs = [make_tokens(p, T, "cuda", offset=5 + i)[0] for i in range(L)]
+        ys, prev = [], None
+        for i, l in enumerate(layers):
+            ys.append(l.forward_chained(xs[i], n_deferred=3 if i < L - 1 else 0, prev=prev))
+            prev = l
+        torch.cuda.synchronize()
+        outs, ties = _chain_oracle(p, ws, xs, [None] * L, [3, 3, 0])
+        keep = np.setdiff1d(np.arange(T), ties)
+        for i in range(L):
+            check_output(f"chain_full/v3/T{T}/layer{i}", ys[i].float().cpu().numpy()[keep], outs[i][keep],
+                         TOL[p.wtype])
     for l in layers:
         l.close()
