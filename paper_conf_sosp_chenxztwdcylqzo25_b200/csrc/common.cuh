@@ -251,6 +251,9 @@ struct moe_layer {
   int F_full = 0, Fs_full = 0;
   void *tp_comm = nullptr;      // ncclComm_t of the TP group (null: in-process group)
   bool pending_use_def = false; // in-process TP group: the last partial forward kept deferred sums
+  // fused decode cluster split: resident clusters per size (index = size), peers' partials
+  int fd_max_clusters[9] = {};
+  float *cl_scratch = nullptr;
   int n_launch = 0, launches_prefill = 0, launches_decode = 0;   // kernel launches per forward
   unsigned long long *trace = nullptr;   // MOE_DEBUG_TRACE timeline buffer (timing experiments)
   // swap-AB CTA-pair GEMM (umma_swap.cu): tiled weights as 128-byte rows (box 128),

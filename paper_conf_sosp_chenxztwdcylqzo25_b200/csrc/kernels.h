@@ -244,8 +244,11 @@ struct FusedDecodeParams {
   int *sched, *done;            // work counter + exit ticket, zero on entry (re-armed by the kernel)
   unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
   int debug;                    // MOE_EXPERIMENTS builds (MOE_DEBUG_FD): 1 no phase-A fold, 2 no phase-A MMAs
+  float *cl_scratch;            // cluster split: [clusters][7][128][32] fp32 partials of the peers (L2)
 };
-cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, cudaStream_t st);
+// csize > 1: clusters of csize CTAs share each unit (the cluster split)
+cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, int csize, cudaStream_t st);
+int fused_decode_max_clusters(bool fp8, int csize);
 cudaError_t launch_decode_finalize(const DecodeFinalizeArgs &a, cudaStream_t st);
 
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);

@@ -67,7 +67,7 @@ void free_all(moe_layer *L) {
                   L->row_token, L->pos, L->sched, L->pairs, L->n_pairs, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
                   L->hsh, L->hsh_s, L->ysh, L->w13_img, L->w2_img, L->ws13_img, L->ws2_img,
                   L->xperm_img, L->h_img, L->xq_img, L->hsh_img, L->dacc, L->trace, L->imm_list, L->def_list,
-                  L->n_lists, L->xcopy};
+                  L->n_lists, L->xcopy, L->cl_scratch};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   void *eps[] = {L->ep.send_x, L->ep.send_idx, L->ep.send_w, L->ep.sendpos, L->ep.cnt_dev, L->ep.recv_x,
@@ -519,6 +519,11 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
       const size_t n = (size_t)2 * L->gemv_max_tokens * H * 4;
       C_TRY(dalloc(L, &L->dacc, n, false));
       C_TRY(cudaMemset(L->dacc, 0, n));
+      // cluster split of the stream (few units): how many clusters of 2 / 4 / 8 fit, and the
+      // L2 scratch the peers hand their fp32 partials to the leader through
+      for (int c = 2; c <= 8; c *= 2) L->fd_max_clusters[c] = fused_decode_max_clusters(f8, c);
+      const int ncl = std::max(L->fd_max_clusters[2], 1);
+      C_TRY(dalloc(L, &L->cl_scratch, (size_t)ncl * 7 * 128 * 32 * 4, false));
       if (!f8) {
         C_TRY(dalloc(L, &L->xcopy, (size_t)L->gemv_max_tokens * H * 2, false));
         C_TRY(cudaMemset(L->xcopy, 0, (size_t)L->gemv_max_tokens * H * 2));
@@ -980,8 +985,20 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     fp.trace = L->trace;
     static const int dbg_fd = experiment_knob("MOE_DEBUG_FD");   // timing experiments (MOE_EXPERIMENTS builds)
     fp.debug = dbg_fd;
+    static const int cluster_override = experiment_knob("MOE_FD_CLUSTER");   // A/B of the cluster size
     const int units = prev_units + Fs / 128 + (int)std::min<int64_t>(E, pairs) * (F / 128);
-    KL_TRY(launch_umma_decode_fused(f8, fp, std::min(L->num_sms, units), st));
+    // few units (expert TP, small layers): split each over a cluster so more SMs stream it --
+    // the largest cluster size whose clusters all fit in one wave (and that leaves every CTA
+    // at least one W13 k-block and one W2 tile)
+    int csize = 1;
+    const int KA = H / (f8 ? 128 : 64), NT = H / 256;
+    for (int c = 8; c >= 2; c /= 2)
+      if (c <= KA && c <= NT && units <= L->fd_max_clusters[c] && units * c <= L->num_sms) { csize = c; break; }
+    if (cluster_override > 0 && units <= L->fd_max_clusters[2] && cluster_override <= std::min(KA, NT))
+      csize = cluster_override;                  // (cluster ids stay within the scratch slots)
+    fp.cl_scratch = L->cl_scratch;
+    const int grid = csize > 1 ? units * csize : std::min(L->num_sms, units);
+    KL_TRY(launch_umma_decode_fused(f8, fp, grid, csize, st));
     mark(L, ST_GEMM1, st);
     if (A.chained) { L->chain_T = n_def > 0 ? T : -1; L->chain_ndef = n_def; }
     else L->chain_T = -1;

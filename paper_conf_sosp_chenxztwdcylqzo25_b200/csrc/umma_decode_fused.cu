@@ -179,23 +179,36 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   uint64_t *accB_empty = accB_full + FD_ACCB;                // [FD_ACCB]
   uint64_t *uq_full = accB_empty + FD_ACCB;                  // [FD_UQ]
   uint64_t *uq_empty = uq_full + FD_UQ;                      // [FD_UQ]
-  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(uq_empty + FD_UQ);
+  uint64_t *part_bar = uq_empty + FD_UQ;                     // cluster leader: the peers' partials are in L2
+  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(part_bar + 1);
   int4 *unit_q = reinterpret_cast<int4 *>((reinterpret_cast<uintptr_t>(tmem_base_smem + 1) + 15) & ~uintptr_t(15));   // [FD_UQ] (expert, chunk, group, valid)
   float *amax = reinterpret_cast<float *>(unit_q + FD_UQ);       // [2 gate warps][16]
   float *hsc = amax + 2 * FD_N;                                  // [2 unit parity][16] h scale per token (FP8)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // Cluster split (csize > 1, few units: expert TP, small layers): the csize CTAs of a
+  // cluster share one unit -- CTA r streams W13 k-blocks [r KA / csize, (r+1) KA / csize)
+  // and W2 tiles [r NT / csize, ...); the peers' fp32 gate/up partials are summed by the
+  // leader (rank 0) through L2, which computes SwiGLU + requant and pushes h_c (and its
+  // scales) into every peer's shared memory with st.async.  The leader claims the units
+  // and forwards them to the peers' queues.
+  const uint32_t csize = cluster_size(), crank = cluster_rank();
+  const bool leader = crank == 0;
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < FD_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     for (int s = 0; s < FD_ACCA_SLOTS; ++s) { mbar_init(&accA_full[s], 1); mbar_init(&accA_empty[s], 4); }
     mbar_init(h_ready, 1);
     for (int s = 0; s < FD_ACCB; ++s) { mbar_init(&accB_full[s], 1); mbar_init(&accB_empty[s], 4); }
-    for (int i = 0; i < FD_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], 5); }
+    // a queue slot is free when the MMA warp and the 4 epilogue warps here and the
+    // producer, MMA and epilogue warps of every peer have read it
+    for (int i = 0; i < FD_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], 5 + 6 * (csize - 1)); }
+    mbar_init(part_bar, 4 * (csize - 1) > 0 ? 4 * (csize - 1) : 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc(tmem_base_smem, FD_TMEM_COLS);
   tc_fence_before();
   __syncthreads();
+  if (csize > 1) cluster_sync();                 // every barrier of the cluster initialised
   tc_fence_after();
   const uint32_t tmem = *tmem_base_smem;
 
@@ -203,6 +216,13 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   constexpr int KBC = 128 / KDIV;                // W2 k-blocks per 128-column chunk
   const int KA = p.H / KDIV;                     // W13 k-blocks
   const int NT = p.H / 256;                      // W2 256-row tiles
+  const int kb0 = (int)(crank * KA / csize), kb1 = (int)((crank + 1) * KA / csize);   // this CTA's share
+  const int nt0 = (int)(crank * NT / csize), nt1 = (int)((crank + 1) * NT / csize);
+  // a consumer is done with queue slot qs (the leader's barrier counts the whole cluster)
+  auto release_slot = [&](int qs_) {
+    if (leader) mbar_arrive(&uq_empty[qs_]);
+    else mbar_arrive_remote(map_to_rank(&uq_empty[qs_], 0));
+  };
 
   if (warp == 0) {
     // ============================ producer ============================
@@ -212,15 +232,34 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       const uint64_t pol = l2_evict_first_policy();   // weights are read once per forward
       int stage = 0; uint32_t phase = 0, qs = 0, qph = 0;
       for (;;) {
-        const int u = atomicAdd(p.sched, 1);
-        if (u >= n_prev && !waited) {
-          pdl_wait();                            // this layer's routing and xq (route kernel)
-          waited = true;
+        FdUnit ui;
+        if (leader) {
+          const int u = atomicAdd(p.sched, 1);
+          if (u >= n_prev && !waited) {
+            pdl_wait();                          // this layer's routing and xq (route kernel)
+            waited = true;
+          }
+          ui = fd_unit(p, u, n_prev);
+          mbar_wait(&uq_empty[qs], qph ^ 1);
+          unit_q[qs] = make_int4(ui.expert, ui.chunk, ui.group, ui.valid);
+          mbar_arrive(&uq_full[qs]);
+          for (uint32_t r = 1; r < csize; ++r) {   // forward the unit to the peers
+            const uint32_t pbar = map_to_rank(&uq_full[qs], r);
+            mbar_arrive_expect_tx_remote(pbar, 16);
+            st_async_v4u32(map_to_rank(&unit_q[qs], r),
+                           make_uint4((uint32_t)ui.expert, (uint32_t)ui.chunk, (uint32_t)ui.group, (uint32_t)ui.valid),
+                           pbar);
+          }
+        } else {
+          mbar_wait(&uq_full[qs], qph);
+          const int4 q4 = unit_q[qs];
+          release_slot(qs);
+          ui.expert = q4.x; ui.chunk = q4.y; ui.group = q4.z; ui.valid = q4.w;
+          if (ui.valid && ui.group != 2 && !waited) {
+            pdl_wait();                          // this layer's xq (TMA-loaded below)
+            waited = true;
+          }
         }
-        const FdUnit ui = fd_unit(p, u, n_prev);
-        mbar_wait(&uq_empty[qs], qph ^ 1);
-        unit_q[qs] = make_int4(ui.expert, ui.chunk, ui.group, ui.valid);
-        mbar_arrive(&uq_full[qs]);
         if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
         if (!ui.valid) {
           // every load of this CTA is issued: let the finalize kernel launch now, so
@@ -231,7 +270,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         const FdGroup &g = p.g[ui.group];
         // ---- phase A: W13 tile `chunk` (256 rows: gate + up of 128 h columns) ----
         const uint8_t *w13 = g.w13 + ((size_t)ui.expert * g.nch + ui.chunk) * (size_t)KA * FD_A_BYTES;
-        for (int kb = 0; kb < KA; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           mbar_expect_tx(&full[stage], FD_A_BYTES + FD_B_BYTES);
           bulk_load_hint(sA + stage * FD_A_BYTES, w13 + (size_t)kb * FD_A_BYTES, FD_A_BYTES, &full[stage], pol);
@@ -241,7 +280,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         // ---- phase B: W2 column block `chunk`, H/256 tiles of 256 rows ----
         const int KB2 = g.nch * KBC;               // W2 k-blocks per tile row
         const uint8_t *w2 = g.w2 + (size_t)ui.expert * NT * KB2 * FD_A_BYTES;
-        for (int n = 0; n < NT; ++n) {
+        for (int n = nt0; n < nt1; ++n) {
           for (int kk = 0; kk < KBC; ++kk) {
             mbar_wait(&empty[stage], phase ^ 1);
             mbar_expect_tx(&full[stage], FD_A_BYTES);
@@ -262,16 +301,17 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       mbar_wait(&uq_full[qs], qph);
       const int4 uq = unit_q[qs];
       __syncwarp();
-      if (lane == 0) mbar_arrive(&uq_empty[qs]);
+      if (lane == 0) release_slot(qs);
       if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
       if (!uq.w) break;
       // ---- phase A ----
-      for (int kb = 0; kb < KA; ++kb) {
+      for (int kb = kb0; kb < kb1; ++kb) {
         if (kExperiments && (p.debug & 2)) {     // timing experiment: phase-A loads only (no MMAs)
+          if (FP8) mbar_wait(&accA_empty[as], asph ^ 1);
           mbar_wait(&full[stage], phase);
           if (lane == 0) {
             mbar_arrive(&empty[stage]);
-            if (FP8 ? true : kb == KA - 1) mbar_arrive(&accA_full[FP8 ? as : 0]);
+            if (FP8 ? true : kb == kb1 - 1) mbar_arrive(&accA_full[FP8 ? as : 0]);
           }
           __syncwarp();
           if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
@@ -296,12 +336,12 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
               if (FP8)
                 mma_f8(tmem + FD_ACCA_COL + as * 32 + t * 16, ad, bd, idesc_f8(128, FD_N), k != 0);
               else   // the accumulator is free: the epilogue read it before h_ready of the previous unit
-                mma_bf16(tmem + FD_ACCA_COL + t * 16, ad, bd, idesc_bf16(128, FD_N), (kb | k) != 0);
+                mma_bf16(tmem + FD_ACCA_COL + t * 16, ad, bd, idesc_bf16(128, FD_N), (kb != kb0) || (k != 0));
             }
           }
           mma_commit(&empty[stage]);
           if (FP8) mma_commit(&accA_full[as]);
-          else if (kb == KA - 1) mma_commit(&accA_full[0]);
+          else if (kb == kb1 - 1) mma_commit(&accA_full[0]);
         }
         __syncwarp();
         if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
@@ -310,9 +350,10 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       // ---- phase B: B operand = h_c in shared memory ----
       mbar_wait(h_ready, hph);
       hph ^= 1;
+      fence_proxy_async_smem();                  // a peer's h_c arrived by st.async
       tc_fence_after();
       const uint32_t h0 = smem_u32(sH);
-      for (int n = 0; n < NT; ++n) {
+      for (int n = nt0; n < nt1; ++n) {
         mbar_wait(&accB_empty[ab], abph ^ 1);
         tc_fence_after();
         for (int kk = 0; kk < KBC; ++kk) {
@@ -351,6 +392,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     int ab = 0; uint32_t abph = 0;
     int as = 0; uint32_t asph = 0;
     int ui_par = 0;
+    uint32_t hph_e = 0, pph = 0;                 // cluster peers: h_ready phase; leader: part_bar phase
     bool waited = false;
     // MOE_DEBUG_TRACE: per-CTA timeline (globaltimer ns) into p.trace[8 + 8 * cta ..] (timing experiments)
     unsigned long long *tr = (p.trace && warp == 2 && lane == 0) ? p.trace + 8 + 8 * blockIdx.x : nullptr;
@@ -380,7 +422,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       mbar_wait(&uq_full[qs], qph);
       const int4 uq = unit_q[qs];
       __syncwarp();
-      if (lane == 0) mbar_arrive(&uq_empty[qs]);
+      if (lane == 0) release_slot(qs);
       if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
       if (!uq.w) break;
       const int expert = uq.x, chunk = uq.y, group = uq.z;
@@ -428,7 +470,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         const float swa = lane < KA ? ws[lane] : 0.f, swb = lane + 32 < KA ? ws[lane + 32] : 0.f;
 #pragma unroll
         for (int t = 0; t < FD_N; ++t) r0[t] = r1[t] = 0.f;
-        for (int kb = 0; kb < KA; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&accA_full[as], asph);
           tc_fence_after();
           if (kExperiments && (p.debug & 1)) {   // timing experiment: no per-k-block fold
@@ -473,13 +515,51 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         for (int t = 0; t < FD_N; ++t) { r0[t] = __uint_as_float(v0[t]); r1[t] = __uint_as_float(v1[t]); }
       }
       if (tr) tr[3] = gtimer();
+      constexpr uint32_t H_TX = FP8 ? 2 * FD_B_BYTES / 2 + 4 * FD_N : FD_H_BYTES;   // h_c (+ FP8 scales) bytes
+      if (csize > 1) {
+        // ---- cluster: the peers' partial gate/up sums -> the leader (through L2) ----
+        float *scr = p.cl_scratch + (size_t)cluster_id_x() * 7 * 128 * 32;
+        if (!leader) {
+          float4 *dst = reinterpret_cast<float4 *>(scr + ((size_t)(crank - 1) * 128 + et) * 32);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            __stcg(dst + j, make_float4(r0[4 * j], r0[4 * j + 1], r0[4 * j + 2], r0[4 * j + 3]));
+            __stcg(dst + 4 + j, make_float4(r1[4 * j], r1[4 * j + 1], r1[4 * j + 2], r1[4 * j + 3]));
+          }
+          __syncwarp();
+          if (lane == 0) mbar_arrive_cluster(map_to_rank(part_bar, 0));   // release.cluster
+          // h_c of this unit comes from the leader (st.async into sH / hsc, complete_tx on h_ready)
+          if (q == 0 && lane == 0) mbar_expect_tx(h_ready, H_TX);
+          mbar_wait(h_ready, hph_e);
+          hph_e ^= 1;
+          if (tr) tr[4] = gtimer();
+          goto phase_b;
+        }
+        mbar_wait_cluster(part_bar, pph);
+        pph ^= 1;
+        for (uint32_t r = 1; r < csize; ++r) {
+          const float4 *src = reinterpret_cast<const float4 *>(scr + ((size_t)(r - 1) * 128 + et) * 32);
+          float4 v[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[j] = __ldcg(src + j);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            r0[4 * j] += v[j].x; r0[4 * j + 1] += v[j].y; r0[4 * j + 2] += v[j].z; r0[4 * j + 3] += v[j].w;
+            r1[4 * j] += v[4 + j].x; r1[4 * j + 1] += v[4 + j].y; r1[4 * j + 2] += v[4 + j].z;
+            r1[4 * j + 3] += v[4 + j].w;
+          }
+        }
+      }
+      {
       // ---- SwiGLU + requant -> h_c (B operand of phase B) ----
       float *xb = xch + qg * (2 * FD_N * 32);
       if (q & 1) {
 #pragma unroll
         for (int t = 0; t < FD_N; ++t) {
-          xb[t * 32 + lane] = r0[t];
-          xb[(FD_N + t) * 32 + lane] = r1[t];
+          if (t < p.T) {                        // (warp-uniform: token columns >= T are never read)
+            xb[t * 32 + lane] = r0[t];
+            xb[(FD_N + t) * 32 + lane] = r1[t];
+          }
         }
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
@@ -494,12 +574,15 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         if (FP8) {
 #pragma unroll
           for (int t = 0; t < FD_N; ++t) {
-            const float m = warp_max(fmaxf(fabsf(h0[t]), fabsf(h1[t])));
-            if (lane == 0) amax[qg * FD_N + t] = m;
+            if (t < p.T) {
+              const float m = warp_max(fmaxf(fabsf(h0[t]), fabsf(h1[t])));
+              if (lane == 0) amax[qg * FD_N + t] = m;
+            }
           }
           asm volatile("bar.sync 2, 64;" ::: "memory");   // the two gate warps
 #pragma unroll
           for (int t = 0; t < FD_N; ++t) {
+            if (t >= p.T) continue;               // (phase B drops token columns >= T)
             const int e = ue8m0_exponent(fmaxf(amax[t], amax[FD_N + t]));
             const float inv = exp2i(-e);
             uint8_t *row = sH + t * 128;
@@ -512,6 +595,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
           // two 64-column k-blocks of bf16: column f0 -> block 0, f0 + 64 -> block 1 (same in-block column)
 #pragma unroll
           for (int t = 0; t < FD_N; ++t) {
+            if (t >= p.T) continue;
             const int off = t * 128 + ((((f0 >> 3) ^ (t & 7)) << 4) | ((f0 & 7) << 1));
             *reinterpret_cast<__nv_bfloat16 *>(sH + off) = __float2bfloat16_rn(h0[t]);
             *reinterpret_cast<__nv_bfloat16 *>(sH + FD_B_BYTES + off) = __float2bfloat16_rn(h1[t]);
@@ -520,8 +604,24 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         fence_proxy_async_smem();                 // generic-proxy h writes -> the MMA's async-proxy reads
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (csize > 1) {
+        // push h_c (and the FP8 h scales) into every peer's shared memory
+        constexpr int HV = (FP8 ? 2 * FD_B_BYTES / 2 : FD_H_BYTES) / 16;   // 16-byte vectors of h_c
+        for (int i = et; i < HV; i += 128) {
+          const uint4 v = *reinterpret_cast<const uint4 *>(sH + 16 * i);
+          for (uint32_t r = 1; r < csize; ++r)
+            st_async_v4u32(map_to_rank(sH + 16 * i, r), v, map_to_rank(h_ready, r));
+        }
+        if (FP8 && et < FD_N / 4) {
+          const uint4 v = *reinterpret_cast<const uint4 *>(hsc + ui_par * FD_N + 4 * et);
+          for (uint32_t r = 1; r < csize; ++r)
+            st_async_v4u32(map_to_rank(hsc + ui_par * FD_N + 4 * et, r), v, map_to_rank(h_ready, r));
+        }
+      }
       if (q == 0 && lane == 0) mbar_arrive(h_ready);
       if (tr) tr[4] = gtimer();
+      }
+    phase_b:
       // ---- phase B epilogue: scaled, weighted partial sums of W2 row tiles ----
       // the unit's W2 block scales (H/128 <= 64 row blocks) into registers up front:
       // a global load per tile would put HBM latency on the epilogue's critical path
@@ -531,7 +631,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         if (lane < p.H / 128) s2a = w2s[(size_t)lane * g.nch];
         if (lane + 32 < p.H / 128) s2b = w2s[(size_t)(lane + 32) * g.nch];
       }
-      for (int nt = 0; nt < NT; ++nt) {
+      for (int nt = nt0; nt < nt1; ++nt) {
         mbar_wait(&accB_full[ab], abph);
         tc_fence_after();
         uint32_t v0[16], v1[16];
@@ -571,6 +671,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   pdl_trigger();
   tc_fence_before();
   __syncthreads();
+  if (csize > 1) cluster_sync();                 // no CTA leaves while a peer may still st.async into it
   if (warp == 1) tmem_dealloc(tmem, FD_TMEM_COLS);
   if (threadIdx.x == 0) {
     // the last CTA out re-arms the work counter for the next forward (graph replay)
@@ -592,16 +693,59 @@ __global__ void decode_finalize_kernel(const __grid_constant__ DecodeFinalizeArg
 }
 
 template <bool FP8>
-static cudaError_t fd_launch(const FusedDecodeParams &p, int grid, cudaStream_t st) {
+static cudaError_t fd_launch(const FusedDecodeParams &p, int grid, int csize, cudaStream_t st) {
   auto k = umma_decode_fused_kernel<FP8>;
   cudaError_t e = set_kernel_attr((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FD_SMEM);
+  if (e == cudaSuccess && csize > 1)
+    e = set_kernel_attr((const void *)k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
   if (e != cudaSuccess) return e;
-  return launch_pdl(k, dim3(grid), dim3(FD_THREADS), FD_SMEM, st, p);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(FD_THREADS);
+  cfg.dynamicSmemBytes = FD_SMEM;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[2];
+  int na = 0;
+  attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[na++].val.programmaticStreamSerializationAllowed = 1;
+  if (csize > 1) {
+    attr[na].id = cudaLaunchAttributeClusterDimension;
+    attr[na].val.clusterDim.x = csize;
+    attr[na].val.clusterDim.y = 1;
+    attr[na++].val.clusterDim.z = 1;
+  }
+  cfg.attrs = attr;
+  cfg.numAttrs = na;
+  return cudaLaunchKernelEx(&cfg, k, p);
 }
 
-cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, cudaStream_t st) {
+cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, int csize, cudaStream_t st) {
   if (grid <= 0) return cudaSuccess;
-  return fp8 ? fd_launch<true>(p, grid, st) : fd_launch<false>(p, grid, st);
+  return fp8 ? fd_launch<true>(p, grid, csize, st) : fd_launch<false>(p, grid, csize, st);
+}
+
+// clusters of `csize` fused-decode CTAs that can be resident at once (0 if none)
+int fused_decode_max_clusters(bool fp8, int csize) {
+  const void *k = fp8 ? (const void *)umma_decode_fused_kernel<true> : (const void *)umma_decode_fused_kernel<false>;
+  if (set_kernel_attr(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FD_SMEM) != cudaSuccess) return 0;
+  if (csize > 8 && set_kernel_attr(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) != cudaSuccess) return 0;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(csize * 16);
+  cfg.blockDim = dim3(FD_THREADS);
+  cfg.dynamicSmemBytes = FD_SMEM;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = csize;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, k, &cfg) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return n;
 }
 
 cudaError_t launch_decode_finalize(const DecodeFinalizeArgs &a, cudaStream_t st) {
