@@ -16,6 +16,7 @@ GROUP_TOP2_SUM = 1
 W_BF16 = 0
 W_FP8 = 1
 W_F32 = 2   # toy config only (BASELINE.json: "fp32 weights")
+W_FP4 = 3   # e2m1 codes (packed 2 per byte) + power-of-two 128x128 block scales
 
 
 @dataclass(frozen=True)
@@ -86,4 +87,12 @@ SMALL = {
     # k-blocks = 2 groups), so both TMEM scale-column sets are exercised
     "v3_m": PRESETS["v3"].with_(name="v3_m", hidden=2048, ffn=1024, n_experts=32,
                                 shared_ffn=1024, prefill_tokens=300),
+    # 4-bit (e2m1) expert weights, DeepSeek-V3 gate (NEXT-3)
+    "v3_s_fp4": PRESETS["v3"].with_(name="v3_s_fp4", hidden=512, ffn=256, n_experts=64, shared_ffn=256,
+                                    prefill_tokens=333, wtype=W_FP4),
+    "v3_m_fp4": PRESETS["v3"].with_(name="v3_m_fp4", hidden=2048, ffn=1024, n_experts=32, shared_ffn=1024,
+                                    prefill_tokens=300, wtype=W_FP4),
 }
+
+# the DeepSeek-V3 layer with 4-bit expert weights (decode bytes halved, NEXT-3)
+PRESETS["v3_fp4"] = PRESETS["v3"].with_(name="v3_fp4", wtype=W_FP4)

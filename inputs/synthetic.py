@@ -12,7 +12,8 @@ Recipe:
                                               "activated in a balanced manner")
   bias ~ U(-0.05, 0.05) fp32 [E]             (DeepSeek-V3 only)
   W1/W3 ~ N(0, 1/H), W2 ~ N(0, 1/F)          (routed and shared)
-      -> bf16, fp32 (toy) or e4m3 + UE8M0 128x128 scales (FP8 presets)
+      -> bf16, fp32 (toy), e4m3 + UE8M0 128x128 scales (FP8 presets) or
+         packed e2m1 + UE8M0 128x128 scales (FP4 presets)
   w_sg ~ N(0, 1/H) -> bf16 [H]              (Qwen2 shared-expert gate)
   skew > 0: per-expert logit offsets via a common direction (hot experts get
       ~4x the mean load at skew=1; "imbalanced expert selection")
@@ -25,7 +26,7 @@ from typing import Optional
 
 import torch
 
-from .presets import LayerPreset, W_BF16, W_F32, W_FP8
+from .presets import LayerPreset, W_BF16, W_F32, W_FP4, W_FP8
 
 E4M3_MAX = 448.0
 
@@ -76,10 +77,34 @@ def fp8_block_encode(w: torch.Tensor):
     return codes.contiguous(), scale.contiguous()
 
 
+E2M1_MAX = 6.0
+
+
+def fp4_block_encode(w: torch.Tensor):
+    """Store fp32 weights [..., R, C] as OCP e2m1 codes (sign bit 3, magnitudes
+    0, .5, 1, 1.5, 2, 3, 4, 6) packed two per byte (element 2i in the low nibble
+    of byte i) with one power-of-two scale per 128x128 block, 2^ceil(log2(amax/6)).
+    Checkpoint preparation (the input format), not hot-path math; rounding is to
+    the nearest magnitude (ties either way: both sides read the stored codes)."""
+    *lead, R, C = w.shape
+    b = w.reshape(*lead, R // 128, 128, C // 128, 128)
+    amax = b.abs().amax(dim=(-3, -1))
+    m, e = torch.frexp(amax / E2M1_MAX)
+    scale = torch.where(m == 0.5, torch.ldexp(torch.ones_like(m), e - 1), torch.ldexp(torch.ones_like(m), e))
+    scale = torch.where(amax > 0, scale, torch.ones_like(scale))
+    q = (b / scale[..., :, None, :, None]).reshape(*lead, R, C)
+    mid = torch.tensor([0.25, 0.75, 1.25, 1.75, 2.5, 3.5, 5.0], device=w.device)
+    code = torch.bucketize(q.abs(), mid).to(torch.uint8) | ((q < 0).to(torch.uint8) << 3)
+    packed = code[..., 0::2] | (code[..., 1::2] << 4)
+    return packed.contiguous(), scale.contiguous()
+
+
 def _weight(shape, std, wtype, g, device):
     w = _normal(shape, std, g, device)
     if wtype == W_FP8:
         return fp8_block_encode(w)
+    if wtype == W_FP4:
+        return fp4_block_encode(w)
     if wtype == W_BF16:
         return w.to(torch.bfloat16), None
     return w, None
@@ -111,8 +136,8 @@ def make_weights(p: LayerPreset, device="cpu", seed: Optional[int] = None,
     w13 = torch.stack(w13_list)
     w2 = torch.stack(w2_list)
     del w13_list, w2_list
-    w13_scale = torch.stack(s13_list) if p.wtype == W_FP8 else None
-    w2_scale = torch.stack(s2_list) if p.wtype == W_FP8 else None
+    w13_scale = torch.stack(s13_list) if p.wtype in (W_FP8, W_FP4) else None
+    w2_scale = torch.stack(s2_list) if p.wtype in (W_FP8, W_FP4) else None
     ws13 = ws13_scale = ws2 = ws2_scale = sgw = None
     if p.shared_ffn:
         Fs = p.shared_ffn

@@ -257,6 +257,44 @@ def dequant_block128(codes: np.ndarray, scales: np.ndarray) -> np.ndarray:
 
 
 # --------------------------------------------------------------------------
+# 4-bit expert weights for decode (SURVEY.md §8(f) NEXT-3; PAPER.md L159
+# "symmetric group-wise linear quantization for Int8 and Int4 ... Int4 tiles
+# are packed into Int8-sized blocks").  B200 reading (DESIGN.md R25): the
+# 4-bit element is OCP FP4 e2m1 -- the type the 5th-gen tensor cores take
+# next to e4m3 -- packed two per byte (element 2i in the low nibble of byte i),
+# with one power-of-two scale per 128x128 block (the group of R10).
+# --------------------------------------------------------------------------
+def unpack_fp4(packed: np.ndarray) -> np.ndarray:
+    """[..., C/2] bytes -> [..., C] 4-bit codes: element 2i = low nibble of byte i."""
+    b = np.asarray(packed, np.uint8)
+    out = np.empty(b.shape[:-1] + (2 * b.shape[-1],), np.uint8)
+    out[..., 0::2] = b & 0x0F
+    out[..., 1::2] = b >> 4
+    return out
+
+
+def e2m1_decode(code: np.ndarray) -> np.ndarray:
+    """OCP e2m1: sign bit 3, exponent bits 2-1 (bias 1), mantissa bit 0; no inf/NaN.
+    exponent 0 is subnormal (0 or 0.5)."""
+    c = np.asarray(code, np.uint8).astype(np.int64)
+    sign = np.where(c & 0x8, -1.0, 1.0)
+    exp = (c >> 1) & 0x3
+    man = c & 0x1
+    val = np.where(exp == 0, man * 0.5, (1.0 + man / 2.0) * np.exp2(exp - 1.0))
+    return sign * val
+
+
+def dequant_fp4_block128(packed: np.ndarray, scales: np.ndarray) -> np.ndarray:
+    """W[r, c] = e2m1(code[r, c]) * scales[r // 128, c // 128], codes unpacked from
+    `packed` [R, C/2] (e2m1_decode evaluated once per code as a 16-entry table)."""
+    table = e2m1_decode(np.arange(16, dtype=np.uint8))
+    w = table[unpack_fp4(packed)]
+    r, c = w.shape
+    w = w.reshape(r // 128, 128, c // 128, 128) * np.asarray(scales, F64)[:, None, :, None]
+    return w.reshape(r, c)
+
+
+# --------------------------------------------------------------------------
 # Expert FFN (SwiGLU; reading R1 -- HF DeepseekV3MLP / Qwen2MoeMLP) and the
 # fused gate+up "one batch" structure of PAPER.md L179 §3.2.
 # --------------------------------------------------------------------------
@@ -294,7 +332,7 @@ class OracleConfig:
     routed_scale: float = 1.0
     shared_ffn: int = 0
     shared_gated: bool = False
-    fp8: bool = False
+    fp8: bool = False          # FP8 activation quantisation (FP8 and FP4 weight storage)
 
 
 class OracleWeights:

@@ -6,17 +6,19 @@ from __future__ import annotations
 import numpy as np
 import torch
 
-from inputs.presets import W_FP8
+from inputs.presets import W_FP4, W_FP8
 from oracle import moe_oracle as O
 
-TOL = {0: 5e-3, 1: 2e-2, 2: 5e-3}   # north_star: BF16 rel-L2 <= 5e-3, FP8 <= 2e-2 (F32 toy: BF16 bar)
+TOL = {0: 5e-3, 1: 2e-2, 2: 5e-3, 3: 2e-2}   # north_star: BF16 rel-L2 <= 5e-3, FP8 <= 2e-2 (F32 toy: BF16 bar;
+                                             # FP4 weights: e4m3 activations as FP8, the FP8 bar)
 
 
 def oracle_cfg(p) -> O.OracleConfig:
     return O.OracleConfig(hidden=p.hidden, ffn=p.ffn, n_experts=p.n_experts, top_k=p.top_k,
                           n_group=p.n_group, topk_group=p.topk_group, group_score=p.group_score,
                           score_fn=p.score_fn, norm_topk=bool(p.norm_topk), routed_scale=p.routed_scale,
-                          shared_ffn=p.shared_ffn, shared_gated=bool(p.shared_gated), fp8=p.wtype == W_FP8)
+                          shared_ffn=p.shared_ffn, shared_gated=bool(p.shared_gated),
+                          fp8=p.wtype in (W_FP8, W_FP4))
 
 
 def _f64(t):
@@ -26,9 +28,11 @@ def _f64(t):
 def oracle_weights(p, w) -> O.OracleWeights:
     """Dequantised fp64 weights, fetched per expert (works for CPU or GPU tensors)."""
     F, Fs = p.ffn, p.shared_ffn
-    fp8 = p.wtype == W_FP8
+    fp8 = p.wtype in (W_FP8, W_FP4)
 
     def deq(codes, scales):
+        if p.wtype == W_FP4:
+            return O.dequant_fp4_block128(codes.detach().cpu().numpy(), scales.detach().cpu().numpy())
         if fp8:
             return O.dequant_block128(codes.detach().cpu().numpy(), scales.detach().cpu().numpy())
         return _f64(codes)

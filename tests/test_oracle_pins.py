@@ -486,3 +486,44 @@ def test_tie_band_group_max_rule():
             [0.9, 0.1, 0.6, 0.1, 0.59, 0.1, 0.05, 0.05]]
     x, W, cfg = _tie_layer(rows, n_group=4, topk_group=2, group_score=O.GROUP_MAX, top_k=2)
     assert list(O.tie_band_tokens(x, W, cfg)) == [0]
+
+
+# ---------------------------------------------------------------- FP4 (e2m1) weights (NEXT-3)
+def test_e2m1_decode_all_codes_match_ml_dtypes():
+    codes = np.arange(16, dtype=np.uint8)
+    ref = codes.view(ml_dtypes.float4_e2m1fn).astype(np.float64)
+    np.testing.assert_array_equal(O.e2m1_decode(codes), ref)
+    # the OCP table, by hand: magnitudes 0, 0.5, 1, 1.5, 2, 3, 4, 6 and their negatives
+    assert list(O.e2m1_decode(codes[:8])) == [0, 0.5, 1, 1.5, 2, 3, 4, 6]
+    assert list(O.e2m1_decode(codes[8:])) == [-0.0, -0.5, -1, -1.5, -2, -3, -4, -6]
+
+
+def test_unpack_fp4_nibble_order():
+    """element 2i is the LOW nibble of byte i: 0x21 -> codes (1, 2) -> (0.5, 1.0)."""
+    np.testing.assert_array_equal(O.unpack_fp4(np.array([[0x21, 0xF7]], np.uint8)), [[1, 2, 7, 15]])
+    np.testing.assert_array_equal(O.e2m1_decode(O.unpack_fp4(np.array([0x21], np.uint8))), [0.5, 1.0])
+
+
+def test_dequant_fp4_block128():
+    rng = np.random.default_rng(12)
+    codes = rng.integers(0, 16, size=(256, 384), dtype=np.uint8)
+    packed = (codes[:, 0::2] | (codes[:, 1::2] << 4)).astype(np.uint8)
+    scales = 2.0 ** rng.integers(-8, 3, size=(2, 3))
+    w = O.dequant_fp4_block128(packed, scales)
+    ref = codes.view(ml_dtypes.float4_e2m1fn).astype(np.float64)
+    for i in range(2):
+        for j in range(3):
+            blk = (slice(128 * i, 128 * (i + 1)), slice(128 * j, 128 * (j + 1)))
+            np.testing.assert_array_equal(w[blk], ref[blk] * scales[i, j])
+
+
+def test_fp4_weights_equal_their_e4m3_expansion():
+    """e2m1 is a subset of e4m3: the FP4 layer equals the FP8 layer built from the
+    same values (the library's prefill path runs on that expansion), exactly."""
+    rng = np.random.default_rng(13)
+    codes = rng.integers(0, 16, size=(128, 256), dtype=np.uint8)
+    packed = (codes[:, 0::2] | (codes[:, 1::2] << 4)).astype(np.uint8)
+    vals = O.e2m1_decode(codes)
+    e4 = vals.astype(np.float32).astype(ml_dtypes.float8_e4m3fn).view(np.uint8)
+    s = np.array([[0.25, 2.0]])
+    np.testing.assert_array_equal(O.dequant_fp4_block128(packed, s), O.dequant_block128(e4, s))
