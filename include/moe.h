@@ -54,7 +54,14 @@ typedef enum { MOE_GROUP_MAX = 0, MOE_GROUP_TOP2_SUM = 1 } moe_group_score;
 /* weight storage: BF16; e4m3 codes + one fp32 power-of-two scale per 128x128
  * block (reading R10: UE8M0 block scaling, north_star "128x128
  * block-scaled FP8"); F32 (toy config only).                                 */
-typedef enum { MOE_W_BF16 = 0, MOE_W_FP8_BLOCK128 = 1, MOE_W_F32 = 2 } moe_wtype;
+typedef enum { MOE_W_BF16 = 0, MOE_W_FP8_BLOCK128 = 1, MOE_W_F32 = 2, MOE_W_FP4_BLOCK128 = 3 } moe_wtype;
+/* MOE_W_FP4_BLOCK128 ("Int4 tiles are
+ * packed into Int8-sized blocks"): OCP FP4 e2m1 codes, two per byte (element 2i
+ * in the LOW nibble of byte i) -- w13 [E, 2F, H/2], w2 [E, H, F/2], shared
+ * likewise -- with the FP8 path's power-of-two scales per 128x128 block.  The
+ * decode stream reads the packed codes (half the bytes of FP8); prefill runs the
+ * FP8 kernels on the exact e4m3 expansion made at create.  Activations are
+ * e4m3-quantised as for FP8 (R25).                                 */
 
 typedef struct {
   int32_t hidden;            /* H, multiple of 128                                   */

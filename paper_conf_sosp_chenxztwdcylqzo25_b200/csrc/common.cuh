@@ -181,6 +181,7 @@ struct moe_layer {
   int e0;       // first global expert owned by this rank
   int k, H, F, Fs;
   bool fp8, f32w;
+  bool fp4 = false;   // 4-bit (e2m1) expert weights: decode streams the packed codes
   int act_bytes;  // bytes per activation element fed to the expert GEMMs (1 fp8, 2 bf16)
   int max_tokens;
   int gemv_max_tokens;
@@ -253,6 +254,9 @@ struct moe_layer {
   bool pending_use_def = false; // in-process TP group: the last partial forward kept deferred sums
   // fused decode cluster split: resident clusters per size (index = size), peers' partials
   int fd_max_clusters[9] = {};
+  // FP4 weights: packed e2m1 codes for the decode stream (W13 rows in the stream's tile order)
+  void *w13_f4 = nullptr, *w2_f4 = nullptr, *ws13_f4 = nullptr, *ws2_f4 = nullptr;
+  CUtensorMap fmap_w13, fmap_w2, fmap_ws13, fmap_ws2;
   float *cl_scratch = nullptr;
   int n_launch = 0, launches_prefill = 0, launches_decode = 0;   // kernel launches per forward
   unsigned long long *trace = nullptr;   // MOE_DEBUG_TRACE timeline buffer (timing experiments)

@@ -216,6 +216,8 @@ cudaError_t launch_tile_weights(const void *src, void *dst, int nexp, int rows, 
 // weighted fp32 partial sums; decode_finalize writes y / deferred_out
 struct FdGroup {                // 0 routed, 1 shared, 2 the previous layer's deferred experts
   CUtensorMap x_map;            // token-order activation rows (xq / bf16 x), K-major SW128, box 16 rows
+  CUtensorMap w13_map4, w2_map4;   // FP4 weights (packed e2m1, 16U4_ALIGN16B, box 128 x 256 rows, SW128):
+                                   // W13 rows in the tile order [expert][F/128][256], W2 rows [expert][H]
   const uint8_t *w13;           // tiled W13 [expert][F/128][H/128 B][256 x 128 B]
   const float *w13_s;           // FP8: [expert][2F/128][H/128] block scales, rows interleaved per 128 (gate, up)
   const float *xs;              // FP8: [T][H/128] activation scales (token order)
@@ -247,11 +249,19 @@ struct FusedDecodeParams {
   float *cl_scratch;            // cluster split: [clusters][7][128][32] fp32 partials of the peers (L2)
 };
 // csize > 1: clusters of csize CTAs share each unit (the cluster split)
-cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, int csize, cudaStream_t st);
+cudaError_t launch_umma_decode_fused(bool fp8, bool w4, const FusedDecodeParams &p, int grid, int csize,
+                                     cudaStream_t st);
 int fused_decode_max_clusters(bool fp8, int csize);
 cudaError_t launch_decode_finalize(const DecodeFinalizeArgs &a, cudaStream_t st);
 
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows);
+// packed e2m1 [rows, cols / 2 bytes] -> shared memory unpacked to 16-byte groups (box 128 x box_rows, SW128)
+bool make_fp4_map(CUtensorMap *m, const void *base, int64_t rows, int64_t cols, int box_rows);
+// FP4 weights at create: e2m1 nibbles -> e4m3 bytes (exact: e2m1 is a subset of e4m3)
+cudaError_t launch_fp4_to_e4m3(const void *packed, void *out, int64_t n_bytes_in, cudaStream_t st);
+// W13 rows [nexp][2F] (W1 rows then W3 rows) -> the 256-row tile order of the decode stream
+// (per tile nb: 128-row halves of [gate | up | gate | up] 32-row quadrants), row_bytes each
+cudaError_t launch_permute_w13_rows(const void *src, void *dst, int nexp, int F, int row_bytes, cudaStream_t st);
 bool make_rows_map(CUtensorMap *m, const void *base, bool u32, int64_t rows, int row_elems, int box_rows);
 bool make_blocks_map(CUtensorMap *m, const void *base, int64_t total_bytes, int row_bytes, int box_rows);
 // prefill grouped expert GEMM, swap-AB on CTA pairs (umma_swap.cu): weights are

@@ -67,7 +67,7 @@ void free_all(moe_layer *L) {
                   L->row_token, L->pos, L->sched, L->pairs, L->n_pairs, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
                   L->hsh, L->hsh_s, L->ysh, L->w13_img, L->w2_img, L->ws13_img, L->ws2_img,
                   L->xperm_img, L->h_img, L->xq_img, L->hsh_img, L->dacc, L->trace, L->imm_list, L->def_list,
-                  L->n_lists, L->xcopy, L->cl_scratch};
+                  L->n_lists, L->xcopy, L->cl_scratch, L->w13_f4, L->w2_f4, L->ws13_f4, L->ws2_f4};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   void *eps[] = {L->ep.send_x, L->ep.send_idx, L->ep.send_w, L->ep.sendpos, L->ep.cnt_dev, L->ep.recv_x,
@@ -239,7 +239,10 @@ moe_status validate(const moe_layer_config *c, const moe_layer_weights *w) {
     return fail(MOE_ERR_INVALID_ARG, "top-2 group score needs >= 2 experts per group");
   if (c->score_fn != MOE_SCORE_SOFTMAX && c->score_fn != MOE_SCORE_SIGMOID) return fail(MOE_ERR_INVALID_ARG, "score_fn");
   if (c->group_score != MOE_GROUP_MAX && c->group_score != MOE_GROUP_TOP2_SUM) return fail(MOE_ERR_INVALID_ARG, "group_score");
-  if (c->wtype != MOE_W_BF16 && c->wtype != MOE_W_FP8_BLOCK128 && c->wtype != MOE_W_F32) return fail(MOE_ERR_INVALID_ARG, "wtype");
+  if (c->wtype != MOE_W_BF16 && c->wtype != MOE_W_FP8_BLOCK128 && c->wtype != MOE_W_F32 && c->wtype != MOE_W_FP4_BLOCK128)
+    return fail(MOE_ERR_INVALID_ARG, "wtype");
+  if (c->wtype == MOE_W_FP4_BLOCK128 && c->hidden % 256)
+    return fail(MOE_ERR_UNSUPPORTED, "FP4 weights need hidden %% 256 == 0 (the tensor-core paths)");
   if (c->max_tokens < 0) return fail(MOE_ERR_INVALID_ARG, "max_tokens");
   if (c->ep_size < 1 || c->ep_size > 32 || c->n_experts % c->ep_size)
     return fail(MOE_ERR_INVALID_ARG, "ep_size %d must be in [1, 32] and divide n_experts", c->ep_size);
@@ -255,10 +258,11 @@ moe_status validate(const moe_layer_config *c, const moe_layer_weights *w) {
       return fail(MOE_ERR_UNSUPPORTED, "expert TP needs the tensor-core decode stream (bf16/fp8, hidden %% 256 == 0)");
   }
   if (!w->gate_w || !w->w13 || !w->w2) return fail(MOE_ERR_INVALID_ARG, "gate_w / w13 / w2 must be non-null");
-  if (c->wtype == MOE_W_FP8_BLOCK128 && (!w->w13_scale || !w->w2_scale))
+  if ((c->wtype == MOE_W_FP8_BLOCK128 || c->wtype == MOE_W_FP4_BLOCK128) && (!w->w13_scale || !w->w2_scale))
     return fail(MOE_ERR_INVALID_ARG, "FP8 weights need w13_scale and w2_scale");
   if (c->shared_ffn > 0 && (!w->ws13 || !w->ws2)) return fail(MOE_ERR_INVALID_ARG, "shared_ffn > 0 needs ws13 / ws2");
-  if (c->shared_ffn > 0 && c->wtype == MOE_W_FP8_BLOCK128 && (!w->ws13_scale || !w->ws2_scale))
+  if (c->shared_ffn > 0 && (c->wtype == MOE_W_FP8_BLOCK128 || c->wtype == MOE_W_FP4_BLOCK128) &&
+      (!w->ws13_scale || !w->ws2_scale))
     return fail(MOE_ERR_INVALID_ARG, "FP8 shared expert needs scales");
   if (c->shared_gated && (!w->shared_gate_w || c->shared_ffn == 0))
     return fail(MOE_ERR_INVALID_ARG, "shared_gated needs shared_gate_w and a shared expert");
@@ -318,7 +322,8 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
     L->F = slice(cfg->ffn);
     L->Fs = cfg->shared_ffn > 0 ? slice(cfg->shared_ffn) : 0;
   }
-  L->fp8 = cfg->wtype == MOE_W_FP8_BLOCK128;
+  L->fp4 = cfg->wtype == MOE_W_FP4_BLOCK128;
+  L->fp8 = cfg->wtype == MOE_W_FP8_BLOCK128 || L->fp4;   // FP4: e4m3 activations, e4m3-expanded prefill weights
   L->f32w = cfg->wtype == MOE_W_F32;
   L->act_bytes = L->fp8 ? 1 : 2;
   L->max_tokens = cfg->max_tokens;
@@ -350,15 +355,50 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
     C_TRY(cudaMemcpy(L->gate_bias, w->gate_bias, (size_t)L->E_glob * 4, cudaMemcpyDeviceToDevice));
   }
   // ---- routed experts ----
+  // FP4 (e2m1, 2 per byte): the decode stream reads the packed codes (W13 rows in its tile
+  // order) through 16U4_ALIGN16B tensor maps; the prefill GEMMs run on the exact e4m3
+  // expansion of the same codes (e2m1 is a subset of e4m3; same power-of-two block scales)
+  struct Expand {
+    void *buf = nullptr;
+    ~Expand() { if (buf) cudaFree(buf); }
+  } ex13, ex2, exs13, exs2;
+  const void *src13 = w->w13, *src2 = w->w2, *srcs13 = w->ws13, *srcs2 = w->ws2;
+  if (L->fp4) {
+    C_TRY(dalloc(L, &L->w13_f4, (size_t)E * 2 * F * H / 2, true));
+    C_TRY(launch_permute_w13_rows(w->w13, L->w13_f4, E, F, H / 2, 0));
+    C_TRY(dalloc(L, &L->w2_f4, (size_t)E * H * F / 2, true));
+    C_TRY(cudaMemcpy(L->w2_f4, w->w2, (size_t)E * H * F / 2, cudaMemcpyDeviceToDevice));
+    C_TRY(cudaMalloc(&ex13.buf, (size_t)E * 2 * F * H));
+    C_TRY(launch_fp4_to_e4m3(w->w13, ex13.buf, (int64_t)E * 2 * F * H / 2, 0));
+    C_TRY(cudaMalloc(&ex2.buf, (size_t)E * H * F));
+    C_TRY(launch_fp4_to_e4m3(w->w2, ex2.buf, (int64_t)E * H * F / 2, 0));
+    src13 = ex13.buf; src2 = ex2.buf;
+    if (Fs > 0) {
+      C_TRY(dalloc(L, &L->ws13_f4, (size_t)2 * Fs * H / 2, true));
+      C_TRY(launch_permute_w13_rows(w->ws13, L->ws13_f4, 1, Fs, H / 2, 0));
+      C_TRY(dalloc(L, &L->ws2_f4, (size_t)H * Fs / 2, true));
+      C_TRY(cudaMemcpy(L->ws2_f4, w->ws2, (size_t)H * Fs / 2, cudaMemcpyDeviceToDevice));
+      C_TRY(cudaMalloc(&exs13.buf, (size_t)2 * Fs * H));
+      C_TRY(launch_fp4_to_e4m3(w->ws13, exs13.buf, (int64_t)Fs * H, 0));
+      C_TRY(cudaMalloc(&exs2.buf, (size_t)H * Fs));
+      C_TRY(launch_fp4_to_e4m3(w->ws2, exs2.buf, (int64_t)H * Fs / 2, 0));
+      srcs13 = exs13.buf; srcs2 = exs2.buf;
+    }
+    bool ok = make_fp4_map(&L->fmap_w13, L->w13_f4, (int64_t)E * 2 * F, H, 256) &&
+              make_fp4_map(&L->fmap_w2, L->w2_f4, (int64_t)E * H, F, 256);
+    if (Fs > 0)
+      ok = ok && make_fp4_map(&L->fmap_ws13, L->ws13_f4, 2 * Fs, H, 256) && make_fp4_map(&L->fmap_ws2, L->ws2_f4, H, Fs, 256);
+    if (!ok) return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for the FP4 weights"));
+  }
   C_TRY(dalloc(L, &L->w13, (size_t)E * 2 * F * H * wes, true));
   L->umma = !L->f32w && (H % 256 == 0);
   // tcgen05 path: weights repacked into 256-row x 128-byte SW128 tiles (one
   // contiguous 32 KB read per k-block); CUDA-core path: row-major, W13 interleaved
-  if (L->umma) C_TRY(launch_tile_weights(w->w13, L->w13, E, 2 * F, H * wes, F, 0));
-  else C_TRY(interleave_w13(w->w13, L->w13, E, F, H, wes));
+  if (L->umma) C_TRY(launch_tile_weights(src13, L->w13, E, 2 * F, H * wes, F, 0));
+  else C_TRY(interleave_w13(src13, L->w13, E, F, H, wes));
   C_TRY(dalloc(L, &L->w2, (size_t)E * H * F * wes, true));
-  if (L->umma) C_TRY(launch_tile_weights(w->w2, L->w2, E, H, F * wes, 0, 0));
-  else C_TRY(cudaMemcpy(L->w2, w->w2, (size_t)E * H * F * wes, cudaMemcpyDeviceToDevice));
+  if (L->umma) C_TRY(launch_tile_weights(src2, L->w2, E, H, F * wes, 0, 0));
+  else C_TRY(cudaMemcpy(L->w2, src2, (size_t)E * H * F * wes, cudaMemcpyDeviceToDevice));
   std::vector<float> hs13, hs2, hss13, hss2;
   if (L->fp8) {
     if (!L->umma) return cleanup(fail(MOE_ERR_UNSUPPORTED, "FP8 weights need hidden %% 256 == 0"));
@@ -367,11 +407,11 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   }
   if (Fs > 0) {
     C_TRY(dalloc(L, &L->ws13, (size_t)2 * Fs * H * wes, true));
-    if (L->umma) C_TRY(launch_tile_weights(w->ws13, L->ws13, 1, 2 * Fs, H * wes, Fs, 0));
-    else C_TRY(interleave_w13(w->ws13, L->ws13, 1, Fs, H, wes));
+    if (L->umma) C_TRY(launch_tile_weights(srcs13, L->ws13, 1, 2 * Fs, H * wes, Fs, 0));
+    else C_TRY(interleave_w13(srcs13, L->ws13, 1, Fs, H, wes));
     C_TRY(dalloc(L, &L->ws2, (size_t)H * Fs * wes, true));
-    if (L->umma) C_TRY(launch_tile_weights(w->ws2, L->ws2, 1, H, Fs * wes, 0, 0));
-    else C_TRY(cudaMemcpy(L->ws2, w->ws2, (size_t)H * Fs * wes, cudaMemcpyDeviceToDevice));
+    if (L->umma) C_TRY(launch_tile_weights(srcs2, L->ws2, 1, H, Fs * wes, 0, 0));
+    else C_TRY(cudaMemcpy(L->ws2, srcs2, (size_t)H * Fs * wes, cudaMemcpyDeviceToDevice));
     if (L->fp8) {
       S_TRY(load_scales(w->ws13_scale, &L->ws13_s, L, 1, 2 * Fs, H, true, "ws13_scale", &hss13));
       S_TRY(load_scales(w->ws2_scale, &L->ws2_s, L, 1, H, Fs, false, "ws2_scale", &hss2));
@@ -850,7 +890,7 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
                   L->gemv_max_tokens);
     if (prev) {
       if (prev == L) return fail(MOE_ERR_INVALID_ARG, "prev is this layer");
-      if (prev->H != L->H || prev->fp8 != L->fp8 || prev->cfg.device != L->cfg.device ||
+      if (prev->H != L->H || prev->fp8 != L->fp8 || prev->fp4 != L->fp4 || prev->cfg.device != L->cfg.device ||
           prev->tp_size != L->tp_size || prev->tp_rank != L->tp_rank || !prev->fused_decode || prev->ep.P > 1)
         return fail(MOE_ERR_INVALID_ARG, "prev has another shape / dtype / device / TP split");
       if (prev->chain_T != T || prev->chain_ndef <= 0)
@@ -951,6 +991,7 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     auto routed = [&](FdGroup &g, const moe_layer *S, const int32_t *list, const int32_t *n_list, int a0, int a1,
                       int a2) {
       g.x_map = S->fp8 ? S->dmap_xq : S->dmap_xc;
+      if (S->fp4) { g.w13_map4 = S->fmap_w13; g.w2_map4 = S->fmap_w2; }
       g.w13 = (const uint8_t *)S->w13; g.w13_s = S->w13_s; g.xs = S->xs;
       g.w2 = (const uint8_t *)S->w2; g.w2_s = S->w2_s; g.nch = S->F / 128;
       g.list = list; g.n_list = n_list; g.topk_idx = S->topk_idx; g.topk_w = S->topk_w; g.k = S->k; g.e0 = S->e0;
@@ -964,6 +1005,7 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     if (Fs > 0) {
       FdGroup &g = fp.g[1];
       g.x_map = f8 ? L->dmap_xq : L->dmap_xc;
+      if (L->fp4) { g.w13_map4 = L->fmap_ws13; g.w2_map4 = L->fmap_ws2; }
       g.w13 = (const uint8_t *)L->ws13; g.w13_s = L->ws13_s; g.xs = L->xs;
       g.w2 = (const uint8_t *)L->ws2; g.w2_s = L->ws2_s; g.nch = Fs / 128;
     } else {
@@ -998,7 +1040,7 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
       csize = cluster_override;                  // (cluster ids stay within the scratch slots)
     fp.cl_scratch = L->cl_scratch;
     const int grid = csize > 1 ? units * csize : std::min(L->num_sms, units);
-    KL_TRY(launch_umma_decode_fused(f8, fp, grid, csize, st));
+    KL_TRY(launch_umma_decode_fused(f8, L->fp4, fp, grid, csize, st));
     mark(L, ST_GEMM1, st);
     if (A.chained) { L->chain_T = n_def > 0 ? T : -1; L->chain_ndef = n_def; }
     else L->chain_T = -1;

@@ -199,6 +199,11 @@ __device__ __forceinline__ void st_async_v4f32(uint32_t cluster_addr, float a, f
                "f"(a), "f"(b), "f"(c), "f"(d), "r"(cluster_mbar)
                : "memory");
 }
+__device__ __forceinline__ void st_async_v2f32(uint32_t cluster_addr, float a, float b, uint32_t cluster_mbar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v2.f32 [%0], {%1, %2}, [%3];" ::"r"(cluster_addr),
+               "f"(a), "f"(b), "r"(cluster_mbar)
+               : "memory");
+}
 __device__ __forceinline__ void st_async_v4u32(uint32_t cluster_addr, uint4 v, uint32_t cluster_mbar) {
   asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
                    cluster_addr),

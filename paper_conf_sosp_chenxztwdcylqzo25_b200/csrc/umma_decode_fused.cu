@@ -61,9 +61,18 @@ constexpr uint32_t FD_TMEM_COLS = 256;
 constexpr uint32_t FD_ACCA_COL = 0, FD_ACCB_COL = 128;   // + 32 per ring slot (two 16-column MMA tiles)
 static_assert(FD_ACCA_SLOTS * 32 <= (int)FD_ACCB_COL && FD_ACCB_COL + FD_ACCB * 32 <= FD_TMEM_COLS, "TMEM map");
 
-// instruction descriptor, kind::f8f6f4 (E4M3 x E4M3 -> F32, no block scale), K-major A and B
-__host__ __device__ constexpr uint32_t idesc_f8(int M, int N) {
-  return (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+// instruction descriptor, kind::f8f6f4 (A E4M3 or E2M1 (a_fmt 5), B E4M3 -> F32, no block scale), K-major A and B
+__host__ __device__ constexpr uint32_t idesc_f8(int M, int N, uint32_t a_fmt = 0) {
+  return (1u << 4) | (a_fmt << 7) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+// TMA tile load with an L2 cache-policy hint (FP4 weights: unpacked to 16-byte
+// aligned 4-bit groups in shared memory by the tensor map's 16U4_ALIGN16B type)
+__device__ __forceinline__ void tma_load_2d_hint(void *dst, const void *map, uint64_t *bar, int c0, int c1, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1, {%2, %3}], [%4], %5;" ::
+          "r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_u32(bar)), "l"(pol)
+      : "memory");
 }
 __device__ __forceinline__ void mma_f8(uint32_t d_tmem, uint64_t a_desc, uint64_t b_desc, uint32_t idesc,
                                        uint32_t accumulate) {
@@ -84,6 +93,10 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
 
 // 128-column chunks of a group this kernel streams
 __device__ __forceinline__ int fd_units_per_expert(const FdGroup &g) { return g.nch; }
+
+// cluster split: the peers' fp32 partials fit the leader's 8 KB exchange buffer
+// ((csize - 1) peers x 128 threads x 2T floats) -> st.async into its shared memory
+__device__ __forceinline__ bool fd_dsmem_partials(uint32_t csize, int T) { return (int)(csize - 1) * T <= 8; }
 
 // unit -> (valid, group, expert, chunk).  Group 2 first (no dependency on this
 // layer's router), then the shared expert (group 1), then the routed experts.
@@ -161,8 +174,13 @@ __device__ __forceinline__ void decode_finalize_range(const DecodeFinalizeArgs &
   }
 }
 
-template <bool FP8>
+// W4: 4-bit (e2m1) expert weights -- streamed packed (half the bytes), unpacked by the
+// TMA into the e4m3 tile geometry, consumed by the same kind::f8f6f4 MMA (A = E2M1)
+template <bool FP8, bool W4>
 __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const __grid_constant__ FusedDecodeParams p) {
+  static_assert(!W4 || FP8, "4-bit weights take e4m3 activations");
+  constexpr uint32_t A_TX = W4 ? FD_A_BYTES / 2 : FD_A_BYTES;   // global bytes of one weight k-block
+  constexpr uint32_t A_FMT = W4 ? 5u : 0u;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t *sA = smem;
@@ -202,7 +220,8 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     // a queue slot is free when the MMA warp and the 4 epilogue warps here and the
     // producer, MMA and epilogue warps of every peer have read it
     for (int i = 0; i < FD_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], 5 + 6 * (csize - 1)); }
-    mbar_init(part_bar, 4 * (csize - 1) > 0 ? 4 * (csize - 1) : 1);
+    // partials through the leader's shared memory (st.async; small T) or through L2
+    mbar_init(part_bar, (csize > 1 && !fd_dsmem_partials(csize, p.T)) ? 4 * (csize - 1) : 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc(tmem_base_smem, FD_TMEM_COLS);
@@ -272,8 +291,12 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         const uint8_t *w13 = g.w13 + ((size_t)ui.expert * g.nch + ui.chunk) * (size_t)KA * FD_A_BYTES;
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          mbar_expect_tx(&full[stage], FD_A_BYTES + FD_B_BYTES);
-          bulk_load_hint(sA + stage * FD_A_BYTES, w13 + (size_t)kb * FD_A_BYTES, FD_A_BYTES, &full[stage], pol);
+          mbar_expect_tx(&full[stage], A_TX + FD_B_BYTES);
+          if (W4)
+            tma_load_2d_hint(sA + stage * FD_A_BYTES, &g.w13_map4, &full[stage], kb * 128,
+                             (ui.expert * g.nch + ui.chunk) * 256, pol);
+          else
+            bulk_load_hint(sA + stage * FD_A_BYTES, w13 + (size_t)kb * FD_A_BYTES, FD_A_BYTES, &full[stage], pol);
           tma_load_2d(sB + stage * FD_B_BYTES, &g.x_map, &full[stage], kb * KDIV, 0);
           if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
         }
@@ -283,9 +306,13 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         for (int n = nt0; n < nt1; ++n) {
           for (int kk = 0; kk < KBC; ++kk) {
             mbar_wait(&empty[stage], phase ^ 1);
-            mbar_expect_tx(&full[stage], FD_A_BYTES);
-            bulk_load_hint(sA + stage * FD_A_BYTES, w2 + ((size_t)n * KB2 + ui.chunk * KBC + kk) * FD_A_BYTES,
-                           FD_A_BYTES, &full[stage], pol);
+            mbar_expect_tx(&full[stage], A_TX);
+            if (W4)
+              tma_load_2d_hint(sA + stage * FD_A_BYTES, &g.w2_map4, &full[stage], ui.chunk * 128,
+                               ui.expert * p.H + n * 256, pol);
+            else
+              bulk_load_hint(sA + stage * FD_A_BYTES, w2 + ((size_t)n * KB2 + ui.chunk * KBC + kk) * FD_A_BYTES,
+                             FD_A_BYTES, &full[stage], pol);
             if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
           }
         }
@@ -334,7 +361,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
             for (int t = 0; t < 2; ++t) {
               const uint64_t ad = sw128_kmajor_desc(a0 + t * 128 * 128 + k * 32);
               if (FP8)
-                mma_f8(tmem + FD_ACCA_COL + as * 32 + t * 16, ad, bd, idesc_f8(128, FD_N), k != 0);
+                mma_f8(tmem + FD_ACCA_COL + as * 32 + t * 16, ad, bd, idesc_f8(128, FD_N, A_FMT), k != 0);
               else   // the accumulator is free: the epilogue read it before h_ready of the previous unit
                 mma_bf16(tmem + FD_ACCA_COL + t * 16, ad, bd, idesc_bf16(128, FD_N), (kb != kb0) || (k != 0));
             }
@@ -369,7 +396,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
               for (int t = 0; t < 2; ++t) {
                 const uint64_t ad = sw128_kmajor_desc(a0 + t * 128 * 128 + k * 32);
                 const uint32_t d = tmem + FD_ACCB_COL + ab * 32 + t * 16;
-                if (FP8) mma_f8(d, ad, bd, idesc_f8(128, FD_N), accum);
+                if (FP8) mma_f8(d, ad, bd, idesc_f8(128, FD_N, A_FMT), accum);
                 else mma_bf16(d, ad, bd, idesc_bf16(128, FD_N), accum);
               }
             }
@@ -519,15 +546,25 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       if (csize > 1) {
         // ---- cluster: the peers' partial gate/up sums -> the leader (through L2) ----
         float *scr = p.cl_scratch + (size_t)cluster_id_x() * 7 * 128 * 32;
+        const bool dsm = fd_dsmem_partials(csize, p.T);
         if (!leader) {
-          float4 *dst = reinterpret_cast<float4 *>(scr + ((size_t)(crank - 1) * 128 + et) * 32);
+          if (dsm) {
+            // (token t of this thread's two rows) -> the leader's xch [peer][thread][2T]
+            float *dst = xch + ((size_t)(crank - 1) * 128 + et) * 2 * p.T;
+            const uint32_t bar = map_to_rank(part_bar, 0);
 #pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            __stcg(dst + j, make_float4(r0[4 * j], r0[4 * j + 1], r0[4 * j + 2], r0[4 * j + 3]));
-            __stcg(dst + 4 + j, make_float4(r1[4 * j], r1[4 * j + 1], r1[4 * j + 2], r1[4 * j + 3]));
+            for (int t = 0; t < FD_N; ++t)
+              if (t < p.T) st_async_v2f32(map_to_rank(dst + 2 * t, 0), r0[t], r1[t], bar);
+          } else {
+            float4 *dst = reinterpret_cast<float4 *>(scr + ((size_t)(crank - 1) * 128 + et) * 32);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              __stcg(dst + j, make_float4(r0[4 * j], r0[4 * j + 1], r0[4 * j + 2], r0[4 * j + 3]));
+              __stcg(dst + 4 + j, make_float4(r1[4 * j], r1[4 * j + 1], r1[4 * j + 2], r1[4 * j + 3]));
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive_cluster(map_to_rank(part_bar, 0));   // release.cluster
           }
-          __syncwarp();
-          if (lane == 0) mbar_arrive_cluster(map_to_rank(part_bar, 0));   // release.cluster
           // h_c of this unit comes from the leader (st.async into sH / hsc, complete_tx on h_ready)
           if (q == 0 && lane == 0) mbar_expect_tx(h_ready, H_TX);
           mbar_wait(h_ready, hph_e);
@@ -535,9 +572,21 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
           if (tr) tr[4] = gtimer();
           goto phase_b;
         }
-        mbar_wait_cluster(part_bar, pph);
-        pph ^= 1;
-        for (uint32_t r = 1; r < csize; ++r) {
+        if (dsm) {
+          if (q == 0 && lane == 0) mbar_expect_tx(part_bar, (csize - 1) * 128 * 2 * p.T * 4);
+          mbar_wait_cluster(part_bar, pph);
+          pph ^= 1;
+          for (uint32_t r = 1; r < csize; ++r) {
+            const float *src = xch + ((size_t)(r - 1) * 128 + et) * 2 * p.T;
+#pragma unroll
+            for (int t = 0; t < FD_N; ++t)
+              if (t < p.T) { r0[t] += src[2 * t]; r1[t] += src[2 * t + 1]; }
+          }
+          asm volatile("bar.sync 1, 128;" ::: "memory");   // xch is the SwiGLU exchange buffer next
+        }
+        if (!dsm) mbar_wait_cluster(part_bar, pph);
+        if (!dsm) pph ^= 1;
+        for (uint32_t r = 1; r < (dsm ? 1u : csize); ++r) {
           const float4 *src = reinterpret_cast<const float4 *>(scr + ((size_t)(r - 1) * 128 + et) * 32);
           float4 v[8];
 #pragma unroll
@@ -692,9 +741,9 @@ __global__ void decode_finalize_kernel(const __grid_constant__ DecodeFinalizeArg
   if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) a.trace[2001] = gtimer();
 }
 
-template <bool FP8>
+template <bool FP8, bool W4>
 static cudaError_t fd_launch(const FusedDecodeParams &p, int grid, int csize, cudaStream_t st) {
-  auto k = umma_decode_fused_kernel<FP8>;
+  auto k = umma_decode_fused_kernel<FP8, W4>;
   cudaError_t e = set_kernel_attr((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FD_SMEM);
   if (e == cudaSuccess && csize > 1)
     e = set_kernel_attr((const void *)k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
@@ -719,14 +768,16 @@ static cudaError_t fd_launch(const FusedDecodeParams &p, int grid, int csize, cu
   return cudaLaunchKernelEx(&cfg, k, p);
 }
 
-cudaError_t launch_umma_decode_fused(bool fp8, const FusedDecodeParams &p, int grid, int csize, cudaStream_t st) {
+cudaError_t launch_umma_decode_fused(bool fp8, bool w4, const FusedDecodeParams &p, int grid, int csize,
+                                     cudaStream_t st) {
   if (grid <= 0) return cudaSuccess;
-  return fp8 ? fd_launch<true>(p, grid, csize, st) : fd_launch<false>(p, grid, csize, st);
+  if (w4) return fd_launch<true, true>(p, grid, csize, st);
+  return fp8 ? fd_launch<true, false>(p, grid, csize, st) : fd_launch<false, false>(p, grid, csize, st);
 }
 
 // clusters of `csize` fused-decode CTAs that can be resident at once (0 if none)
 int fused_decode_max_clusters(bool fp8, int csize) {
-  const void *k = fp8 ? (const void *)umma_decode_fused_kernel<true> : (const void *)umma_decode_fused_kernel<false>;
+  const void *k = fp8 ? (const void *)umma_decode_fused_kernel<true, false> : (const void *)umma_decode_fused_kernel<false, false>;
   if (set_kernel_attr(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FD_SMEM) != cudaSuccess) return 0;
   if (csize > 8 && set_kernel_attr(k, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) != cudaSuccess) return 0;
   cudaLaunchConfig_t cfg{};

@@ -286,6 +286,58 @@ bool make_blocks_map(CUtensorMap *m, const void *base, int64_t total_bytes, int 
   return r == CUDA_SUCCESS;
 }
 
+bool make_fp4_map(CUtensorMap *m, const void *base, int64_t rows, int64_t cols, int box_rows) {
+  auto enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)(cols / 2)};
+  cuuint32_t box[2] = {128, (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_16U4_ALIGN16B, 2, const_cast<void *>(base), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+// e2m1 code -> e4m3 byte: magnitudes 0, .5, 1, 1.5, 2, 3, 4, 6 are e4m3 values exactly
+__global__ void fp4_to_e4m3_kernel(const uint8_t *__restrict__ in, uint16_t *__restrict__ out, int64_t n) {
+  const uint8_t lut[8] = {0x00, 0x30, 0x38, 0x3C, 0x40, 0x44, 0x48, 0x4C};
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint8_t b = in[i];
+    const uint8_t lo = b & 0xF, hi = b >> 4;
+    const uint16_t e0 = lut[lo & 7] | ((lo & 8) << 4), e1 = lut[hi & 7] | ((hi & 8) << 4);
+    out[i] = (uint16_t)(e0 | (e1 << 8));          // element 2i (low nibble) first
+  }
+}
+
+cudaError_t launch_fp4_to_e4m3(const void *packed, void *out, int64_t n_bytes_in, cudaStream_t st) {
+  if (n_bytes_in <= 0) return cudaSuccess;
+  fp4_to_e4m3_kernel<<<148 * 8, 256, 0, st>>>(reinterpret_cast<const uint8_t *>(packed),
+                                             reinterpret_cast<uint16_t *>(out), n_bytes_in);
+  return cudaGetLastError();
+}
+
+// dst row (e, nb, r) <- src row of W1 / W3 with the swap-AB tile interleave (tile_weights_kernel)
+__global__ void permute_w13_rows_kernel(const uint8_t *__restrict__ src, uint8_t *__restrict__ dst, int nexp, int F,
+                                        int row_bytes) {
+  const int64_t chunks = (int64_t)row_bytes / 16, total = (int64_t)nexp * 2 * F * chunks;
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < total; c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t row = c / chunks, j = c % chunks;
+    const int64_t e = row / (2 * F);
+    const int rr = (int)(row % (2 * F)), nb = rr / 256, r = rr % 256;
+    const int h = r >> 7, q = (r >> 5) & 3, i = r & 31;
+    const int f = nb * 128 + h * 64 + (q >> 1) * 32 + i;
+    const int64_t srow = e * 2 * F + ((q & 1) ? F + f : f);
+    reinterpret_cast<uint4 *>(dst + row * row_bytes)[j] = reinterpret_cast<const uint4 *>(src + srow * row_bytes)[j];
+  }
+}
+
+cudaError_t launch_permute_w13_rows(const void *src, void *dst, int nexp, int F, int row_bytes, cudaStream_t st) {
+  permute_w13_rows_kernel<<<148 * 8, 256, 0, st>>>(reinterpret_cast<const uint8_t *>(src), reinterpret_cast<uint8_t *>(dst),
+                                                  nexp, F, row_bytes);
+  return cudaGetLastError();
+}
+
 // 2-D row-major [rows, cols] K-major operand, box = (128 bytes of K, box_rows), 128B swizzle
 bool make_kmajor_map(CUtensorMap *m, const void *base, bool fp8, int64_t rows, int64_t cols, int box_rows) {
   auto enc = get_encode();

@@ -20,7 +20,7 @@ STATUS = {0: "MOE_OK", -1: "MOE_ERR_INVALID_ARG", -2: "MOE_ERR_UNSUPPORTED", -3:
           -4: "MOE_ERR_CUDA", -5: "MOE_ERR_NCCL", -6: "MOE_ERR_CAPACITY"}
 SCORE_SOFTMAX, SCORE_SIGMOID = 0, 1
 GROUP_MAX, GROUP_TOP2_SUM = 0, 1
-W_BF16, W_FP8, W_F32 = 0, 1, 2
+W_BF16, W_FP8, W_F32, W_FP4 = 0, 1, 2, 3
 
 EXPORTED = ["moe_ep_group_forward", "moe_get_unique_id", "moe_layer_create", "moe_layer_forward", "moe_layer_forward_deferred",
             "moe_layer_forward_chained", "moe_tp_group_forward", "moe_layer_destroy", "moe_status_string",
@@ -260,8 +260,9 @@ def slice_tp(weights, rank: int, tp_size: int, ffn: int, shared_ffn: int):
 
     w = copy.copy(weights)
     c0, c1 = cols(ffn)
+    pk = 2 if weights.w2.shape[-1] * 2 == ffn else 1        # FP4: W2 columns are packed 2 per byte
     w.w13 = torch.cat([weights.w13[:, c0:c1], weights.w13[:, ffn + c0:ffn + c1]], dim=1).contiguous()
-    w.w2 = weights.w2[:, :, c0:c1].contiguous()
+    w.w2 = weights.w2[:, :, c0 // pk:c1 // pk].contiguous()
     if weights.w13_scale is not None:
         b0, b1, fb = c0 // 128, c1 // 128, ffn // 128
         w.w13_scale = torch.cat([weights.w13_scale[:, b0:b1], weights.w13_scale[:, fb + b0:fb + b1]], dim=1).contiguous()
@@ -269,7 +270,7 @@ def slice_tp(weights, rank: int, tp_size: int, ffn: int, shared_ffn: int):
     if shared_ffn and weights.ws13 is not None:
         s0, s1 = cols(shared_ffn)
         w.ws13 = torch.cat([weights.ws13[s0:s1], weights.ws13[shared_ffn + s0:shared_ffn + s1]], dim=0).contiguous()
-        w.ws2 = weights.ws2[:, s0:s1].contiguous()
+        w.ws2 = weights.ws2[:, s0 // pk:s1 // pk].contiguous()
         if weights.ws13_scale is not None:
             b0, b1, fb = s0 // 128, s1 // 128, shared_ffn // 128
             w.ws13_scale = torch.cat([weights.ws13_scale[b0:b1], weights.ws13_scale[fb + b0:fb + b1]],

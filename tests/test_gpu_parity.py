@@ -69,7 +69,7 @@ def test_small_layer_parity(lib, name):
     check_output(f"small/{name}/T{T}", res["y"], out["y"], TOL[p.wtype], ties=len(ties))
 
 
-@pytest.mark.parametrize("name", ["toy", "v3_s", "v2lite_s", "v2lite_h384"])
+@pytest.mark.parametrize("name", ["toy", "v3_s", "v2lite_s", "v2lite_h384", "v3_s_fp4"])
 @pytest.mark.parametrize("T", [1, 3, 17])
 def test_small_decode_shapes(lib, name, T):
     p = SMALL[name]
@@ -175,7 +175,7 @@ def _full(lib, name, T, n_def=0, sample=6, rows=None, min_experts=0):
 
 
 @pytest.mark.parametrize("name,T", [("v3", 1), ("v25", 4), ("v2lite", 1), ("v2lite", 512), ("qwen2", 2048),
-                                    ("qwen2", 1), ("v3", 16)])
+                                    ("qwen2", 1), ("v3", 16), ("v3_fp4", 1), ("v3_fp4", 16)])
 def test_full_size(lib, name, T):
     _full(lib, name, T, sample=8 if T > 1 else 1)
 
@@ -208,19 +208,20 @@ def test_full_v3_decode_deferral(lib):
     _full(lib, "v3", 1, n_def=3, sample=1)
 
 
+@pytest.mark.parametrize("name", ["v3_m", "v3_m_fp4"])
 @pytest.mark.parametrize("T", [1, 16, 300])
-def test_mid_size_fp8_elementwise(lib, T):
+def test_mid_size_fp8_elementwise(lib, name, T):
     """Mid-size FP8 preset (H = 2048, F = 1024: 16 W13 k-blocks = 4 scale groups,
     8 W2 k-blocks = 2 groups, so both TMEM scale-column sets of the swap GEMM and
     the fused decode stream are used) compared element by element on all tokens."""
-    p = SMALL["v3_m"]
+    p = SMALL[name]
     res = _run(lib, p, T, max_tokens=max(T, 16))
     out, ties, idx, w = _oracle(p, res)
     g = res["routing"]
     check_tie_fraction(ties, T)
     check_routing(g["topk_idx"], g["topk_w"], idx, w, ties, p.routed_scale, p.norm_topk)
     check_permutation(g["expert_counts"], g["perm"], idx, p.n_experts)
-    check_output(f"mid/v3_m/T{T}", res["y"], out["y"], TOL[p.wtype], ties=len(ties))
+    check_output(f"mid/{name}/T{T}", res["y"], out["y"], TOL[p.wtype], ties=len(ties))
 
 
 @pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v3_m"])

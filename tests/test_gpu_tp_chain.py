@@ -31,7 +31,7 @@ def _din(T, H, seed=7):
 
 # ------------------------------------------------------------------ expert TP
 @pytest.mark.parametrize("name,P", [("v3_s", 2), ("qwen2_s", 2), ("v25_s", 2), ("v2lite_s", 2), ("v2lite_s", 3),
-                                    ("v3_m", 4), ("v3_m", 3)])
+                                    ("v3_m", 4), ("v3_m", 3), ("v3_m_fp4", 4)])
 @pytest.mark.parametrize("T", [1, 6, 16])
 def test_tp_group_matches_oracle(lib, name, P, T):
     """Every rank's y (and deferred_out) equals the whole layer's (Eq. L241 middle
@@ -129,7 +129,7 @@ def _chain_oracle(p, ws, xs, rs, n_defs):
     return outs, sorted(ties)
 
 
-@pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v2lite_s", "v3_m", "v25_s"])
+@pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v2lite_s", "v3_m", "v25_s", "v3_s_fp4"])
 @pytest.mark.parametrize("T", [1, 5, 16])
 def test_chained_deferral_matches_eq_L241(lib, name, T):
     """A 3-layer chain (k = 1: no deferred input; k = L: n_def = 0) against Eq.
