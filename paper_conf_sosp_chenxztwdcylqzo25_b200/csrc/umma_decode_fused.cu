@@ -386,6 +386,15 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         for (int kk = 0; kk < KBC; ++kk) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
+          if (kExperiments && (p.debug & 8)) {   // timing experiment: phase-B loads only (no MMAs)
+            if (lane == 0) {
+              mbar_arrive(&empty[stage]);
+              if (kk == KBC - 1) mbar_arrive(&accB_full[ab]);
+            }
+            __syncwarp();
+            if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
+            continue;
+          }
           if (lane == 0) {
             const uint32_t a0 = smem_u32(sA + stage * FD_A_BYTES);
 #pragma unroll
@@ -683,6 +692,12 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       for (int nt = nt0; nt < nt1; ++nt) {
         mbar_wait(&accB_full[ab], abph);
         tc_fence_after();
+        if (kExperiments && (p.debug & 4)) {     // timing experiment: no phase-B epilogue work
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&accB_empty[ab]);
+          if (++ab == FD_ACCB) { ab = 0; abph ^= 1; }
+          continue;
+        }
         uint32_t v0[16], v1[16];
         tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCB_COL + ab * 32, v0);
         tmem_ld_32x32b_x16(tmem + lane_base + FD_ACCB_COL + ab * 32 + 16, v1);
