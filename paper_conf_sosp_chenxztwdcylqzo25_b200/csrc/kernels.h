@@ -118,6 +118,8 @@ struct RouteSmallArgs {
   void *xq; float *xs;
   void *xcopy;
   unsigned long long *trace;     // MOE_DEBUG_TRACE: [0] CTA 0 entry, [1..4] tail start / select / permute / end
+  int early_trigger;            // let the decode stream launch at once (it has the previous layer's deferred
+                                // units to stream meanwhile); else only when routing is complete
   // The tail writes the active-expert list (p.act_list: any slot) and, for chained
   // Expert Deferral, the experts of the immediate slots [0, n_imm) and of the
   // deferred slots [n_imm, k) (ascending local ids); the full counts and
@@ -247,6 +249,7 @@ struct FusedDecodeParams {
   unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
   int debug;                    // MOE_EXPERIMENTS builds (MOE_DEBUG_FD): 1 no phase-A fold, 2 no phase-A MMAs
   float *cl_scratch;            // cluster split: [clusters][7][128][32] fp32 partials of the peers (L2)
+  int ts;                       // FP8 weights: MMA A operand staged in TMEM (TS form) instead of read from smem
 };
 // csize > 1: clusters of csize CTAs share each unit (the cluster split)
 cudaError_t launch_umma_decode_fused(bool fp8, bool w4, const FusedDecodeParams &p, int grid, int csize,

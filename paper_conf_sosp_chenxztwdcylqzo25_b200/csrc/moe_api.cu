@@ -947,6 +947,7 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     if (L->fp8) { rs.xq = L->xq; rs.xs = L->xs; }
     else rs.xcopy = L->xcopy;
     rs.n_imm = A.chained ? k - n_def : k;
+    rs.early_trigger = prev != nullptr;
     rs.imm_list = L->imm_list; rs.def_list = L->def_list; rs.n_imm_list = L->n_lists; rs.n_def_list = L->n_lists + 1;
     KL_TRY(launch_route_small(rs, st));
     mark(L, ST_PERMUTE, st);
@@ -1039,6 +1040,8 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     if (cluster_override > 0 && units <= L->fd_max_clusters[2] && cluster_override <= std::min(KA, NT))
       csize = cluster_override;                  // (cluster ids stay within the scratch slots)
     fp.cl_scratch = L->cl_scratch;
+    static const int ts_off = experiment_knob("MOE_FD_SS");   // A/B: the SS form (A read from smem)
+    fp.ts = !ts_off;
     const int grid = csize > 1 ? units * csize : std::min(L->num_sms, units);
     KL_TRY(launch_umma_decode_fused(f8, L->fp4, fp, grid, csize, st));
     mark(L, ST_GEMM1, st);

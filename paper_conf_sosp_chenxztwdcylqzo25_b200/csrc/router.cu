@@ -547,9 +547,10 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
     const int e = (threadIdx.x & 31) * 8 + i;
     bpre[i] = (r.bias && e < r.E) ? __ldg(r.bias + e) : 0.f;
   }
-  // the decode stream may launch now: its CTAs become resident beside ours (no launch gap after
-  // routing); MOE_DEBUG_ROUTE bit 16 (experiments): launch it only when routing is complete
-  if (!(kExperiments && (a.debug & 16))) pdl_trigger();
+  // chained deferral: the decode stream may launch now and stream the previous layer's deferred
+  // experts beside us; otherwise it launches when every CTA here has exited (measured ~1 us/layer
+  // faster: CTAs waiting in griddepcontrol.wait beside ours slow the routing down)
+  if (a.early_trigger) pdl_trigger();
   pdl_wait();                                    // x (the previous layer's output) and our workspaces
   if (a.trace && threadIdx.x == 0 && blockIdx.x == 0) a.trace[0] = gtimer_ns();
   // ---- logits of router rows `row` for all T tokens ----
