@@ -249,7 +249,8 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     mbar_init(&a_free[1], 1);
     fence_barrier_init();
   }
-  if (warp == 1) tmem_alloc(tmem_base_smem, FD_TMEM_COLS);
+  const uint32_t tmem_cols = p.ts ? FD_TMEM_COLS : FD_ASTAGE_COL;   // the TS stage only when used
+  if (warp == 1) tmem_alloc(tmem_base_smem, tmem_cols);
   tc_fence_before();
   __syncthreads();
   if (csize > 1) cluster_sync();                 // every barrier of the cluster initialised
@@ -784,7 +785,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   tc_fence_before();
   __syncthreads();
   if (csize > 1) cluster_sync();                 // no CTA leaves while a peer may still st.async into it
-  if (warp == 1) tmem_dealloc(tmem, FD_TMEM_COLS);
+  if (warp == 1) tmem_dealloc(tmem, tmem_cols);
   if (threadIdx.x == 0) {
     // the last CTA out re-arms the work counter for the next forward (graph replay)
     asm volatile("fence.acq_rel.gpu;" ::: "memory");
