@@ -182,6 +182,8 @@ struct moe_layer {
   int k, H, F, Fs;
   bool fp8, f32w;
   bool fp4 = false;   // 4-bit (e2m1) expert weights: decode streams the packed codes
+  bool scale_nonpow2 = false;   // some FP8 block scale is not a power of two (decode-only layer)
+  char nonpow2_what[96] = {};
   int act_bytes;  // bytes per activation element fed to the expert GEMMs (1 fp8, 2 bf16)
   int max_tokens;
   int gemv_max_tokens;

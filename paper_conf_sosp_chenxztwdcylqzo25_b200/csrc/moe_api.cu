@@ -128,17 +128,22 @@ cudaError_t interleave_w13(const void *src, void *dst, int nexp, int F, int H, i
   return cudaSuccess;
 }
 
-// scales: copy to host, check powers of two, optionally interleave like W13
+// scales: copy to host, check them (positive, finite; note any that is not a power of
+// two -- the prefill GEMMs take UE8M0 scales only), optionally interleave like W13
 moe_status load_scales(const float *src, float **dst, moe_layer *L, int nexp, int rows, int cols, bool inter,
                        const char *name, std::vector<float> *host_out = nullptr) {
   const int rb = rows / 128, cb = cols / 128;
   const size_t n = (size_t)nexp * rb * cb;
   std::vector<float> h(n), o(n);
   CUDA_TRY(cudaMemcpy(h.data(), src, n * sizeof(float), cudaMemcpyDeviceToHost));
-  for (size_t i = 0; i < n; ++i)
-    if (!is_pow2(h[i]))
-      return fail(MOE_ERR_UNSUPPORTED, "%s[%zu] = %g is not a power of two (UE8M0 block scales only, DESIGN.md R10)",
-                  name, i, (double)h[i]);
+  for (size_t i = 0; i < n; ++i) {
+    if (!(h[i] > 0.f) || !std::isfinite(h[i]))
+      return fail(MOE_ERR_INVALID_ARG, "%s[%zu] = %g is not a positive finite scale", name, i, (double)h[i]);
+    if (!is_pow2(h[i]) && !L->scale_nonpow2) {
+      L->scale_nonpow2 = true;
+      snprintf(L->nonpow2_what, sizeof L->nonpow2_what, "%s[%zu] = %g", name, i, (double)h[i]);
+    }
+  }
   if (inter) {
     const int half = rb / 2;
     for (int e = 0; e < nexp; ++e)
@@ -571,6 +576,16 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
           return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for the decode x copy"));
       }
     }
+  }
+  if (L->scale_nonpow2) {
+    // arbitrary fp32 block scales (e.g. the released DeepSeek-V3/V2.5 FP8 checkpoints' weight_scale_inv):
+    // the decode stream applies the weight scales in its epilogues (any fp32 value is exact there);
+    // the prefill GEMMs' block-scaled MMAs take UE8M0 (power-of-two) scales only
+    if (!(L->fused_decode && L->E_glob <= 256 && cfg->ep_size == 1 && cfg->max_tokens <= L->gemv_max_tokens))
+      return cleanup(fail(MOE_ERR_UNSUPPORTED,
+                          "%s is not a power of two: non-UE8M0 block scales are served by the decode stream only "
+                          "(max_tokens <= %d, no expert parallelism); the prefill GEMMs need UE8M0 scales "
+                          "(DESIGN.md R10)", L->nonpow2_what, L->gemv_max_tokens));
   }
   if (L->tp_size > 1) {
     if (!L->fused_decode) return cleanup(fail(MOE_ERR_UNSUPPORTED, "expert TP needs the fused decode stream"));

@@ -23,7 +23,10 @@ def lib():
 
 
 def _run(lib, p, T, n_def=0, with_deferred_in=False, residual=False, max_tokens=None, gemv=0, seed_off=0):
-    w_cpu = make_weights(p, "cpu")
+    return _run_w(lib, p, make_weights(p, "cpu"), T, n_def, with_deferred_in, residual, max_tokens, gemv, seed_off)
+
+
+def _run_w(lib, p, w_cpu, T, n_def=0, with_deferred_in=False, residual=False, max_tokens=None, gemv=0, seed_off=0):
     x_cpu, r_cpu = make_tokens(p, T, "cpu", offset=seed_off)
     w = w_cpu.to("cuda")
     layer = lib.MoELayer(p, w, max_tokens=max_tokens or max(T, 1), gemv_max_tokens=gemv)
@@ -121,13 +124,35 @@ def test_zero_tokens_and_capacity(lib):
     assert e.value.status == -1
 
 
-def test_non_pow2_scales_rejected(lib):
+def test_non_pow2_scales_prefill_rejected(lib):
+    """The prefill GEMMs' block-scaled MMAs take UE8M0 scales only (reading R10): a layer
+    that can run prefill (max_tokens > the decode limit) refuses other fp32 scales."""
     p = SMALL["v3_s"]
     w = make_weights(p, "cpu")
     w.w13_scale[0, 0, 0] = 0.3
     with pytest.raises(lib.MoEError) as e:
-        lib.MoELayer(p, w.to("cuda"), max_tokens=8)
+        lib.MoELayer(p, w.to("cuda"), max_tokens=64)
     assert e.value.status == -2
+    w.w13_scale[0, 0, 0] = -1.0
+    with pytest.raises(lib.MoEError) as e:
+        lib.MoELayer(p, w.to("cuda"), max_tokens=8)
+    assert e.value.status == -1
+
+
+@pytest.mark.parametrize("name", ["v3_s", "v3_m"])
+@pytest.mark.parametrize("T", [1, 7, 16])
+def test_non_pow2_scales_decode(lib, name, T):
+    """Arbitrary fp32 128x128 block scales (the released DeepSeek-V3/V2.5 FP8 checkpoints
+    store weight_scale_inv as plain fp32): a decode-only layer (max_tokens <= 16) applies
+    them exactly in the stream's epilogues; the oracle dequantises with the same scales."""
+    p = SMALL[name]
+    w = make_weights(p, "cpu")
+    g = torch.Generator().manual_seed(3)
+    for t in (w.w13_scale, w.w2_scale, w.ws13_scale, w.ws2_scale):
+        t.mul_(1.0 + torch.rand(t.shape, generator=g))            # mantissas in [1, 2)
+    res = _run_w(lib, p, w, T, max_tokens=16)
+    out, ties, idx, wt = _oracle(p, res)
+    check_output(f"nonpow2/{name}/T{T}", res["y"], out["y"], TOL[p.wtype], ties=len(ties))
 
 
 def test_deterministic(lib):
