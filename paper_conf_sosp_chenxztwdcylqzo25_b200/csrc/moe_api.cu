@@ -435,6 +435,7 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   L->nchunk_max = (int)((Tr + kChunkTokens - 1) / kChunkTokens);
   const int ab = L->act_bytes;
   C_TRY(dalloc(L, &L->logits, (size_t)Tm * L->gate_rows * 4, false));
+  C_TRY(cudaMemset(L->logits, 0, (size_t)Tm * L->gate_rows * 4));   // finite for the router's warm-up pass
   if (cfg->ep_size > 1 || (cfg->nccl_unique_id && L->tp_size == 1)) S_TRY(ep_create(L, cfg));
   C_TRY(dalloc(L, &L->topk_idx, (size_t)pairs * 4, false));
   C_TRY(dalloc(L, &L->topk_w, (size_t)pairs * 4, false));
