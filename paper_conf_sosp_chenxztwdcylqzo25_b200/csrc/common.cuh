@@ -276,13 +276,14 @@ struct moe_layer {
   struct Ep {
     int P = 1, rank = 0;
     void *comm = nullptr;       // ncclComm_t (NCCL transport) or null (in-process group)
-    __nv_bfloat16 *send_x = nullptr;   // [P][Tm][H]
+    uint8_t *send_x = nullptr;         // [P][Tm] rows of row_bytes: bf16 x, or FP8 codes + exponent bytes
+    int row_bytes = 0;
     int32_t *send_idx = nullptr;       // [P][Tm][k]
     float *send_w = nullptr;           // [P][Tm][k]
     int32_t *sendpos = nullptr;        // [Tm][P]
     int32_t *cnt_dev = nullptr;        // [2P] send counts, recv counts
     int32_t *cnt_host = nullptr;       // pinned [2P]
-    __nv_bfloat16 *recv_x = nullptr;   // [P*Tm][H]
+    uint8_t *recv_x = nullptr;         // [P*Tm] rows of row_bytes
     __nv_bfloat16 *partial = nullptr;  // [P*Tm][H] expert-side weighted sums (immediate)
     __nv_bfloat16 *partial_def = nullptr;
     __nv_bfloat16 *back = nullptr;     // [P][Tm][H] partial sums returned to this rank

@@ -72,6 +72,74 @@ __global__ void __launch_bounds__(128) ep_pack_kernel(const __nv_bfloat16 *__res
   }
 }
 
+// FP8 layers: the token's e4m3 row (quantised once on the origin, 1x128 UE8M0, reading
+// R10) + its H/128 exponent bytes -- H + H/128 bytes instead of 2H (round-2 EP v2)
+__global__ void __launch_bounds__(128) ep_pack_fp8_kernel(const uint8_t *__restrict__ xq, const float *__restrict__ xs,
+                                                          int H, int k, const int32_t *__restrict__ idx,
+                                                          const float *__restrict__ w, int E_loc, int P, int Tm,
+                                                          int row_bytes, const int32_t *__restrict__ sendpos,
+                                                          uint8_t *__restrict__ send_x, int32_t *__restrict__ send_idx,
+                                                          float *__restrict__ send_w) {
+  const int t = blockIdx.x;
+  const uint4 *src = reinterpret_cast<const uint4 *>(xq + (size_t)t * H);
+  for (int d = 0; d < P; ++d) {
+    const int sp = sendpos[(int64_t)t * P + d];
+    if (sp < 0) continue;
+    const int64_t row = (int64_t)d * Tm + sp;
+    uint8_t *dst = send_x + row * row_bytes;
+    for (int c = threadIdx.x; c < H / 16; c += blockDim.x) reinterpret_cast<uint4 *>(dst)[c] = __ldg(src + c);
+    for (int b = threadIdx.x; b < H / 128; b += blockDim.x)
+      dst[H + b] = (uint8_t)((__float_as_uint(xs[(size_t)t * (H / 128) + b]) >> 23) & 0xFF);
+    if (threadIdx.x < k) {
+      const int e = idx[(int64_t)t * k + threadIdx.x];
+      send_idx[row * k + threadIdx.x] = (e / E_loc) == d ? e : -1;
+      send_w[row * k + threadIdx.x] = w[(int64_t)t * k + threadIdx.x];
+    }
+  }
+}
+
+// expert side, FP8: a received row's codes into its k sorted rows (pos, -1 = not local)
+// and its exponents into their scale images (one 32-bit word per 4 k-blocks, sf_img_off)
+__global__ void __launch_bounds__(128) ep_scatter_fp8_kernel(const uint8_t *__restrict__ recv, int H, int k,
+                                                             int row_bytes, const int32_t *__restrict__ pos,
+                                                             uint8_t *__restrict__ xperm, uint8_t *__restrict__ img,
+                                                             int img_stride) {
+  const int r = blockIdx.x;
+  __shared__ int sp[32];
+  if (threadIdx.x < k) sp[threadIdx.x] = pos[(int64_t)r * k + threadIdx.x];
+  __syncthreads();
+  const uint8_t *src = recv + (int64_t)r * row_bytes;
+  const int nb = H / 128, ng = (nb + 3) / 4;
+  for (int j = 0; j < k; ++j) {
+    const int rw = sp[j];
+    if (rw < 0) continue;
+    uint4 *dst = reinterpret_cast<uint4 *>(xperm + (int64_t)rw * H);
+    for (int c = threadIdx.x; c < H / 16; c += blockDim.x) dst[c] = reinterpret_cast<const uint4 *>(src)[c];
+    for (int g = threadIdx.x; g < ng; g += blockDim.x) {
+      uint32_t wd = 0;
+      for (int q = 0; q < 4; ++q) wd |= (4 * g + q < nb ? (uint32_t)src[H + 4 * g + q] : 127u) << (8 * q);
+      *reinterpret_cast<uint32_t *>(img + sf_img_off(rw, 4 * g, img_stride)) = wd;
+    }
+  }
+}
+
+cudaError_t launch_ep_pack_fp8(const void *xq, const float *xs, int T, int H, int k, const int32_t *idx,
+                               const float *w, int E_loc, int P, int Tm, int row_bytes, const int32_t *sendpos,
+                               void *send_x, int32_t *send_idx, float *send_w, cudaStream_t st) {
+  if (T <= 0) return cudaSuccess;
+  ep_pack_fp8_kernel<<<T, 128, 0, st>>>(reinterpret_cast<const uint8_t *>(xq), xs, H, k, idx, w, E_loc, P, Tm,
+                                        row_bytes, sendpos, reinterpret_cast<uint8_t *>(send_x), send_idx, send_w);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_ep_scatter_fp8(const void *recv, int R, int H, int k, int row_bytes, const int32_t *pos,
+                                  void *xperm, uint8_t *img, int img_stride, cudaStream_t st) {
+  if (R <= 0) return cudaSuccess;
+  ep_scatter_fp8_kernel<<<R, 128, 0, st>>>(reinterpret_cast<const uint8_t *>(recv), H, k, row_bytes, pos,
+                                           reinterpret_cast<uint8_t *>(xperm), img, img_stride);
+  return cudaGetLastError();
+}
+
 // ------------------------------------------------------------------ final combine
 // y[t] = residual + g_t * ys[t] + sum_d back[d][sendpos[t][d]] + deferred_in;
 // deferred_out[t] = sum_d back_def[d][sendpos[t][d]]   (fp32 accumulation)

@@ -182,6 +182,12 @@ cudaError_t launch_ep_pack(const void *x, int T, int H, int k, const int32_t *id
                            int Tm, const int32_t *sendpos, void *send_x, int32_t *send_idx, float *send_w,
                            cudaStream_t st);
 cudaError_t launch_ep_final_combine(const EpCombineArgs &a, cudaStream_t st);
+// FP8 dispatch: rows of [H e4m3 codes | H/128 UE8M0 exponent bytes], row_bytes apart
+cudaError_t launch_ep_pack_fp8(const void *xq, const float *xs, int T, int H, int k, const int32_t *idx,
+                               const float *w, int E_loc, int P, int Tm, int row_bytes, const int32_t *sendpos,
+                               void *send_x, int32_t *send_idx, float *send_w, cudaStream_t st);
+cudaError_t launch_ep_scatter_fp8(const void *recv, int R, int H, int k, int row_bytes, const int32_t *pos,
+                                  void *xperm, uint8_t *img, int img_stride, cudaStream_t st);
 int ep_nccl_get_unique_id(void *out128);
 int ep_nccl_init(void **comm, int P, int rank, const void *uid128);
 void ep_nccl_destroy(void *comm);

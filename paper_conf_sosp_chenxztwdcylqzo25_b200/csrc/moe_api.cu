@@ -89,12 +89,14 @@ moe_status ep_create(moe_layer *L, const moe_layer_config *cfg) {
   L->ep.P = P;
   L->ep.rank = cfg->ep_rank;
   const size_t rows = (size_t)P * Tm;
-  CUDA_TRY(dalloc(L, &L->ep.send_x, rows * H * 2, false));
+  // dispatched token rows: bf16 (2H bytes) or, FP8 layers, [H e4m3 codes | H/128 UE8M0 bytes]
+  L->ep.row_bytes = L->fp8 ? ((H + H / 128 + 15) / 16) * 16 : 2 * H;
+  CUDA_TRY(dalloc(L, &L->ep.send_x, rows * L->ep.row_bytes, false));
   CUDA_TRY(dalloc(L, &L->ep.send_idx, rows * k * 4, false));
   CUDA_TRY(dalloc(L, &L->ep.send_w, rows * k * 4, false));
   CUDA_TRY(dalloc(L, &L->ep.sendpos, Tm * P * 4, false));
   CUDA_TRY(dalloc(L, &L->ep.cnt_dev, 2 * P * 4, false));
-  CUDA_TRY(dalloc(L, &L->ep.recv_x, rows * H * 2, false));
+  CUDA_TRY(dalloc(L, &L->ep.recv_x, rows * L->ep.row_bytes, false));
   CUDA_TRY(dalloc(L, &L->ep.partial, rows * H * 2, false));
   CUDA_TRY(dalloc(L, &L->ep.partial_def, rows * H * 2, false));
   CUDA_TRY(dalloc(L, &L->ep.back, rows * H * 2, false));
@@ -757,8 +759,18 @@ static moe_status ep_phase_a(moe_layer *L, const void *x, int T, cudaStream_t st
   if (s != MOE_OK) return s;
   const int P = L->ep.P, Tm = std::max(1, L->max_tokens);
   KL_TRY(launch_ep_plan(L->topk_idx, T, L->k, L->E, P, L->ep.sendpos, L->ep.cnt_dev, st));
-  KL_TRY(launch_ep_pack(x, T, L->H, L->k, L->topk_idx, L->topk_w, L->E, P, Tm, L->ep.sendpos, L->ep.send_x,
+  if (L->fp8) {
+    // quantise the own tokens once (1x128 UE8M0 + e4m3, reading R10): the dispatched rows and
+    // the shared expert's input (xq) -- half the bytes of a bf16 row on the wire
+    ScatterDst q{};
+    q.fp8 = 1; q.xq = L->xq; q.xs = L->xs; q.xq_img = L->xq_img; q.xq_img_stride = L->img_tiles_sh;
+    KL_TRY(launch_scatter_rows(x, T, L->H, 0, L->pos, q, st));
+    KL_TRY(launch_ep_pack_fp8(L->xq, L->xs, T, L->H, L->k, L->topk_idx, L->topk_w, L->E, P, Tm, L->ep.row_bytes,
+                              L->ep.sendpos, L->ep.send_x, L->ep.send_idx, L->ep.send_w, st));
+  } else {
+    KL_TRY(launch_ep_pack(x, T, L->H, L->k, L->topk_idx, L->topk_w, L->E, P, Tm, L->ep.sendpos, L->ep.send_x,
                           L->ep.send_idx, L->ep.send_w, st));
+  }
   return MOE_OK;
 }
 
@@ -795,19 +807,15 @@ static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_d
     CUDA_TRY(cudaMemsetAsync(L->n_tiles, 0, 4, st));
     CUDA_TRY(cudaMemsetAsync(L->n_pairs, 0, 4, st));
   }
-  ScatterDst d{};
-  d.fp8 = L->fp8; d.xperm = L->xperm;
   if (L->fp8) {
-    d.xperm_img = L->umma ? L->xperm_img : nullptr; d.xperm_img_stride = L->max_tiles;
-    d.xperm_s = L->umma ? nullptr : L->xperm_s;
-  }
-  KL_TRY(launch_scatter_rows(L->ep.recv_x, R, H, k, L->pos, d, st));
-  if (Fs > 0 && L->fp8 && T_own > 0) {
-    // the shared expert runs on this rank's own tokens: quantise them into xq
-    ScatterDst s{};
-    s.fp8 = 1; s.xq = L->xq; s.xs = L->xs; s.xq_img = L->umma ? L->xq_img : nullptr;
-    s.xq_img_stride = L->img_tiles_sh;
-    KL_TRY(launch_scatter_rows(x_own, T_own, H, 0, L->pos, s, st));
+    // received e4m3 rows + exponents -> the expert-sorted rows and their scale images (the
+    // own tokens' xq for the shared expert was quantised in phase A)
+    KL_TRY(launch_ep_scatter_fp8(L->ep.recv_x, R, H, k, L->ep.row_bytes, L->pos, L->xperm, L->xperm_img,
+                                 L->max_tiles, st));
+  } else {
+    ScatterDst d{};
+    d.fp8 = 0; d.xperm = L->xperm;
+    KL_TRY(launch_scatter_rows(L->ep.recv_x, R, H, k, L->pos, d, st));
   }
   const int64_t pairs = (int64_t)R * k;
   const int64_t R_bound = std::min<int64_t>(L->R_max, pairs + (int64_t)std::min<int64_t>(E, pairs) * kPadM);
@@ -856,7 +864,7 @@ static moe_status ep_forward_nccl(moe_layer *L, const void *x, const void *resid
   {
     const void *snd[3] = {L->ep.send_x, L->ep.send_idx, L->ep.send_w};
     void *rcv[3] = {L->ep.recv_x, L->topk_idx, L->topk_w};
-    const int64_t rb[3] = {(int64_t)H * 2, (int64_t)k * 4, (int64_t)k * 4};
+    const int64_t rb[3] = {(int64_t)L->ep.row_bytes, (int64_t)k * 4, (int64_t)k * 4};
     NCCL_TRY(ep_nccl_rows(L->ep.comm, P, scnt, soff, rcnt, roff, 3, snd, rcv, rb, st));
   }
   const bool want_def = dout != nullptr && n_def > 0;
@@ -1180,7 +1188,8 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
       const int64_t n = layers[src]->ep.cnt_host[d];
       if (!n) continue;
       const int64_t ro = layers[d]->ep.roff[src], so = (int64_t)d * Tm;
-      CUDA_TRY(cudaMemcpyAsync(layers[d]->ep.recv_x + ro * H, layers[src]->ep.send_x + so * H, n * H * 2,
+      const int64_t rbytes = layers[d]->ep.row_bytes;
+      CUDA_TRY(cudaMemcpyAsync(layers[d]->ep.recv_x + ro * rbytes, layers[src]->ep.send_x + so * rbytes, n * rbytes,
                                cudaMemcpyDefault, st));
       CUDA_TRY(cudaMemcpyAsync(layers[d]->topk_idx + ro * k, layers[src]->ep.send_idx + so * k, n * k * 4,
                                cudaMemcpyDefault, st));
