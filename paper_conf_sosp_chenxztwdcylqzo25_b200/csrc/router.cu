@@ -551,11 +551,11 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   // experts beside us; otherwise it launches when every CTA here has exited (measured ~1 us/layer
   // faster: CTAs waiting in griddepcontrol.wait beside ours slow the routing down)
   if (a.early_trigger) pdl_trigger();
-  // warm this SM's instruction cache with one dry run of the selection code (stores off):
-  // only the last CTA to finish routes, its SM is not known in advance, and a cold
-  // instruction cache -- not the arithmetic -- sets the latency of the serial selection.
-  // It runs before the dependency wait, under the previous layer's tail.
-  if (!(kExperiments && (a.debug & 32)) && threadIdx.x < 32)
+  // (an instruction-cache warm-up -- a dry run of the selection before the dependency wait --
+  //  was measured: the window before the wait is ~1-2 us, so the dry run lands on the
+  //  critical path, +1 us/layer plain, worse with deferral; MOE_DEBUG_ROUTE bit 32 in
+  //  experiments builds re-enables it)
+  if (kExperiments && (a.debug & 32) && threadIdx.x < 32)
     select_token_regs(r, 0, rsm, nullptr, threadIdx.x & 31, false, bpre);
   pdl_wait();                                    // x (the previous layer's output) and our workspaces
   if (a.trace && threadIdx.x == 0 && blockIdx.x == 0) a.trace[0] = gtimer_ns();

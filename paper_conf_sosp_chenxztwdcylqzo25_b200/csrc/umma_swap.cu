@@ -121,7 +121,8 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
   }
   if (warp == 1) tmem_alloc_pair(tmem_base_smem, SW_TMEM_COLS);
   tc_fence_before();
-  cluster_sync();
+  __syncthreads();                               // the allocated TMEM address, CTA-local
+  cluster_sync();                                // barriers of both CTAs initialised
   tc_fence_after();
   const uint32_t tmem = *tmem_base_smem;
 
@@ -369,20 +370,20 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
 #pragma unroll
         for (int c = 0; c < 128 / SW_XCH; ++c) {
           if (c < nx) {
+            // (both warps reach each named barrier at the same instruction)
             if (up) {
 #pragma unroll
               for (int j = 0; j < SW_XCH; ++j) xb[j * 32 + lane] = __uint_as_float(r[c * SW_XCH + j]);
-              asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
-              asm volatile("bar.sync %0, 64;" ::"r"(5 + pi) : "memory");
-            } else {
-              asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
+            }
+            asm volatile("bar.sync %0, 64;" ::"r"(1 + pi) : "memory");
+            if (!up) {
 #pragma unroll
               for (int j = 0; j < SW_XCH; ++j) {
                 const float gt = __uint_as_float(r[c * SW_XCH + j]);
                 r[c * SW_XCH + j] = __float_as_uint(silu_f(gt) * xb[j * 32 + lane]);
               }
-              asm volatile("bar.sync %0, 64;" ::"r"(5 + pi) : "memory");
             }
+            asm volatile("bar.sync %0, 64;" ::"r"(5 + pi) : "memory");
           }
         }
         if (up) { ++tile_i; continue; }
