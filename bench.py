@@ -204,8 +204,9 @@ def run_reference(args):
 def algorithmic(p, T, n_distinct):
     """Algorithmic FLOPs / bytes per stage."""
     H, F, Fs, k, E = p.hidden, p.ffn, p.shared_ffn, p.top_k, p.n_experts
-    wb = 1 if p.wtype == 1 else 2
-    exp_bytes = 3 * H * F * wb + (3 * (H // 128) * (F // 128) * 4 if p.wtype == 1 else 0)
+    wb = {0: 2, 1: 1, 2: 4, 3: 0.5}[p.wtype]           # bf16, e4m3, f32, packed e2m1 bytes per weight
+    blocked = p.wtype in (1, 3)                          # + one fp32 scale per 128x128 block
+    exp_bytes = 3 * H * F * wb + (3 * (H // 128) * (F // 128) * 4 if blocked else 0)
     # one launch computes the routed experts AND the shared expert (two operand groups)
     return {
         "gemm1_swiglu": {"flops": 2.0 * T * k * 2 * F * H + 2.0 * T * 2 * Fs * H,

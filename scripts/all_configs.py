@@ -1,6 +1,8 @@
 """Every BASELINE.json configuration on one B200: prefill tokens/s + TFLOP/s and decode
-us/layer + GB/s (CUDA graph over a chain of distinct layers, L2 flushed), each against the
-measured peaks.  Writes one JSON line per measurement and a markdown table (argv[1])."""
+us/layer + GB/s (CUDA graph over a chain of 8 distinct layers, L2 flushed), each against the
+measured peaks (tensor: the burst bf16 figure, x 2 for FP8 -- as bench.py); decode also with
+chained Expert Deferral (moe_layer_forward_chained) and the V3 layer with 4-bit (e2m1) weights.
+Writes one JSON line per measurement and a markdown table (argv[1])."""
 import json, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
@@ -28,20 +30,20 @@ def prefill(name, T):
     layer.forward(x, y=y, routing=routing)
     nd = int((routing["expert_counts"] > 0).sum())
     alg = bench.algorithmic(p, T, nd)
-    fp8 = p.wtype == 1
-    peak_tf = (2 if fp8 else 1) * peaks["bf16_tflops_sustained"]
+    fp8 = p.wtype in (1, 3)
+    peak_tf = (2 if fp8 else 1) * peaks["bf16_tflops"]
     tf = alg["layer_flops"] / (ms * 1e-3) / 1e12
     gbs = alg["layer_bytes"] / (ms * 1e-3) / 1e9
     r = {"config": name, "phase": "prefill", "T": T, "ms": ms, "tokens_per_s": T / (ms * 1e-3), "tflops": tf,
          "tensor_frac": tf / peak_tf, "gbs": gbs, "hbm_frac": gbs / peaks["hbm_gbs"], "distinct_experts": nd,
-         "dtype": "e4m3" if fp8 else ("bf16" if p.wtype == 0 else "f32")}
+         "dtype": {0: "bf16", 1: "e4m3", 2: "f32", 3: "e2m1 weights"}[p.wtype]}
     layer.close()
     del w
     torch.cuda.empty_cache()
     return r
 
 
-def decode(name, T, L=4, n_def=0):
+def decode(name, T, L=8, n_def=0):
     p = PRESETS[name]
     w = make_weights(p, "cuda")
     layers = [moe.MoELayer(p, w, max_tokens=16) for _ in range(L)]
@@ -53,13 +55,12 @@ def decode(name, T, L=4, n_def=0):
     dbufs = [torch.zeros_like(rows[0]), torch.zeros_like(rows[0])]
 
     def step():
+        prev = None
         for i, l in enumerate(layers):
             a, b = bufs[i % 2], bufs[(i + 1) % 2]
-            if n_def:
-                din = None if i == 0 else dbufs[(i + 1) % 2]
-                dout = None if i == L - 1 else dbufs[i % 2]
-                l.forward(a, residual=a, y=b, n_deferred=n_def if dout is not None else 0, deferred_in=din,
-                          deferred_out=dout)
+            if n_def:       # Eq. L241 across the chain: layer i computes layer i-1's deferred experts
+                l.forward_chained(a, residual=a, n_deferred=n_def if i < L - 1 else 0, prev=prev, y=b)
+                prev = l
             else:
                 l.forward(a, residual=a, y=b)
     s = torch.cuda.Stream(); s.wait_stream(torch.cuda.current_stream())
@@ -93,14 +94,13 @@ def decode(name, T, L=4, n_def=0):
     return r
 
 
-plan = [("prefill", "v2lite", 512), ("decode", "v2lite", 1), ("prefill", "qwen2", 2048), ("decode", "qwen2", 1),
-        ("prefill", "v25", 4096), ("decode", "v25", 4), ("prefill", "v3", 8192), ("decode", "v3", 1)]
-for kind, name, T in plan:
-    r = prefill(name, T) if kind == "prefill" else decode(name, T)
-    print(json.dumps(r), flush=True)
-    rows_out.append(r)
-for nd_ in (3, 6):
-    r = decode("v3", 1, n_def=nd_)
+plan = [("prefill", "v2lite", 512, 0), ("decode", "v2lite", 1, 0), ("decode", "v2lite", 1, 3),
+        ("prefill", "qwen2", 2048, 0), ("decode", "qwen2", 1, 0), ("decode", "qwen2", 1, 3),
+        ("prefill", "v25", 4096, 0), ("decode", "v25", 4, 0), ("decode", "v25", 4, 3),
+        ("prefill", "v3", 8192, 0), ("decode", "v3", 1, 0), ("decode", "v3", 1, 3), ("decode", "v3", 1, 6),
+        ("prefill", "v3_fp4", 8192, 0), ("decode", "v3_fp4", 1, 0), ("decode", "v3_fp4", 1, 3)]
+for kind, name, T, nd_ in plan:
+    r = prefill(name, T) if kind == "prefill" else decode(name, T, n_def=nd_)
     print(json.dumps(r), flush=True)
     rows_out.append(r)
 
