@@ -255,7 +255,6 @@ struct FusedDecodeParams {
   unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
   int debug;                    // MOE_EXPERIMENTS builds (MOE_DEBUG_FD): 1 no phase-A fold, 2 no phase-A MMAs
   float *cl_scratch;            // cluster split: [clusters][7][128][32] fp32 partials of the peers (L2)
-  int ts;                       // FP8 weights: MMA A operand staged in TMEM (TS form) instead of read from smem
 };
 // csize > 1: clusters of csize CTAs share each unit (the cluster split)
 cudaError_t launch_umma_decode_fused(bool fp8, bool w4, const FusedDecodeParams &p, int grid, int csize,

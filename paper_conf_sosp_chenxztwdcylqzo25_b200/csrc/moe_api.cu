@@ -1064,11 +1064,6 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     if (cluster_override > 0 && units <= L->fd_max_clusters[2] && cluster_override <= std::min(KA, NT))
       csize = cluster_override;                  // (cluster ids stay within the scratch slots)
     fp.cl_scratch = L->cl_scratch;
-    // A/B only (MOE_EXPERIMENTS builds): the TS form -- weights copied into TMEM by tcgen05.cp and
-    // read there by the MMA -- is correct but measured 1.45x slower per k-block than the SS form
-    // (profiles/r02/decode_ts_vs_ss.md)
-    static const int ts_on = experiment_knob("MOE_FD_TS");
-    fp.ts = ts_on;
     const int grid = csize > 1 ? units * csize : std::min(L->num_sms, units);
     KL_TRY(launch_umma_decode_fused(f8, L->fp4, fp, grid, csize, st));
     mark(L, ST_GEMM1, st);

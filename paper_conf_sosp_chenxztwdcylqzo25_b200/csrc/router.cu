@@ -591,13 +591,43 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
         red[half][w4][t] = acc0;
         if (two) red[half][w4][t + 1] = acc1;
       }
+      // FP8: the x rows are in registers already -- CTA u < nv/128 quantises the 128-chunk slice u
+      // (chunks tid + 128 u) of token t (half 0) / t + 1 (half 1): 1x128 UE8M0 over 16 lanes,
+      // e4m3 RNE satfinite (reading R10), no second read of x
+      if (a.fp8 && a.xq && (half == 0 || two)) {
+#pragma unroll 1
+        for (int u = blockIdx.x; u < 8 && u * 128 < nv; u += gridDim.x) {
+          const int c = tid + u * 128, tt = t + half;
+          uint4 xv = xv0[0];
+#pragma unroll
+          for (int uu = 0; uu < 8; ++uu) xv = uu == u ? (half ? xv1[uu] : xv0[uu]) : xv;
+          float f[8];
+          bf16x8_to_f32(xv, f);
+          float am = 0.f;
+#pragma unroll
+          for (int j = 0; j < 8; ++j) am = fmaxf(am, fabsf(f[j]));
+#pragma unroll
+          for (int o = 8; o > 0; o >>= 1) am = fmaxf(am, __shfl_xor_sync(0xffffffffu, am, o));
+          if (c < nv) {
+            const int ex = ue8m0_exponent(am);
+            const float inv = exp2i(-ex);
+            uint2 q;
+            q.x = (uint32_t)f32_to_e4m3(f[0] * inv) | ((uint32_t)f32_to_e4m3(f[1] * inv) << 8) |
+                  ((uint32_t)f32_to_e4m3(f[2] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[3] * inv) << 24);
+            q.y = (uint32_t)f32_to_e4m3(f[4] * inv) | ((uint32_t)f32_to_e4m3(f[5] * inv) << 8) |
+                  ((uint32_t)f32_to_e4m3(f[6] * inv) << 16) | ((uint32_t)f32_to_e4m3(f[7] * inv) << 24);
+            *reinterpret_cast<uint2 *>(reinterpret_cast<uint8_t *>(a.xq) + (size_t)tt * H + c * 8) = q;
+            if ((lane & 15) == 0) a.xs[(size_t)tt * (H / 128) + (c >> 4)] = exp2i(ex);
+          }
+        }
+      }
     }
     __syncthreads();
     if (row < a.rows && tid < T)
       const_cast<float *>(r.logits)[(size_t)tid * r.ldl + row] = red[half][0][tid] + red[half][1][tid] + red[half][2][tid] + red[half][3][tid];
   }
-  // ---- FP8: quantise x -> xq (token order) across all CTAs, in parallel with routing ----
-  if (a.fp8 && a.xq) {
+  // ---- FP8, H > 8192 only (x slices beyond 8 x 128 chunks): quantise x -> xq from global ----
+  if (a.fp8 && a.xq && nv > 8 * 128) {
     const int nc = H / 8;                       // 8-element chunks per row; a 1x128 block = 16 chunks
     const int64_t total = (int64_t)T * nc;
     const int lane = threadIdx.x & 31;

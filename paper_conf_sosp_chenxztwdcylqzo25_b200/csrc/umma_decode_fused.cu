@@ -57,11 +57,9 @@ constexpr size_t FD_SMEM = 1024 + (size_t)FD_STAGES * (FD_A_BYTES + FD_B_BYTES) 
                            2 * 2 * FD_N * 32 * 4 +     // up -> gate exchange [gate warp][acc][token][lane]
                            2 * FD_MAX_KB * FD_N * 4 +  // activation scales [this layer | previous layer][kb][token]
                            1024;                       // barriers, queue, amax, scales
-constexpr uint32_t FD_TMEM_COLS = 512;
+constexpr uint32_t FD_TMEM_COLS = 256;
 constexpr uint32_t FD_ACCA_COL = 0, FD_ACCB_COL = 128;   // + 32 per ring slot (two 16-column MMA tiles)
-constexpr uint32_t FD_ASTAGE_COL = 256;                  // TS form: weight k-block staged in TMEM, 2 x 64 columns
-static_assert(FD_ACCA_SLOTS * 32 <= (int)FD_ACCB_COL && FD_ACCB_COL + FD_ACCB * 32 <= FD_ASTAGE_COL &&
-              FD_ASTAGE_COL + 2 * 64 <= FD_TMEM_COLS, "TMEM map");
+static_assert(FD_ACCA_SLOTS * 32 <= (int)FD_ACCB_COL && FD_ACCB_COL + FD_ACCB * 32 <= FD_TMEM_COLS, "TMEM map");
 
 // instruction descriptor, kind::f8f6f4 (A E4M3 or E2M1 (a_fmt 5), B E4M3 -> F32, no block scale), K-major A and B
 __host__ __device__ constexpr uint32_t idesc_f8(int M, int N, uint32_t a_fmt = 0) {
@@ -83,20 +81,6 @@ __device__ __forceinline__ void mma_f8(uint32_t d_tmem, uint64_t a_desc, uint64_
       "tcgen05.mma.cta_group::1.kind::f8f6f4 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
       "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
       : "memory");
-}
-// TS form: A (the weights) read from TMEM, B (tokens / h) from shared memory.  The A
-// operand gets there by tcgen05.cp 128x256b (one 32-byte K slice of 128 rows per copy,
-// read through the same SW128 K-major descriptor the SS form uses)
-__device__ __forceinline__ void mma_f8_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
-                                          uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f8f6f4 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
-      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
-      : "memory");
-}
-__device__ __forceinline__ void tmem_cp_128x256b(uint32_t taddr, uint64_t sdesc) {
-  asm volatile("tcgen05.cp.cta_group::1.128x256b [%0], %1;" ::"r"(taddr), "l"(sdesc) : "memory");
 }
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
@@ -220,8 +204,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   uint64_t *uq_full = accB_empty + FD_ACCB;                  // [FD_UQ]
   uint64_t *uq_empty = uq_full + FD_UQ;                      // [FD_UQ]
   uint64_t *part_bar = uq_empty + FD_UQ;                     // cluster leader: the peers' partials are in L2
-  uint64_t *a_free = part_bar + 1;                           // [2] TS form: the TMEM weight stage is free
-  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(a_free + 2);
+  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(part_bar + 1);
   int4 *unit_q = reinterpret_cast<int4 *>((reinterpret_cast<uintptr_t>(tmem_base_smem + 1) + 15) & ~uintptr_t(15));   // [FD_UQ] (expert, chunk, group, valid)
   float *amax = reinterpret_cast<float *>(unit_q + FD_UQ);       // [2 gate warps][16]
   float *hsc = amax + 2 * FD_N;                                  // [2 unit parity][16] h scale per token (FP8)
@@ -245,12 +228,9 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     for (int i = 0; i < FD_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], 5 + 6 * (csize - 1)); }
     // partials through the leader's shared memory (st.async; small T) or through L2
     mbar_init(part_bar, (csize > 1 && !fd_dsmem_partials(csize, p.T)) ? 4 * (csize - 1) : 1);
-    mbar_init(&a_free[0], 1);
-    mbar_init(&a_free[1], 1);
     fence_barrier_init();
   }
-  const uint32_t tmem_cols = p.ts ? FD_TMEM_COLS : FD_ASTAGE_COL;   // the TS stage only when used
-  if (warp == 1) tmem_alloc(tmem_base_smem, tmem_cols);
+  if (warp == 1) tmem_alloc(tmem_base_smem, FD_TMEM_COLS);
   tc_fence_before();
   __syncthreads();
   if (csize > 1) cluster_sync();                 // every barrier of the cluster initialised
@@ -350,45 +330,6 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     int stage = 0; uint32_t phase = 0, qs = 0, qph = 0, hph = 0;
     int ab = 0; uint32_t abph = 0;
     int as = 0; uint32_t asph = 0;
-    int tsb = 0; uint32_t tsph = 0;              // TS form: TMEM weight-stage ring (2 buffers)
-    const bool ts = FP8 && !W4 && p.ts;
-    // one 256-row weight k-block (two 128-row tiles x 4 K slices of 32 B) against B: TS form --
-    // copy it into TMEM stage tsb, then 8 MMAs reading A there; SS form -- 8 MMAs from smem
-    auto mma_kblock = [&](uint32_t a0, uint32_t b0, uint32_t dcol, bool zero_first) {
-      if (ts) {
-        const uint32_t abuf = tmem + FD_ASTAGE_COL + tsb * 64;
-#pragma unroll
-        for (int t = 0; t < 2; ++t)
-#pragma unroll
-          for (int k = 0; k < 4; ++k)
-            tmem_cp_128x256b(abuf + t * 32 + k * 8, sw128_kmajor_desc(a0 + t * 128 * 128 + k * 32));
-#pragma unroll
-        for (int k = 0; k < 4; ++k)
-#pragma unroll
-          for (int t = 0; t < 2; ++t)
-            mma_f8_ts(dcol + t * 16, abuf + t * 32 + k * 8, sw128_kmajor_desc(b0 + k * 32),
-                      idesc_f8(128, FD_N, A_FMT), (k != 0) || !zero_first);
-      } else {
-#pragma unroll
-        for (int k = 0; k < 4; ++k)
-#pragma unroll
-          for (int t = 0; t < 2; ++t) {
-            const uint64_t ad = sw128_kmajor_desc(a0 + t * 128 * 128 + k * 32);
-            const uint64_t bd = sw128_kmajor_desc(b0 + k * 32);
-            if (FP8) mma_f8(dcol + t * 16, ad, bd, idesc_f8(128, FD_N, A_FMT), (k != 0) || !zero_first);
-            else mma_bf16(dcol + t * 16, ad, bd, idesc_bf16(128, FD_N), (k != 0) || !zero_first);
-          }
-      }
-    };
-    auto ts_acquire = [&]() {                    // the stage's previous MMAs are done reading it
-      if (ts) { mbar_wait(&a_free[tsb], tsph ^ 1); tc_fence_after(); }
-    };
-    auto ts_release = [&]() {                    // (lane 0, after the k-block's MMAs)
-      if (ts) mma_commit(&a_free[tsb]);
-    };
-    auto ts_advance = [&]() {
-      if (ts && ++tsb == 2) { tsb = 0; tsph ^= 1; }
-    };
     for (;;) {
       mbar_wait(&uq_full[qs], qph);
       const int4 uq = unit_q[qs];
@@ -414,21 +355,28 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
           mbar_wait(&accA_empty[as], asph ^ 1);
           tc_fence_after();
         }
-        ts_acquire();
         mbar_wait(&full[stage], phase);
         tc_fence_after();
         if (lane == 0) {
-          // FP8: a fresh accumulator slot per k-block; BF16: the accumulator is free (the
-          // epilogue read it before h_ready of the previous unit) and sums over all of K
-          mma_kblock(smem_u32(sA + stage * FD_A_BYTES), smem_u32(sB + stage * FD_B_BYTES),
-                     tmem + FD_ACCA_COL + (FP8 ? as * 32 : 0), FP8 || kb == kb0);
+          const uint32_t a0 = smem_u32(sA + stage * FD_A_BYTES);
+          const uint32_t b0 = smem_u32(sB + stage * FD_B_BYTES);
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const uint64_t bd = sw128_kmajor_desc(b0 + k * 32);
+#pragma unroll
+            for (int t = 0; t < 2; ++t) {
+              const uint64_t ad = sw128_kmajor_desc(a0 + t * 128 * 128 + k * 32);
+              if (FP8)     // a fresh accumulator slot per k-block
+                mma_f8(tmem + FD_ACCA_COL + as * 32 + t * 16, ad, bd, idesc_f8(128, FD_N, A_FMT), k != 0);
+              else         // the accumulator is free: the epilogue read it before h_ready of the previous unit
+                mma_bf16(tmem + FD_ACCA_COL + t * 16, ad, bd, idesc_bf16(128, FD_N), (kb != kb0) || (k != 0));
+            }
+          }
           mma_commit(&empty[stage]);
-          ts_release();
           if (FP8) mma_commit(&accA_full[as]);
           else if (kb == kb1 - 1) mma_commit(&accA_full[0]);
         }
         __syncwarp();
-        ts_advance();
         if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
         if (FP8 && ++as == FD_ACCA_SLOTS) { as = 0; asph ^= 1; }
       }
@@ -453,15 +401,24 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
             if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
             continue;
           }
-          ts_acquire();
           if (lane == 0) {
-            mma_kblock(smem_u32(sA + stage * FD_A_BYTES), h0 + kk * FD_B_BYTES, tmem + FD_ACCB_COL + ab * 32, kk == 0);
+            const uint32_t a0 = smem_u32(sA + stage * FD_A_BYTES);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+              const uint64_t bd = sw128_kmajor_desc(h0 + kk * FD_B_BYTES + k * 32);
+              const uint32_t accum = (kk | k) != 0;
+#pragma unroll
+              for (int t = 0; t < 2; ++t) {
+                const uint64_t ad = sw128_kmajor_desc(a0 + t * 128 * 128 + k * 32);
+                const uint32_t d = tmem + FD_ACCB_COL + ab * 32 + t * 16;
+                if (FP8) mma_f8(d, ad, bd, idesc_f8(128, FD_N, A_FMT), accum);
+                else mma_bf16(d, ad, bd, idesc_bf16(128, FD_N), accum);
+              }
+            }
             mma_commit(&empty[stage]);
-            ts_release();
             if (kk == KBC - 1) mma_commit(&accB_full[ab]);
           }
           __syncwarp();
-          ts_advance();
           if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
         }
         if (++ab == FD_ACCB) { ab = 0; abph ^= 1; }
@@ -785,7 +742,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   tc_fence_before();
   __syncthreads();
   if (csize > 1) cluster_sync();                 // no CTA leaves while a peer may still st.async into it
-  if (warp == 1) tmem_dealloc(tmem, tmem_cols);
+  if (warp == 1) tmem_dealloc(tmem, FD_TMEM_COLS);
   if (threadIdx.x == 0) {
     // the last CTA out re-arms the work counter for the next forward (graph replay)
     asm volatile("fence.acq_rel.gpu;" ::: "memory");

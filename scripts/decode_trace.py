@@ -43,6 +43,7 @@ if NL > 1:
     g = torch.cuda.CUDAGraph()
     with torch.cuda.graph(g):
         step()
+allb = [np.zeros(4096, dtype=np.uint64) for _ in layers]
 for it in range(4):
     fw.zero_(); torch.sum(fr, 0, out=sink)
     if NL > 1:
@@ -50,7 +51,19 @@ for it in range(4):
     else:
         layer.forward(x, y=y)
     torch.cuda.synchronize()
-    assert lib.moe_layer_debug_trace(layer._h, buf.ctypes.data, 4096) == 0
+    for l, b in zip(layers, allb):
+        assert lib.moe_layer_debug_trace(l._h, b.ctypes.data, 4096) == 0
+buf = allb[NL // 2]
+if NL > 1:
+    # the chain's period: route entry of every layer, its finalize end, and the gap to the next layer
+    base = int(allb[0][0])
+    ent = [(int(b[0]) - base) / 1e3 for b in allb]
+    fin = [(int(b[2001]) - base) / 1e3 for b in allb]
+    print("chain: route entry / finalize end per layer (us):",
+          " ".join(f"{e:.1f}/{f:.1f}" for e, f in zip(ent, fin)))
+    print("chain: period per layer (route entry to next route entry):",
+          " ".join(f"{ent[i + 1] - ent[i]:.1f}" for i in range(NL - 1)),
+          "| finalize end -> next route entry:", " ".join(f"{ent[i + 1] - fin[i]:.1f}" for i in range(NL - 1)))
 t0 = int(buf[0])
 rel = lambda v: (int(v) - t0) / 1e3
 if buf[6]:
