@@ -59,6 +59,34 @@ dec.close(); gem.close()
 del w
 torch.cuda.empty_cache()
 
+# (3) tokens per expert {1 .. 512} (SURVEY.md §8(d) E1/E4 analog): the grouped-GEMM layer from
+#     T = 32 (1 token per expert at k/E = 1/32) to T = 16384 (512 per expert) -- where the
+#     tensor-core path becomes compute-efficient (the paper's ARI switch, L170)
+peaks = bench.load_peaks()
+w = make_weights(p, "cuda")
+big = moe.MoELayer(p, w, max_tokens=16384)
+for tpe in (() if os.environ.get("SWEEP_SKIP_TPE") == "1" else (1, 2, 4, 8, 16, 32, 64, 128, 256, 512)):
+    T = tpe * p.n_experts // p.top_k
+    x, _ = make_tokens(p, T, "cuda", offset=33)
+    y = torch.empty_like(x)
+    times, stages = bench.timed_steps(big, [x], y, 5, 3, flush, profile=True)
+    times.sort()
+    ms = times[len(times) // 2]
+    routing = {}
+    big.forward(x, y=y, routing=routing)
+    nd = int((routing["expert_counts"] > 0).sum())
+    alg = bench.algorithmic(p, T, nd)
+    tf = alg["layer_flops"] / (ms * 1e-3) / 1e12
+    r = {"sweep": "tokens_per_expert", "tokens_per_expert": tpe, "T": T, "ms": ms, "tokens_per_s": T / (ms * 1e-3),
+         "tflops": tf, "tensor_frac": tf / (2 * peaks["bf16_tflops"]),
+         "hbm_frac": alg["layer_bytes"] / (ms * 1e-3) / 1e9 / peaks["hbm_gbs"], "distinct_experts": nd,
+         "gemm1_ms": stages.get("gemm1_swiglu"), "gemm2_ms": stages.get("gemm2")}
+    print(json.dumps(r), flush=True)
+    out.append(r)
+big.close()
+del w
+torch.cuda.empty_cache()
+
 for skew in (() if os.environ.get("SWEEP_SKIP_SKEW") == "1" else (0.0, 1.0)):
     w = make_weights(p, "cuda", skew=skew)
     x, _ = make_tokens(p, 8192, "cuda", skew=skew, weights=w if skew > 0 else None)
@@ -84,6 +112,12 @@ with open(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/sweeps.md", "w") as 
         if r["sweep"] == "decode_vs_gemm":
             f.write(f"| {r['T']} | {r['distinct_experts']} | {r.get('decode_stream_us', float('nan')):.1f} us | "
                     f"{r.get('grouped_gemm_us', float('nan')):.1f} us |\n")
+    f.write("\nTokens per expert (grouped-GEMM layer, V3, one forward, L2 flushed; tensor fraction of 2 x burst bf16):\n\n"
+            "| tokens/expert | T | layer ms | M tokens/s | TFLOP/s | tensor frac | HBM frac |\n|---|---|---|---|---|---|---|\n")
+    for r in out:
+        if r["sweep"] == "tokens_per_expert":
+            f.write(f"| {r['tokens_per_expert']} | {r['T']} | {r['ms']:.3f} | {r['tokens_per_s'] / 1e6:.3f} | "
+                    f"{r['tflops']:.0f} | {r['tensor_frac']:.3f} | {r['hbm_frac']:.3f} |\n")
     f.write("\nPrefill, T = 8192, balanced vs skewed routing:\n\n| skew | max/mean expert load | layer ms | GEMM1 ms | GEMM2 ms |\n|---|---|---|---|---|\n")
     for r in out:
         if r["sweep"] == "prefill_skew":
