@@ -971,7 +971,8 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     if (L->fp8) { rs.xq = L->xq; rs.xs = L->xs; }
     else rs.xcopy = L->xcopy;
     rs.n_imm = A.chained ? k - n_def : k;
-    rs.early_trigger = prev != nullptr;
+    static const int early_knob = experiment_knob("MOE_ROUTE_EARLY");   // A/B (MOE_EXPERIMENTS builds)
+    rs.early_trigger = prev != nullptr || early_knob == 1;
     rs.imm_list = L->imm_list; rs.def_list = L->def_list; rs.n_imm_list = L->n_lists; rs.n_def_list = L->n_lists + 1;
     KL_TRY(launch_route_small(rs, st));
     mark(L, ST_PERMUTE, st);
