@@ -249,6 +249,21 @@ def test_mid_size_fp8_elementwise(lib, name, T):
     check_output(f"mid/{name}/T{T}", res["y"], out["y"], TOL[p.wtype], ties=len(ties))
 
 
+@pytest.mark.parametrize("name", ["v3_m", "v3_m_fp4"])
+@pytest.mark.parametrize("T", [2, 5, 8])
+def test_split_shared_decode(lib, name, T):
+    """Decode launch with the shared expert's chunks as cluster-split units that start as soon
+    as the router has quantised x (used when the routed units fill the GPU; v3_m at T >= 2),
+    the routed units independent -- element by element against the oracle."""
+    p = SMALL[name]
+    res = _run(lib, p, T, max_tokens=16, residual=True)
+    out, ties, idx, w = _oracle(p, res, residual=False)
+    g = res["routing"]
+    check_routing(g["topk_idx"], g["topk_w"], idx, w, ties, p.routed_scale, p.norm_topk)
+    rr = res["r"].to(torch.float64).numpy()
+    check_output(f"split_shared/{name}/T{T}", res["y"] - rr, out["y"], TOL[p.wtype], ties=len(ties))
+
+
 @pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v3_m"])
 def test_skewed_routing(lib, name):
     """Imbalanced expert selection: a Zipf-like hot-expert logit
