@@ -126,7 +126,6 @@ struct RouteSmallArgs {
   // permutation only when dbg_perm / dbg_counts ask for them (parity outputs).
   int n_imm;
   int32_t *imm_list, *n_imm_list, *def_list, *n_def_list;
-  int *xq_ready;                // null, or incremented by every CTA that quantised a slice of x (release)
 };
 cudaError_t launch_route_small(const RouteSmallArgs &a, cudaStream_t st);
 
@@ -256,12 +255,6 @@ struct FusedDecodeParams {
   unsigned long long *trace;     // MOE_DEBUG_TRACE: per-CTA globaltimer timeline (timing experiments only)
   int debug;                    // MOE_EXPERIMENTS builds (MOE_DEBUG_FD): 1 no phase-A fold, 2 no phase-A MMAs
   float *cl_scratch;            // cluster split: [clusters][7][128][32] fp32 partials of the peers (L2)
-  // split shared expert (FP8, many units): the shared chunks are cluster-split units started
-  // as soon as the route kernel has quantised x (xq_ready reaches xq_target), the rest independent
-  int split_shared;
-  int *sched_s;                 // the split units' counter (re-armed by the kernel)
-  int *xq_ready;                // route CTAs that finished quantising x this forward (re-armed by the kernel)
-  int xq_target;
 };
 // csize > 1: clusters of csize CTAs share each unit (the cluster split)
 cudaError_t launch_umma_decode_fused(bool fp8, bool w4, const FusedDecodeParams &p, int grid, int csize,

@@ -882,26 +882,6 @@ static moe_status ep_forward_nccl(moe_layer *L, const void *x, const void *resid
 // deferred slots -> deferred_out) and chained deferral (moe_layer_forward_chained:
 // deferred slots left for the next layer, `prev`'s deferred slots computed here).
 // skip_finalize: leave the fp32 partial sums in L->dacc (in-process TP group).
-// Split shared expert (decode, FP8/FP4, one GPU, many units): the shared expert's chunks run
-// as cluster-split units while the router selects (they need only the quantised x).  Used
-// when the launch would otherwise be C = 1 and clusters of 8 (or 4) can hold every chunk.
-static int split_shared_csize(const moe_layer *L) {
-  const int n = L->Fs / 128;
-  if (L->fd_max_clusters[8] >= n && L->fd_max_clusters[8] * 8 >= 96) return 8;
-  if (L->fd_max_clusters[4] >= n) return 4;
-  return 0;
-}
-static bool split_shared_ok(const moe_layer *L, int T, bool has_prev) {
-  static const int off = experiment_knob("MOE_NO_SPLIT_SHARED");   // A/B (MOE_EXPERIMENTS builds)
-  if (off || !L->fp8 || L->Fs == 0 || L->cfg.shared_gated || L->tp_size > 1 || T > 8) return false;
-  const int KA = L->H / 128, NT = L->H / 256;
-  const int cs = split_shared_csize(L);
-  if (cs == 0 || cs > KA || cs > NT) return false;
-  // the launch must otherwise be one CTA per unit (C = 1): many routed units
-  const int64_t routed = std::min<int64_t>(L->E, (int64_t)T * L->k) * (L->F / 128);
-  return routed + L->Fs / 128 > L->num_sms / 2;
-}
-
 struct FwdArgs {
   const void *x, *residual;
   int32_t T, n_def;
@@ -980,7 +960,6 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
   pa.pairs = L->pairs; pa.n_pairs = L->n_pairs;
   pa.dbg_perm = dbg ? dbg->perm : nullptr;
   pa.dbg_counts = dbg ? dbg->expert_counts : nullptr;
-  bool split_shared = false;
   if (tc_decode) {
     // 1-3 (decode). logits + select + count/scan/assign in one launch
     RouteSmallArgs rs{};
@@ -993,11 +972,7 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     else rs.xcopy = L->xcopy;
     rs.n_imm = A.chained ? k - n_def : k;
     static const int early_knob = experiment_knob("MOE_ROUTE_EARLY");   // A/B (MOE_EXPERIMENTS builds)
-    // the decode stream's launch shape is decided below (fused branch); the route kernel only
-    // needs to know whether it has work before the routing is done
-    split_shared = fused && split_shared_ok(L, T, prev != nullptr);
-    rs.early_trigger = prev != nullptr || split_shared || early_knob == 1;
-    rs.xq_ready = split_shared ? L->sched + 4 : nullptr;
+    rs.early_trigger = prev != nullptr || early_knob == 1;
     rs.imm_list = L->imm_list; rs.def_list = L->def_list; rs.n_imm_list = L->n_lists; rs.n_def_list = L->n_lists + 1;
     KL_TRY(launch_route_small(rs, st));
     mark(L, ST_PERMUTE, st);
@@ -1087,23 +1062,10 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     const int KA = H / (f8 ? 128 : 64), NT = H / 256;
     for (int c = 8; c >= 2; c /= 2)
       if (c <= KA && c <= NT && units <= L->fd_max_clusters[c] && units * c <= L->num_sms) { csize = c; break; }
-    int grid = csize > 1 ? units * csize : std::min(L->num_sms, units);
-    fp.split_shared = 0;
-    fp.sched_s = L->sched + 3;
-    fp.xq_ready = L->sched + 4;
-    fp.xq_target = std::min((L->gate_rows + 1) / 2, (H / 8 + 127) / 128);   // route CTAs that quantise x
-    if (split_shared && csize == 1) {
-      // many units on one GPU: the shared expert's chunks as cluster-split units that start as
-      // soon as x is quantised (the router's idle HBM), the rest independent; every CTA of
-      // the launch is in a resident cluster
-      const int cs = split_shared_csize(L);
-      csize = cs;
-      grid = std::min(L->fd_max_clusters[cs], L->num_sms / cs) * cs;
-      fp.split_shared = 1;
-    }
     if (cluster_override > 0 && units <= L->fd_max_clusters[2] && cluster_override <= std::min(KA, NT))
       csize = cluster_override;                  // (cluster ids stay within the scratch slots)
     fp.cl_scratch = L->cl_scratch;
+    const int grid = csize > 1 ? units * csize : std::min(L->num_sms, units);
     KL_TRY(launch_umma_decode_fused(f8, L->fp4, fp, grid, csize, st));
     mark(L, ST_GEMM1, st);
     if (A.chained) { L->chain_T = n_def > 0 ? T : -1; L->chain_ndef = n_def; }

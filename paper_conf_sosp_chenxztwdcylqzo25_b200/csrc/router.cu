@@ -674,9 +674,6 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   __syncthreads();
   if (threadIdx.x == 0) {
     asm volatile("fence.acq_rel.gpu;" ::: "memory");
-    // the CTAs that quantised a slice of x announce it (the decode stream's split shared units
-    // start on it before the routing is done)
-    if (a.xq_ready && a.fp8 && blockIdx.x < 8 && (int)blockIdx.x * 128 < H / 8) atomicAdd(a.xq_ready, 1);
     const int tk = atomicAdd(a.done, 1);
     is_last = tk == (int)gridDim.x - 1;
     if (is_last) asm volatile("fence.acq_rel.gpu;" ::: "memory");

@@ -113,7 +113,7 @@ __device__ __forceinline__ int fd_prev_units(const FusedDecodeParams &p) {
   return p.has_prev ? (*p.g[2].n_list) * p.g[2].nch : 0;
 }
 // this layer's units (valid only after griddepcontrol.wait: n_list is the router's)
-__device__ __forceinline__ FdUnit fd_unit(const FusedDecodeParams &p, int u, int n_prev, bool skip_shared = false) {
+__device__ __forceinline__ FdUnit fd_unit(const FusedDecodeParams &p, int u, int n_prev) {
   FdUnit r{};
   if (u < n_prev) {
     const FdGroup &g = p.g[2];
@@ -121,7 +121,7 @@ __device__ __forceinline__ FdUnit fd_unit(const FusedDecodeParams &p, int u, int
     return r;
   }
   u -= n_prev;
-  const int ns = (p.has_shared && !skip_shared) ? p.g[1].nch : 0;
+  const int ns = p.has_shared ? p.g[1].nch : 0;
   if (u < ns) {
     r.valid = 1; r.group = 1; r.expert = 0; r.chunk = u;
     return r;
@@ -204,12 +204,9 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   uint64_t *uq_full = accB_empty + FD_ACCB;                  // [FD_UQ]
   uint64_t *uq_empty = uq_full + FD_UQ;                      // [FD_UQ]
   uint64_t *part_bar = uq_empty + FD_UQ;                     // cluster leader: the peers' partials are in L2
-  uint64_t *uqI_full = part_bar + 1;                         // [FD_UQ] this CTA's own units (independent)
-  uint64_t *uqI_empty = uqI_full + FD_UQ;                    // [FD_UQ]
-  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(uqI_empty + FD_UQ);
+  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(part_bar + 1);
   int4 *unit_q = reinterpret_cast<int4 *>((reinterpret_cast<uintptr_t>(tmem_base_smem + 1) + 15) & ~uintptr_t(15));   // [FD_UQ] (expert, chunk, group, valid)
-  int4 *unit_qI = unit_q + FD_UQ;                                // [FD_UQ]
-  float *amax = reinterpret_cast<float *>(unit_qI + FD_UQ);      // [2 gate warps][16]
+  float *amax = reinterpret_cast<float *>(unit_q + FD_UQ);       // [2 gate warps][16]
   float *hsc = amax + 2 * FD_N;                                  // [2 unit parity][16] h scale per token (FP8)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -221,15 +218,6 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   // and forwards them to the peers' queues.
   const uint32_t csize = cluster_size(), crank = cluster_rank();
   const bool leader = crank == 0;
-  // Unit queues: S = split units (csize > 1), claimed by the cluster leader and forwarded to
-  // the peers; I = independent units, each CTA claims its own.  All units are split when the
-  // whole launch is few units (expert TP); with p.split_shared (many units, FP8, one GPU) only
-  // the shared expert's chunks are split -- they need only this layer's quantised x, so they
-  // start on every cluster while the router is still selecting, and use the HBM the router
-  // leaves idle -- and the previous layer's deferred and this layer's routed units follow as
-  // independent units.
-  const bool splitS = p.split_shared && csize > 1;
-  const bool phaseS = csize > 1, phaseI = csize == 1 || splitS;
   if (warp == 0 && lane == 0) {
     for (int s = 0; s < FD_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
     for (int s = 0; s < FD_ACCA_SLOTS; ++s) { mbar_init(&accA_full[s], 1); mbar_init(&accA_empty[s], 4); }
@@ -240,7 +228,6 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     for (int i = 0; i < FD_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], 5 + 6 * (csize - 1)); }
     // partials through the leader's shared memory (st.async; small T) or through L2
     mbar_init(part_bar, (csize > 1 && !fd_dsmem_partials(csize, p.T)) ? 4 * (csize - 1) : 1);
-    for (int i = 0; i < FD_UQ; ++i) { mbar_init(&uqI_full[i], 1); mbar_init(&uqI_empty[i], 5); }
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc(tmem_base_smem, FD_TMEM_COLS);
@@ -254,98 +241,30 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   constexpr int KBC = 128 / KDIV;                // W2 k-blocks per 128-column chunk
   const int KA = p.H / KDIV;                     // W13 k-blocks
   const int NT = p.H / 256;                      // W2 256-row tiles
-  const int skb0 = (int)(crank * KA / csize), skb1 = (int)((crank + 1) * KA / csize);   // this CTA's share
-  const int snt0 = (int)(crank * NT / csize), snt1 = (int)((crank + 1) * NT / csize);   // of a split unit
+  const int kb0 = (int)(crank * KA / csize), kb1 = (int)((crank + 1) * KA / csize);   // this CTA's share
+  const int nt0 = (int)(crank * NT / csize), nt1 = (int)((crank + 1) * NT / csize);
   // a consumer is done with queue slot qs (the leader's barrier counts the whole cluster)
   auto release_slot = [&](int qs_) {
     if (leader) mbar_arrive(&uq_empty[qs_]);
     else mbar_arrive_remote(map_to_rank(&uq_empty[qs_], 0));
-  };
-  // consumers (MMA warp, epilogue warps): the next unit -- queue S until its end marker, then
-  // queue I; returns whether it is a split unit (uq.w == 0: no more units)
-  struct QState { uint32_t qs = 0, qph = 0, qsI = 0, qphI = 0; bool inS = true; };
-  auto next_unit = [&](QState &q, int4 &uq) -> bool {
-    if (q.inS && phaseS) {
-      mbar_wait(&uq_full[q.qs], q.qph);
-      uq = unit_q[q.qs];
-      __syncwarp();
-      if (lane == 0) release_slot(q.qs);
-      if (++q.qs == FD_UQ) { q.qs = 0; q.qph ^= 1; }
-      if (uq.w) return true;
-      q.inS = false;
-      if (!phaseI) return false;
-    }
-    q.inS = false;
-    mbar_wait(&uqI_full[q.qsI], q.qphI);
-    uq = unit_qI[q.qsI];
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&uqI_empty[q.qsI]);
-    if (++q.qsI == FD_UQ) { q.qsI = 0; q.qphI ^= 1; }
-    return false;
   };
 
   if (warp == 0) {
     // ============================ producer ============================
     if (lane == 0) {
       const int n_prev = fd_prev_units(p);       // the previous layer's routing is complete
-      bool waited = false, have_x = false;
+      bool waited = false;
       const uint64_t pol = l2_evict_first_policy();   // weights are read once per forward
-      int stage = 0; uint32_t phase = 0, qs = 0, qph = 0, qsI = 0, qphI = 0;
-      auto wait_routing = [&]() {
-        if (!waited) { pdl_wait(); waited = true; }   // this layer's routing and xq (route kernel)
-      };
-      auto wait_x = [&]() {                      // split shared units: only this layer's xq
-        if (!have_x) {
-          while (ld_acquire_gpu(p.xq_ready) < p.xq_target) __nanosleep(128);
-          asm volatile("fence.proxy.async.global;" ::: "memory");   // generic writes -> TMA reads
-          have_x = true;
-        }
-      };
-      auto loads = [&](const FdUnit &ui, bool split) {
-        const FdGroup &g = p.g[ui.group];
-        const int ka0 = split ? skb0 : 0, ka1 = split ? skb1 : KA, na0 = split ? snt0 : 0, na1 = split ? snt1 : NT;
-        // ---- phase A: W13 tile `chunk` (256 rows: gate + up of 128 h columns) ----
-        const uint8_t *w13 = g.w13 + ((size_t)ui.expert * g.nch + ui.chunk) * (size_t)KA * FD_A_BYTES;
-        for (int kb = ka0; kb < ka1; ++kb) {
-          mbar_wait(&empty[stage], phase ^ 1);
-          mbar_expect_tx(&full[stage], A_TX + FD_B_BYTES);
-          if (W4)
-            tma_load_2d_hint(sA + stage * FD_A_BYTES, &g.w13_map4, &full[stage], kb * 128,
-                             (ui.expert * g.nch + ui.chunk) * 256, pol);
-          else
-            bulk_load_hint(sA + stage * FD_A_BYTES, w13 + (size_t)kb * FD_A_BYTES, FD_A_BYTES, &full[stage], pol);
-          tma_load_2d(sB + stage * FD_B_BYTES, &g.x_map, &full[stage], kb * KDIV, 0);
-          if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
-        }
-        // ---- phase B: W2 column block `chunk`, H/256 tiles of 256 rows ----
-        const int KB2 = g.nch * KBC;               // W2 k-blocks per tile row
-        const uint8_t *w2 = g.w2 + (size_t)ui.expert * NT * KB2 * FD_A_BYTES;
-        for (int n = na0; n < na1; ++n) {
-          for (int kk = 0; kk < KBC; ++kk) {
-            mbar_wait(&empty[stage], phase ^ 1);
-            mbar_expect_tx(&full[stage], A_TX);
-            if (W4)
-              tma_load_2d_hint(sA + stage * FD_A_BYTES, &g.w2_map4, &full[stage], ui.chunk * 128,
-                               ui.expert * p.H + n * 256, pol);
-            else
-              bulk_load_hint(sA + stage * FD_A_BYTES, w2 + ((size_t)n * KB2 + ui.chunk * KBC + kk) * FD_A_BYTES,
-                             FD_A_BYTES, &full[stage], pol);
-            if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
-          }
-        }
-      };
-      // ---- queue S: split units ----
-      for (; phaseS;) {
-        FdUnit ui{};
+      int stage = 0; uint32_t phase = 0, qs = 0, qph = 0;
+      for (;;) {
+        FdUnit ui;
         if (leader) {
-          if (splitS) {
-            const int u = atomicAdd(p.sched_s, 1);
-            if (u < p.g[1].nch) { ui.valid = 1; ui.group = 1; ui.expert = 0; ui.chunk = u; }
-          } else {
-            const int u = atomicAdd(p.sched, 1);
-            if (u >= n_prev) wait_routing();
-            ui = fd_unit(p, u, n_prev);
+          const int u = atomicAdd(p.sched, 1);
+          if (u >= n_prev && !waited) {
+            pdl_wait();                          // this layer's routing and xq (route kernel)
+            waited = true;
           }
+          ui = fd_unit(p, u, n_prev);
           mbar_wait(&uq_empty[qs], qph ^ 1);
           unit_q[qs] = make_int4(ui.expert, ui.chunk, ui.group, ui.valid);
           mbar_arrive(&uq_full[qs]);
@@ -361,41 +280,63 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
           const int4 q4 = unit_q[qs];
           release_slot(qs);
           ui.expert = q4.x; ui.chunk = q4.y; ui.group = q4.z; ui.valid = q4.w;
-          if (ui.valid && ui.group != 2 && !splitS) wait_routing();   // (xq TMA-loaded below)
+          if (ui.valid && ui.group != 2 && !waited) {
+            pdl_wait();                          // this layer's xq (TMA-loaded below)
+            waited = true;
+          }
         }
         if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
-        if (!ui.valid) break;
-        if (splitS) wait_x();
-        loads(ui, true);
+        if (!ui.valid) {
+          // every load of this CTA is issued: let the finalize kernel launch now, so
+          // its launch latency overlaps the last stages (it waits for our completion)
+          pdl_trigger();
+          break;
+        }
+        const FdGroup &g = p.g[ui.group];
+        // ---- phase A: W13 tile `chunk` (256 rows: gate + up of 128 h columns) ----
+        const uint8_t *w13 = g.w13 + ((size_t)ui.expert * g.nch + ui.chunk) * (size_t)KA * FD_A_BYTES;
+        for (int kb = kb0; kb < kb1; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          mbar_expect_tx(&full[stage], A_TX + FD_B_BYTES);
+          if (W4)
+            tma_load_2d_hint(sA + stage * FD_A_BYTES, &g.w13_map4, &full[stage], kb * 128,
+                             (ui.expert * g.nch + ui.chunk) * 256, pol);
+          else
+            bulk_load_hint(sA + stage * FD_A_BYTES, w13 + (size_t)kb * FD_A_BYTES, FD_A_BYTES, &full[stage], pol);
+          tma_load_2d(sB + stage * FD_B_BYTES, &g.x_map, &full[stage], kb * KDIV, 0);
+          if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
+        }
+        // ---- phase B: W2 column block `chunk`, H/256 tiles of 256 rows ----
+        const int KB2 = g.nch * KBC;               // W2 k-blocks per tile row
+        const uint8_t *w2 = g.w2 + (size_t)ui.expert * NT * KB2 * FD_A_BYTES;
+        for (int n = nt0; n < nt1; ++n) {
+          for (int kk = 0; kk < KBC; ++kk) {
+            mbar_wait(&empty[stage], phase ^ 1);
+            mbar_expect_tx(&full[stage], A_TX);
+            if (W4)
+              tma_load_2d_hint(sA + stage * FD_A_BYTES, &g.w2_map4, &full[stage], ui.chunk * 128,
+                               ui.expert * p.H + n * 256, pol);
+            else
+              bulk_load_hint(sA + stage * FD_A_BYTES, w2 + ((size_t)n * KB2 + ui.chunk * KBC + kk) * FD_A_BYTES,
+                             FD_A_BYTES, &full[stage], pol);
+            if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
+          }
+        }
       }
-      // ---- queue I: this CTA's own units ----
-      for (; phaseI;) {
-        const int u = atomicAdd(p.sched, 1);
-        if (u >= n_prev) wait_routing();
-        const FdUnit ui = fd_unit(p, u, n_prev, splitS);
-        mbar_wait(&uqI_empty[qsI], qphI ^ 1);
-        unit_qI[qsI] = make_int4(ui.expert, ui.chunk, ui.group, ui.valid);
-        mbar_arrive(&uqI_full[qsI]);
-        if (++qsI == FD_UQ) { qsI = 0; qphI ^= 1; }
-        if (!ui.valid) break;
-        loads(ui, false);
-      }
-      // every load of this CTA is issued: let the finalize kernel launch now, so
-      // its launch latency overlaps the last stages (it waits for our completion)
-      pdl_trigger();
     }
   } else if (warp == 1) {
     // ============================ MMA issuer ============================
     // (touches only shared memory and TMEM: no griddepcontrol.wait needed)
-    int stage = 0; uint32_t phase = 0, hph = 0;
+    int stage = 0; uint32_t phase = 0, qs = 0, qph = 0, hph = 0;
     int ab = 0; uint32_t abph = 0;
     int as = 0; uint32_t asph = 0;
-    QState qst;
     for (;;) {
-      int4 uq;
-      const bool split = next_unit(qst, uq);
+      mbar_wait(&uq_full[qs], qph);
+      const int4 uq = unit_q[qs];
+      __syncwarp();
+      if (lane == 0) release_slot(qs);
+      if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
       if (!uq.w) break;
-      const int kb0 = split ? skb0 : 0, kb1 = split ? skb1 : KA, nt0 = split ? snt0 : 0, nt1 = split ? snt1 : NT;
       // ---- phase A ----
       for (int kb = kb0; kb < kb1; ++kb) {
         if (kExperiments && (p.debug & 2)) {     // timing experiment: phase-A loads only (no MMAs)
@@ -489,13 +430,12 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     const int qg = q >> 1;
     const int et = threadIdx.x - 64;             // 0..127
     const uint32_t lane_base = (uint32_t)(q * 32) << 16;
-    uint32_t aph = 0;
+    uint32_t qs = 0, qph = 0, aph = 0;
     int ab = 0; uint32_t abph = 0;
     int as = 0; uint32_t asph = 0;
     int ui_par = 0;
     uint32_t hph_e = 0, pph = 0;                 // cluster peers: h_ready phase; leader: part_bar phase
-    bool waited = false, xs_loaded = false;
-    QState qst;
+    bool waited = false;
     // MOE_DEBUG_TRACE: per-CTA timeline (globaltimer ns) into p.trace[8 + 8 * cta ..] (timing experiments)
     unsigned long long *tr = (p.trace && warp == 2 && lane == 0) ? p.trace + 8 + 8 * blockIdx.x : nullptr;
     if (tr) {
@@ -521,25 +461,19 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     if (FP8 && p.has_prev) load_xs(p.g[2].xs, xs_s + FD_MAX_KB * FD_N);   // previous layer: complete
     asm volatile("bar.sync 3, 128;" ::: "memory");
     for (;;) {
-      int4 uq;
-      const bool split = next_unit(qst, uq);
+      mbar_wait(&uq_full[qs], qph);
+      const int4 uq = unit_q[qs];
+      __syncwarp();
+      if (lane == 0) release_slot(qs);
+      if (++qs == FD_UQ) { qs = 0; qph ^= 1; }
       if (!uq.w) break;
       const int expert = uq.x, chunk = uq.y, group = uq.z;
-      const int kb0 = split ? skb0 : 0, kb1 = split ? skb1 : KA, nt0 = split ? snt0 : 0, nt1 = split ? snt1 : NT;
-      if (group == 1 && splitS) {
-        if (!xs_loaded) {                        // split shared units: this layer's x scales only
-          while (ld_acquire_gpu(p.xq_ready) < p.xq_target) __nanosleep(128);
-          if (FP8) load_xs(p.g[0].xs, xs_s);
-          asm volatile("bar.sync 3, 128;" ::: "memory");
-          xs_loaded = true;
-        }
-      } else if (group != 2 && !waited) {
+      if (group != 2 && !waited) {
         pdl_wait();                              // this layer's routing results and activation scales
         if (tr) tr[1] = gtimer();
-        if (FP8 && !xs_loaded) load_xs(p.g[0].xs, xs_s);
+        if (FP8) load_xs(p.g[0].xs, xs_s);
         asm volatile("bar.sync 3, 128;" ::: "memory");
         waited = true;
-        xs_loaded = true;
       }
       const FdGroup &g = p.g[group];
       const float *xsg = xs_s + (group == 2 ? FD_MAX_KB * FD_N : 0);
@@ -624,7 +558,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       }
       if (tr) tr[3] = gtimer();
       constexpr uint32_t H_TX = FP8 ? 2 * FD_B_BYTES / 2 + 4 * FD_N : FD_H_BYTES;   // h_c (+ FP8 scales) bytes
-      if (split) {
+      if (csize > 1) {
         // ---- cluster: the peers' partial gate/up sums -> the leader (through L2) ----
         float *scr = p.cl_scratch + (size_t)cluster_id_x() * 7 * 128 * 32;
         const bool dsm = fd_dsmem_partials(csize, p.T);
@@ -734,7 +668,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         fence_proxy_async_smem();                 // generic-proxy h writes -> the MMA's async-proxy reads
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
-      if (split) {
+      if (csize > 1) {
         // push h_c (and the FP8 h scales) into every peer's shared memory
         constexpr int HV = (FP8 ? 2 * FD_B_BYTES / 2 : FD_H_BYTES) / 16;   // 16-byte vectors of h_c
         for (int i = et; i < HV; i += 128) {
@@ -815,8 +749,6 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     if (atomicAdd(p.done, 1) == (int)gridDim.x - 1) {
       asm volatile("fence.acq_rel.gpu;" ::: "memory");
       atomicExch(p.sched, 0);
-      atomicExch(p.sched_s, 0);
-      if (p.xq_ready) atomicExch(p.xq_ready, 0);   // (the route's increments of this forward are done)
       atomicExch(p.done, 0);
     }
   }
