@@ -380,6 +380,131 @@ __global__ void __launch_bounds__(RT_WARPS * 32) router_select_regs_kernel(const
   if (t < a.T) select_token_regs(a, t, scratch[warp], nullptr, lane, true);
 }
 
+// ---- one token, the whole CTA (decode at T = 1) ----
+// Sigmoid scores, groups of exactly 32 experts (or no group limit), k <= 8: warp w scores
+// experts 32w .. 32w+31 (one per lane), takes its group's score and its best k with warp
+// max-reductions (redux.sync) on order-preserving bits -- ties to the lowest lane = the lower
+// id -- and warp 0 merges the kept groups' candidates.  Same rules, tie-breaks and float
+// operations (sigmoid, the sequential weight sum, one reciprocal) as select_token_regs, so
+// both give bit-identical routing.
+__device__ __forceinline__ uint32_t ord_bits(float v) {
+  const uint32_t u = __float_as_uint(v);
+  return (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+}
+__device__ __forceinline__ float ord_float(uint32_t o) {
+  return __uint_as_float((o & 0x80000000u) ? (o & 0x7FFFFFFFu) : ~o);
+}
+__device__ __forceinline__ bool route_one_fast_ok(const RouterArgs &r) {
+  const int E = r.E, G = r.n_group;
+  const int ng = G > 1 ? r.topk_group : E / 32;
+  return r.T == 1 && r.score_fn == MOE_SCORE_SIGMOID && r.k <= 8 && E % 32 == 0 && E <= RS_MAX_E &&
+         (G <= 1 || E == 32 * G) && ng * r.k <= 32;
+}
+// Writes topk_idx / topk_w / sgate and ids_s[0 .. k) (canonical order).  With lists = true
+// (all experts local, no debug outputs) also the fused decode's active / immediate / deferred
+// expert lists (ascending ids) and re-arms the CTA counter.
+__device__ void route_one_fast(const RouteSmallArgs &a, int *ids_s, bool lists) {
+  const RouterArgs &r = a.r;
+  const int E = r.E, G = r.n_group, k = r.k;
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+  const int NW = E / 32;
+  __shared__ float s_all[RS_MAX_E], gsc_s[8], sv_s[8];
+  __shared__ uint32_t cand_o[32];
+  __shared__ int cand_id[32], id_s[8], rc_s[8];
+  const bool act = w < NW;                       // warp-uniform
+  const int e = w * 32 + lane;
+  uint32_t o = 0u;
+  if (act) {
+    const float l = r.logits[e];
+    const float b = r.bias ? r.bias[e] : 0.f;
+    const float s = __fdividef(1.f, 1.f + __expf(-l));
+    s_all[e] = s;
+    o = ord_bits(s + b);
+  }
+  unsigned long long *tr = a.trace ? a.trace + 1900 : nullptr;     // MOE_DEBUG_TRACE: phase stamps
+  if (tr && tid == 0) tr[0] = gtimer_ns();
+  int slot0 = w * k;                             // this group's place in the candidate list
+  bool keep = true;
+  if (G > 1) {
+    if (act) {
+      const uint32_t m1 = __reduce_max_sync(0xffffffffu, o);
+      const uint32_t one = __ballot_sync(0xffffffffu, o == m1);
+      const uint32_t m2 = __reduce_max_sync(0xffffffffu, lane == __ffs(one) - 1 ? 0u : o);
+      if (lane == 0)
+        gsc_s[w] = r.group_score == MOE_GROUP_TOP2_SUM ? ord_float(m1) + ord_float(m2) : ord_float(m1);
+    }
+    __syncthreads();
+    if (tr && tid == 0) tr[1] = gtimer_ns();
+    if (act) {
+      const float mine = gsc_s[w];
+      int rk = 0;
+      for (int j = 0; j < G; ++j) rk += better(gsc_s[j], j, mine, w);
+      keep = rk < r.topk_group;
+      slot0 = rk * k;                            // group rank: unique among the kept groups
+    }
+  }
+  if (act && keep) {
+    uint32_t c = o;
+#pragma unroll 1
+    for (int i = 0; i < k; ++i) {
+      const uint32_t m = __reduce_max_sync(0xffffffffu, c);
+      const int win = __ffs(__ballot_sync(0xffffffffu, c == m)) - 1;
+      if (lane == win) c = 0u;
+      if (lane == 0) { cand_o[slot0 + i] = m; cand_id[slot0 + i] = w * 32 + win; }
+    }
+  }
+  __syncthreads();
+  if (tr && tid == 0) tr[2] = gtimer_ns();
+  if (w != 0) return;
+  const int nc = (G > 1 ? r.topk_group : NW) * k;
+  const bool has = lane < nc;
+  const uint32_t mo = has ? cand_o[lane] : 0u;
+  const int mid = has ? cand_id[lane] : 0x7fffffff;
+  int rank = 0;
+  for (int j = 0; j < nc; ++j) {
+    const uint32_t oj = cand_o[j];
+    rank += (oj > mo) | ((oj == mo) & (cand_id[j] < mid));
+  }
+  if (has && rank < k) { id_s[rank] = mid; sv_s[rank] = s_all[mid]; }
+  __syncwarp();
+  float sum = 0.f;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) sum += i < k ? sv_s[i] : 0.f;
+  const float cmul = (r.norm_topk ? 1.f / sum : 1.f) * r.routed_scale;
+  int rc = 0, my_id = 0;
+  if (lane < k) {
+    my_id = id_s[lane];
+    const float my_w = sv_s[lane] * cmul;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) rc += (i < k) & (i != lane) & better(sv_s[i] * cmul, id_s[i], my_w, my_id);
+    r.topk_idx[rc] = my_id;
+    r.topk_w[rc] = my_w;
+    ids_s[rc] = my_id;
+    rc_s[lane] = rc;
+  }
+  if (r.shared_gated && lane == 0) r.sgate[0] = 1.f / (1.f + expf(-r.logits[E]));
+  if (tr && lane == 0) tr[3] = gtimer_ns();
+  if (!lists) return;
+  __syncwarp();
+  if (lane < k) {
+    // T = 1: the k experts are distinct -- a list position is a count of smaller ids
+    const bool imm = rc < a.n_imm;
+    int below = 0, below_same = 0;
+    for (int i = 0; i < k; ++i) {
+      const bool lt = id_s[i] < my_id;
+      below += lt;
+      below_same += lt & ((rc_s[i] < a.n_imm) == imm);
+    }
+    a.p.act_list[below] = my_id;
+    if (a.imm_list) (imm ? a.imm_list : a.def_list)[below_same] = my_id;
+  }
+  if (lane == 0) {
+    *a.p.n_active = k;
+    if (a.imm_list) { *a.n_imm_list = min(a.n_imm, k); *a.n_def_list = k - min(a.n_imm, k); }
+    *a.done = 0;                                 // re-arm the CTA counter (graph replay)
+  }
+}
+
 // The last router CTA: route every token (one warp per token), then the
 // expert-sorted order for T <= 16 tokens -- with at most T <= kPadM rows per
 // expert every active expert's padded segment is one 128-row tile, so its
@@ -398,11 +523,21 @@ __device__ void route_small_tail(const RouteSmallArgs &a, float *rsm, const floa
   long long ck[4];
   ck[0] = clock64();
   if (a.trace && tid == 0) a.trace[1] = gtimer_ns();
+  const bool fast = route_one_fast_ok(r) && !(kExperiments && (a.debug & 16));   // MOE_DEBUG_ROUTE=16: general select
+  if (fast) {
+    const bool lists = p.e0 == 0 && p.E == r.E && !p.dbg_perm && !p.dbg_counts;
+    route_one_fast(a, ids_s, lists);
+    if (lists) {
+      if (a.trace && tid == 0) { a.trace[2] = gtimer_ns(); a.trace[3] = a.trace[4] = a.trace[2]; }
+      return;
+    }
+    __syncthreads();
+  }
   for (int e = tid; e < p.E; e += RS_THREADS) cnt_s[e] = 0;
   if (tid < RS_MAX_E / 32) bm[tid] = bmi[tid] = bmd[tid] = 0u;
   // one warp per token; warps past the last token skip (warp-uniform branch)
 #pragma unroll 1
-  for (int t0 = 0; t0 < T; t0 += RS_THREADS / 32) {
+  for (int t0 = 0; t0 < T && !fast; t0 += RS_THREADS / 32) {
     const int t = __shfl_sync(0xffffffffu, t0 + warp, 0);
     if (t < T) select_token_regs(r, t, rsm + warp * 2 * RS_MAX_E, ids_s, lane, true, bias_pre);
   }

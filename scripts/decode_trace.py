@@ -68,6 +68,9 @@ t0 = int(buf[0])
 rel = lambda v: (int(v) - t0) / 1e3
 if buf[6]:
     print(f"route select cycles: first pass {int(buf[5])}, warm second pass {int(buf[6])}")
+if buf[1900]:
+    print("route one-token select (us): scores " + " ".join(f"{rel(buf[1900 + i]):.2f}" for i in range(4)) +
+          "  (scores, groups, candidates, merged)")
 print(f"route: entry 0, tail start {rel(buf[1]):.1f}, select done {rel(buf[2]):.1f}, permute done {rel(buf[3]):.1f}, end {rel(buf[4]):.1f} us")
 cta = buf[8:8 + 8 * 148].reshape(148, 8).astype(np.int64)
 act = cta[cta[:, 5] > 0]

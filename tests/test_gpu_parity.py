@@ -341,3 +341,23 @@ def test_fused_decode_repeats(lib, name):
     assert d <= 2 ** -6 * max(1.0, ya.abs().max().item()), d
     fused.close()
     gemm.close()
+
+
+def test_full_v3_single_token_decode_calls(lib):
+    """T = 1 forwards without routing outputs -- the router's one-token select and its
+    active-expert list (router.cu route_one_fast) -- on 4 separate tokens, each against the
+    oracle with the residual."""
+    p = PRESETS["v3"]
+    w = make_weights(p, "cuda")
+    x, r = make_tokens(p, 4, "cuda", offset=21)
+    layer = lib.MoELayer(p, w, max_tokens=16)
+    ys = [layer.forward(x[i:i + 1].contiguous(), residual=r[i:i + 1].contiguous()) for i in range(4)]
+    torch.cuda.synchronize()
+    y = torch.cat(ys).float().cpu().numpy()
+    cfg, W = oracle_cfg(p), oracle_weights(p, w)
+    x64 = x.cpu().to(torch.float64).numpy()
+    ties = O.tie_band_tokens(x64, W, cfg)
+    keep = np.setdiff1d(np.arange(4), ties)
+    out = O.moe_layer(x64[keep], W, cfg, residual=r.cpu().to(torch.float64).numpy()[keep])
+    check_output("full/v3/T1x4/no_routing_out", y[keep], out["y"], TOL[p.wtype], ties=len(ties))
+    layer.close()
