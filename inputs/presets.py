@@ -83,6 +83,10 @@ SMALL = {
                                            shared_ffn=512, prefill_tokens=77),
     "v3_s": PRESETS["v3"].with_(name="v3_s", hidden=512, ffn=256, n_experts=64,
                                 shared_ffn=256, prefill_tokens=333),
+    # DeepSeek-V3 gate with two groups of exactly 32 experts (the router's one-token CTA path
+    # takes one group per warp)
+    "v3_g32": PRESETS["v3"].with_(name="v3_g32", hidden=512, ffn=256, n_experts=64, n_group=2, topk_group=1,
+                                  shared_ffn=256, prefill_tokens=200),
     # mid-size FP8: H = 2048 (16 W13 k-blocks = 4 scale groups), F = 1024 (8 W2
     # k-blocks = 2 groups), so both TMEM scale-column sets are exercised
     "v3_m": PRESETS["v3"].with_(name="v3_m", hidden=2048, ffn=1024, n_experts=32,

@@ -381,11 +381,11 @@ __global__ void __launch_bounds__(RT_WARPS * 32) router_select_regs_kernel(const
 }
 
 // ---- one token, the whole CTA (decode at T = 1) ----
-// Sigmoid scores, groups of exactly 32 experts (or no group limit), k <= 8: warp w scores
+// Groups of exactly 32 experts (or no group limit), k <= 8, E <= 256: warp w scores
 // experts 32w .. 32w+31 (one per lane), takes its group's score and its best k with warp
 // max-reductions (redux.sync) on order-preserving bits -- ties to the lowest lane = the lower
 // id -- and warp 0 merges the kept groups' candidates.  Same rules, tie-breaks and float
-// operations (sigmoid, the sequential weight sum, one reciprocal) as select_token_regs, so
+// operations (sigmoid / softmax, the sequential weight sum, one reciprocal) as select_token_regs, so
 // both give bit-identical routing.
 __device__ __forceinline__ uint32_t ord_bits(float v) {
   const uint32_t u = __float_as_uint(v);
@@ -397,7 +397,7 @@ __device__ __forceinline__ float ord_float(uint32_t o) {
 __device__ __forceinline__ bool route_one_fast_ok(const RouterArgs &r) {
   const int E = r.E, G = r.n_group;
   const int ng = G > 1 ? r.topk_group : E / 32;
-  return r.T == 1 && r.score_fn == MOE_SCORE_SIGMOID && r.k <= 8 && E % 32 == 0 && E <= RS_MAX_E &&
+  return r.T == 1 && r.k <= 8 && E % 32 == 0 && E <= RS_MAX_E &&
          (G <= 1 || E == 32 * G) && ng * r.k <= 32;
 }
 // Writes topk_idx / topk_w / sgate and ids_s[0 .. k) (canonical order).  With lists = true
@@ -414,7 +414,28 @@ __device__ void route_one_fast(const RouteSmallArgs &a, int *ids_s, bool lists) 
   const bool act = w < NW;                       // warp-uniform
   const int e = w * 32 + lane;
   uint32_t o = 0u;
-  if (act) {
+  if (r.score_fn == MOE_SCORE_SOFTMAX) {
+    // warp 0 computes the softmax in select_token_regs's layout and order (lane l: experts
+    // 8l .. 8l+7; lane max, warp max, lane sum, warp sum, one reciprocal) -- bit-identical s
+    if (w == 0) {
+      float lv[8], m = -INFINITY, sum = 0.f, sv[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        lv[i] = lane * 8 + i < E ? r.logits[lane * 8 + i] : -INFINITY;
+        m = i ? fmaxf(m, lv[i]) : lv[i];
+      }
+      m = warp_max(m);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) { sv[i] = lane * 8 + i < E ? __expf(lv[i] - m) : 0.f; sum += sv[i]; }
+      sum = warp_sum(sum);
+      const float inv = 1.f / sum;
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        if (lane * 8 + i < E) s_all[lane * 8 + i] = sv[i] * inv;
+    }
+    __syncthreads();
+    if (act) o = ord_bits(s_all[e] + (r.bias ? r.bias[e] : 0.f));
+  } else if (act) {
     const float l = r.logits[e];
     const float b = r.bias ? r.bias[e] : 0.f;
     const float s = __fdividef(1.f, 1.f + __expf(-l));

@@ -72,7 +72,7 @@ def test_small_layer_parity(lib, name):
     check_output(f"small/{name}/T{T}", res["y"], out["y"], TOL[p.wtype], ties=len(ties))
 
 
-@pytest.mark.parametrize("name", ["toy", "v3_s", "v2lite_s", "v2lite_h384", "v3_s_fp4"])
+@pytest.mark.parametrize("name", ["toy", "v3_s", "v2lite_s", "v2lite_h384", "v3_s_fp4", "v3_g32"])
 @pytest.mark.parametrize("T", [1, 3, 17])
 def test_small_decode_shapes(lib, name, T):
     p = SMALL[name]

@@ -129,7 +129,7 @@ def _chain_oracle(p, ws, xs, rs, n_defs):
     return outs, sorted(ties)
 
 
-@pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v2lite_s", "v3_m", "v25_s", "v3_s_fp4"])
+@pytest.mark.parametrize("name", ["v3_s", "qwen2_s", "v2lite_s", "v3_m", "v25_s", "v3_s_fp4", "v3_g32"])
 @pytest.mark.parametrize("T", [1, 5, 16])
 def test_chained_deferral_matches_eq_L241(lib, name, T):
     """A 3-layer chain (k = 1: no deferred input; k = L: n_def = 0) against Eq.
