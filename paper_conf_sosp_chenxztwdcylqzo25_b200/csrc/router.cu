@@ -704,8 +704,9 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
     bpre[i] = (r.bias && e < r.E) ? __ldg(r.bias + e) : 0.f;
   }
   // chained deferral: the decode stream may launch now and stream the previous layer's deferred
-  // experts beside us; otherwise it launches when every CTA here has exited (measured ~1 us/layer
-  // faster: CTAs waiting in griddepcontrol.wait beside ours slow the routing down)
+  // experts beside us; otherwise it launches once only the last CTA's tail is left (a launch
+  // here measured ~1 us/layer slower: CTAs waiting in griddepcontrol.wait beside all 128 router
+  // CTAs slow the logits phase down)
   if (a.early_trigger) pdl_trigger();
   // (an instruction-cache warm-up -- a dry run of the selection before the dependency wait --
   //  was measured: the window before the wait is ~1-2 us, so the dry run lands on the
@@ -836,6 +837,9 @@ __global__ void __launch_bounds__(RS_THREADS) route_small_kernel(const __grid_co
   }
   __syncthreads();
   if (!is_last) return;
+  // every other CTA has exited: the decode stream may launch now, so its launch latency and
+  // prologue overlap this tail (its griddepcontrol.wait still waits for the whole grid)
+  if (!a.early_trigger && !(kExperiments && (a.debug & 64))) pdl_trigger();   // MOE_DEBUG_ROUTE=64: at exit
   if (kExperiments && (a.debug & 2)) { if (threadIdx.x == 0) *a.done = 0; return; }
   route_small_tail(a, rsm, bpre);
 }
