@@ -271,7 +271,10 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             const uint32_t a0 = smem_u32(sW + stage * SW_W_BYTES);
             const uint32_t b0 = smem_u32(sX + stage * SW_X_BYTES);
             // one scale image covers 4 k-blocks (sf id = kb & 3); two TMEM column
-            // sets alternate so a copy never overwrites scales in use
+            // sets alternate so a copy never overwrites scales in use.  The copy and the
+            // MMAs are issued by this one thread into the tensor pipe, which executes its
+            // tcgen05.cp / tcgen05.mma in issue order: the copy into set s at kb = 4j + 8 runs
+            // after the MMAs of kb = 4j .. 4j + 3 that read set s, whatever SW_STAGES is
             const uint32_t set = FP8 ? ((kb >> 2) & 1) * 16 : 0;
             if (FP8 && (kb & 3) == 0) {
               tmem_cp_32x128b_x4_pair(tmem + SW_SFA_COL + set, sf_desc(smem_u32(sSFW + stage * SW_SFW_BYTES)));
