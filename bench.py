@@ -355,19 +355,24 @@ def run_ours(args):
         rows = [xd[i:i + 1].contiguous() for i in range(xd.shape[0])]
         st = torch.cuda.current_stream()
 
-        def time_chain(dlayers, n_def=0, chained=False):
+        def time_chain(dlayers, n_def=0, chained=False, cyclic=False):
+            # cyclic (chained only): every layer defers and layer 0 takes the last layer's deferred
+            # experts of the previous replay -- a deep stack's steady state, without the two end
+            # layers of a finite chain (the first streams 5 experts, the last 8 + 3)
             bufs = [rows[0].clone(), torch.empty_like(rows[0])]
+            first = [True]
 
             def dstep():
-                prev = None
+                prev = dlayers[-1] if (cyclic and not first[0]) else None
                 for i, l in enumerate(dlayers):
                     a_, b_ = bufs[i % 2], bufs[(i + 1) % 2]
                     if chained:
-                        nd = n_def if i < len(dlayers) - 1 else 0
+                        nd = n_def if (cyclic or i < len(dlayers) - 1) else 0
                         l.forward_chained(a_, residual=a_, n_deferred=nd, prev=prev, y=b_)
                         prev = l
                     else:
                         l.forward(a_, residual=a_, y=b_)
+                first[0] = False
 
             side = torch.cuda.Stream()
             side.wait_stream(torch.cuda.current_stream())
@@ -413,10 +418,17 @@ def run_ours(args):
             decode["roofline"]["stage_us_eager"] = {k: round(v * 1e3, 2) for k, v in dstages.items()}
             if not args.no_deferral and p.top_k > 3:
                 dd = time_chain(dlayers, n_def=3, chained=True)
+                dc = time_chain(dlayers, n_def=3, chained=True, cyclic=True)
                 decode["deferral"] = {"n_deferred": 3, "us_per_layer": dd, "speedup_vs_no_deferral": dus / dd,
                                       "roofline": hbm(dd),
                                       "mode": "moe_layer_forward_chained: layer i streams layer i-1's deferred "
-                                              "experts while its own router runs (PAPER.md L241)"}
+                                              "experts while its own router runs (PAPER.md L241); finite chain, "
+                                              "last layer n_def = 0",
+                                      "steady_state": {"us_per_layer": dc, "speedup_vs_no_deferral": dus / dc,
+                                                       "roofline": hbm(dc),
+                                                       "mode": "cyclic chain: every layer defers, layer 0 takes "
+                                                               "the last layer's deferred experts of the previous "
+                                                               "replay (same bytes per layer as plain)"}}
             for l in dlayers[1:]:
                 l.close()
             del dlayers

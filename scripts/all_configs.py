@@ -43,7 +43,7 @@ def prefill(name, T):
     return r
 
 
-def decode(name, T, L=8, n_def=0):
+def decode(name, T, L=8, n_def=0, cyclic=False):
     p = PRESETS[name]
     w = make_weights(p, "cuda")
     layers = [moe.MoELayer(p, w, max_tokens=16) for _ in range(L)]
@@ -54,15 +54,20 @@ def decode(name, T, L=8, n_def=0):
     bufs = [rows[0].clone(), torch.empty_like(rows[0])]
     dbufs = [torch.zeros_like(rows[0]), torch.zeros_like(rows[0])]
 
+    first = [True]
+
     def step():
-        prev = None
+        # cyclic: every layer defers and layer 0 takes the last layer's deferred experts of the
+        # previous replay (a deep stack's steady state, no end layers)
+        prev = layers[-1] if (cyclic and not first[0]) else None
         for i, l in enumerate(layers):
             a, b = bufs[i % 2], bufs[(i + 1) % 2]
             if n_def:       # Eq. L241 across the chain: layer i computes layer i-1's deferred experts
-                l.forward_chained(a, residual=a, n_deferred=n_def if i < L - 1 else 0, prev=prev, y=b)
+                l.forward_chained(a, residual=a, n_deferred=n_def if (cyclic or i < L - 1) else 0, prev=prev, y=b)
                 prev = l
             else:
                 l.forward(a, residual=a, y=b)
+        first[0] = False
     s = torch.cuda.Stream(); s.wait_stream(torch.cuda.current_stream())
     with torch.cuda.stream(s):
         for _ in range(2):
@@ -94,13 +99,16 @@ def decode(name, T, L=8, n_def=0):
     return r
 
 
-plan = [("prefill", "v2lite", 512, 0), ("decode", "v2lite", 1, 0), ("decode", "v2lite", 1, 3),
-        ("prefill", "qwen2", 2048, 0), ("decode", "qwen2", 1, 0), ("decode", "qwen2", 1, 3),
-        ("prefill", "v25", 4096, 0), ("decode", "v25", 4, 0), ("decode", "v25", 4, 3),
-        ("prefill", "v3", 8192, 0), ("decode", "v3", 1, 0), ("decode", "v3", 1, 3), ("decode", "v3", 1, 6),
-        ("prefill", "v3_fp4", 8192, 0), ("decode", "v3_fp4", 1, 0), ("decode", "v3_fp4", 1, 3)]
+# decode rows: (n_def, cyclic) -- cyclic = the steady state of a deep stack (every layer defers)
+plan = [("prefill", "v2lite", 512, 0), ("decode", "v2lite", 1, 0), ("decode", "v2lite", 1, 3), ("cyc", "v2lite", 1, 3),
+        ("prefill", "qwen2", 2048, 0), ("decode", "qwen2", 1, 0), ("decode", "qwen2", 1, 3), ("cyc", "qwen2", 1, 3),
+        ("prefill", "v25", 4096, 0), ("decode", "v25", 4, 0), ("decode", "v25", 4, 3), ("cyc", "v25", 4, 3),
+        ("prefill", "v3", 8192, 0), ("decode", "v3", 1, 0), ("decode", "v3", 1, 3), ("cyc", "v3", 1, 3),
+        ("decode", "v3", 1, 6),
+        ("prefill", "v3_fp4", 8192, 0), ("decode", "v3_fp4", 1, 0), ("decode", "v3_fp4", 1, 3), ("cyc", "v3_fp4", 1, 3)]
 for kind, name, T, nd_ in plan:
-    r = prefill(name, T) if kind == "prefill" else decode(name, T, n_def=nd_)
+    r = prefill(name, T) if kind == "prefill" else decode(name, T, n_def=nd_, cyclic=kind == "cyc")
+    r["cyclic"] = kind == "cyc"
     print(json.dumps(r), flush=True)
     rows_out.append(r)
 
@@ -112,7 +120,8 @@ with open(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/all_configs.md", "w"
                     f"{r['tflops']:.0f} TFLOP/s | {r['tensor_frac']*100:.1f} % of tensor peak, {r['hbm_frac']*100:.1f} % of HBM "
                     f"({r['distinct_experts']} experts hit) |\n")
         else:
-            f.write(f"| {r['config']} | decode{' n_def=%d' % r['n_deferred'] if r['n_deferred'] else ''} | {r['T']} | "
+            f.write(f"| {r['config']} | decode{' n_def=%d' % r['n_deferred'] if r['n_deferred'] else ''}"
+                    f"{' steady state (cyclic chain)' if r.get('cyclic') else ''} | {r['T']} | "
                     f"{r['us_per_layer']:.1f} us/layer | {r['gbs']:.0f} GB/s | {r['hbm_frac']*100:.1f} % of HBM "
                     f"({r['distinct_experts']} experts, {r['layer_bytes']/1e6:.1f} MB) |\n")
 print(open(sys.argv[1] if len(sys.argv) > 1 else "gpurun_out/all_configs.md").read())

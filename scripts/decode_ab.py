@@ -2,6 +2,8 @@
 the 8-layer chained CUDA graph (distinct V3 layers, L2 flushed before each replay),
   plain     -- moe_layer_forward per layer
   deferral  -- moe_layer_forward_chained, n_def = 3 (last layer 0)
+  deferral3_cyclic -- every layer defers; layer 0 takes the last layer's deferred experts of the
+              previous replay (the steady state of a deep stack: no end layers)
 Prints per-layer µs for each variant and round."""
 import json, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -21,16 +23,22 @@ bufs = [x0.clone(), torch.empty_like(x0)]
 flush = (torch.empty(64 << 20, device="cuda"), torch.zeros(64 << 20, device="cuda"), torch.zeros((), device="cuda"))
 
 
-def make_graph(n_def):
+def make_graph(n_def, cyclic=False):
+    # cyclic: every layer defers, and layer 0 takes the last layer's deferred experts from the
+    # previous replay -- the steady state of a deep stack, without the chain's two end layers
+    first = [True]
+
     def step():
-        prev = None
+        prev = layers[-1] if (cyclic and not first[0]) else None
         for i, l in enumerate(layers):
             a_, b_ = bufs[i % 2], bufs[(i + 1) % 2]
             if n_def:
-                l.forward_chained(a_, residual=a_, n_deferred=n_def if i < NL - 1 else 0, prev=prev, y=b_)
+                nd = n_def if (cyclic or i < NL - 1) else 0
+                l.forward_chained(a_, residual=a_, n_deferred=nd, prev=prev, y=b_)
                 prev = l
             else:
                 l.forward(a_, residual=a_, y=b_)
+        first[0] = False
     s = torch.cuda.Stream()
     s.wait_stream(torch.cuda.current_stream())
     with torch.cuda.stream(s):
@@ -43,7 +51,7 @@ def make_graph(n_def):
     return g
 
 
-graphs = {"plain": make_graph(0), "deferral3": make_graph(3)}
+graphs = {"plain": make_graph(0), "deferral3": make_graph(3), "deferral3_cyclic": make_graph(3, cyclic=True)}
 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
 res = {k: [] for k in graphs}
 for r in range(ROUNDS):
