@@ -55,6 +55,7 @@ constexpr int FD_H_BYTES = 2 * FD_B_BYTES;     // h_c: FP8 one k-block, BF16 two
 constexpr int FD_MAX_KB = 64;                  // H <= 8192: FP8 k-blocks of W13
 constexpr size_t FD_SMEM = 1024 + (size_t)FD_STAGES * (FD_A_BYTES + FD_B_BYTES) + FD_H_BYTES +
                            2 * 2 * FD_N * 32 * 4 +     // up -> gate exchange [gate warp][acc][token][lane]
+                           2 * 2 * FD_N * 32 * 4 +     // gate values, then h, [gate warp][acc][token][lane]
                            2 * FD_MAX_KB * FD_N * 4 +  // activation scales [this layer | previous layer][kb][token]
                            1024;                       // barriers, queue, amax, scales
 constexpr uint32_t FD_TMEM_COLS = 256;
@@ -194,7 +195,8 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
   uint8_t *sB = sH + FD_H_BYTES;
   float *xch = reinterpret_cast<float *>(sB + FD_STAGES * FD_B_BYTES);   // [2][2][16][32]
   float *xs_s = xch + 2 * 2 * FD_N * 32;                     // [2: this layer, previous layer][FD_MAX_KB][16]
-  uint64_t *full = reinterpret_cast<uint64_t *>(xs_s + 2 * FD_MAX_KB * FD_N);
+  float *gbuf = xs_s + 2 * FD_MAX_KB * FD_N;                 // [2][2][16][32] gate values -> h (SwiGLU)
+  uint64_t *full = reinterpret_cast<uint64_t *>(gbuf + 2 * 2 * FD_N * 32);
   uint64_t *empty = full + FD_STAGES;
   uint64_t *accA_full = empty + FD_STAGES;                   // [FD_ACCA_SLOTS]
   uint64_t *accA_empty = accA_full + FD_ACCA_SLOTS;          // [FD_ACCA_SLOTS]
@@ -587,9 +589,11 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
           if (tr) tr[4] = gtimer();
           goto phase_b;
         }
+        unsigned long long *tl = (p.trace && warp == 2 && lane == 0) ? p.trace + 1300 + 4 * blockIdx.x : nullptr;
         if (dsm) {
           if (q == 0 && lane == 0) mbar_expect_tx(part_bar, (csize - 1) * 128 * 2 * p.T * 4);
           mbar_wait_cluster(part_bar, pph);
+          if (tl) tl[0] = gtimer();
           pph ^= 1;
           for (uint32_t r = 1; r < csize; ++r) {
             const float *src = xch + ((size_t)(r - 1) * 128 + et) * 2 * p.T;
@@ -615,59 +619,70 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         }
       }
       {
+      unsigned long long *tl = (p.trace && csize > 1 && warp == 2 && lane == 0) ? p.trace + 1300 + 4 * blockIdx.x : nullptr;
+      if (tl) tl[1] = gtimer();
       // ---- SwiGLU + requant -> h_c (B operand of phase B) ----
-      float *xb = xch + qg * (2 * FD_N * 32);
-      if (q & 1) {
+      // The accumulators go to shared memory once (unrolled: one store per live token), then
+      // rolled loops over the T live tokens: this code runs once per unit with a cold
+      // instruction cache while the weight streams load L2, so its footprint -- not its
+      // instruction count -- is what the unit waits for (the 16-way unrolled form with
+      // predicated-off token columns measured ~3.5 us here at T = 1).
+      float *xb = xch + qg * (2 * FD_N * 32);      // up values
+      float *gb = gbuf + qg * (2 * FD_N * 32);     // gate values, then h
+      {
+        float *dst = (q & 1) ? xb : gb;
 #pragma unroll
         for (int t = 0; t < FD_N; ++t) {
           if (t < p.T) {                        // (warp-uniform: token columns >= T are never read)
-            xb[t * 32 + lane] = r0[t];
-            xb[(FD_N + t) * 32 + lane] = r1[t];
+            dst[t * 32 + lane] = r0[t];
+            dst[(FD_N + t) * 32 + lane] = r1[t];
           }
         }
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
+      unsigned long long *tq = (p.trace && csize > 1 && !(q & 1) && lane == 0) ? p.trace + 2100 + 8 * blockIdx.x + 4 * qg : nullptr;
+      if (tq) tq[0] = gtimer();
       const int f0 = qg * 32 + lane;             // h column within the chunk (accumulator 1: + 64)
       if (!(q & 1)) {
-        float h0[FD_N], h1[FD_N];
-#pragma unroll
-        for (int t = 0; t < FD_N; ++t) {
-          h0[t] = t < p.T ? silu_f(r0[t]) * xb[t * 32 + lane] : 0.f;
-          h1[t] = t < p.T ? silu_f(r1[t]) * xb[(FD_N + t) * 32 + lane] : 0.f;
-        }
-        if (FP8) {
-#pragma unroll
-          for (int t = 0; t < FD_N; ++t) {
-            if (t < p.T) {
-              const float m = warp_max(fmaxf(fabsf(h0[t]), fabsf(h1[t])));
-              if (lane == 0) amax[qg * FD_N + t] = m;
-            }
+#pragma unroll 1
+        for (int t = 0; t < p.T; ++t) {
+          const float h0 = silu_f(gb[t * 32 + lane]) * xb[t * 32 + lane];
+          const float h1 = silu_f(gb[(FD_N + t) * 32 + lane]) * xb[(FD_N + t) * 32 + lane];
+          gb[t * 32 + lane] = h0;
+          gb[(FD_N + t) * 32 + lane] = h1;
+          if (FP8) {
+            const float m = warp_max(fmaxf(fabsf(h0), fabsf(h1)));
+            if (lane == 0) amax[qg * FD_N + t] = m;
           }
+        }
+        if (tq) tq[1] = gtimer();
+        if (FP8) {
           asm volatile("bar.sync 2, 64;" ::: "memory");   // the two gate warps
-#pragma unroll
-          for (int t = 0; t < FD_N; ++t) {
-            if (t >= p.T) continue;               // (phase B drops token columns >= T)
+          if (tq) tq[2] = gtimer();
+          const int f1 = f0 + 64;
+#pragma unroll 1
+          for (int t = 0; t < p.T; ++t) {
             const int e = ue8m0_exponent(fmaxf(amax[t], amax[FD_N + t]));
             const float inv = exp2i(-e);
             uint8_t *row = sH + t * 128;
-            row[(((f0 >> 4) ^ (t & 7)) << 4) | (f0 & 15)] = f32_to_e4m3(h0[t] * inv);
-            const int f1 = f0 + 64;
-            row[(((f1 >> 4) ^ (t & 7)) << 4) | (f1 & 15)] = f32_to_e4m3(h1[t] * inv);
+            row[(((f0 >> 4) ^ (t & 7)) << 4) | (f0 & 15)] = f32_to_e4m3(gb[t * 32 + lane] * inv);
+            row[(((f1 >> 4) ^ (t & 7)) << 4) | (f1 & 15)] = f32_to_e4m3(gb[(FD_N + t) * 32 + lane] * inv);
             if (qg == 0 && lane == 0) hsc[ui_par * FD_N + t] = exp2i(e);
           }
         } else {
           // two 64-column k-blocks of bf16: column f0 -> block 0, f0 + 64 -> block 1 (same in-block column)
-#pragma unroll
-          for (int t = 0; t < FD_N; ++t) {
-            if (t >= p.T) continue;
+#pragma unroll 1
+          for (int t = 0; t < p.T; ++t) {
             const int off = t * 128 + ((((f0 >> 3) ^ (t & 7)) << 4) | ((f0 & 7) << 1));
-            *reinterpret_cast<__nv_bfloat16 *>(sH + off) = __float2bfloat16_rn(h0[t]);
-            *reinterpret_cast<__nv_bfloat16 *>(sH + FD_B_BYTES + off) = __float2bfloat16_rn(h1[t]);
+            *reinterpret_cast<__nv_bfloat16 *>(sH + off) = __float2bfloat16_rn(gb[t * 32 + lane]);
+            *reinterpret_cast<__nv_bfloat16 *>(sH + FD_B_BYTES + off) = __float2bfloat16_rn(gb[(FD_N + t) * 32 + lane]);
           }
         }
+        if (tq) tq[3] = gtimer();
         fence_proxy_async_smem();                 // generic-proxy h writes -> the MMA's async-proxy reads
       }
       asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (tl) tl[2] = gtimer();
       if (csize > 1) {
         // push h_c (and the FP8 h scales) into every peer's shared memory
         constexpr int HV = (FP8 ? 2 * FD_B_BYTES / 2 : FD_H_BYTES) / 16;   // 16-byte vectors of h_c
@@ -684,6 +699,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
       }
       if (q == 0 && lane == 0) mbar_arrive(h_ready);
       if (tr) tr[4] = gtimer();
+      if (tl) tl[3] = gtimer();
       }
     phase_b:
       // ---- phase B epilogue: scaled, weighted partial sums of W2 row tiles ----

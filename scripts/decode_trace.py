@@ -89,3 +89,18 @@ for i in order:
     u = act[i]
     print(f"  slowest: sm {u[7]:3d} grp {u[6] >> 30} exp {(u[6] >> 16) & 0x3fff:3d} chunk {u[6] & 0xffff:2d} unit {(u[2]-t0)/1e3:6.1f} accA {(u[3]-t0)/1e3:6.1f} h {(u[4]-t0)/1e3:6.1f} end {(u[5]-t0)/1e3:6.1f}")
 print(f"finalize: past pdl {rel(buf[2000]):.1f}, end {rel(buf[2001]):.1f} us")
+lead = buf[1300:1300 + 4 * 148].reshape(148, 4).astype(np.int64)
+ld = lead[lead[:, 0] > 0]
+if len(ld):
+    acc = cta[:, 3]
+    print("cluster leaders (us): partials in " + st(np.array([rel(v) for v in ld[:, 0]])) +
+          " | summed " + st(np.array([rel(v) for v in ld[:, 1]])) + " | swiglu " + st(np.array([rel(v) for v in ld[:, 2]])) +
+          " | pushed " + st(np.array([rel(v) for v in ld[:, 3]])))
+gq = buf[2100:2100 + 8 * 148].reshape(148, 8).astype(np.int64)
+gq = gq[gq[:, 0] > 0]
+if len(gq):
+    for w in range(2):
+        g4 = gq[:, 4 * w:4 * w + 4]
+        print(f"leader gate warp {w} (us): exchanged " + st(np.array([rel(v) for v in g4[:, 0]])) + " | h " +
+              st(np.array([rel(v) for v in g4[:, 1]])) + " | amax " + st(np.array([rel(v) for v in g4[:, 2]])) +
+              " | quant " + st(np.array([rel(v) for v in g4[:, 3]])))

@@ -158,6 +158,33 @@ def test_chained_deferral_matches_eq_L241(lib, name, T):
         l.close()
 
 
+@pytest.mark.parametrize("name", ["v3_s", "v3_g32"])
+@pytest.mark.parametrize("T", [1, 5])
+def test_cyclic_chain_matches_eq_L241(lib, name, T):
+    """Two layers used cyclically, A B A B, every call deferring (the steady state bench.py's
+    decode.deferral.steady_state times): the second A takes B's deferred experts, so the
+    sequence is the Eq. L241 chain over [wA, wB, wA, wB] whose last layer keeps its deferred
+    slots pending."""
+    p = SMALL[name]
+    n_def = 3
+    wA, wB = make_weights(p, "cpu", seed=4100), make_weights(p, "cpu", seed=4117)
+    A = lib.MoELayer(p, wA.to("cuda"), max_tokens=16)
+    B = lib.MoELayer(p, wB.to("cuda"), max_tokens=16)
+    seq = [A, B, A, B]
+    xs = [make_tokens(p, T, "cuda", offset=41 + i)[0] for i in range(4)]
+    ys, prev = [], None
+    for i, l in enumerate(seq):
+        ys.append(l.forward_chained(xs[i], n_deferred=n_def, prev=prev))
+        prev = l
+    torch.cuda.synchronize()
+    outs, ties = _chain_oracle(p, [wA, wB, wA, wB], xs, [None] * 4, [n_def] * 4)
+    keep = np.setdiff1d(np.arange(T), ties)
+    for i in range(4):
+        check_output(f"cyclic/{name}/T{T}/call{i}", ys[i].float().cpu().numpy()[keep], outs[i][keep], TOL[p.wtype])
+    A.close()
+    B.close()
+
+
 def test_chained_without_deferral_is_the_plain_forward(lib):
     p = SMALL["v3_s"]
     w = make_weights(p, "cpu").to("cuda")
@@ -192,6 +219,30 @@ def test_chained_errors(lib):
     torch.cuda.synchronize()
     a.close()
     b.close()
+
+
+def test_full_v25_cyclic_chain_decode(lib):
+    """Full DeepSeek-V2.5 layers (FP8, 160 experts, softmax + group-limited gate), T = 4,
+    used cyclically A B A (every call defers 3 of 6 slots) -- the configuration whose
+    steady-state deferral timing (profiles/r02/all_configs.md) is the fastest -- against
+    the Eq. L241 oracle chain over [wA, wB, wA]."""
+    p = PRESETS["v25"]
+    T, n_def = 4, 3
+    wA, wB = make_weights(p, "cuda", seed=5100), make_weights(p, "cuda", seed=5101)
+    A = lib.MoELayer(p, wA, max_tokens=16)
+    B = lib.MoELayer(p, wB, max_tokens=16)
+    xs = [make_tokens(p, T, "cuda", offset=51 + i)[0] for i in range(3)]
+    ys, prev = [], None
+    for i, l in enumerate([A, B, A]):
+        ys.append(l.forward_chained(xs[i], n_deferred=n_def, prev=prev))
+        prev = l
+    torch.cuda.synchronize()
+    outs, ties = _chain_oracle(p, [wA, wB, wA], xs, [None] * 3, [n_def] * 3)
+    keep = np.setdiff1d(np.arange(T), ties)
+    for i in range(3):
+        check_output(f"cyclic_full/v25/T{T}/call{i}", ys[i].float().cpu().numpy()[keep], outs[i][keep], TOL[p.wtype])
+    A.close()
+    B.close()
 
 
 def test_full_v3_chain_decode(lib):
