@@ -278,6 +278,7 @@ struct SwapGroup {              // one operand set: 0 = routed experts, 1 = shar
   CUtensorMap w_map;            // tiled weights as 128-byte rows, box 128 rows
   CUtensorMap x_map;            // token rows, K-major SW128, box 32 rows (ragged tails)
   CUtensorMap x_map128;         // the same, box 128 rows (full halves)
+  CUtensorMap x_map64;          // the same, box 64 rows (a half split between 2 multicasting pairs)
   CUtensorMap sfw_map;          // FP8: weight scale images as 512-byte rows, box 1
   CUtensorMap sfx_map;          // FP8: token scale images as 512-byte rows, box 2
   int w_nblk;                   // 256-row weight blocks per expert
@@ -299,6 +300,8 @@ struct SwapParams {
   int debug_mode;               // 0; (MOE_DEBUG_GEMM) 2 = no epilogue math -- timing experiments
   unsigned long long *trace;     // MOE_DEBUG_TRACE: MMA-warp cycle breakdown per CTA pair (timing experiments)
 };
-cudaError_t launch_umma_swap_gemm(bool fp8, int epi, const SwapParams &p, int grid, cudaStream_t st);
+// np = 1: grid = CTAs (pairs of 2); np = 2: grid = clusters of 2 pairs sharing token boxes (multicast)
+cudaError_t launch_umma_swap_gemm(bool fp8, int epi, const SwapParams &p, int grid, int np, cudaStream_t st);
+int umma_swap_max_clusters4(bool fp8);   // co-resident clusters of 4 CTAs (0: not available)
 
 }  // namespace moe

@@ -482,6 +482,7 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
 
   // ---- tcgen05 path: scale images and tensor maps ----
   C_TRY(cudaDeviceGetAttribute(&L->num_sms, cudaDevAttrMultiProcessorCount, cfg->device));
+  if (L->umma) L->swap_clusters4 = umma_swap_max_clusters4(L->fp8);
   if (!make_kmajor_map(&L->map_gate, L->gate_w, false, L->gate_rows, H, 256))
     return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for the router weights"));
   {
@@ -537,12 +538,16 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
       ok = ok && make_blocks_map(&L->tmap_w13, L->w13, (int64_t)E * 2 * F * H * es, 2048, 8) &&
            make_blocks_map(&L->tmap_w2, L->w2, (int64_t)E * H * F * es, 2048, 8) &&
            make_kmajor_map(&L->xmap_xperm, L->xperm, f8, L->R_max, H, 32) &&
-           make_kmajor_map(&L->xmap_h, L->hbuf, f8, L->R_max, F, 32);
+           make_kmajor_map(&L->xmap_h, L->hbuf, f8, L->R_max, F, 32) &&
+           make_kmajor_map(&L->x64map_xperm, L->xperm, f8, L->R_max, H, 64) &&
+           make_kmajor_map(&L->x64map_h, L->hbuf, f8, L->R_max, F, 64);
       if (Fs) {
         ok = ok && make_blocks_map(&L->tmap_ws13, L->ws13, (int64_t)2 * Fs * H * es, 2048, 8) &&
              make_blocks_map(&L->tmap_ws2, L->ws2, (int64_t)H * Fs * es, 2048, 8) &&
-             make_kmajor_map(&L->xmap_hsh, L->hsh, f8, Tm, Fs, 32);
-        if (f8) ok = ok && make_kmajor_map(&L->xmap_xq, L->xq, true, Tm, H, 32);
+             make_kmajor_map(&L->xmap_hsh, L->hsh, f8, Tm, Fs, 32) &&
+             make_kmajor_map(&L->x64map_hsh, L->hsh, f8, Tm, Fs, 64);
+        if (f8) ok = ok && make_kmajor_map(&L->xmap_xq, L->xq, true, Tm, H, 32) &&
+                     make_kmajor_map(&L->x64map_xq, L->xq, true, Tm, H, 64);
       }
       if (f8) {
         const int64_t g1 = (H / 128 + 3) / 4, g2 = (F / 128 + 3) / 4, gs = (Fs / 128 + 3) / 4;
@@ -617,6 +622,19 @@ static inline void mark(moe_layer *L, int stage, cudaStream_t st) {
 // Prefill-shaped expert GEMMs: routed experts over the sorted rows described by
 // L->tiles (built by the permutation) and the shared expert over T_shared token
 // rows (FP8: L->xq, quantised by the scatter; BF16: x_shared).
+// CTA pairs per cluster of the swap GEMM: 2 (token boxes multicast to two pairs that take
+// adjacent weight blocks) when both groups' weight-block counts are even and enough clusters
+// of 4 fit, else 1.  MOE_SWAP_NP1 / MOE_SWAP_NP2 = 1 or 2 choose per GEMM (A/B experiments).
+static int swap_np(const moe_layer *L, int gemm, int nb_r, int nb_s, int dbg_mode) {
+  // default: pairs for both GEMMs.  Clusters of 4 fit only 33 times on a B200 (132 of 148 SMs):
+  // per unit 7 % faster, per launch 2-5 % slower (interleaved A/B, profiles/r02/swap_np.txt)
+  static const int force1 = getenv("MOE_SWAP_NP1") ? atoi(getenv("MOE_SWAP_NP1")) : 1;
+  static const int force2 = getenv("MOE_SWAP_NP2") ? atoi(getenv("MOE_SWAP_NP2")) : 1;
+  if ((gemm == 1 ? force1 : force2) == 1 || dbg_mode != 0) return 1;
+  if ((nb_r & 1) || (nb_s & 1) || 4 * L->swap_clusters4 < L->num_sms * 3 / 4) return 1;
+  return 2;
+}
+
 static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_shared, int T_shared,
                                    cudaStream_t st) {
   const int H = L->H, F = L->F, Fs = T_shared > 0 ? L->Fs : 0;
@@ -634,7 +652,8 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     SwapParams p1{};
     {
       SwapGroup &g = p1.g[0];
-      g.w_map = L->tmap_w13; g.x_map = L->xmap_xperm; g.x_map128 = L->map_xperm; g.sfw_map = L->smap_w13; g.sfx_map = L->smap_xperm;
+      g.w_map = L->tmap_w13; g.x_map = L->xmap_xperm; g.x_map128 = L->map_xperm; g.x_map64 = L->x64map_xperm;
+      g.sfw_map = L->smap_w13; g.sfx_map = L->smap_xperm;
       g.w_nblk = F / 128; g.kblocks = H / kdiv; g.sfw_per_cta = 0; g.sfx_tile_stride = L->max_tiles;
       g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
     }
@@ -642,8 +661,9 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
       SwapGroup &g = p1.g[1];
       g.w_map = L->tmap_ws13; g.sfw_map = L->smap_ws13; g.sfx_map = L->smap_xq;
       if (f8) {
-        g.x_map = L->xmap_xq; g.x_map128 = L->map_xq;
-      } else if (!make_kmajor_map(&g.x_map, x, false, T, H, 32) || !make_kmajor_map(&g.x_map128, x, false, T, H, 128)) {
+        g.x_map = L->xmap_xq; g.x_map128 = L->map_xq; g.x_map64 = L->x64map_xq;
+      } else if (!make_kmajor_map(&g.x_map, x, false, T, H, 32) || !make_kmajor_map(&g.x_map128, x, false, T, H, 128) ||
+                 !make_kmajor_map(&g.x_map64, x, false, T, H, 64)) {
         return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
       }
       g.w_nblk = Fs / 128; g.kblocks = H / kdiv; g.sfw_per_cta = 0; g.sfx_tile_stride = L->img_tiles_sh;
@@ -651,28 +671,33 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     } else {
       p1.g[1] = p1.g[0];
     }
-    p1.tiles = L->pairs; p1.n_tiles = L->n_pairs; p1.nb_r = F / 128;
-    p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = Fs / 128; p1.sched = L->sched; p1.debug_mode = dbg_mode; p1.trace = L->trace;
-    KL_TRY(launch_umma_swap_gemm(f8, GEMM_SWIGLU, p1, L->num_sms, st));
+    // clusters of 2 CTA pairs (adjacent weight blocks, token boxes multicast to both pairs)
+    // when every operand group has an even number of weight blocks
+    const int np1 = swap_np(L, 1, F / 128, Fs / 128, dbg_mode), np2 = swap_np(L, 2, H / 256, Fs > 0 ? H / 256 : 0, dbg_mode);
+    p1.tiles = L->pairs; p1.n_tiles = L->n_pairs; p1.nb_r = F / 128 / np1;
+    p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = Fs / 128 / np1; p1.sched = L->sched; p1.debug_mode = dbg_mode; p1.trace = L->trace;
+    KL_TRY(launch_umma_swap_gemm(f8, GEMM_SWIGLU, p1, np1 == 2 ? L->swap_clusters4 : L->num_sms, np1, st));
     mark(L, ST_GEMM1, st);
     SwapParams p2{};
     {
       SwapGroup &g = p2.g[0];
-      g.w_map = L->tmap_w2; g.x_map = L->xmap_h; g.x_map128 = L->map_h; g.sfw_map = L->smap_w2; g.sfx_map = L->smap_h;
+      g.w_map = L->tmap_w2; g.x_map = L->xmap_h; g.x_map128 = L->map_h; g.x_map64 = L->x64map_h;
+      g.sfw_map = L->smap_w2; g.sfx_map = L->smap_h;
       g.w_nblk = H / 256; g.kblocks = F / kdiv; g.sfw_per_cta = 1; g.sfx_tile_stride = L->max_tiles;
       g.out = L->yperm; g.ldc = H;
     }
     if (Fs > 0) {
       SwapGroup &g = p2.g[1];
-      g.w_map = L->tmap_ws2; g.x_map = L->xmap_hsh; g.x_map128 = L->map_hsh; g.sfw_map = L->smap_ws2; g.sfx_map = L->smap_hsh;
+      g.w_map = L->tmap_ws2; g.x_map = L->xmap_hsh; g.x_map128 = L->map_hsh; g.x_map64 = L->x64map_hsh;
+      g.sfw_map = L->smap_ws2; g.sfx_map = L->smap_hsh;
       g.w_nblk = H / 256; g.kblocks = Fs / kdiv; g.sfw_per_cta = 1; g.sfx_tile_stride = L->img_tiles_sh;
       g.out = L->ysh; g.ldc = H;
     } else {
       p2.g[1] = p2.g[0];
     }
-    p2.tiles = L->pairs; p2.n_tiles = L->n_pairs; p2.nb_r = H / 256;
-    p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256; p2.sched = L->sched + 1; p2.debug_mode = dbg_mode; p2.trace = L->trace ? L->trace + 2048 : nullptr;
-    KL_TRY(launch_umma_swap_gemm(f8, GEMM_PLAIN, p2, L->num_sms, st));
+    p2.tiles = L->pairs; p2.n_tiles = L->n_pairs; p2.nb_r = H / 256 / np2;
+    p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256 / np2; p2.sched = L->sched + 1; p2.debug_mode = dbg_mode; p2.trace = L->trace ? L->trace + 2048 : nullptr;
+    KL_TRY(launch_umma_swap_gemm(f8, GEMM_PLAIN, p2, np2 == 2 ? L->swap_clusters4 : L->num_sms, np2, st));
     mark(L, ST_GEMM2, st);
   } else {
     // 5. routed experts: GEMM1 + SwiGLU, GEMM2 (CUDA-core path: F32 weights, H % 256 != 0)

@@ -39,6 +39,13 @@ namespace moe {
 using namespace sm100;
 
 constexpr int SW_STAGES = 6, SW_THREADS = 320, SW_UQ = 4;
+// stages are released in groups of SW_CE by one MMA commit: a tcgen05.commit costs the tensor
+// pipe ~100 cycles at N = 256 (profiles/r02/mma_ring.txt: block-scaled pair MMA 153.5 cycles
+// with a commit per k-block, 132.8 per 2, 128.0 per 4) -- but in this kernel SW_CE = 2
+// measured 1-2 % slower than 1 (interleaved A/B, GEMM1 2.50 vs 2.47 ms): the coarser
+// release shortens the producer's run-ahead, and the pipe is not what binds here
+constexpr int SW_CE = 1;
+static_assert(SW_STAGES % SW_CE == 0, "stage groups");
 constexpr int SW_W_BYTES = 128 * 128;          // this CTA's 128 weight rows x 128 B
 constexpr int SW_X_BYTES = 128 * 128;          // up to 128 token rows (half of N <= 256)
 constexpr int SW_SFW_BYTES = 512, SW_SFX_BYTES = 1024;
@@ -77,7 +84,7 @@ __device__ __forceinline__ SwapUnit swap_unit(const SwapParams &p, int u, int n_
   return r;
 }
 
-template <bool FP8, int EPI>
+template <bool FP8, int EPI, int NP>
 __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_constant__ SwapParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -102,8 +109,13 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
   int *unit_q = reinterpret_cast<int *>(tmem_base_smem + 4);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // NP CTA pairs per cluster: pair `pair` = cluster ranks 2*pair, 2*pair + 1 (the MMA
+  // peers); with NP = 2 the pairs work on adjacent weight blocks of the same token tile
+  // and each token box is loaded once and multicast to both pairs
   const uint32_t crank = cluster_rank();
-  const bool leader = crank == 0;
+  const uint32_t prank = crank & 1, pair = crank >> 1;
+  const bool leader = crank == 0;                  // cluster leader: claims units
+  const bool pleader = prank == 0;                 // pair leader: issues the MMAs
   const int n_routed_units = p.tiles ? (*p.n_tiles) * p.nb_r : 0;
 
   if (warp == 0 && lane == 0) {
@@ -111,11 +123,17 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
       prefetch_tmap(&p.g[i].w_map); prefetch_tmap(&p.g[i].x_map); prefetch_tmap(&p.g[i].x_map128);
       if (FP8) { prefetch_tmap(&p.g[i].sfw_map); prefetch_tmap(&p.g[i].sfx_map); }
     }
-    for (int s = 0; s < SW_STAGES; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+    // a stage is released by every pair's MMA commit (its token box is in every pair's smem)
+    for (int s = 0; s < SW_STAGES; ++s) mbar_init(&full[s], 1);
+    for (int s = 0; s < SW_STAGES / SW_CE; ++s) mbar_init(&empty[s], NP);
     mbar_init(tmem_full, 1);
     mbar_init(tmem_empty, 16);                   // 8 epilogue warps x 2 CTAs (the leader's copy is used)
-    // leader's uq_empty: MMA warp + 8 epilogue warps (leader) + producer + 8 epilogue warps (peer)
-    for (int i = 0; i < SW_UQ; ++i) { mbar_init(&uq_full[i], 1); mbar_init(&uq_empty[i], (kExperiments && p.debug_mode >= 4) ? 19 : 18); }
+    // leader's uq_empty: per pair an MMA warp + 8 epilogue warps per CTA; the other CTAs' producers
+    constexpr int kUqArrivals = NP * 17 + 2 * NP - 1;
+    for (int i = 0; i < SW_UQ; ++i) {
+      mbar_init(&uq_full[i], 1);
+      mbar_init(&uq_empty[i], (kExperiments && p.debug_mode >= 4) ? kUqArrivals + 1 : kUqArrivals);
+    }
     for (int i = 0; i < 4; ++i) mbar_init(&am_bar[i], 64);    // 2 gate warps here, per lane (+ peer bytes)
     fence_barrier_init();
   }
@@ -156,9 +174,12 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
           mbar_wait(&uq_empty[qs], qph ^ 1);
           unit_q[qs] = u;
           mbar_arrive(&uq_full[qs]);
-          const uint32_t pbar = map_to_rank(&uq_full[qs], 1);
-          mbar_arrive_expect_tx_remote(pbar, 4);
-          st_async_u32(map_to_rank(&unit_q[qs], 1), (uint32_t)u, pbar);
+#pragma unroll
+          for (uint32_t r = 1; r < 2 * NP; ++r) {
+            const uint32_t pbar = map_to_rank(&uq_full[qs], r);
+            mbar_arrive_expect_tx_remote(pbar, 4);
+            st_async_u32(map_to_rank(&unit_q[qs], r), (uint32_t)u, pbar);
+          }
           if (++qs == SW_UQ) { qs = 0; qph ^= 1; }
         } else {
           mbar_wait(&uq_full[qs], qph);
@@ -169,16 +190,17 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         const SwapUnit ui = swap_unit(p, u, n_routed_units);
         if (!ui.valid) break;
         const SwapGroup &g = p.g[ui.group];
+        const int nb = ui.nb * NP + (int)pair;                 // this pair's weight block
         const int half_n = ((ui.n + 15) & ~15) >> 1;          // token rows per CTA
         const int nbox0 = (half_n + SW_XBOX - 1) / SW_XBOX;
         const int nbox = nbox0 > 2 ? 4 : nbox0;                // > 64 rows: one 128-row box (4 x 32 rows of bytes)
-        const int xrow = ui.row0 + (int)crank * half_n;
-        const int64_t wtile = ((int64_t)ui.expert * g.w_nblk + ui.nb) * g.kblocks;
+        const int xrow = ui.row0 + (int)prank * half_n;
+        const int64_t wtile = ((int64_t)ui.expert * g.w_nblk + nb) * g.kblocks;
         const int G = (g.kblocks + 3) >> 2;
         for (int kb = 0; kb < g.kblocks; ++kb) {
-          mbar_wait(&empty[stage], phase ^ 1);
+          if (stage % SW_CE == 0) mbar_wait(&empty[stage / SW_CE], phase ^ 1);   // the group's release
           if (kExperiments && p.debug_mode == 3) {                 // timing experiment: MMAs on stale smem, no loads
-            if (leader) mbar_arrive(&full[stage]);
+            if (pleader) mbar_arrive(&full[stage]);
             if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
             continue;
           }
@@ -188,7 +210,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             const bool dw = p.debug_mode != 5, dx = p.debug_mode != 4;
             const uint32_t b1 = (dw ? SW_W_BYTES : 0) + (dx ? nbox * (SW_XBOX * 128) : 0);
             mbar_expect_tx(&full[stage], b1);
-            if (dw) tma_load_2d(sW + stage * SW_W_BYTES, &g.w_map, &full[stage], 0, (int)((wtile + kb) * 16 + crank * 8));
+            if (dw) tma_load_2d(sW + stage * SW_W_BYTES, &g.w_map, &full[stage], 0, (int)((wtile + kb) * 16 + prank * 8));
             if (dx) {
               if (nbox > 2)
                 tma_load_2d(sX + stage * SW_X_BYTES, &g.x_map128, &full[stage], kc, xrow);
@@ -200,20 +222,32 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             continue;
           }
           const uint32_t bytes = SW_W_BYTES + nbox * (SW_XBOX * 128) + (sf ? SW_SFW_BYTES + SW_SFX_BYTES : 0);
-          if (leader) mbar_expect_tx(&full[stage], 2 * bytes);
+          if (pleader) mbar_expect_tx(&full[stage], 2 * bytes);
           // the CTA's 16 KB half of the 256-row tile: 8 rows of 2 KB
           tma_load_2d_pair(sW + stage * SW_W_BYTES, &g.w_map, &full[stage], 0,
-                           (int)((wtile + kb) * 16 + crank * 8));
-          if (nbox > 2)                            // one 128-row box (rows past the half are never read)
-            tma_load_2d_pair(sX + stage * SW_X_BYTES, &g.x_map128, &full[stage], kc, xrow);
-          else
-            for (int i = 0; i < nbox; ++i)
-              tma_load_2d_pair(sX + stage * SW_X_BYTES + i * (SW_XBOX * 128), &g.x_map, &full[stage], kc,
-                               xrow + i * SW_XBOX);
+                           (int)((wtile + kb) * 16 + prank * 8));
+          if constexpr (NP == 1) {
+            if (nbox > 2)                          // one 128-row box (rows past the half are never read)
+              tma_load_2d_pair(sX + stage * SW_X_BYTES, &g.x_map128, &full[stage], kc, xrow);
+            else
+              for (int i = 0; i < nbox; ++i)
+                tma_load_2d_pair(sX + stage * SW_X_BYTES + i * (SW_XBOX * 128), &g.x_map, &full[stage], kc,
+                                 xrow + i * SW_XBOX);
+          } else {
+            // token half split between the two pairs, each part multicast to the CTA with
+            // the same pair rank in both pairs: > 64 rows as 2 x 64-row boxes, else 32-row boxes
+            const uint16_t mask = (uint16_t)(0x5u << prank);
+            if (nbox > 2)
+              tma_load_2d_pair_mc(sX + stage * SW_X_BYTES + pair * (64 * 128), &g.x_map64, &full[stage], kc,
+                                  xrow + (int)pair * 64, mask);
+            else if ((int)pair < nbox)
+              tma_load_2d_pair_mc(sX + stage * SW_X_BYTES + pair * (SW_XBOX * 128), &g.x_map, &full[stage], kc,
+                                  xrow + (int)pair * SW_XBOX, mask);
+          }
           if (sf) {
             const int kg = kb >> 2;
-            const int wr = g.sfw_per_cta ? (int)((((int64_t)ui.expert * G + kg) * g.w_nblk + ui.nb) * 2 + crank)
-                                         : (int)(((int64_t)ui.expert * G + kg) * g.w_nblk + ui.nb);
+            const int wr = g.sfw_per_cta ? (int)((((int64_t)ui.expert * G + kg) * g.w_nblk + nb) * 2 + prank)
+                                         : (int)(((int64_t)ui.expert * G + kg) * g.w_nblk + nb);
             tma_load_2d_pair(sSFW + stage * SW_SFW_BYTES, &g.sfw_map, &full[stage], 0, wr);
             tma_load_2d_pair(sSFX + stage * SW_SFX_BYTES, &g.sfx_map, &full[stage], 0,
                              kg * g.sfx_tile_stride + (ui.row0 >> 7));
@@ -235,15 +269,17 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         for (int kb = 0; kb < kblocks; ++kb) {
           mbar_wait(&full[stage], phase);
           if (lane == 0) {
-            mbar_arrive(&empty[stage]);
+            if (stage % SW_CE == SW_CE - 1) mbar_arrive(&empty[stage / SW_CE]);
             if (kb == kblocks - 1) mbar_arrive(tmem_full);
           }
           __syncwarp();
           if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
         }
       }
-    } else if (leader) {
+    } else if (pleader) {
       int stage = 0; uint32_t phase = 0; uint32_t acc_phase = 0;
+      constexpr uint16_t kAllPairs = NP == 1 ? 0x3 : 0xF;
+      const uint16_t my_pair = (uint16_t)(0x3u << (2 * pair));
       int qs = 0; uint32_t qph = 0;
       // MOE_DEBUG_TRACE: cycles waiting for a unit / the accumulator / loaded stages, and issuing
       long long c_unit = 0, c_tmem = 0, c_full = 0, c_issue = 0, n_units = 0, n_flop16 = 0;
@@ -265,7 +301,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
           if (trc) { const long long c = clock64(); c_full += c - c0; c0 = c; }
           tc_fence_after();
           if (kExperiments && lane == 0 && p.debug_mode == 1) {    // timing experiment: loads only (commit releases the stage)
-            mma_commit_pair(&empty[stage]);
+            if (stage % SW_CE == SW_CE - 1) mma_commit_pair(&empty[stage / SW_CE]);
             if (kb == kblocks - 1) mma_commit_pair(tmem_full);
           } else if (lane == 0) {
             const uint32_t a0 = smem_u32(sW + stage * SW_W_BYTES);
@@ -293,8 +329,8 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
               else
                 mma_bf16_pair(tmem, ad, bd, idesc_bf16(256, N), acc);
             }
-            mma_commit_pair(&empty[stage]);
-            if (kb == kblocks - 1) mma_commit_pair(tmem_full);
+            if (stage % SW_CE == SW_CE - 1) mma_commit_pair_mc(&empty[stage / SW_CE], kAllPairs);
+            if (kb == kblocks - 1) mma_commit_pair_mc(tmem_full, my_pair);
           }
           __syncwarp();
           if (trc) { const long long c = clock64(); c_issue += c - c0; c0 = c; }
@@ -303,7 +339,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         acc_phase ^= 1;
       }
       if (trc) {
-        unsigned long long *o = p.trace + 8 * (blockIdx.x >> 1);
+        unsigned long long *o = p.trace + 8 * (blockIdx.x >> 1);   // one record per CTA pair
         o[0] = c_unit; o[1] = c_tmem; o[2] = c_full; o[3] = c_issue; o[4] = n_units; o[5] = n_flop16;
         o[6] = clock64() - c_start;
       }
@@ -337,16 +373,17 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
       tc_fence_before();
       __syncwarp();
       if (lane == 0) {
-        if (leader) mbar_arrive(tmem_empty);
-        else mbar_arrive_remote(map_to_rank(tmem_empty, 0));
+        if (pleader) mbar_arrive(tmem_empty);
+        else mbar_arrive_remote(map_to_rank(tmem_empty, crank & ~1u));
       }
       acc_phase ^= 1;
       const int64_t rbase = (int64_t)ui.row0 + c0;          // token row of this half's column 0
+      const int nb = ui.nb * NP + (int)pair;                 // this pair's weight block
       if (kExperiments && p.debug_mode >= 1) { ++tile_i; continue; }        // timing experiments: no epilogue math
       if constexpr (EPI == GEMM_PLAIN) {
         // transpose 32 tokens x 32 H rows per step through a per-warp smem tile,
         // then 16-byte row stores (token t: 64 contiguous bytes of its y row)
-        const int h0 = ui.nb * 256 + (int)crank * 128 + q * 32;
+        const int h0 = nb * 256 + (int)prank * 128 + q * 32;
         __nv_bfloat16 *tr = reinterpret_cast<__nv_bfloat16 *>(reinterpret_cast<uint8_t *>(xbuf) + ew * 2048);
 #pragma unroll
         for (int c = 0; c < 4; ++c) {
@@ -391,7 +428,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         }
         if (up) { ++tile_i; continue; }
         const int qg = q >> 1;                                // gate warp 0 / 1 of this half
-        const int f = ui.nb * 128 + (int)crank * 64 + qg * 32 + lane;
+        const int f = nb * 128 + (int)prank * 64 + qg * 32 + lane;
         const int f0 = f - lane;
         uint8_t *trw = trbuf + (half * 2 + qg) * 2048;
         if constexpr (!FP8) {
@@ -461,8 +498,8 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
               const int col = 32 * c + lane;
               const int e = ue8m0_exponent(mx[c]);
               sc[col] = exp2i(-e);
-              if (leader && qg == 0 && col < nvalid)
-                g.out_sf[sf_img_off(rbase + col, ui.nb, g.out_sf_tile_stride)] = (uint8_t)(e + 127);
+              if (pleader && qg == 0 && col < nvalid)
+                g.out_sf[sf_img_off(rbase + col, nb, g.out_sf_tile_stride)] = (uint8_t)(e + 127);
             }
           }
           __syncwarp();
@@ -494,19 +531,40 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
   if (warp == 1) tmem_dealloc_pair(tmem, SW_TMEM_COLS);
 }
 
-template <bool FP8, int EPI>
+// clusters of NP CTA pairs that can be co-resident (persistent grid = that many clusters)
+template <bool FP8, int EPI, int NP>
+static int swap_max_clusters() {
+  auto k = umma_swap_gemm<FP8, EPI, NP>;
+  if (set_kernel_attr((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SW_SMEM) != cudaSuccess) return 0;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(2 * NP);
+  cfg.blockDim = dim3(SW_THREADS);
+  cfg.dynamicSmemBytes = SW_SMEM;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2 * NP;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, (const void *)k, &cfg) != cudaSuccess) { cudaGetLastError(); return 0; }
+  return n;
+}
+
+template <bool FP8, int EPI, int NP>
 static cudaError_t launch_swap(const SwapParams &p, int grid, cudaStream_t st) {
-  auto k = umma_swap_gemm<FP8, EPI>;
+  auto k = umma_swap_gemm<FP8, EPI, NP>;
   cudaError_t e = set_kernel_attr((const void *)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SW_SMEM);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg{};
-  cfg.gridDim = dim3(grid & ~1);
+  cfg.gridDim = dim3(grid & ~(2 * NP - 1));
   cfg.blockDim = dim3(SW_THREADS);
   cfg.dynamicSmemBytes = SW_SMEM;
   cfg.stream = st;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = 2;
+  attr[0].val.clusterDim.x = 2 * NP;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
@@ -514,10 +572,21 @@ static cudaError_t launch_swap(const SwapParams &p, int grid, cudaStream_t st) {
   return cudaLaunchKernelEx(&cfg, k, p);
 }
 
-cudaError_t launch_umma_swap_gemm(bool fp8, int epi, const SwapParams &p, int grid, cudaStream_t st) {
+cudaError_t launch_umma_swap_gemm(bool fp8, int epi, const SwapParams &p, int grid, int np, cudaStream_t st) {
+  if (np == 2) {
+    grid = 4 * grid;                               // grid = clusters of 2 pairs (host: umma_swap_max_clusters4)
+    if (fp8) return epi == GEMM_SWIGLU ? launch_swap<true, GEMM_SWIGLU, 2>(p, grid, st) : launch_swap<true, GEMM_PLAIN, 2>(p, grid, st);
+    return epi == GEMM_SWIGLU ? launch_swap<false, GEMM_SWIGLU, 2>(p, grid, st) : launch_swap<false, GEMM_PLAIN, 2>(p, grid, st);
+  }
   if (grid < 2) grid = 2;
-  if (fp8) return epi == GEMM_SWIGLU ? launch_swap<true, GEMM_SWIGLU>(p, grid, st) : launch_swap<true, GEMM_PLAIN>(p, grid, st);
-  return epi == GEMM_SWIGLU ? launch_swap<false, GEMM_SWIGLU>(p, grid, st) : launch_swap<false, GEMM_PLAIN>(p, grid, st);
+  if (fp8) return epi == GEMM_SWIGLU ? launch_swap<true, GEMM_SWIGLU, 1>(p, grid, st) : launch_swap<true, GEMM_PLAIN, 1>(p, grid, st);
+  return epi == GEMM_SWIGLU ? launch_swap<false, GEMM_SWIGLU, 1>(p, grid, st) : launch_swap<false, GEMM_PLAIN, 1>(p, grid, st);
+}
+
+int umma_swap_max_clusters4(bool fp8) {
+  const int a = fp8 ? swap_max_clusters<true, GEMM_SWIGLU, 2>() : swap_max_clusters<false, GEMM_SWIGLU, 2>();
+  const int b = fp8 ? swap_max_clusters<true, GEMM_PLAIN, 2>() : swap_max_clusters<false, GEMM_PLAIN, 2>();
+  return a < b ? a : b;
 }
 
 size_t umma_swap_smem_bytes() { return SW_SMEM; }
