@@ -279,6 +279,7 @@ struct SwapGroup {              // one operand set: 0 = routed experts, 1 = shar
   CUtensorMap x_map;            // token rows, K-major SW128, box 32 rows (ragged tails)
   CUtensorMap x_map128;         // the same, box 128 rows (full halves)
   CUtensorMap x_map64;          // the same, box 64 rows (a half split between 2 multicasting pairs)
+  CUtensorMap x_map16;          // the same, box 16 rows
   CUtensorMap sfw_map;          // FP8: weight scale images as 512-byte rows, box 1
   CUtensorMap sfx_map;          // FP8: token scale images as 512-byte rows, box 2
   int w_nblk;                   // 256-row weight blocks per expert

@@ -652,7 +652,7 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     SwapParams p1{};
     {
       SwapGroup &g = p1.g[0];
-      g.w_map = L->tmap_w13; g.x_map = L->xmap_xperm; g.x_map128 = L->map_xperm; g.x_map64 = L->x64map_xperm;
+      g.w_map = L->tmap_w13; g.x_map = L->xmap_xperm; g.x_map128 = L->map_xperm; g.x_map64 = L->x64map_xperm; g.x_map16 = L->dmap_xperm;
       g.sfw_map = L->smap_w13; g.sfx_map = L->smap_xperm;
       g.w_nblk = F / 128; g.kblocks = H / kdiv; g.sfw_per_cta = 0; g.sfx_tile_stride = L->max_tiles;
       g.out = L->hbuf; g.ldc = F; g.out_sf = L->h_img; g.out_sf_tile_stride = L->max_tiles;
@@ -661,9 +661,9 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
       SwapGroup &g = p1.g[1];
       g.w_map = L->tmap_ws13; g.sfw_map = L->smap_ws13; g.sfx_map = L->smap_xq;
       if (f8) {
-        g.x_map = L->xmap_xq; g.x_map128 = L->map_xq; g.x_map64 = L->x64map_xq;
+        g.x_map = L->xmap_xq; g.x_map128 = L->map_xq; g.x_map64 = L->x64map_xq; g.x_map16 = L->dmap_xq;
       } else if (!make_kmajor_map(&g.x_map, x, false, T, H, 32) || !make_kmajor_map(&g.x_map128, x, false, T, H, 128) ||
-                 !make_kmajor_map(&g.x_map64, x, false, T, H, 64)) {
+                 !make_kmajor_map(&g.x_map64, x, false, T, H, 64) || !make_kmajor_map(&g.x_map16, x, false, T, H, 16)) {
         return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for x");
       }
       g.w_nblk = Fs / 128; g.kblocks = H / kdiv; g.sfw_per_cta = 0; g.sfx_tile_stride = L->img_tiles_sh;
@@ -681,14 +681,14 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     SwapParams p2{};
     {
       SwapGroup &g = p2.g[0];
-      g.w_map = L->tmap_w2; g.x_map = L->xmap_h; g.x_map128 = L->map_h; g.x_map64 = L->x64map_h;
+      g.w_map = L->tmap_w2; g.x_map = L->xmap_h; g.x_map128 = L->map_h; g.x_map64 = L->x64map_h; g.x_map16 = L->dmap_h;
       g.sfw_map = L->smap_w2; g.sfx_map = L->smap_h;
       g.w_nblk = H / 256; g.kblocks = F / kdiv; g.sfw_per_cta = 1; g.sfx_tile_stride = L->max_tiles;
       g.out = L->yperm; g.ldc = H;
     }
     if (Fs > 0) {
       SwapGroup &g = p2.g[1];
-      g.w_map = L->tmap_ws2; g.x_map = L->xmap_hsh; g.x_map128 = L->map_hsh; g.x_map64 = L->x64map_hsh;
+      g.w_map = L->tmap_ws2; g.x_map = L->xmap_hsh; g.x_map128 = L->map_hsh; g.x_map64 = L->x64map_hsh; g.x_map16 = L->dmap_hsh;
       g.sfw_map = L->smap_ws2; g.sfx_map = L->smap_hsh;
       g.w_nblk = H / 256; g.kblocks = Fs / kdiv; g.sfw_per_cta = 1; g.sfx_tile_stride = L->img_tiles_sh;
       g.out = L->ysh; g.ldc = H;

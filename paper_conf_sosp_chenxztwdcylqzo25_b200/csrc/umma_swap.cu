@@ -195,6 +195,13 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         const int nbox0 = (half_n + SW_XBOX - 1) / SW_XBOX;
         const int nbox = nbox0 > 2 ? 4 : nbox0;                // > 64 rows: one 128-row box (4 x 32 rows of bytes)
         const int xrow = ui.row0 + (int)prank * half_n;
+        // NP = 1: the half in at most two boxes of 128 / 64 / 32 / 16 rows, at most 32 rows
+        // over-read (one 128-row box above 96 rows, 64 + 32, 64, 32 + 16, 32, 16)
+        const int xb0 = half_n > 96 ? 128 : half_n > 48 ? 64 : half_n > 16 ? 32 : 16;
+        const int xb1 = (half_n > 64 && half_n <= 96) ? 32 : (half_n > 32 && half_n <= 48) ? 16 : 0;
+        const CUtensorMap *xm0 = xb0 == 128 ? &g.x_map128 : xb0 == 64 ? &g.x_map64 : xb0 == 32 ? &g.x_map : &g.x_map16;
+        const CUtensorMap *xm1 = xb1 == 32 ? &g.x_map : &g.x_map16;
+        const uint32_t xbytes = NP == 1 ? (uint32_t)(xb0 + xb1) * 128 : (uint32_t)nbox * (SW_XBOX * 128);
         const int64_t wtile = ((int64_t)ui.expert * g.w_nblk + nb) * g.kblocks;
         const int G = (g.kblocks + 3) >> 2;
         for (int kb = 0; kb < g.kblocks; ++kb) {
@@ -221,18 +228,14 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
             continue;
           }
-          const uint32_t bytes = SW_W_BYTES + nbox * (SW_XBOX * 128) + (sf ? SW_SFW_BYTES + SW_SFX_BYTES : 0);
+          const uint32_t bytes = SW_W_BYTES + xbytes + (sf ? SW_SFW_BYTES + SW_SFX_BYTES : 0);
           if (pleader) mbar_expect_tx(&full[stage], 2 * bytes);
           // the CTA's 16 KB half of the 256-row tile: 8 rows of 2 KB
           tma_load_2d_pair(sW + stage * SW_W_BYTES, &g.w_map, &full[stage], 0,
                            (int)((wtile + kb) * 16 + prank * 8));
-          if constexpr (NP == 1) {
-            if (nbox > 2)                          // one 128-row box (rows past the half are never read)
-              tma_load_2d_pair(sX + stage * SW_X_BYTES, &g.x_map128, &full[stage], kc, xrow);
-            else
-              for (int i = 0; i < nbox; ++i)
-                tma_load_2d_pair(sX + stage * SW_X_BYTES + i * (SW_XBOX * 128), &g.x_map, &full[stage], kc,
-                                 xrow + i * SW_XBOX);
+          if constexpr (NP == 1) {                 // (rows past the half are never read)
+            tma_load_2d_pair(sX + stage * SW_X_BYTES, xm0, &full[stage], kc, xrow);
+            if (xb1) tma_load_2d_pair(sX + stage * SW_X_BYTES + xb0 * 128, xm1, &full[stage], kc, xrow + xb0);
           } else {
             // token half split between the two pairs, each part multicast to the CTA with
             // the same pair rank in both pairs: > 64 rows as 2 x 64-row boxes, else 32-row boxes
