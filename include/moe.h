@@ -86,6 +86,9 @@ typedef struct {
                                 tp_size > 1 (the group's communicator)              */
   int32_t tp_rank, tp_size;  /* tensor parallelism within every expert (decode):
                                 tp_size 1 => off; see "Tensor parallelism" below    */
+  int32_t ep_fixed_capacity; /* ep_size > 1: 1 => fixed-capacity exchange, no host
+                                synchronisation (CUDA-Graph capturable); 0 => exact
+                                row counts learned on the host (fewer bytes moved) */
 } moe_layer_config;
 
 /* Tensor parallelism within every expert (the B200
@@ -150,8 +153,13 @@ moe_status moe_get_unique_id(void *out128);
  * to NULL on failure.  With ep_size > 1 and a unique id this initialises the
  * NCCL communicator and is collective over the EP group; with ep_size > 1 and
  * nccl_unique_id == NULL the layer is one rank of an in-process group
- * (moe_ep_group_forward).  Expert-parallel forwards synchronise the stream to
- * learn the received row counts (not CUDA-Graph capturable).                 */
+ * (moe_ep_group_forward).  Expert-parallel forwards with ep_fixed_capacity = 0
+ * synchronise the stream to learn the received row counts and move exactly
+ * those rows (not CUDA-Graph capturable).  With ep_fixed_capacity = 1 every
+ * (source, destination) transfer moves the whole max_tokens-row block (rows
+ * past the source's count carry expert ids -1 and are skipped by the expert
+ * side), both ways: no host synchronisation, capturable, at the cost of
+ * P * max_tokens rows per direction per rank instead of the routed rows.     */
 moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights *w,
                             moe_layer **out);
 

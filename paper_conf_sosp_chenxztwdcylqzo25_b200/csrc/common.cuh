@@ -290,6 +290,7 @@ struct moe_layer {
     __nv_bfloat16 *partial_def = nullptr;
     __nv_bfloat16 *back = nullptr;     // [P][Tm][H] partial sums returned to this rank
     __nv_bfloat16 *back_def = nullptr;
+    bool fixed = false;                // ep_fixed_capacity: whole [P][Tm] blocks, no host sync
     int R = 0;                         // rows received this step
     int roff[33] = {};                 // receive offsets per source
   } ep;

@@ -88,6 +88,7 @@ moe_status ep_create(moe_layer *L, const moe_layer_config *cfg) {
   const size_t Tm = std::max(1, cfg->max_tokens);
   L->ep.P = P;
   L->ep.rank = cfg->ep_rank;
+  L->ep.fixed = cfg->ep_fixed_capacity != 0;
   const size_t rows = (size_t)P * Tm;
   // dispatched token rows: bf16 (2H bytes) or, FP8 layers, [H e4m3 codes | H/128 UE8M0 bytes]
   L->ep.row_bytes = L->fp8 ? ((H + H / 128 + 15) / 16) * 16 : 2 * H;
@@ -254,6 +255,8 @@ moe_status validate(const moe_layer_config *c, const moe_layer_weights *w) {
   if (c->ep_size < 1 || c->ep_size > 32 || c->n_experts % c->ep_size)
     return fail(MOE_ERR_INVALID_ARG, "ep_size %d must be in [1, 32] and divide n_experts", c->ep_size);
   if (c->ep_rank < 0 || c->ep_rank >= c->ep_size) return fail(MOE_ERR_INVALID_ARG, "ep_rank %d", c->ep_rank);
+  if (c->ep_fixed_capacity != 0 && c->ep_fixed_capacity != 1)
+    return fail(MOE_ERR_INVALID_ARG, "ep_fixed_capacity %d (0 or 1)", c->ep_fixed_capacity);
   if (c->tp_size < 0 || c->tp_size > 32 || c->tp_rank < 0 || (c->tp_size > 1 && c->tp_rank >= c->tp_size))
     return fail(MOE_ERR_INVALID_ARG, "tp rank %d / size %d", c->tp_rank, c->tp_size);
   if (c->tp_size > 1) {
@@ -784,6 +787,9 @@ static moe_status ep_phase_a(moe_layer *L, const void *x, int T, cudaStream_t st
   if (s != MOE_OK) return s;
   const int P = L->ep.P, Tm = std::max(1, L->max_tokens);
   KL_TRY(launch_ep_plan(L->topk_idx, T, L->k, L->E, P, L->ep.sendpos, L->ep.cnt_dev, st));
+  // fixed-capacity exchange: every [P][Tm] send block travels whole, so the rows past a
+  // destination's count must carry no expert ids (-1: the expert side skips them)
+  if (L->ep.fixed) CUDA_TRY(cudaMemsetAsync(L->ep.send_idx, 0xff, (size_t)P * Tm * L->k * 4, st));
   if (L->fp8) {
     // quantise the own tokens once (1x128 UE8M0 + e4m3, reading R10): the dispatched rows and
     // the shared expert's input (xq) -- half the bytes of a bf16 row on the wire
@@ -797,6 +803,13 @@ static moe_status ep_phase_a(moe_layer *L, const void *x, int T, cudaStream_t st
                           L->ep.send_idx, L->ep.send_w, st));
   }
   return MOE_OK;
+}
+
+// fixed-capacity exchange: source p's rows land in block [p Tm, (p+1) Tm) whatever its count
+static void ep_fixed_layout(moe_layer *L) {
+  const int P = L->ep.P, Tm = std::max(1, L->max_tokens);
+  for (int p = 0; p <= P; ++p) L->ep.roff[p] = p * Tm;
+  L->ep.R = P * Tm;
 }
 
 // send counts (cnt_dev[0:P]) and received counts (cnt_dev[P:2P]) -> host
@@ -881,11 +894,19 @@ static moe_status ep_forward_nccl(moe_layer *L, const void *x, const void *resid
   const int64_t Tm = std::max(1, L->max_tokens);
   moe_status s = ep_phase_a(L, x, T, st);
   if (s != MOE_OK) return s;
-  NCCL_TRY(ep_nccl_counts(L->ep.comm, L->ep.cnt_dev, L->ep.cnt_dev + P, P, st));
-  if ((s = ep_counts_to_host(L, st)) != MOE_OK) return s;
+  int32_t full_cnt[32];
+  const int32_t *scnt = L->ep.cnt_host, *rcnt = L->ep.cnt_host + P;
+  if (L->ep.fixed) {
+    // no host synchronisation (CUDA-Graph capturable): whole Tm-row blocks both ways
+    ep_fixed_layout(L);
+    for (int p = 0; p < P; ++p) full_cnt[p] = (int32_t)Tm;
+    scnt = rcnt = full_cnt;
+  } else {
+    NCCL_TRY(ep_nccl_counts(L->ep.comm, L->ep.cnt_dev, L->ep.cnt_dev + P, P, st));
+    if ((s = ep_counts_to_host(L, st)) != MOE_OK) return s;
+  }
   int64_t soff[32], roff[32];
   for (int p = 0; p < P; ++p) { soff[p] = p * Tm; roff[p] = L->ep.roff[p]; }
-  const int32_t *scnt = L->ep.cnt_host, *rcnt = L->ep.cnt_host + P;
   {
     const void *snd[3] = {L->ep.send_x, L->ep.send_idx, L->ep.send_w};
     void *rcv[3] = {L->ep.recv_x, L->topk_idx, L->topk_w};
@@ -1199,14 +1220,23 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
   for (int r = 0; r < P; ++r)
     if ((s = ep_phase_a(layers[r], x[r], T[r], st)) != MOE_OK) return s;
   // counts: rank d receives cnt_dev[d] of every source
-  for (int d = 0; d < P; ++d)
-    for (int src = 0; src < P; ++src)
-      CUDA_TRY(cudaMemcpyAsync(layers[d]->ep.cnt_dev + P + src, layers[src]->ep.cnt_dev + d, 4, cudaMemcpyDefault, st));
-  for (int r = 0; r < P; ++r)
-    if ((s = ep_counts_to_host(layers[r], st)) != MOE_OK) return s;
+  const bool fixed = layers[0]->ep.fixed;
+  for (int r = 1; r < P; ++r)
+    if (layers[r]->ep.fixed != fixed) return fail(MOE_ERR_INVALID_ARG, "ep_fixed_capacity differs across the group");
+  // rows sent from src to d: the exact count (host-synchronised) or the whole Tm block (fixed)
+  auto nrows = [&](int src, int d) -> int64_t { return fixed ? Tm : layers[src]->ep.cnt_host[d]; };
+  if (fixed) {
+    for (int r = 0; r < P; ++r) ep_fixed_layout(layers[r]);
+  } else {
+    for (int d = 0; d < P; ++d)
+      for (int src = 0; src < P; ++src)
+        CUDA_TRY(cudaMemcpyAsync(layers[d]->ep.cnt_dev + P + src, layers[src]->ep.cnt_dev + d, 4, cudaMemcpyDefault, st));
+    for (int r = 0; r < P; ++r)
+      if ((s = ep_counts_to_host(layers[r], st)) != MOE_OK) return s;
+  }
   for (int d = 0; d < P; ++d)
     for (int src = 0; src < P; ++src) {
-      const int64_t n = layers[src]->ep.cnt_host[d];
+      const int64_t n = nrows(src, d);
       if (!n) continue;
       const int64_t ro = layers[d]->ep.roff[src], so = (int64_t)d * Tm;
       const int64_t rbytes = layers[d]->ep.row_bytes;
@@ -1223,7 +1253,7 @@ moe_status moe_ep_group_forward(moe_layer *const *layers, int32_t P, const void 
   }
   for (int src = 0; src < P; ++src)       // partial rows back to their origin
     for (int d = 0; d < P; ++d) {
-      const int64_t n = layers[src]->ep.cnt_host[d];
+      const int64_t n = nrows(src, d);
       if (!n) continue;
       const int64_t ro = layers[d]->ep.roff[src], so = (int64_t)d * Tm;
       CUDA_TRY(cudaMemcpyAsync(layers[src]->ep.back + so * H, layers[d]->ep.partial + ro * H, n * H * 2,

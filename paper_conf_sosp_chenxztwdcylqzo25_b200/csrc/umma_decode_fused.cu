@@ -49,6 +49,7 @@ namespace moe {
 using namespace sm100;
 
 constexpr int FD_N = 16, FD_STAGES = 5, FD_THREADS = 192, FD_UQ = 4, FD_ACCB = 4, FD_ACCA_SLOTS = 4;
+static_assert(FD_STAGES > FD_ACCA_SLOTS, "phase-A epilogue waits on the stage barriers (no parity aliasing)");
 constexpr int FD_A_BYTES = 256 * 128;          // one 256-row weight tile k-block (two 128-row MMA tiles)
 constexpr int FD_B_BYTES = FD_N * 128;         // 16 token rows x 128 B
 constexpr int FD_H_BYTES = 2 * FD_B_BYTES;     // h_c: FP8 one k-block, BF16 two
@@ -346,7 +347,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
           mbar_wait(&full[stage], phase);
           if (lane == 0) {
             mbar_arrive(&empty[stage]);
-            if (FP8 ? true : kb == kb1 - 1) mbar_arrive(&accA_full[FP8 ? as : 0]);
+            if (!FP8 && kb == kb1 - 1) mbar_arrive(&accA_full[0]);
           }
           __syncwarp();
           if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
@@ -374,9 +375,11 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
                 mma_bf16(tmem + FD_ACCA_COL + t * 16, ad, bd, idesc_bf16(128, FD_N), (kb != kb0) || (k != 0));
             }
           }
+          // FP8: one commit per k-block serves the producer (stage free) and the epilogue
+          // (slot `as` complete) -- a tcgen05.commit costs the tensor pipe ~100 cycles
+          // (profiles/r02/mma_ring.txt), so the second commit per k-block was a bubble
           mma_commit(&empty[stage]);
-          if (FP8) mma_commit(&accA_full[as]);
-          else if (kb == kb1 - 1) mma_commit(&accA_full[0]);
+          if (!FP8 && kb == kb1 - 1) mma_commit(&accA_full[0]);
         }
         __syncwarp();
         if (++stage == FD_STAGES) { stage = 0; phase ^= 1; }
@@ -435,6 +438,7 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
     uint32_t qs = 0, qph = 0, aph = 0;
     int ab = 0; uint32_t abph = 0;
     int as = 0; uint32_t asph = 0;
+    int es = 0; uint32_t eph = 0;                // FP8: the smem stage ring, followed (phase A waits)
     int ui_par = 0;
     uint32_t hph_e = 0, pph = 0;                 // cluster peers: h_ready phase; leader: part_bar phase
     bool waited = false;
@@ -515,7 +519,13 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
 #pragma unroll
         for (int t = 0; t < FD_N; ++t) r0[t] = r1[t] = 0.f;
         for (int kb = kb0; kb < kb1; ++kb) {
-          mbar_wait(&accA_full[as], asph);
+          // the k-block's MMAs are complete when its smem stage is released (the MMA warp's
+          // single commit per k-block); this warp group follows the stage ring: phase A takes
+          // one stage per k-block, phase B (nt1 - nt0) * KBC (advanced below).  No parity
+          // aliasing: the stage is reused only FD_STAGES > FD_ACCA_SLOTS k-blocks later, which
+          // needs slot `as` released by this warp group first
+          mbar_wait(&empty[es], eph);
+          if (++es == FD_STAGES) { es = 0; eph ^= 1; }
           tc_fence_after();
           if (kExperiments && (p.debug & 1)) {   // timing experiment: no per-k-block fold
             __syncwarp();
@@ -747,6 +757,8 @@ __global__ void __launch_bounds__(FD_THREADS, 1) umma_decode_fused_kernel(const 
         }
       }
       ui_par ^= 1;
+      for (int i = (nt1 - nt0) * KBC; i > 0; --i)   // the stages phase B consumed
+        if (++es == FD_STAGES) { es = 0; eph ^= 1; }
       if (tr) tr[5] = gtimer();
     }
     if (!waited) pdl_wait();                     // (a CTA that only saw group-2 units: nothing left to read)

@@ -36,7 +36,7 @@ class MoEConfig(ctypes.Structure):
                 ("shared_gated", ctypes.c_int32), ("wtype", ctypes.c_int32), ("max_tokens", ctypes.c_int32),
                 ("gemv_max_tokens", ctypes.c_int32), ("device", ctypes.c_int32), ("ep_rank", ctypes.c_int32),
                 ("ep_size", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p), ("tp_rank", ctypes.c_int32),
-                ("tp_size", ctypes.c_int32)]
+                ("tp_size", ctypes.c_int32), ("ep_fixed_capacity", ctypes.c_int32)]
 
 
 class MoEWeights(ctypes.Structure):
@@ -128,7 +128,7 @@ class MoELayer:
 
     def __init__(self, preset, weights, max_tokens: int, device: int = 0, gemv_max_tokens: int = 0,
                  ep_rank: int = 0, ep_size: int = 1, unique_id: Optional[bytes] = None, tp_rank: int = 0,
-                 tp_size: int = 1):
+                 tp_size: int = 1, ep_fixed: bool = False):
         lib = load_library()
         self.p = preset
         self.max_tokens = max_tokens
@@ -142,7 +142,7 @@ class MoELayer:
                         shared_gated=int(preset.shared_gated), wtype=preset.wtype, max_tokens=max_tokens,
                         gemv_max_tokens=gemv_max_tokens, device=device, ep_rank=ep_rank, ep_size=ep_size,
                         nccl_unique_id=ctypes.cast(self._uid, ctypes.c_void_p) if self._uid else None,
-                        tp_rank=tp_rank, tp_size=tp_size)
+                        tp_rank=tp_rank, tp_size=tp_size, ep_fixed_capacity=int(ep_fixed))
         self.tp_size = tp_size
         w = MoEWeights(**{n: _ptr(getattr(weights, n)) for n, _ in MoEWeights._fields_})
         h = ctypes.c_void_p()
@@ -311,7 +311,7 @@ class MoEGroup:
     """In-process expert-parallel group on one GPU (moe_ep_group_forward): P ranks,
     one MoELayer each, owning E/P experts (the NCCL transport runs one process per GPU)."""
 
-    def __init__(self, preset, weights, ep_size: int, max_tokens: int, device: int = 0):
+    def __init__(self, preset, weights, ep_size: int, max_tokens: int, device: int = 0, ep_fixed: bool = False):
         devices = [device] * ep_size
         self.P = ep_size
         self.layers = []
@@ -320,14 +320,15 @@ class MoEGroup:
             if devices[r] != weights.w13.device.index:
                 wr = wr.to(f"cuda:{devices[r]}")
             self.layers.append(MoELayer(preset, wr, max_tokens=max_tokens, device=devices[r], ep_rank=r,
-                                        ep_size=ep_size))
+                                        ep_size=ep_size, ep_fixed=ep_fixed))
         self._lib = load_library()
 
-    def forward(self, xs, residuals=None, n_deferred=0, deferred_in=None, want_deferred_out=False, stream=None):
+    def forward(self, xs, residuals=None, n_deferred=0, deferred_in=None, want_deferred_out=False, stream=None,
+                ys=None):
         P = self.P
         vp = ctypes.c_void_p
         arr = lambda ts: (vp * P)(*[None if t is None else _ptr(t) for t in ts]) if ts is not None else None
-        ys = [torch.empty_like(x) for x in xs]
+        ys = ys if ys is not None else [torch.empty_like(x) for x in xs]
         douts = [torch.empty_like(x) for x in xs] if want_deferred_out else None
         T = (ctypes.c_int32 * P)(*[x.shape[0] for x in xs])
         st = (stream or torch.cuda.current_stream(xs[0].device)).cuda_stream

@@ -78,3 +78,74 @@ def test_ep_nccl_single_rank(lib):
     torch.cuda.synchronize()
     _oracle_check(p, w_cpu, x, y)
     layer.close()
+
+
+@pytest.mark.parametrize("name,P,Ts", [("v3_s", 2, [40, 33]), ("v3_s", 4, [25, 0, 61, 7]),
+                                       ("qwen2_s", 2, [50, 19]), ("v3_s", 8, [5, 9, 1, 0, 3, 17, 2, 8])])
+def test_ep_group_fixed_capacity(lib, name, P, Ts):
+    """ep_fixed_capacity: whole max_tokens-row blocks both ways, no host synchronisation."""
+    p = SMALL[name]
+    w_cpu = make_weights(p, "cpu")
+    group = lib.MoEGroup(p, w_cpu.to("cuda"), ep_size=P, max_tokens=max(Ts) or 1, ep_fixed=True)
+    xs = [make_tokens(p, t, "cpu", offset=r)[0] for r, t in enumerate(Ts)]
+    ys = group.forward([x.cuda() for x in xs])
+    torch.cuda.synchronize()
+    for x, y in zip(xs, ys):
+        _oracle_check(p, w_cpu, x, y)
+    group.close()
+
+
+def test_ep_group_fixed_capacity_graph(lib):
+    """The fixed-capacity EP forward captured in a CUDA graph and replayed on new tokens."""
+    p = SMALL["v3_s"]
+    P, Ts = 4, [24, 31, 0, 17]
+    w_cpu = make_weights(p, "cpu")
+    group = lib.MoEGroup(p, w_cpu.to("cuda"), ep_size=P, max_tokens=32, ep_fixed=True)
+    xin = [torch.zeros(t, p.hidden, dtype=torch.bfloat16, device="cuda") for t in Ts]
+    yout = [torch.empty_like(x) for x in xin]
+    side = torch.cuda.Stream()
+    side.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(side):
+        group.forward(xin, ys=yout, stream=side)          # warm-up outside the capture
+    torch.cuda.current_stream().wait_stream(side)
+    torch.cuda.synchronize()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph):
+        group.forward(xin, ys=yout, stream=torch.cuda.current_stream())
+    for rep in range(2):
+        xs = [make_tokens(p, t, "cpu", offset=10 * rep + r)[0] for r, t in enumerate(Ts)]
+        for dst, src in zip(xin, xs):
+            dst.copy_(src)
+        graph.replay()
+        torch.cuda.synchronize()
+        for x, y in zip(xs, yout):
+            _oracle_check(p, w_cpu, x, y)
+    del graph
+    group.close()
+
+
+def test_ep_nccl_single_rank_fixed_graph(lib):
+    """The NCCL transport in fixed-capacity mode, captured in a CUDA graph (1-rank communicator)."""
+    p = SMALL["v3_s"]
+    w_cpu = make_weights(p, "cpu")
+    uid = lib.get_unique_id()
+    layer = lib.MoELayer(p, w_cpu.to("cuda"), max_tokens=64, ep_rank=0, ep_size=1, unique_id=uid, ep_fixed=True)
+    xin = torch.zeros(57, p.hidden, dtype=torch.bfloat16, device="cuda")
+    yout = torch.empty_like(xin)
+    side = torch.cuda.Stream()
+    side.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(side):
+        layer.forward(xin, y=yout)
+    torch.cuda.current_stream().wait_stream(side)
+    torch.cuda.synchronize()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph):
+        layer.forward(xin, y=yout)
+    for rep in range(2):
+        x, _ = make_tokens(p, 57, "cpu", offset=rep)
+        xin.copy_(x)
+        graph.replay()
+        torch.cuda.synchronize()
+        _oracle_check(p, w_cpu, x, yout)
+    del graph
+    layer.close()
