@@ -281,7 +281,8 @@ def run_ours(args):
         dist.broadcast_object_list(uid, src=0)
         w = moe.slice_experts(w, rank, ws)
         torch.cuda.empty_cache()
-        layer = moe.MoELayer(p, w, max_tokens=T, device=local, ep_rank=rank, ep_size=ws, unique_id=uid[0])
+        layer = moe.MoELayer(p, w, max_tokens=T, device=local, ep_rank=rank, ep_size=ws, unique_id=uid[0],
+                             ep_fixed=args.ep_fixed)
     else:
         layer = moe.MoELayer(p, w, max_tokens=T, device=local)
     flush = (torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda"),
@@ -558,7 +559,9 @@ def run_ours(args):
                 "config": {"workload": f"{p.name}_moe_layer_prefill", "tokens_per_gpu": T, "hidden": p.hidden,
                            "ffn": p.ffn, "experts": p.n_experts, "top_k": p.top_k, "shared_ffn": p.shared_ffn,
                            "weights": "fp8_e4m3_block128_ue8m0" if fp8 else "bf16", "parallelism":
-                           (f"ep{ws} (NCCL all-to-all-v dispatch/combine)" if ep else f"replica x{ws}")
+                           (f"ep{ws} (NCCL " + ("fixed-capacity all-to-all, no host sync" if args.ep_fixed
+                                                else "all-to-all-v, counts via the host") + " dispatch/combine)"
+                            if ep else f"replica x{ws}")
                            if ws > 1 else "single", "l2": "flushed before every step (256 MiB write, then 256 MiB read so the dirty lines are written back "
                            "before the events, "
                            "outside the timed events); inputs resident in HBM",
@@ -591,6 +594,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-tokens", type=int, default=16, help="tokens of the cpu_baseline oracle call")
     ap.add_argument("--replicas", action="store_true", help="N>1: independent replicas instead of expert parallel")
+    ap.add_argument("--ep-fixed", action="store_true",
+                    help="N>1: fixed-capacity EP exchange (no host sync, capturable; more bytes on the wire)")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "ours":
         args.warmup = 3
