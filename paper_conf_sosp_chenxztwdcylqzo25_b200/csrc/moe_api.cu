@@ -1099,19 +1099,28 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     fp.trace = L->trace;
     static const int dbg_fd = experiment_knob("MOE_DEBUG_FD");   // timing experiments (MOE_EXPERIMENTS builds)
     fp.debug = dbg_fd;
-    static const int cluster_override = experiment_knob("MOE_FD_CLUSTER");   // A/B of the cluster size
     const int units = prev_units + Fs / 128 + (int)std::min<int64_t>(E, pairs) * (F / 128);
-    // few units (expert TP, small layers): split each over a cluster so more SMs stream it --
-    // the largest cluster size whose clusters all fit in one wave (and that leaves every CTA
-    // at least one W13 k-block and one W2 tile)
-    int csize = 1;
+    // Cluster split: each unit over C = 1/2/4/8 CTAs (C <= the W13 k-blocks and W2 tiles), the
+    // clusters taking units from the device queue.  Cost model per layer: rounds x (unit time / C +
+    // per-unit split overhead), rounds = ceil(units / resident clusters), unit time = its weight
+    // bytes at the per-SM streaming rate -- one wave of whole units when units fill the GPU (V3,
+    // T = 1), wider splits when units are few (expert TP, small layers) or leave a ragged last
+    // round (Qwen2: 320 units on 148 SMs).  MOE_FD_CSIZE forces C (A/B experiments).
+    static const int force_c = getenv("MOE_FD_CSIZE") ? atoi(getenv("MOE_FD_CSIZE")) : 0;
     const int KA = H / (f8 ? 128 : 64), NT = H / 256;
-    for (int c = 8; c >= 2; c /= 2)
-      if (c <= KA && c <= NT && units <= L->fd_max_clusters[c] && units * c <= L->num_sms) { csize = c; break; }
-    if (cluster_override > 0 && units <= L->fd_max_clusters[2] && cluster_override <= std::min(KA, NT))
-      csize = cluster_override;                  // (cluster ids stay within the scratch slots)
+    const double wb = L->fp4 ? 0.5 : (f8 ? 1.0 : 2.0);
+    const double unit_us = (256.0 * H + 128.0 * H) * wb / 45e3;      // ~45 GB/s per SM
+    constexpr double kSplitUs = 1.5;                                   // leader reduce + h exchange
+    int csize = 1, ncl = L->num_sms;
+    double best = 1e30;
+    for (int c = 1; c <= 8; c *= 2) {
+      if (c > 1 && (c > KA || c > NT || L->fd_max_clusters[c] < 1)) continue;
+      const int nc = c == 1 ? L->num_sms : L->fd_max_clusters[c];
+      const double cost = (double)((units + nc - 1) / nc) * (unit_us / c + (c > 1 ? kSplitUs : 0.0));
+      if (cost < best - 1e-9 || (force_c == c)) { best = force_c == c ? -1.0 : cost; csize = c; ncl = nc; }
+    }
     fp.cl_scratch = L->cl_scratch;
-    const int grid = csize > 1 ? units * csize : std::min(L->num_sms, units);
+    const int grid = csize > 1 ? std::min(units, ncl) * csize : std::min(L->num_sms, units);
     KL_TRY(launch_umma_decode_fused(f8, L->fp4, fp, grid, csize, st));
     mark(L, ST_GEMM1, st);
     if (A.chained) { L->chain_T = n_def > 0 ? T : -1; L->chain_ndef = n_def; }
