@@ -1100,25 +1100,37 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     static const int dbg_fd = experiment_knob("MOE_DEBUG_FD");   // timing experiments (MOE_EXPERIMENTS builds)
     fp.debug = dbg_fd;
     const int units = prev_units + Fs / 128 + (int)std::min<int64_t>(E, pairs) * (F / 128);
-    // Cluster split: each unit over C = 1/2/4/8 CTAs (C <= the W13 k-blocks and W2 tiles), the
-    // clusters taking units from the device queue.  Cost model per layer: rounds x (unit time / C +
-    // per-unit split overhead), rounds = ceil(units / resident clusters), unit time = its weight
-    // bytes at the per-SM streaming rate -- one wave of whole units when units fill the GPU (V3,
-    // T = 1), wider splits when units are few (expert TP, small layers) or leave a ragged last
-    // round (Qwen2: 320 units on 148 SMs).  MOE_FD_CSIZE forces C (A/B experiments).
+    // Cluster split: each unit over C = 1/2/4/8 CTAs (C <= the W13 k-blocks and W2 tiles).
+    // (1) Few units (expert TP, small layers): the largest C whose clusters all fit in one wave.
+    // (2) Otherwise C = 2 when a cost model of the part after the router says so -- this
+    //     layer's routed + shared units (a chained layer's group-2 units run beside the router):
+    //     rounds x (unit time / C + split overhead), rounds = ceil(units / resident clusters),
+    //     unit time = its weight bytes at ~56 GB/s per SM, overhead 2.3 us, and >= 5 % cheaper
+    //     than C = 1.  Routed units use the expected number of distinct experts of T tokens.
+    //     (Fitted to profiles/r02/decode_csize.txt: C = 2 wins when the post-router units fit
+    //     one round of pairs -- V2-Lite / V2.5 chained deferral -- or leave a ragged third round
+    //     at C = 1 -- Qwen2, 320 units; C = 4 / 8 beyond one wave lost everywhere.)
+    // Clusters take units from the device queue.  MOE_FD_CSIZE forces C (A/B experiments).
     static const int force_c = getenv("MOE_FD_CSIZE") ? atoi(getenv("MOE_FD_CSIZE")) : 0;
     const int KA = H / (f8 ? 128 : 64), NT = H / 256;
-    const double wb = L->fp4 ? 0.5 : (f8 ? 1.0 : 2.0);
-    const double unit_us = (256.0 * H + 128.0 * H) * wb / 45e3;      // ~45 GB/s per SM
-    constexpr double kSplitUs = 1.5;                                   // leader reduce + h exchange
-    int csize = 1, ncl = L->num_sms;
-    double best = 1e30;
-    for (int c = 1; c <= 8; c *= 2) {
-      if (c > 1 && (c > KA || c > NT || L->fd_max_clusters[c] < 1)) continue;
-      const int nc = c == 1 ? L->num_sms : L->fd_max_clusters[c];
-      const double cost = (double)((units + nc - 1) / nc) * (unit_us / c + (c > 1 ? kSplitUs : 0.0));
-      if (cost < best - 1e-9 || (force_c == c)) { best = force_c == c ? -1.0 : cost; csize = c; ncl = nc; }
+    auto c_ok = [&](int c) { return c == 1 || (c <= KA && c <= NT && L->fd_max_clusters[c] >= 1); };
+    auto n_cl = [&](int c) { return c == 1 ? L->num_sms : L->fd_max_clusters[c]; };
+    int csize = 1;
+    for (int c = 8; c >= 2; c /= 2)
+      if (c_ok(c) && units <= n_cl(c) && units * c <= L->num_sms) { csize = c; break; }
+    if (csize == 1 && c_ok(2)) {
+      const double wb = L->fp4 ? 0.5 : (f8 ? 1.0 : 2.0);
+      const double unit_us = (256.0 * H + 128.0 * H) * wb / 56e3;
+      const int k_now = (A.chained && n_def > 0) ? k - n_def : k;
+      const double e_exp = T <= 1 ? (double)k_now
+                                  : std::min((double)E, std::ceil(E * (1.0 - std::pow(1.0 - (double)k_now / E, T))));
+      const int post = Fs / 128 + (int)e_exp * (F / 128);
+      const double c1 = (double)((post + n_cl(1) - 1) / n_cl(1)) * unit_us;
+      const double c2 = (double)((post + n_cl(2) - 1) / n_cl(2)) * (unit_us / 2 + 2.3);
+      if (c2 < 0.95 * c1) csize = 2;
     }
+    if (force_c == 1 || ((force_c == 2 || force_c == 4 || force_c == 8) && c_ok(force_c))) csize = force_c;
+    const int ncl = n_cl(csize);
     fp.cl_scratch = L->cl_scratch;
     const int grid = csize > 1 ? std::min(units, ncl) * csize : std::min(L->num_sms, units);
     KL_TRY(launch_umma_decode_fused(f8, L->fp4, fp, grid, csize, st));
