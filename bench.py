@@ -164,8 +164,20 @@ def cpu_cores():
         return os.cpu_count()
 
 
+def prefill_config(p, T, parallelism):
+    """The `config` object of the prefill line (shared by both arms)."""
+    weights = {0: "bf16", 1: "fp8_e4m3_block128_ue8m0", 2: "f32", 3: "fp4_e2m1_block128_ue8m0"}[p.wtype]
+    return {"workload": f"{p.name}_moe_layer_prefill", "tokens_per_gpu": T, "hidden": p.hidden, "ffn": p.ffn,
+            "experts": p.n_experts, "top_k": p.top_k, "shared_ffn": p.shared_ffn,
+            "weights": weights, "parallelism": parallelism}
+
+
 def run_reference(args):
-    """--impl reference: the oracle timed on the host cores, same metric/config."""
+    """--impl reference: the oracle (the reference is a paper, no installable code) timed on
+    the host cores, on our arm's metric and config.  Each step is one full-layer oracle call
+    (as it stands: every expert the batch hits is dequantised in the call) on a bounded
+    sample of the workload's tokens -- `--ref-tokens` per step -- so the default run ends
+    within a few minutes.  Under torchrun only rank 0 runs."""
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -174,28 +186,30 @@ def run_reference(args):
     from inputs.presets import PRESETS
     from inputs.synthetic import make_tokens, make_weights
     p = PRESETS[args.config]
+    T = args.tokens or p.prefill_tokens
     dev = "cuda" if torch.cuda.is_available() else "cpu"
     w = make_weights(p, dev)
-    x, _ = make_tokens(p, args.steps + args.warmup, dev)
-    from oracle import moe_oracle as O
-    from tests.parity import oracle_cfg, oracle_weights
-    cfg, W = oracle_cfg(p), oracle_weights(p, w)
+    nt = max(1, min(args.ref_tokens, T))
+    x, _ = make_tokens(p, nt * (args.steps + args.warmup), dev)
     for i in range(args.warmup):
-        O.moe_layer(x[i:i + 1].cpu().to(torch.float64).numpy(), W, cfg)
-    t0 = time.perf_counter()
+        oracle_layer_call(p, w, x[i * nt:(i + 1) * nt])
+    dts, nexps = [], []
     for i in range(args.steps):
         j = args.warmup + i
-        O.moe_layer(x[j:j + 1].cpu().to(torch.float64).numpy(), W, cfg)
-    dt = time.perf_counter() - t0
-    v = args.steps / dt
+        _, nexp, dt = oracle_layer_call(p, w, x[j * nt:(j + 1) * nt])
+        dts.append(dt)
+        nexps.append(nexp)
+    dt = sum(dts)
+    v = nt * args.steps / dt
+    cfg = prefill_config(p, T, "single")
+    cfg["sample"] = (f"{nt} tokens per step of the {T}-token workload (one full-layer oracle call per step, "
+                     f"{min(nexps)}-{max(nexps)} distinct experts dequantised in the call)")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "tokens/s", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic",
-            "config": {"workload": f"{p.name}_moe_layer_prefill", "tokens_per_step": 1},
-            "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": cpu_cores(), "kind": "oracle",
-                             "sample": f"1 token per step of the {p.name} layer (fp64 numpy oracle, "
-                                       "experts dequantised per call)"},
+            "data": "synthetic", "config": cfg,
+            "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": cpu_cores(), "cpu_model": cpu_model(),
+                             "kind": "oracle", "sample": cfg["sample"]},
             "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -556,16 +570,12 @@ def run_ours(args):
         line = {"metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": ws, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
                 "vs_baseline": None, "dtype": "e4m3" if fp8 else "bf16", "data": "synthetic",
-                "config": {"workload": f"{p.name}_moe_layer_prefill", "tokens_per_gpu": T, "hidden": p.hidden,
-                           "ffn": p.ffn, "experts": p.n_experts, "top_k": p.top_k, "shared_ffn": p.shared_ffn,
-                           "weights": "fp8_e4m3_block128_ue8m0" if fp8 else "bf16", "parallelism":
-                           (f"ep{ws} (NCCL " + ("fixed-capacity all-to-all, no host sync" if args.ep_fixed
-                                                else "all-to-all-v, counts via the host") + " dispatch/combine)"
-                            if ep else f"replica x{ws}")
-                           if ws > 1 else "single", "l2": "flushed before every step (256 MiB write, then 256 MiB read so the dirty lines are written back "
-                           "before the events, "
-                           "outside the timed events); inputs resident in HBM",
-                           "distinct_experts_hit": n_distinct},
+                "config": dict(prefill_config(p, T, (f"ep{ws} (NCCL " + (
+                    "fixed-capacity all-to-all, no host sync" if args.ep_fixed else "all-to-all-v, counts via the host")
+                    + " dispatch/combine)" if ep else f"replica x{ws}") if ws > 1 else "single"),
+                    l2="flushed before every step (256 MiB write, then 256 MiB read so the dirty lines are written "
+                       "back before the events, outside the timed events); inputs resident in HBM",
+                    distinct_experts_hit=n_distinct),
                 "layer_tflops": layer_tflops,
                 "roofline": roofline, "decode": decode, "e2e": e2e, "cpu_baseline": cpu,
                 "gpu_launches": pinfo.kernels_per_forward_prefill * args.steps,
@@ -593,6 +603,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-tokens", type=int, default=16, help="tokens of the cpu_baseline oracle call")
+    ap.add_argument("--ref-tokens", type=int, default=8, help="--impl reference: tokens per step (oracle call)")
     ap.add_argument("--replicas", action="store_true", help="N>1: independent replicas instead of expert parallel")
     ap.add_argument("--ep-fixed", action="store_true",
                     help="N>1: fixed-capacity EP exchange (no host sync, capturable; more bytes on the wire)")
