@@ -318,8 +318,9 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             if (FP8 && (kb & 3) == 0) {
               tmem_cp_32x128b_x4_pair(tmem + SW_SFA_COL + set, sf_desc(smem_u32(sSFW + stage * SW_SFW_BYTES)));
               tmem_cp_32x128b_x4_pair(tmem + SW_SFB_COL + set, sf_desc(smem_u32(sSFX + stage * SW_SFX_BYTES)));
-              tmem_cp_32x128b_x4_pair(tmem + SW_SFB_COL + set + 4,
-                                      sf_desc(smem_u32(sSFX + stage * SW_SFX_BYTES + 512)));
+              if (N > 128)                         // tokens 128..255 (a cp costs the pipe ~100 cycles)
+                tmem_cp_32x128b_x4_pair(tmem + SW_SFB_COL + set + 4,
+                                        sf_desc(smem_u32(sSFX + stage * SW_SFX_BYTES + 512)));
             }
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
