@@ -42,8 +42,9 @@ constexpr int SW_STAGES = 6, SW_THREADS = 320, SW_UQ = 4;
 // stages are released in groups of SW_CE by one MMA commit: a tcgen05.commit costs the tensor
 // pipe ~100 cycles at N = 256 (profiles/r02/mma_ring.txt: block-scaled pair MMA 153.5 cycles
 // with a commit per k-block, 132.8 per 2, 128.0 per 4) -- but in this kernel SW_CE = 2
-// measured 1-2 % slower than 1 (interleaved A/B, GEMM1 2.50 vs 2.47 ms): the coarser
-// release shortens the producer's run-ahead, and the pipe is not what binds here
+// measured 1-2 % slower than 1 twice (interleaved A/B: GEMM1 2.50 vs 2.47 ms, and 2.42 vs 2.37 ms
+// after the two-box token halves): the coarser release shortens the producer's run-ahead, and
+// the commit is not what binds inside this kernel (profiles/r02/swap_np.txt)
 constexpr int SW_CE = 1;
 static_assert(SW_STAGES % SW_CE == 0, "stage groups");
 constexpr int SW_W_BYTES = 128 * 128;          // this CTA's 128 weight rows x 128 B
