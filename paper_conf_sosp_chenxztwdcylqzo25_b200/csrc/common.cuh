@@ -240,6 +240,7 @@ struct moe_layer {
   CUtensorMap map_xperm, map_h, map_xq, map_hsh, map_gate;   // activation rows (box 128), router rows
   CUtensorMap dmap_xperm, dmap_h, dmap_xq, dmap_hsh;           // decode: activation rows (box 16)
   float *dacc = nullptr;        // fused decode: [2][gemv_max_tokens, H] fp32 sums (immediate, deferred), kept zero
+  int32_t *zero_i32 = nullptr; // [0] a device 0 (an empty routed list), [1..2] the EP shared launch's work counter
   bool fused_decode = false;
   // chained Expert Deferral (moe_layer_forward_chained): expert lists of the
   // immediate / deferred canonical slots, and what the last chained call left

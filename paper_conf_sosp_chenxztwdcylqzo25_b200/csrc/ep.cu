@@ -123,6 +123,24 @@ __global__ void __launch_bounds__(128) ep_scatter_fp8_kernel(const uint8_t *__re
   }
 }
 
+// expert side, FP8 decode: received rows in arrival order -> e4m3 codes [R, H] (the fused
+// decode stream's token operand) + fp32 scales [R, H/128] (2^(e - 127) from the UE8M0 bytes)
+__global__ void __launch_bounds__(128) ep_unpack_fp8_kernel(const uint8_t *__restrict__ recv, int H, int row_bytes,
+                                                            uint8_t *__restrict__ xq, float *__restrict__ xs) {
+  const int r = blockIdx.x;
+  const uint8_t *src = recv + (int64_t)r * row_bytes;
+  uint4 *dst = reinterpret_cast<uint4 *>(xq + (int64_t)r * H);
+  for (int c = threadIdx.x; c < H / 16; c += blockDim.x) dst[c] = reinterpret_cast<const uint4 *>(src)[c];
+  for (int b = threadIdx.x; b < H / 128; b += blockDim.x) xs[(int64_t)r * (H / 128) + b] = exp2i((int)src[H + b] - 127);
+}
+
+cudaError_t launch_ep_unpack_fp8(const void *recv, int R, int H, int row_bytes, void *xq, float *xs, cudaStream_t st) {
+  if (R <= 0) return cudaSuccess;
+  ep_unpack_fp8_kernel<<<R, 128, 0, st>>>(reinterpret_cast<const uint8_t *>(recv), H, row_bytes,
+                                          reinterpret_cast<uint8_t *>(xq), xs);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_ep_pack_fp8(const void *xq, const float *xs, int T, int H, int k, const int32_t *idx,
                                const float *w, int E_loc, int P, int Tm, int row_bytes, const int32_t *sendpos,
                                void *send_x, int32_t *send_idx, float *send_w, cudaStream_t st) {

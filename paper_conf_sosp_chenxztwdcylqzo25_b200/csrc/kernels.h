@@ -188,6 +188,7 @@ cudaError_t launch_ep_pack_fp8(const void *xq, const float *xs, int T, int H, in
                                void *send_x, int32_t *send_idx, float *send_w, cudaStream_t st);
 cudaError_t launch_ep_scatter_fp8(const void *recv, int R, int H, int k, int row_bytes, const int32_t *pos,
                                   void *xperm, uint8_t *img, int img_stride, cudaStream_t st);
+cudaError_t launch_ep_unpack_fp8(const void *recv, int R, int H, int row_bytes, void *xq, float *xs, cudaStream_t st);
 int ep_nccl_get_unique_id(void *out128);
 int ep_nccl_init(void **comm, int P, int rank, const void *uid128);
 void ep_nccl_destroy(void *comm);

@@ -67,7 +67,7 @@ void free_all(moe_layer *L) {
                   L->row_token, L->pos, L->sched, L->pairs, L->n_pairs, L->xq, L->xs, L->xperm, L->xperm_s, L->hbuf, L->h_s, L->yperm,
                   L->hsh, L->hsh_s, L->ysh, L->w13_img, L->w2_img, L->ws13_img, L->ws2_img,
                   L->xperm_img, L->h_img, L->xq_img, L->hsh_img, L->dacc, L->trace, L->imm_list, L->def_list,
-                  L->n_lists, L->xcopy, L->cl_scratch, L->w13_f4, L->w2_f4, L->ws13_f4, L->ws2_f4};
+                  L->n_lists, L->xcopy, L->cl_scratch, L->zero_i32, L->w13_f4, L->w2_f4, L->ws13_f4, L->ws2_f4};
   for (void *p : ptrs)
     if (p) cudaFree(p);
   void *eps[] = {L->ep.send_x, L->ep.send_idx, L->ep.send_w, L->ep.sendpos, L->ep.cnt_dev, L->ep.recv_x,
@@ -575,6 +575,8 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
       const size_t n = (size_t)2 * L->gemv_max_tokens * H * 4;
       C_TRY(dalloc(L, &L->dacc, n, false));
       C_TRY(cudaMemset(L->dacc, 0, n));
+      C_TRY(dalloc(L, &L->zero_i32, 16, false));   // [0] = 0, [1..2] a second stream work counter
+      C_TRY(cudaMemset(L->zero_i32, 0, 16));
       // cluster split of the stream (few units): how many clusters of 2 / 4 / 8 fit, and the
       // L2 scratch the peers hand their fp32 partials to the leader through
       for (int c = 2; c <= 8; c *= 2) L->fd_max_clusters[c] = fused_decode_max_clusters(f8, c);
@@ -828,6 +830,79 @@ static moe_status ep_counts_to_host(moe_layer *L, cudaStream_t st) {
   return MOE_OK;
 }
 
+static int fd_cluster_size(const moe_layer *L, int units, int k_used, int T, bool with_shared, int *ncl_out);
+
+// Expert side at decode sizes (R received rows and T_own own tokens <= gemv_max_tokens): the
+// fused decode stream instead of the prefill grouped GEMMs -- (A) the routed experts over the
+// received rows (arrival order, expert ids masked to this rank) -> fp32 sums -> the bf16 partial
+// rows returned to the origins; (B) the shared expert over the own tokens -> ysh (ungated: the
+// origin's final combine applies the Qwen2 gate).  Two stream launches + finalizes, in order.
+static moe_status ep_decode_stream(moe_layer *L, const void *x_own, int T_own, int n_def, bool want_def,
+                                   cudaStream_t st) {
+  const int R = L->ep.R, k = L->k, H = L->H, Fs = L->Fs;
+  const bool f8 = L->fp8;
+  float *acc_imm = L->dacc, *acc_def = L->dacc + (size_t)L->gemv_max_tokens * H;
+  // (B may launch while A's last CTAs still run -- finalize A triggers it through PDL -- so
+  // the two launches take units from separate work counters)
+  auto launch = [&](FusedDecodeParams &fp, int T, int units, int k_used, bool shared, int *ctr) -> moe_status {
+    fp.H = H; fp.T = T; fp.has_shared = shared; fp.has_prev = 0; fp.sgate = nullptr;
+    fp.acc_imm = acc_imm; fp.acc_def = acc_def;
+    fp.sched = ctr; fp.done = ctr + 1;
+    fp.cl_scratch = L->cl_scratch;
+    int ncl = 0;
+    const int csize = fd_cluster_size(L, units, k_used, T, shared, &ncl);
+    const int grid = csize > 1 ? std::min(units, ncl) * csize : std::min(L->num_sms, units);
+    KL_TRY(launch_umma_decode_fused(f8, L->fp4, fp, grid, csize, st));
+    return MOE_OK;
+  };
+  if (R > 0) {
+    // (A) routed experts over the received rows
+    FusedDecodeParams fp{};
+    FdGroup &g = fp.g[0];
+    if (f8) {
+      KL_TRY(launch_ep_unpack_fp8(L->ep.recv_x, R, H, L->ep.row_bytes, L->xperm, L->xperm_s, st));
+      g.x_map = L->dmap_xperm;
+      g.xs = L->xperm_s;
+    } else if (!make_kmajor_map(&g.x_map, L->ep.recv_x, false, (int64_t)L->ep.P * std::max(1, L->max_tokens), H, 16)) {
+      return fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for the received rows");
+    }
+    if (L->fp4) { g.w13_map4 = L->fmap_w13; g.w2_map4 = L->fmap_w2; }
+    g.w13 = (const uint8_t *)L->w13; g.w13_s = L->w13_s;
+    g.w2 = (const uint8_t *)L->w2; g.w2_s = L->w2_s; g.nch = L->F / 128;
+    g.list = L->act_list; g.n_list = L->n_active; g.topk_idx = L->topk_idx; g.topk_w = L->topk_w;
+    g.k = k; g.e0 = L->e0;
+    g.a0 = 0; g.a1 = want_def ? k - n_def : k; g.a2 = k;
+    fp.g[1] = fp.g[2] = g;
+    const int units = (int)std::min<int64_t>(L->E, (int64_t)R * k) * (L->F / 128);
+    moe_status s = launch(fp, R, units, k, false, L->sched + 5);
+    if (s != MOE_OK) return s;
+    DecodeFinalizeArgs fa{};
+    fa.T = R; fa.H = H; fa.use_def = want_def; fa.acc_imm = acc_imm; fa.acc_def = acc_def;
+    fa.y = L->ep.partial; fa.deferred_out = want_def ? L->ep.partial_def : nullptr;
+    KL_TRY(launch_decode_finalize(fa, st));
+  }
+  if (Fs > 0 && T_own > 0) {
+    // (B) the shared expert over the own tokens (FP8: xq / xs quantised in phase A)
+    FusedDecodeParams fp{};
+    FdGroup &g = fp.g[1];
+    if (!f8) CUDA_TRY(cudaMemcpyAsync(L->xcopy, x_own, (size_t)T_own * H * 2, cudaMemcpyDeviceToDevice, st));
+    g.x_map = f8 ? L->dmap_xq : L->dmap_xc;
+    if (L->fp4) { g.w13_map4 = L->fmap_ws13; g.w2_map4 = L->fmap_ws2; }
+    g.w13 = (const uint8_t *)L->ws13; g.w13_s = L->ws13_s; g.xs = L->xs;
+    g.w2 = (const uint8_t *)L->ws2; g.w2_s = L->ws2_s; g.nch = Fs / 128;
+    fp.g[0] = g;
+    fp.g[0].list = L->act_list; fp.g[0].n_list = L->zero_i32;   // no routed units
+    fp.g[0].nch = L->F / 128;
+    fp.g[2] = fp.g[0];
+    moe_status s = launch(fp, T_own, Fs / 128, 0, true, L->zero_i32 + 1);
+    if (s != MOE_OK) return s;
+    DecodeFinalizeArgs fa{};
+    fa.T = T_own; fa.H = H; fa.use_def = 0; fa.acc_imm = acc_imm; fa.acc_def = acc_def; fa.y = L->ysh;
+    KL_TRY(launch_decode_finalize(fa, st));
+  }
+  return MOE_OK;
+}
+
 static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_def, bool want_def,
                              cudaStream_t st) {
   const int R = L->ep.R, k = L->k, H = L->H, Fs = L->Fs, E = L->E;
@@ -845,6 +920,9 @@ static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_d
     CUDA_TRY(cudaMemsetAsync(L->n_tiles, 0, 4, st));
     CUDA_TRY(cudaMemsetAsync(L->n_pairs, 0, 4, st));
   }
+  static const bool ep_gemm = getenv("MOE_EP_DECODE_GEMM") && atoi(getenv("MOE_EP_DECODE_GEMM")) == 1;  // A/B
+  if (!ep_gemm && L->fused_decode && L->umma && R <= L->gemv_max_tokens && T_own <= L->gemv_max_tokens)
+    return ep_decode_stream(L, x_own, T_own, n_def, want_def, st);
   if (L->fp8) {
     // received e4m3 rows + exponents -> the expert-sorted rows and their scale images (the
     // own tokens' xq for the shared expert was quantised in phase A)
@@ -922,6 +1000,45 @@ static moe_status ep_forward_nccl(moe_layer *L, const void *x, const void *resid
     NCCL_TRY(ep_nccl_rows(L->ep.comm, P, rcnt, roff, scnt, soff, want_def ? 2 : 1, snd, rcv, rb, st));
   }
   return ep_phase_d(L, residual, T, din, y, want_def ? dout : nullptr, st);
+}
+
+// Cluster size of the fused decode stream for `units` queued units (k_used slots per token of T
+// tokens routed here, with / without the shared expert's units after the router).
+static int fd_cluster_size(const moe_layer *L, int units, int k_used, int T, bool with_shared, int *ncl_out) {
+  const int H = L->H, E = L->E;
+  const bool f8 = L->fp8;
+  // Cluster split: each unit over C = 1/2/4/8 CTAs (C <= the W13 k-blocks and W2 tiles).
+  // (1) Few units (expert TP, small layers): the largest C whose clusters all fit in one wave.
+  // (2) Otherwise C = 2 when a cost model of the part after the router says so -- this
+  //     layer's routed + shared units (a chained layer's group-2 units run beside the router):
+  //     rounds x (unit time / C + split overhead), rounds = ceil(units / resident clusters),
+  //     unit time = its weight bytes at ~56 GB/s per SM, overhead 2.3 us, and >= 5 % cheaper
+  //     than C = 1.  Routed units use the expected number of distinct experts of T tokens.
+  //     (Fitted to profiles/r02/decode_csize.txt: C = 2 wins when the post-router units fit
+  //     one round of pairs -- V2-Lite / V2.5 chained deferral -- or leave a ragged third round
+  //     at C = 1 -- Qwen2, 320 units; C = 4 / 8 beyond one wave lost everywhere.)
+  // Clusters take units from the device queue.  MOE_FD_CSIZE forces C (A/B experiments).
+  static const int force_c = getenv("MOE_FD_CSIZE") ? atoi(getenv("MOE_FD_CSIZE")) : 0;
+  const int KA = H / (f8 ? 128 : 64), NT = H / 256;
+  auto c_ok = [&](int c) { return c == 1 || (c <= KA && c <= NT && L->fd_max_clusters[c] >= 1); };
+  auto n_cl = [&](int c) { return c == 1 ? L->num_sms : L->fd_max_clusters[c]; };
+  int csize = 1;
+  for (int c = 8; c >= 2; c /= 2)
+    if (c_ok(c) && units <= n_cl(c) && units * c <= L->num_sms) { csize = c; break; }
+  if (csize == 1 && c_ok(2)) {
+    const double wb = L->fp4 ? 0.5 : (f8 ? 1.0 : 2.0);
+    const double unit_us = (256.0 * H + 128.0 * H) * wb / 56e3;
+    const int k_now = k_used;
+    const double e_exp = T <= 1 ? (double)k_now
+                                : std::min((double)E, std::ceil(E * (1.0 - std::pow(1.0 - (double)k_now / E, T))));
+    const int post = (with_shared ? L->Fs / 128 : 0) + (int)e_exp * (L->F / 128);
+    const double c1 = (double)((post + n_cl(1) - 1) / n_cl(1)) * unit_us;
+    const double c2 = (double)((post + n_cl(2) - 1) / n_cl(2)) * (unit_us / 2 + 2.3);
+    if (c2 < 0.95 * c1) csize = 2;
+  }
+  if (force_c == 1 || ((force_c == 2 || force_c == 4 || force_c == 8) && c_ok(force_c))) csize = force_c;
+  *ncl_out = n_cl(csize);
+  return csize;
 }
 
 // One forward.  Modes: plain / split deferral (moe_layer_forward[_deferred]:
@@ -1100,37 +1217,8 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
     static const int dbg_fd = experiment_knob("MOE_DEBUG_FD");   // timing experiments (MOE_EXPERIMENTS builds)
     fp.debug = dbg_fd;
     const int units = prev_units + Fs / 128 + (int)std::min<int64_t>(E, pairs) * (F / 128);
-    // Cluster split: each unit over C = 1/2/4/8 CTAs (C <= the W13 k-blocks and W2 tiles).
-    // (1) Few units (expert TP, small layers): the largest C whose clusters all fit in one wave.
-    // (2) Otherwise C = 2 when a cost model of the part after the router says so -- this
-    //     layer's routed + shared units (a chained layer's group-2 units run beside the router):
-    //     rounds x (unit time / C + split overhead), rounds = ceil(units / resident clusters),
-    //     unit time = its weight bytes at ~56 GB/s per SM, overhead 2.3 us, and >= 5 % cheaper
-    //     than C = 1.  Routed units use the expected number of distinct experts of T tokens.
-    //     (Fitted to profiles/r02/decode_csize.txt: C = 2 wins when the post-router units fit
-    //     one round of pairs -- V2-Lite / V2.5 chained deferral -- or leave a ragged third round
-    //     at C = 1 -- Qwen2, 320 units; C = 4 / 8 beyond one wave lost everywhere.)
-    // Clusters take units from the device queue.  MOE_FD_CSIZE forces C (A/B experiments).
-    static const int force_c = getenv("MOE_FD_CSIZE") ? atoi(getenv("MOE_FD_CSIZE")) : 0;
-    const int KA = H / (f8 ? 128 : 64), NT = H / 256;
-    auto c_ok = [&](int c) { return c == 1 || (c <= KA && c <= NT && L->fd_max_clusters[c] >= 1); };
-    auto n_cl = [&](int c) { return c == 1 ? L->num_sms : L->fd_max_clusters[c]; };
-    int csize = 1;
-    for (int c = 8; c >= 2; c /= 2)
-      if (c_ok(c) && units <= n_cl(c) && units * c <= L->num_sms) { csize = c; break; }
-    if (csize == 1 && c_ok(2)) {
-      const double wb = L->fp4 ? 0.5 : (f8 ? 1.0 : 2.0);
-      const double unit_us = (256.0 * H + 128.0 * H) * wb / 56e3;
-      const int k_now = (A.chained && n_def > 0) ? k - n_def : k;
-      const double e_exp = T <= 1 ? (double)k_now
-                                  : std::min((double)E, std::ceil(E * (1.0 - std::pow(1.0 - (double)k_now / E, T))));
-      const int post = Fs / 128 + (int)e_exp * (F / 128);
-      const double c1 = (double)((post + n_cl(1) - 1) / n_cl(1)) * unit_us;
-      const double c2 = (double)((post + n_cl(2) - 1) / n_cl(2)) * (unit_us / 2 + 2.3);
-      if (c2 < 0.95 * c1) csize = 2;
-    }
-    if (force_c == 1 || ((force_c == 2 || force_c == 4 || force_c == 8) && c_ok(force_c))) csize = force_c;
-    const int ncl = n_cl(csize);
+    int ncl = 0;
+    const int csize = fd_cluster_size(L, units, (A.chained && n_def > 0) ? k - n_def : k, T, Fs > 0, &ncl);
     fp.cl_scratch = L->cl_scratch;
     const int grid = csize > 1 ? std::min(units, ncl) * csize : std::min(L->num_sms, units);
     KL_TRY(launch_umma_decode_fused(f8, L->fp4, fp, grid, csize, st));

@@ -149,3 +149,36 @@ def test_ep_nccl_single_rank_fixed_graph(lib):
         _oracle_check(p, w_cpu, x, yout)
     del graph
     layer.close()
+
+
+@pytest.mark.parametrize("name,P,Ts,fixed", [("v3_s", 2, [3, 5], False), ("v3_s", 4, [1, 0, 2, 1], False),
+                                             ("qwen2_s", 2, [4, 1], False), ("v2lite_s", 4, [2, 2, 1, 3], False),
+                                             ("v3_s", 4, [1, 1, 0, 2], True), ("v3_s_fp4", 2, [2, 3], False)])
+def test_ep_group_decode_stream(lib, name, P, Ts, fixed):
+    """Decode-sized EP (received rows and own tokens <= gemv_max_tokens): the expert side runs the
+    fused decode stream (routed experts over the received rows, shared expert over the own tokens)."""
+    p = SMALL[name]
+    w_cpu = make_weights(p, "cpu")
+    group = lib.MoEGroup(p, w_cpu.to("cuda"), ep_size=P, max_tokens=max(max(Ts), 1), ep_fixed=fixed)
+    xs = [make_tokens(p, t, "cpu", offset=r)[0] for r, t in enumerate(Ts)]
+    ys = group.forward([x.cuda() for x in xs])
+    torch.cuda.synchronize()
+    for x, y in zip(xs, ys):
+        _oracle_check(p, w_cpu, x, y)
+    group.close()
+
+
+def test_ep_group_decode_stream_deferral(lib):
+    p = SMALL["v3_s"]
+    P, Ts = 2, [3, 4]
+    w_cpu = make_weights(p, "cpu")
+    group = lib.MoEGroup(p, w_cpu.to("cuda"), ep_size=P, max_tokens=4)
+    xs, rs = zip(*[make_tokens(p, t, "cpu", offset=r) for r, t in enumerate(Ts)])
+    dins = [(torch.randn(t, p.hidden, generator=torch.Generator().manual_seed(r)) * 0.5).to(torch.bfloat16)
+            for r, t in enumerate(Ts)]
+    ys, douts = group.forward([x.cuda() for x in xs], residuals=[r.cuda() for r in rs], n_deferred=3,
+                              deferred_in=[d.cuda() for d in dins], want_deferred_out=True)
+    torch.cuda.synchronize()
+    for x, r, d, y, do in zip(xs, rs, dins, ys, douts):
+        _oracle_check(p, w_cpu, x, y, residual=r, n_def=3, din=d, dout=do)
+    group.close()
