@@ -70,7 +70,8 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(const __grid_constan
   if (e == 0) *a.n_active = total;
   __syncthreads();
   // 2-CTA work list: pairs of consecutive 128-row tiles of one expert
-  const int npair = (ntile + 1) / 2;
+  const int prow = a.pair_rows > 0 ? a.pair_rows : 256;  // multiple of 128 (entries stay tile-aligned)
+  const int npair = (cnt + prow - 1) / prow;
   int pair_off;
   Scan(tmp).ExclusiveSum(npair, pair_off, total);
   if (e == 0 && a.n_pairs) *a.n_pairs = total;
@@ -84,7 +85,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(const __grid_constan
       a.tiles[tile_off + m] = make_int4(e, off_pad + m * kPadM, off_pad + cnt, tile_off | (ntile << 16));
     if (a.pairs)
       for (int m = 0; m < npair; ++m)
-        a.pairs[pair_off + m] = make_int4(e, off_pad + m * 2 * kPadM, off_pad + cnt, pair_off | (npair << 16));
+        a.pairs[pair_off + m] = make_int4(e, off_pad + m * prow, off_pad + cnt, pair_off | (npair << 16));
     if (cnt > 0) a.act_list[act_off] = e;
   }
   if (e == 0) {
