@@ -92,8 +92,8 @@ struct PermuteArgs {
   int32_t *chunk_cnt, *chunk_base;  // [nchunk, E]
   int32_t *counts, *offs, *offs_pad;
   int4 *tiles; int32_t *n_tiles;
-  int4 *pairs; int32_t *n_pairs;   // 2-CTA work list (null = not needed)
-  int pair_rows;                    // rows per work-list entry: 256 (one token tile) or 384 (dual unit)
+  int4 *pairs; int32_t *n_pairs;   // 2-CTA work list (expert, row0, entry end, t0 | nt << 16); null = not needed
+  int pair_rows;                    // > 256: dual units for experts of 257 .. pair_rows tokens (else 256)
   int32_t *act_list; int32_t *n_active;
   int32_t *row_token;       // [R_max]
   int64_t R_max;

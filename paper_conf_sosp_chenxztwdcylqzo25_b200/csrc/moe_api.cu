@@ -490,6 +490,8 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   // token tile plus a <= 128-row one that share each weight k-block's load (MOE_SWAP_DUAL=0: 256)
   L->swap_dual = L->umma && !(getenv("MOE_SWAP_DUAL") && atoi(getenv("MOE_SWAP_DUAL")) == 0) &&
                  experiment_knob("MOE_DEBUG_GEMM") == 0;
+  // experts of 257 .. 256 + dual_tail tokens run as one dual unit (MOE_SWAP_DUAL_TAIL, default 64, <= 128)
+  L->dual_tail = getenv("MOE_SWAP_DUAL_TAIL") ? std::max(16, std::min(128, atoi(getenv("MOE_SWAP_DUAL_TAIL")))) : 64;
   if (!make_kmajor_map(&L->map_gate, L->gate_w, false, L->gate_rows, H, 256))
     return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for the router weights"));
   {
@@ -918,7 +920,7 @@ static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_d
   pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
   pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
   pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
-  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs; pa.pair_rows = L->swap_dual ? 384 : 256;
+  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs; pa.pair_rows = L->swap_dual ? 256 + L->dual_tail : 256;
   if (R > 0) {
     KL_TRY(launch_permute(pa, st));
     L->n_launch += 2;                            // count + scan + assign kernels
@@ -1126,7 +1128,7 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
   pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
   pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
   pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
-  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs; pa.pair_rows = L->swap_dual ? 384 : 256;
+  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs; pa.pair_rows = L->swap_dual ? 256 + L->dual_tail : 256;
   pa.dbg_perm = dbg ? dbg->perm : nullptr;
   pa.dbg_counts = dbg ? dbg->expert_counts : nullptr;
   if (tc_decode) {
