@@ -38,7 +38,7 @@
 namespace moe {
 using namespace sm100;
 
-constexpr int SW_STAGES = 6, SW_THREADS = 320, SW_UQ = 4;
+constexpr int SW_STAGES = 6, SW_THREADS = 320, SW_UQ = 8;
 // stages are released in groups of SW_CE by one MMA commit: a tcgen05.commit costs the tensor
 // pipe ~100 cycles at N = 256 (profiles/r02/mma_ring.txt: block-scaled pair MMA 153.5 cycles
 // with a commit per k-block, 132.8 per 2, 128.0 per 4) -- but in this kernel SW_CE = 2
