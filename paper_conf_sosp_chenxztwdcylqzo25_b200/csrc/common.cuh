@@ -269,8 +269,6 @@ struct moe_layer {
   CUtensorMap xmap_xperm, xmap_h, xmap_xq, xmap_hsh;
   CUtensorMap x64map_xperm, x64map_h, x64map_xq, x64map_hsh;   // box 64 rows (token boxes split between 2 pairs)
   int swap_clusters4 = 0;       // co-resident clusters of 2 CTA pairs (0: pair kernel only)
-  bool swap_dual = false;       // swap GEMM work list of dual units (384 rows: 256-row + <= 128-row tiles)
-  int dual_tail = 64;           // dual units for experts of 257 .. 256 + dual_tail tokens
   CUtensorMap smap_w13, smap_w2, smap_ws13, smap_ws2, smap_xperm, smap_h, smap_xq, smap_hsh;
   int4 *pairs = nullptr;        // [max_tiles] work list of 256-token tiles (2 x 128-row tiles)
   int32_t *n_pairs = nullptr;

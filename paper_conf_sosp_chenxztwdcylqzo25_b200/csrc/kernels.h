@@ -92,8 +92,7 @@ struct PermuteArgs {
   int32_t *chunk_cnt, *chunk_base;  // [nchunk, E]
   int32_t *counts, *offs, *offs_pad;
   int4 *tiles; int32_t *n_tiles;
-  int4 *pairs; int32_t *n_pairs;   // 2-CTA work list (expert, row0, entry end, t0 | nt << 16); null = not needed
-  int pair_rows;                    // > 256: dual units for experts of 257 .. pair_rows tokens (else 256)
+  int4 *pairs; int32_t *n_pairs;   // 2-CTA work list (null = not needed)
   int32_t *act_list; int32_t *n_active;
   int32_t *row_token;       // [R_max]
   int64_t R_max;
@@ -212,7 +211,6 @@ struct LogitsParams {
   int n_valid;                  // columns < n_valid are written
   int T;                        // token rows
   int nb;                       // 256-row blocks of router rows
-  int dual;                     // 1: routed units of up to 384 rows (two token tiles, one weight stream)
   int *sched;                   // device work counter, zero at launch
 };
 cudaError_t launch_umma_logits(const LogitsParams &p, int grid, cudaStream_t st);
@@ -300,7 +298,6 @@ struct SwapParams {
   const int32_t *n_tiles;
   int nb_r, nb_s;               // weight blocks per unit group
   int T_shared;                 // shared-expert tokens (0 = none)
-  int dual;                     // 1: routed units of up to 384 rows (two token tiles, one weight stream)
   int *sched;                   // device work counter, zero at launch
   int debug_mode;               // 0; (MOE_DEBUG_GEMM) 2 = no epilogue math -- timing experiments
   unsigned long long *trace;     // MOE_DEBUG_TRACE: MMA-warp cycle breakdown per CTA pair (timing experiments)

@@ -486,12 +486,6 @@ moe_status moe_layer_create(const moe_layer_config *cfg, const moe_layer_weights
   // ---- tcgen05 path: scale images and tensor maps ----
   C_TRY(cudaDeviceGetAttribute(&L->num_sms, cudaDevAttrMultiProcessorCount, cfg->device));
   if (L->umma) L->swap_clusters4 = umma_swap_max_clusters4(L->fp8);
-  // dual units (default): an expert's work-list entries cover up to 384 sorted rows, a 256-row
-  // token tile plus a <= 128-row one that share each weight k-block's load (MOE_SWAP_DUAL=0: 256)
-  L->swap_dual = L->umma && !(getenv("MOE_SWAP_DUAL") && atoi(getenv("MOE_SWAP_DUAL")) == 0) &&
-                 experiment_knob("MOE_DEBUG_GEMM") == 0;
-  // experts of 257 .. 256 + dual_tail tokens run as one dual unit (MOE_SWAP_DUAL_TAIL, default 64, <= 128)
-  L->dual_tail = getenv("MOE_SWAP_DUAL_TAIL") ? std::max(16, std::min(128, atoi(getenv("MOE_SWAP_DUAL_TAIL")))) : 64;
   if (!make_kmajor_map(&L->map_gate, L->gate_w, false, L->gate_rows, H, 256))
     return cleanup(fail(MOE_ERR_CUDA, "cuTensorMapEncodeTiled failed for the router weights"));
   {
@@ -641,7 +635,7 @@ static int swap_np(const moe_layer *L, int gemm, int nb_r, int nb_s, int dbg_mod
   // per unit 7 % faster, per launch 2-5 % slower (interleaved A/B, profiles/r02/swap_np.txt)
   static const int force1 = getenv("MOE_SWAP_NP1") ? atoi(getenv("MOE_SWAP_NP1")) : 1;
   static const int force2 = getenv("MOE_SWAP_NP2") ? atoi(getenv("MOE_SWAP_NP2")) : 1;
-  if ((gemm == 1 ? force1 : force2) == 1 || dbg_mode != 0 || L->swap_dual) return 1;
+  if ((gemm == 1 ? force1 : force2) == 1 || dbg_mode != 0) return 1;
   if ((nb_r & 1) || (nb_s & 1) || 4 * L->swap_clusters4 < L->num_sms * 3 / 4) return 1;
   return 2;
 }
@@ -685,7 +679,6 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     // clusters of 2 CTA pairs (adjacent weight blocks, token boxes multicast to both pairs)
     // when every operand group has an even number of weight blocks
     const int np1 = swap_np(L, 1, F / 128, Fs / 128, dbg_mode), np2 = swap_np(L, 2, H / 256, Fs > 0 ? H / 256 : 0, dbg_mode);
-    p1.dual = L->swap_dual;
     p1.tiles = L->pairs; p1.n_tiles = L->n_pairs; p1.nb_r = F / 128 / np1;
     p1.T_shared = Fs > 0 ? T : 0; p1.nb_s = Fs / 128 / np1; p1.sched = L->sched; p1.debug_mode = dbg_mode; p1.trace = L->trace;
     KL_TRY(launch_umma_swap_gemm(f8, GEMM_SWIGLU, p1, np1 == 2 ? L->swap_clusters4 : L->num_sms, np1, st));
@@ -707,7 +700,6 @@ static moe_status run_expert_gemms(moe_layer *L, int tile_bound, const void *x_s
     } else {
       p2.g[1] = p2.g[0];
     }
-    p2.dual = L->swap_dual;
     p2.tiles = L->pairs; p2.n_tiles = L->n_pairs; p2.nb_r = H / 256 / np2;
     p2.T_shared = Fs > 0 ? T : 0; p2.nb_s = H / 256 / np2; p2.sched = L->sched + 1; p2.debug_mode = dbg_mode; p2.trace = L->trace ? L->trace + 2048 : nullptr;
     KL_TRY(launch_umma_swap_gemm(f8, GEMM_PLAIN, p2, np2 == 2 ? L->swap_clusters4 : L->num_sms, np2, st));
@@ -920,7 +912,7 @@ static moe_status ep_phase_c(moe_layer *L, const void *x_own, int T_own, int n_d
   pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
   pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
   pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
-  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs; pa.pair_rows = L->swap_dual ? 256 + L->dual_tail : 256;
+  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs;
   if (R > 0) {
     KL_TRY(launch_permute(pa, st));
     L->n_launch += 2;                            // count + scan + assign kernels
@@ -1128,7 +1120,7 @@ static moe_status forward_impl(moe_layer *L, const FwdArgs &A, void *stream) {
   pa.chunk_cnt = L->chunk_cnt; pa.chunk_base = L->chunk_base; pa.counts = L->counts; pa.offs = L->offs;
   pa.offs_pad = L->offs_pad; pa.tiles = L->tiles; pa.n_tiles = L->n_tiles; pa.act_list = L->act_list;
   pa.n_active = L->n_active; pa.row_token = L->row_token; pa.R_max = L->R_max; pa.pos = L->pos;
-  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs; pa.pair_rows = L->swap_dual ? 256 + L->dual_tail : 256;
+  pa.pairs = L->pairs; pa.n_pairs = L->n_pairs;
   pa.dbg_perm = dbg ? dbg->perm : nullptr;
   pa.dbg_counts = dbg ? dbg->expert_counts : nullptr;
   if (tc_decode) {

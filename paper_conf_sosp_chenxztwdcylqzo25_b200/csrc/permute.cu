@@ -70,12 +70,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(const __grid_constan
   if (e == 0) *a.n_active = total;
   __syncthreads();
   // 2-CTA work list: pairs of consecutive 128-row tiles of one expert
-  // work-list entries of 256 rows (one token tile each); with pair_rows > 256 (dual units) an
-  // expert whose count exceeds 256 by at most pair_rows - 256 gets ONE entry covering all its rows
-  // (a 256-row tile + a short tile sharing the weight loads); larger experts keep 256-row entries
-  const int dual_tail = a.pair_rows > 256 ? a.pair_rows - 256 : 0;
-  const bool one_dual = cnt > 256 && cnt <= 256 + dual_tail;
-  const int npair = one_dual ? 1 : (cnt + 255) / 256;
+  const int npair = (ntile + 1) / 2;
   int pair_off;
   Scan(tmp).ExclusiveSum(npair, pair_off, total);
   if (e == 0 && a.n_pairs) *a.n_pairs = total;
@@ -89,8 +84,7 @@ __global__ void __launch_bounds__(SCAN_THREADS) scan_kernel(const __grid_constan
       a.tiles[tile_off + m] = make_int4(e, off_pad + m * kPadM, off_pad + cnt, tile_off | (ntile << 16));
     if (a.pairs)
       for (int m = 0; m < npair; ++m)
-        a.pairs[pair_off + m] = make_int4(e, off_pad + m * 256, off_pad + (one_dual ? cnt : min(cnt, (m + 1) * 256)),
-                                          pair_off | (npair << 16));
+        a.pairs[pair_off + m] = make_int4(e, off_pad + m * 2 * kPadM, off_pad + cnt, pair_off | (npair << 16));
     if (cnt > 0) a.act_list[act_off] = e;
   }
   if (e == 0) {

@@ -38,7 +38,7 @@
 namespace moe {
 using namespace sm100;
 
-constexpr int SW_STAGES = 6, SW_THREADS = 320, SW_UQ = 8;
+constexpr int SW_STAGES = 6, SW_THREADS = 320, SW_UQ = 4;
 // stages are released in groups of SW_CE by one MMA commit: a tcgen05.commit costs the tensor
 // pipe ~100 cycles at N = 256 (profiles/r02/mma_ring.txt: block-scaled pair MMA 153.5 cycles
 // with a commit per k-block, 132.8 per 2, 128.0 per 4) -- but in this kernel SW_CE = 2
@@ -46,16 +46,13 @@ constexpr int SW_STAGES = 6, SW_THREADS = 320, SW_UQ = 8;
 // after the two-box token halves): the coarser release shortens the producer's run-ahead, and
 // the commit is not what binds inside this kernel (profiles/r02/swap_np.txt)
 constexpr int SW_CE = 1;
-static_assert(SW_CE == 1, "dual units release their two stages with one commit each");
 static_assert(SW_STAGES % SW_CE == 0, "stage groups");
 constexpr int SW_W_BYTES = 128 * 128;          // this CTA's 128 weight rows x 128 B
 constexpr int SW_X_BYTES = 128 * 128;          // up to 128 token rows (half of N <= 256)
 constexpr int SW_SFW_BYTES = 512, SW_SFX_BYTES = 1024;
 constexpr int SW_XBOX = 32;                    // token rows per TMA box
 constexpr uint32_t SW_TMEM_COLS = 512;
-// TMEM: accumulator of the 256-row token tile at columns [0, 256), of a dual unit's second
-// (<= 128-row) tile at [256, 384); scale images at 384.. (two alternating sets 24 apart)
-constexpr uint32_t SW_ACC1_COL = 256, SW_SFA_COL = 384, SW_SFB_COL = 392, SW_SFB1_COL = 400, SW_SF_SET = 24;
+constexpr uint32_t SW_SFA_COL = 256, SW_SFB_COL = 264;   // + 16 for the second scale set
 constexpr int SW_XCH = 8;                      // columns per up->gate exchange chunk
 constexpr size_t SW_SMEM = 1024 + (size_t)SW_STAGES * (SW_W_BYTES + SW_X_BYTES + SW_SFW_BYTES + SW_SFX_BYTES) +
                            4 * 32 * SW_XCH * 4 +      // up -> gate exchange
@@ -76,9 +73,7 @@ __device__ __forceinline__ SwapUnit swap_unit(const SwapParams &p, int u, int n_
     const int t0 = any.w & 0xFFFF, nt = any.w >> 16;
     const int local = u - t0 * nb_r;
     const int4 tl = p.tiles[t0 + local % nt];
-    // dual units (p.dual): up to 384 rows = a 256-row tile + a <= 128-row tile sharing the weight loads
-    r.valid = 1; r.group = 0; r.expert = tl.x; r.row0 = tl.y; r.n = min(p.dual ? 384 : 256, tl.z - tl.y);
-    r.nb = local / nt;
+    r.valid = 1; r.group = 0; r.expert = tl.x; r.row0 = tl.y; r.n = min(256, tl.z - tl.y); r.nb = local / nt;
     return r;
   }
   const int us = u - n_routed_units;
@@ -111,8 +106,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
   uint64_t *uq_full = tmem_empty + 1;
   uint64_t *uq_empty = uq_full + SW_UQ;
   uint64_t *am_bar = uq_empty + SW_UQ;                                        // [2 parity][2 half]
-  uint64_t *tmem_empty1 = am_bar + 4;                                         // a dual unit's second tile read
-  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(tmem_empty1 + 1);
+  uint32_t *tmem_base_smem = reinterpret_cast<uint32_t *>(am_bar + 4);
   int *unit_q = reinterpret_cast<int *>(tmem_base_smem + 4);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -135,7 +129,6 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
     for (int s = 0; s < SW_STAGES / SW_CE; ++s) mbar_init(&empty[s], NP);
     mbar_init(tmem_full, 1);
     mbar_init(tmem_empty, 16);                   // 8 epilogue warps x 2 CTAs (the leader's copy is used)
-    mbar_init(tmem_empty1, 16);                  // the same, for the columns of a dual unit's second tile
     // leader's uq_empty: per pair an MMA warp + 8 epilogue warps per CTA; the other CTAs' producers
     constexpr int kUqArrivals = NP * 17 + 2 * NP - 1;
     for (int i = 0; i < SW_UQ; ++i) {
@@ -199,7 +192,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         if (!ui.valid) break;
         const SwapGroup &g = p.g[ui.group];
         const int nb = ui.nb * NP + (int)pair;                 // this pair's weight block
-        const int half_n = ((min(ui.n, 256) + 15) & ~15) >> 1;   // token rows per CTA (the 256-row tile)
+        const int half_n = ((ui.n + 15) & ~15) >> 1;          // token rows per CTA
         const int nbox0 = (half_n + SW_XBOX - 1) / SW_XBOX;
         const int nbox = nbox0 > 2 ? 4 : nbox0;                // > 64 rows: one 128-row box (4 x 32 rows of bytes)
         const int xrow = ui.row0 + (int)prank * half_n;
@@ -212,20 +205,8 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         const uint32_t xbytes = NP == 1 ? (uint32_t)(xb0 + xb1) * 128 : (uint32_t)nbox * (SW_XBOX * 128);
         const int64_t wtile = ((int64_t)ui.expert * g.w_nblk + nb) * g.kblocks;
         const int G = (g.kblocks + 3) >> 2;
-        // dual unit: the second tile's token half (<= 64 rows) in the next stage's X slot (the
-        // weights of this k-block serve both tiles), its bytes completing on this stage's barrier
-        const bool du = NP == 1 && ui.n > 256;
-        const int half1 = du ? ((ui.n - 256 + 15) & ~15) >> 1 : 0;
-        const int xrow1 = ui.row0 + 256 + (int)prank * half1;
-        const int yb0 = half1 > 48 ? 64 : half1 > 16 ? 32 : 16;
-        const int yb1 = (half1 > 32 && half1 <= 48) ? 16 : 0;
-        const CUtensorMap *ym0 = yb0 == 64 ? &g.x_map64 : yb0 == 32 ? &g.x_map : &g.x_map16;
-        const uint32_t xbytes1 = du ? (uint32_t)(yb0 + yb1) * 128 : 0;
         for (int kb = 0; kb < g.kblocks; ++kb) {
           if (stage % SW_CE == 0) mbar_wait(&empty[stage / SW_CE], phase ^ 1);   // the group's release
-          const int s1 = stage + 1 == SW_STAGES ? 0 : stage + 1;
-          const uint32_t ph1 = stage + 1 == SW_STAGES ? phase ^ 1 : phase;
-          if (du) mbar_wait(&empty[s1], ph1 ^ 1);
           if (kExperiments && p.debug_mode == 3) {                 // timing experiment: MMAs on stale smem, no loads
             if (pleader) mbar_arrive(&full[stage]);
             if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
@@ -248,17 +229,8 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
             continue;
           }
-          const uint32_t bytes = SW_W_BYTES + xbytes + (sf ? SW_SFW_BYTES + SW_SFX_BYTES : 0) +
-                                 (du ? xbytes1 + (sf ? SW_SFX_BYTES : 0) : 0);
+          const uint32_t bytes = SW_W_BYTES + xbytes + (sf ? SW_SFW_BYTES + SW_SFX_BYTES : 0);
           if (pleader) mbar_expect_tx(&full[stage], 2 * bytes);
-          if (du) {
-            tma_load_2d_pair(sX + s1 * SW_X_BYTES, ym0, &full[stage], kc, xrow1);
-            if (yb1) tma_load_2d_pair(sX + s1 * SW_X_BYTES + yb0 * 128, &g.x_map16, &full[stage], kc, xrow1 + yb0);
-            if (sf)
-              tma_load_2d_pair(sSFX + s1 * SW_SFX_BYTES, &g.sfx_map, &full[stage], 0,
-                               (kb >> 2) * g.sfx_tile_stride + ((ui.row0 + 256) >> 7));
-            if (pleader) mbar_arrive(&full[s1]);        // the second stage carries no bytes of its own
-          }
           // the CTA's 16 KB half of the 256-row tile: 8 rows of 2 KB
           tma_load_2d_pair(sW + stage * SW_W_BYTES, &g.w_map, &full[stage], 0,
                            (int)((wtile + kb) * 16 + prank * 8));
@@ -285,7 +257,6 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
                              kg * g.sfx_tile_stride + (ui.row0 >> 7));
           }
           if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
-          if (du && ++stage == SW_STAGES) { stage = 0; phase ^= 1; }
         }
       }
     }
@@ -310,7 +281,7 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         }
       }
     } else if (pleader) {
-      int stage = 0; uint32_t phase = 0; uint32_t acc_phase = 0, acc1_phase = 0;
+      int stage = 0; uint32_t phase = 0; uint32_t acc_phase = 0;
       constexpr uint16_t kAllPairs = NP == 1 ? 0x3 : 0xF;
       const uint16_t my_pair = (uint16_t)(0x3u << (2 * pair));
       int qs = 0; uint32_t qph = 0;
@@ -325,18 +296,12 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         if (trc) { const long long c = clock64(); c_unit += c - c0; c0 = c; }
         if (!ui.valid) break;
         const int kblocks = p.g[ui.group].kblocks;
-        const bool du = NP == 1 && ui.n > 256;                // dual unit (two token tiles, one weight stream)
-        const int N = (min(ui.n, 256) + 15) & ~15;
-        const int N1 = du ? (ui.n - 256 + 15) & ~15 : 0;
+        const int N = (ui.n + 15) & ~15;
         mbar_wait(tmem_empty, acc_phase ^ 1);
-        if (du) { mbar_wait(tmem_empty1, acc1_phase ^ 1); acc1_phase ^= 1; }
         if (trc) { const long long c = clock64(); c_tmem += c - c0; c0 = c; ++n_units; n_flop16 += N / 16; }
         tc_fence_after();
         for (int kb = 0; kb < kblocks; ++kb) {
-          const int s1 = stage + 1 == SW_STAGES ? 0 : stage + 1;
-          const uint32_t ph1 = stage + 1 == SW_STAGES ? phase ^ 1 : phase;
           mbar_wait(&full[stage], phase);
-          if (du) mbar_wait(&full[s1], ph1);
           if (trc) { const long long c = clock64(); c_full += c - c0; c0 = c; }
           tc_fence_after();
           if (kExperiments && lane == 0 && p.debug_mode == 1) {    // timing experiment: loads only (commit releases the stage)
@@ -350,15 +315,13 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
             // MMAs are issued by this one thread into the tensor pipe, which executes its
             // tcgen05.cp / tcgen05.mma in issue order: the copy into set s at kb = 4j + 8 runs
             // after the MMAs of kb = 4j .. 4j + 3 that read set s, whatever SW_STAGES is
-            const uint32_t set = FP8 ? ((kb >> 2) & 1) * SW_SF_SET : 0;
+            const uint32_t set = FP8 ? ((kb >> 2) & 1) * 16 : 0;
             if (FP8 && (kb & 3) == 0) {
               tmem_cp_32x128b_x4_pair(tmem + SW_SFA_COL + set, sf_desc(smem_u32(sSFW + stage * SW_SFW_BYTES)));
               tmem_cp_32x128b_x4_pair(tmem + SW_SFB_COL + set, sf_desc(smem_u32(sSFX + stage * SW_SFX_BYTES)));
               if (N > 128)                         // tokens 128..255 (a cp costs the pipe ~100 cycles)
                 tmem_cp_32x128b_x4_pair(tmem + SW_SFB_COL + set + 4,
                                         sf_desc(smem_u32(sSFX + stage * SW_SFX_BYTES + 512)));
-              if (du)                              // the second tile's tokens (one 128-row image)
-                tmem_cp_32x128b_x4_pair(tmem + SW_SFB1_COL + set, sf_desc(smem_u32(sSFX + s1 * SW_SFX_BYTES)));
             }
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
@@ -371,28 +334,12 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
               else
                 mma_bf16_pair(tmem, ad, bd, idesc_bf16(256, N), acc);
             }
-            if (du) {
-              const uint32_t b1 = smem_u32(sX + s1 * SW_X_BYTES);
-#pragma unroll
-              for (int k = 0; k < 4; ++k) {
-                const uint64_t ad = sw128_kmajor_desc(a0 + k * 32);
-                const uint64_t bd = sw128_kmajor_desc(b1 + k * 32);
-                const uint32_t acc = (kb | k) != 0;
-                if (FP8)
-                  mma_mxf8_pair(tmem + SW_ACC1_COL, ad, bd, idesc_mxf8(256, N1, kb & 3, kb & 3), acc,
-                                tmem + SW_SFA_COL + set, tmem + SW_SFB1_COL + set);
-                else
-                  mma_bf16_pair(tmem + SW_ACC1_COL, ad, bd, idesc_bf16(256, N1), acc);
-              }
-            }
             if (stage % SW_CE == SW_CE - 1) mma_commit_pair_mc(&empty[stage / SW_CE], kAllPairs);
-            if (du) mma_commit_pair_mc(&empty[s1], kAllPairs);
             if (kb == kblocks - 1) mma_commit_pair_mc(tmem_full, my_pair);
           }
           __syncwarp();
           if (trc) { const long long c = clock64(); c_issue += c - c0; c0 = c; }
           if (++stage == SW_STAGES) { stage = 0; phase ^= 1; }
-          if (du && ++stage == SW_STAGES) { stage = 0; phase ^= 1; }
         }
         acc_phase ^= 1;
       }
@@ -418,33 +365,25 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
       const SwapUnit ui = swap_unit(p, u, n_routed_units);
       if (!ui.valid) break;
       const SwapGroup &g = p.g[ui.group];
-      const int nb = ui.nb * NP + (int)pair;                 // this pair's weight block
-      // dual unit: the second (<= 128-row) tile first, 64 columns per warp half, its TMEM columns
-      // released at once (the next dual unit's second-tile MMAs wait only for that), then the
-      // 256-row tile as for a single unit
-      const bool du = ui.n > 256;
       mbar_wait(tmem_full, acc_phase);
       tc_fence_after();
-      for (int tt = du ? 1 : 0; tt >= 0; --tt) {
-      const int cw = tt ? 64 : 128;                          // columns per warp half
-      const int c0 = half * cw;
-      const int nvalid = max(0, min(cw, (tt == 0 ? min(ui.n, 256) : ui.n - 256) - c0));
+      const int c0 = half * 128;
+      const int nvalid = max(0, min(128, ui.n - c0));
       const int nch = (nvalid + 31) >> 5;
       uint32_t r[128];
 #pragma unroll
       for (int c = 0; c < 4; ++c)
-        if (c < nch)
-          tmem_ld_32x32b_x32(tmem + lane_base + tt * SW_ACC1_COL + c0 + c * 32, *reinterpret_cast<uint32_t(*)[32]>(r + 32 * c));
+        if (c < nch) tmem_ld_32x32b_x32(tmem + lane_base + c0 + c * 32, *reinterpret_cast<uint32_t(*)[32]>(r + 32 * c));
       tmem_ld_wait();
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) {                                       // this tile's accumulator columns are read
-        uint64_t *bar = tt ? tmem_empty1 : tmem_empty;
-        if (pleader) mbar_arrive(bar);
-        else mbar_arrive_remote(map_to_rank(bar, crank & ~1u));
+      if (lane == 0) {
+        if (pleader) mbar_arrive(tmem_empty);
+        else mbar_arrive_remote(map_to_rank(tmem_empty, crank & ~1u));
       }
-      if (tt == 0) acc_phase ^= 1;
-      const int64_t rbase = (int64_t)ui.row0 + tt * 256 + c0;   // token row of this half's column 0
+      acc_phase ^= 1;
+      const int64_t rbase = (int64_t)ui.row0 + c0;          // token row of this half's column 0
+      const int nb = ui.nb * NP + (int)pair;                 // this pair's weight block
       if (kExperiments && p.debug_mode >= 1) { ++tile_i; continue; }        // timing experiments: no epilogue math
       if constexpr (EPI == GEMM_PLAIN) {
         // transpose 32 tokens x 32 H rows per step through a per-warp smem tile,
@@ -590,7 +529,6 @@ __global__ void __launch_bounds__(SW_THREADS, 1) umma_swap_gemm(const __grid_con
         }
       }
       ++tile_i;
-      }
     }
   }
   tc_fence_before();

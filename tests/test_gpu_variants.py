@@ -1,9 +1,7 @@
 """Runtime-selectable kernel variants (environment knobs read once per process, so each
 runs the parity subset in a subprocess of its own):
-  MOE_SWAP_NP1/2=2  (with MOE_SWAP_DUAL=0) prefill grouped GEMMs on clusters of 2 CTA pairs, multicast token boxes
+  MOE_SWAP_NP1/2=2  prefill grouped GEMMs on clusters of 2 CTA pairs with multicast token boxes
                     (opt-in: measured slower on a B200, profiles/r02/swap_np.txt)
-  MOE_SWAP_DUAL=0   single token tiles only (no dual units); MOE_SWAP_DUAL_TAIL=128: dual units
-                    for experts of up to 384 tokens
   MOE_FD_CSIZE=C    the fused decode stream split over clusters of C CTAs, each cluster
                     taking several units from the queue (the cost model picks C otherwise)"""
 import os
@@ -18,9 +16,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 @pytest.mark.parametrize("env,select", [
-    ({"MOE_SWAP_NP1": "2", "MOE_SWAP_NP2": "2", "MOE_SWAP_DUAL": "0"}, "small_layer or swap_pair or prefill_8k"),
-    ({"MOE_SWAP_DUAL": "0"}, "small_layer or swap_pair or full_size"),
-    ({"MOE_SWAP_DUAL_TAIL": "128"}, "small_layer or swap_pair or prefill_8k or skewed"),
+    ({"MOE_SWAP_NP1": "2", "MOE_SWAP_NP2": "2"}, "small_layer or swap_pair or prefill_8k"),
     ({"MOE_FD_CSIZE": "2"}, "decode_shapes or fused_decode"),
     ({"MOE_FD_CSIZE": "4"}, "decode_shapes or fused_decode or mid_size_decode"),
     ({"MOE_FD_CSIZE": "8"}, "decode_shapes or fused_decode"),
