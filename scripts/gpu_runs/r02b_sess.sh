@@ -1,4 +1,4 @@
-# this session's net change: HEAD vs the session's starting commit 2d1588e (oldref_tmp), interleaved, every config (prefill)
+# this session net change, final: HEAD vs the session start 2d1588e (oldref_tmp), interleaved, every config (prefill)
 cd $GRAFT_REPO_ROOT
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || exit 1
 (cd oldref_tmp && python -c "import __graft_entry__ as g; g.build()" > ../gpurun_out/build_old.log 2>&1) || exit 1
