@@ -1012,7 +1012,7 @@ static int fd_cluster_size(const moe_layer *L, int units, int k_used, int T, boo
   // (2) Otherwise C = 2 when a cost model of the part after the router says so -- this
   //     layer's routed + shared units (a chained layer's group-2 units run beside the router):
   //     rounds x (unit time / C + split overhead), rounds = ceil(units / resident clusters),
-  //     unit time = its weight bytes at ~56 GB/s per SM, overhead 2.3 us, and >= 5 % cheaper
+  //     unit time = its weight bytes at ~56 GB/s per SM, overhead 1.5 us, and >= 2 % cheaper
   //     than C = 1.  Routed units use the expected number of distinct experts of T tokens.
   //     (Fitted to profiles/r02/decode_csize.txt: C = 2 wins when the post-router units fit
   //     one round of pairs -- V2-Lite / V2.5 chained deferral -- or leave a ragged third round
@@ -1033,8 +1033,8 @@ static int fd_cluster_size(const moe_layer *L, int units, int k_used, int T, boo
                                 : std::min((double)E, std::ceil(E * (1.0 - std::pow(1.0 - (double)k_now / E, T))));
     const int post = (with_shared ? L->Fs / 128 : 0) + (int)e_exp * (L->F / 128);
     const double c1 = (double)((post + n_cl(1) - 1) / n_cl(1)) * unit_us;
-    const double c2 = (double)((post + n_cl(2) - 1) / n_cl(2)) * (unit_us / 2 + 2.3);
-    if (c2 < 0.95 * c1) csize = 2;
+    const double c2 = (double)((post + n_cl(2) - 1) / n_cl(2)) * (unit_us / 2 + 1.5);
+    if (c2 < 0.98 * c1) csize = 2;
   }
   if (force_c == 1 || ((force_c == 2 || force_c == 4 || force_c == 8) && c_ok(force_c))) csize = force_c;
   *ncl_out = n_cl(csize);

@@ -4,7 +4,7 @@ the 8-layer chained CUDA graph (distinct V3 layers, L2 flushed before each repla
   deferral  -- moe_layer_forward_chained, n_def = 3 (last layer 0)
   deferral3_cyclic -- every layer defers; layer 0 takes the last layer's deferred experts of the
               previous replay (the steady state of a deep stack: no end layers)
-Prints per-layer µs for each variant and round."""
+Prints per-layer µs for each variant and round.  python scripts/decode_ab.py CONFIG ROUNDS [TOKENS]"""
 import json, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
@@ -17,8 +17,9 @@ NL, ROUNDS, STEPS = 8, int(sys.argv[2]) if len(sys.argv) > 2 else 4, 10
 p = PRESETS[cfg]
 w = make_weights(p, "cuda")
 layers = [moe.MoELayer(p, w, max_tokens=16) for _ in range(NL)]
-xd, _ = make_tokens(p, 4, "cuda", offset=1000)
-x0 = xd[:1].contiguous()
+TOK = int(sys.argv[3]) if len(sys.argv) > 3 else 1          # tokens per decode step
+xd, _ = make_tokens(p, max(4, TOK), "cuda", offset=1000)
+x0 = xd[:TOK].contiguous()
 bufs = [x0.clone(), torch.empty_like(x0)]
 flush = (torch.empty(64 << 20, device="cuda"), torch.zeros(64 << 20, device="cuda"), torch.zeros((), device="cuda"))
 
